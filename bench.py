@@ -1,0 +1,429 @@
+#!/usr/bin/env python
+"""bench.py -- BASELINE.json's metric on B200: effective HBM GB/s of the
+input-adaptive TMV/MV path (Adaptic, PLDI'12), printed as ONE JSON line.
+
+Workloads (``--workload``):
+  sweep    (default, BJ:configs[1]) one step = the selector-chosen kernel on all 42
+           problems of the fixed-256-MiB shape sweep: R x C = 2^k x 2^(26-k),
+           k = 3..23, in both layouts (MV: A row-major R x C; TMV: B = A^T).
+  rowshard (BJ:configs[3]) MV 131072 x 32768 fp32, rows sharded over ranks.
+  splitk   (BJ:configs[4]) TMV 1024 x 16M fp32, C split over ranks + NCCL all-reduce.
+  dot      (BJ:configs[2]) scalar product N = 1, L = 2^10..2^30 (fp32).
+Multi-GPU: one process per GPU (torchrun), barrier + synchronize around the
+timed region, max elapsed over ranks; ``value`` = bytes of all ranks / that time.
+
+``--impl reference`` times the CPU oracle (there is no reference code; see
+DESIGN.md) on a bounded sample of the same workload, rank 0 only.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "TMV/MV effective HBM GB/s and % of B200 peak across rows×cols sweep, 1/2/4/8 GPU"
+UNIT = "GB/s"
+GiB = 1 << 30
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", choices=["adaptic", "reference"], default="adaptic")
+    ap.add_argument("--workload", choices=["sweep", "rowshard", "splitk", "dot"], default="sweep")
+    ap.add_argument("--variant", default="AUTO", help="force one variant (fixed-variant sweeps)")
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--detail", default=None, help="write per-problem JSONL here")
+    return ap.parse_args()
+
+
+# ------------------------------------------------------------------------------ helpers
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class Clocks:
+    """nvidia-smi sampler running during the timed region (the recipe's clocks line)."""
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                 "-lms", "50"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+            time.sleep(0.15)
+        except FileNotFoundError:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"], "samples": 0}
+        time.sleep(0.1)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [p.strip() for p in ln.split(",")]
+            if len(parts) < 7:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                mx.append(float(parts[1]))
+            except ValueError:
+                continue
+            for n, v in zip(names, parts[3:7]):
+                if v.lower() in ("active", "1", "yes"):
+                    reasons.add(n)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def dist_setup():
+    import torch
+    import torch.distributed as dist
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    else:
+        torch.cuda.set_device(0)
+    return world, rank, local
+
+
+def barrier(world):
+    import torch.distributed as dist
+    if world > 1:
+        dist.barrier()
+
+
+def max_over_ranks(v: float, world: int) -> float:
+    if world == 1:
+        return v
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([v], dtype=torch.float64, device="cuda")
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+# ------------------------------------------------------------------------------ problems
+class Problem:
+    """One (op, R, C) instance, resident in HBM, with its selected plan."""
+
+    def __init__(self, op, R, C, cfg, variant="AUTO", shard=None, full=None):
+        import torch
+        import synth
+        import paper_conf_pldi_samadihmlm12_b200 as adaptic
+        from paper_conf_pldi_samadihmlm12_b200 import _lib as L
+        self.op, self.R, self.C = op, R, C
+        dev = torch.device("cuda", torch.cuda.current_device())
+        Rf, Cf = full if full else (R, C)           # logical full problem (shards are slices)
+        rows, cols = shard if shard else ((0, R), (0, C))
+        self.M = torch.empty(R * C, dtype=torch.float32, device=dev)
+        layout = "tmv" if op == "tmv" else "mv"
+        synth.device_matrix(self.M, Rf, Cf, layout, "uniform", synth.seed(cfg, "A"), rows=rows, cols=cols)
+        if op == "dot":
+            self.X = torch.empty(R * C, dtype=torch.float32, device=dev)
+            synth.device_matrix(self.X, Rf, Cf, "mv", "uniform", synth.seed(cfg, "b"), rows=rows, cols=cols)
+        else:
+            self.X = torch.empty(C, dtype=torch.float32, device=dev)
+            synth.device_vector(self.X, "uniform", synth.seed(cfg, "x"), start=cols[0])
+        self.y = torch.empty(R, dtype=torch.float32, device=dev)
+        opc = {"mv": L.OP_MV, "tmv": L.OP_TMV, "dot": L.OP_DOT}[op]
+        self.stream = torch.cuda.current_stream().cuda_stream
+        self.plan = adaptic.get_plan(opc, R, C, L.F32, dev, variant, None, self.stream)
+        self.desc = self.plan.describe()
+        self.bytes = 4 * (R * C + C + R) if op != "dot" else 4 * (2 * R * C + R)   # algorithmic
+        self.ptrs = (self.M.data_ptr(), self.X.data_ptr(), self.y.data_ptr())
+
+    def launch(self):
+        self.plan.run(*self.ptrs, self.stream)
+
+    def key(self):
+        return f"{self.op}:{self.R}x{self.C}:{self.desc['variant']}"
+
+
+def build_problems(args, world, rank):
+    if args.workload == "sweep":
+        return [Problem(op, 1 << k, 1 << (26 - k), 1, args.variant)
+                for k in range(3, 24) for op in ("mv", "tmv")], \
+            {"workload": "configs[1]: TMV/MV fp32 shape sweep at 256 MiB, 8Mx8 .. 8192x8192 .. 8x8M, "
+                         "both layouts, variant selector", "shapes": 42, "per_gpu": "full sweep (weak)"}
+    if args.workload == "dot":
+        return [Problem("dot", 1, 1 << k, 2, args.variant) for k in range(10, 31)], \
+            {"workload": "configs[2]: scalar product fp32 N=1, L=2^10..2^30", "shapes": 21}
+    from paper_conf_pldi_samadihmlm12_b200.dist import shard_range
+    if args.workload == "rowshard":
+        R, C = 131072, 32768
+        r0, r1 = shard_range(R, world, rank)
+        return [Problem("mv", r1 - r0, C, 3, args.variant, shard=((r0, r1), (0, C)), full=(R, C))], \
+            {"workload": "configs[3]: MV fp32 131072x32768 row-sharded, no collective", "rows_per_rank": r1 - r0}
+    R, C = 1024, 1 << 24
+    c0, c1 = shard_range(C, world, rank)
+    return [Problem("tmv", R, c1 - c0, 4, args.variant, shard=((0, R), (c0, c1)), full=(R, C))], \
+        {"workload": "configs[4]: TMV fp32 1024x16M split-K + NCCL all_reduce", "cols_per_rank": c1 - c0}
+
+
+# ------------------------------------------------------------------------------ adaptic arm
+def run_adaptic(args):
+    import torch
+    import torch.distributed as dist
+    world, rank, local = dist_setup()
+    probs, config = build_problems(args, world, rank)
+    splitk = args.workload == "splitk" and world > 1
+    torch.cuda.synchronize()
+    n = len(probs)
+    step_bytes = sum(p.bytes for p in probs)
+
+    def one_step(evs=None):
+        for i, p in enumerate(probs):
+            if evs is not None:
+                evs[i].record()
+            p.launch()
+        if evs is not None:
+            evs[n].record()
+        if splitk:
+            dist.all_reduce(probs[0].y, op=dist.ReduceOp.SUM)
+
+    for _ in range(max(3, args.warmup)):
+        one_step()
+    torch.cuda.synchronize()
+
+    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(n + 1)] for _ in range(args.steps)]
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    clocks = Clocks(torch.cuda.current_device())
+    clocks.start()
+    barrier(world)
+    torch.cuda.synchronize()
+    t0.record()
+    for s in range(args.steps):
+        one_step(evs[s])
+    t1.record()
+    torch.cuda.synchronize()
+    barrier(world)
+    clk = clocks.stop()
+    elapsed_ms = max_over_ranks(t0.elapsed_time(t1), world)
+    value = world * step_bytes * args.steps / (elapsed_ms / 1e3) / 1e9
+
+    # per-kernel durations (CUDA events on the launching stream)
+    dur = [[evs[s][i].elapsed_time(evs[s][i + 1]) for s in range(args.steps)] for i in range(n)]
+    mean_ms = [statistics.mean(d) for d in dur]
+    peak, peak_src = peaks()
+    per = []
+    for i, p in enumerate(probs):
+        gbs = p.bytes / (mean_ms[i] / 1e3) / 1e9
+        per.append({"op": p.op, "R": p.R, "C": p.C, "variant": p.desc["variant"], "us": mean_ms[i] * 1e3,
+                    "us_median": statistics.median(dur[i]) * 1e3, "GBps": gbs, "frac": gbs / peak,
+                    "bytes": p.bytes, "share": mean_ms[i] / sum(mean_ms), "plan": p.desc})
+    dom = max(range(n), key=lambda i: mean_ms[i])
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(tpath):
+        with open(tpath) as f:
+            traffic = json.load(f).get(probs[dom].key())
+    roofline = {"bound": "hbm", "achieved": per[dom]["GBps"], "peak": peak, "unit": "GB/s",
+                "frac": per[dom]["GBps"] / peak, "traffic": traffic,
+                "kernel": probs[dom].key(), "peak_source": peak_src,
+                "step_frac": value / world / peak,
+                "min_frac": min(q["frac"] for q in per), "min_kernel": min(per, key=lambda q: q["frac"])["variant"]
+                + f" {min(per, key=lambda q: q['frac'])['op']} {min(per, key=lambda q: q['frac'])['R']}x"
+                f"{min(per, key=lambda q: q['frac'])['C']}",
+                "median_frac": statistics.median(q["frac"] for q in per)}
+
+    e2e = None
+    if not args.no_e2e and args.e2e_steps > 0:
+        e2e = measure_e2e(args, probs, world)
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline(probs, args)
+    if args.detail and rank == 0:
+        with open(args.detail, "w") as f:
+            for q in per:
+                f.write(json.dumps(q) + "\n")
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": elapsed_ms / args.steps, "higher_is_better": True,
+                "scaling": "weak" if args.workload in ("sweep", "dot") else "strong",
+                "vs_baseline": None, "dtype": "f32", "data": "synthetic (seeded splitmix64, U[-1,1))",
+                "config": dict(config, bytes_per_step_per_gpu=step_bytes, variant=args.variant,
+                               l2="every input >= 256 MiB > 126 MB L2 and problems alternate; no flush needed"
+                               if args.workload == "sweep" else "inputs > L2; no flush needed"),
+                "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
+                "gpu_launches": n * args.steps, "clocks": clk,
+                "selected": {q["op"] + f" {q['R']}x{q['C']}": [q["variant"], round(q["frac"], 3)] for q in per}}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def measure_e2e(args, probs, world):
+    """Same metric through the C ABI with HOST buffers: every step copies each problem's
+    inputs host->device (pinned), runs the kernel, and reads y back."""
+    import torch
+    import psutil
+    need = sum(p.M.numel() * 4 + p.X.numel() * 4 for p in probs)
+    sel = probs
+    if need > 0.5 * psutil.virtual_memory().available:
+        k = max(1, int(len(probs) * 0.5 * psutil.virtual_memory().available / need))
+        sel = probs[:: max(1, len(probs) // k)]
+    hosts = []
+    for p in sel:
+        Mh = torch.empty(p.M.numel(), dtype=torch.float32, pin_memory=True)
+        Xh = torch.empty(p.X.numel(), dtype=torch.float32, pin_memory=True)
+        Mh.copy_(p.M)
+        Xh.copy_(p.X)
+        yh = torch.empty(p.R, dtype=torch.float32, pin_memory=True)
+        hosts.append((Mh.data_ptr(), Xh.data_ptr(), yh.data_ptr(), Mh, Xh, yh))
+    torch.cuda.synchronize()
+
+    def step():
+        for p, h in zip(sel, hosts):
+            p.plan.run_host(h[0], h[1], h[2], p.ptrs[0], p.ptrs[1], p.ptrs[2], p.stream)
+
+    step()
+    torch.cuda.synchronize()
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    barrier(world)
+    torch.cuda.synchronize()
+    t0.record()
+    for _ in range(args.e2e_steps):
+        step()
+    t1.record()
+    torch.cuda.synchronize()
+    barrier(world)
+    ms = max_over_ranks(t0.elapsed_time(t1), world)
+    b = sum(p.bytes for p in sel)
+    h2d = sum(p.M.numel() * 4 + p.X.numel() * 4 for p in sel)
+    d2h = sum(p.R * 4 for p in sel)
+    return {"value": world * b * args.e2e_steps / (ms / 1e3) / 1e9, "unit": UNIT,
+            "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h, "steps": args.e2e_steps,
+            "problems": len(sel), "api": "adaptic_run_host (C ABI, pinned host buffers)"}
+
+
+def cpu_baseline(probs, args, budget_s: float = 20.0):
+    """The fp64 oracle as it stands, single-threaded, on the box's host cores, over a
+    bounded sample of the workload's problems (inputs copied from HBM)."""
+    import numpy as np
+    import oracle
+    t_total, b_total, names = 0.0, 0, []
+    order = sorted(range(len(probs)), key=lambda i: (i * 7) % len(probs))
+    for i in order:
+        p = probs[i]
+        M = p.M.cpu().numpy()
+        X = p.X.cpu().numpy()
+        t = time.perf_counter()
+        if p.op == "mv":
+            oracle.mv(M.reshape(p.R, p.C), X)
+        elif p.op == "tmv":
+            oracle.tmv(M.reshape(p.C, p.R), X)
+        else:
+            oracle.dot(M.reshape(p.R, p.C), X.reshape(p.R, p.C))
+        t_total += time.perf_counter() - t
+        b_total += p.bytes
+        names.append(f"{p.op} {p.R}x{p.C}")
+        del M, X
+        if t_total > budget_s:
+            break
+    return {"value": b_total / t_total / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "seconds": t_total, "host_cores_available": os.cpu_count(),
+            "sample": f"{len(names)} of {len(probs)} problems, full size: " + ", ".join(names[:6])
+                      + (" ..." if len(names) > 6 else "")}
+
+
+# ------------------------------------------------------------------------------ reference arm
+def run_reference(args):
+    """The CPU oracle on a bounded sample of the same workload (rank 0 only)."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import numpy as np
+    import oracle
+    import synth
+    if args.workload == "sweep":
+        pool = [("mv", 1 << 13, 1 << 13), ("tmv", 1 << 13, 1 << 13), ("mv", 1 << 20, 64), ("tmv", 64, 1 << 20)]
+        cfg = 1
+    elif args.workload == "dot":
+        pool = [("dot", 1, 1 << 26)]
+        cfg = 2
+    elif args.workload == "rowshard":
+        pool = [("mv", 2048, 32768)]
+        cfg = 3
+    else:
+        pool = [("tmv", 1024, 1 << 16)]
+        cfg = 4
+    data = []
+    for op, R, C in pool:
+        if op == "dot":
+            a = synth.matrix(R, C, "mv", np.float32, "uniform", synth.seed(cfg, "A"))
+            b = synth.matrix(R, C, "mv", np.float32, "uniform", synth.seed(cfg, "b"))
+            data.append((op, R, C, a, b, 4 * (2 * R * C + R)))
+        else:
+            M = synth.matrix(R, C, op, np.float32, "uniform", synth.seed(cfg, "A"))
+            x = synth.vector(C, np.float32, "uniform", synth.seed(cfg, "x"))
+            data.append((op, R, C, M, x, 4 * (R * C + R + C)))
+    fns = {"mv": oracle.mv, "tmv": oracle.tmv, "dot": oracle.dot}
+    for s in range(args.warmup):
+        op, R, C, M, X, _ = data[s % len(data)]
+        fns[op](M, X)
+    t = time.perf_counter()
+    nbytes = 0
+    for s in range(args.steps):
+        op, R, C, M, X, b = data[s % len(data)]
+        fns[op](M, X)
+        nbytes += b
+    el = time.perf_counter() - t
+    value = nbytes / el / 1e9
+    sample = "one problem per step, cycling: " + ", ".join(f"{op} {R}x{C}" for op, R, C, *_ in data)
+    print(json.dumps({
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": el / args.steps * 1e3,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64 (oracle)",
+        "data": "synthetic (seeded splitmix64, U[-1,1))",
+        "config": {"workload": f"{args.workload} (bounded CPU sample)", "note": "no reference code exists; "
+                   "the reference arm is the single-threaded fp64 CPU oracle (oracle/oracle.c)"},
+        "cpu_baseline": {"value": value, "unit": UNIT, "kind": "oracle", "cores": 1, "sample": sample},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}), flush=True)
+
+
+if __name__ == "__main__":
+    a = parse()
+    if a.impl == "reference":
+        run_reference(a)
+    else:
+        run_adaptic(a)

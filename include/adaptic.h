@@ -1,0 +1,216 @@
+/*
+ * adaptic.h -- C ABI of the B200-native input-adaptive reduction library.
+ *
+ * What it computes (P:N = line N of the paper text, PAPER.md, Samadi et al.,
+ * "Adaptive Input-aware Compilation for Graphics Engines", PLDI'12):
+ *
+ *   The hot path is the paper's stream-reduction actor (Sec. 4.2.1): a kernel
+ *   that "receives N_arrays different arrays with N_elements elements each as
+ *   input, and produces one element per array as output", evaluated by
+ *   a tree over an associative and commutative operator -- here
+ *   multiply-accumulate.  Three operations use it:
+ *
+ *     ADAPTIC_OP_MV   y[r] = sum_c A[r*C + c] * x[c]     A row-major R x C
+ *                     (each output is "the dot product of one row with the
+ *                     input vector"; reductions are contiguous)
+ *     ADAPTIC_OP_TMV  y[r] = sum_c B[c*R + r] * x[c]     B row-major C x R, B = A^T
+ *                     (the paper's memory-restructured layout, Fig. 3 /
+ *                     thread t's k-th pop reads word T*k + t; outputs
+ *                     are contiguous, reductions are strided).  TMV(B) == MV(B^T).
+ *     ADAPTIC_OP_DOT  y[n] = sum_e a[n*L + e] * b[n*L + e]  (Scalar Product,
+ *                     "scalar products of pairs of vectors"; Sdot is
+ *                     N = 1).  rows = N, cols = L, x := b (N x L).
+ *
+ *   For every op, `rows` (R) is the number of outputs and `cols` (C) is the
+ *   reduction length (reading R1).
+ *
+ * The input-adaptive part (Fig. 2): adaptic_plan() is the paper's
+ * "runtime kernel management" -- on the CPU, from the actual input dimensions,
+ * it selects one of several hand-written kernels and fixes its launch
+ * parameters (blocks, threads, shared memory).  The selection comes from
+ * a threshold table fitted on B200 sweeps (not from the paper, whose break-even
+ * points were for a Tesla C2050).  The variants map to the paper's five TMV
+ * kernels:
+ *
+ *     MV_TPR      K5  thread per row; rows staged in shared memory by the TMA
+ *                     bulk-copy engine (the paper's shared-memory alternative to
+ *                     restructuring)
+ *     MV_SUBWARP  K4  g lanes per row (g = 1..16), shuffle reduction
+ *     MV_WPR      K3  warp per row, several rows per CTA (horizontal thread
+ *                     integration)
+ *     MV_CPR      K2  CTA per row, single-kernel reduction (Fig. 7b)
+ *     MV_SPLIT    K1  several CTAs per row + merge (two-phase reduction, P:480,
+ *                     Fig. 7c); the merge is done in the same kernel by the last
+ *                     CTA to finish a row (atomic ticket), in fixed order
+ *     TMV_COL     K5 on the restructured layout: thread per 4 outputs, loop over c
+ *     TMV_SPLITK  2-D tiles of outputs x c-ranges, CTA combine + ticket merge
+ *     TMV_REGTILE TMV_SPLITK whose tile holds every output (R <= 1024)
+ *   DOT uses the MV variants with a per-row second operand.
+ *
+ * Arithmetic (readings R4, R5):
+ *   ADAPTIC_F32: fp32 inputs, fp32 accumulation, round-to-nearest-even, FMA
+ *     contraction allowed, no FTZ / fast-math.  Summation order is a tree
+ *     whose serial chain per accumulator is <= 1024 terms, so every output is
+ *     within 1e-4 * sum_c |a(r,c) x_c| of the exact value.  Different variants
+ *     may return different roundings; a given plan is deterministic (it does not
+ *     depend on CTA arrival order).
+ *   ADAPTIC_I32: int32 inputs; products and sums modulo 2^32 (two's
+ *     complement wrap).  Bit-exact for every variant.
+ *   alpha = 1, beta = 0: y is fully overwritten; A and x are never written.
+ *
+ * Conventions:
+ *   - Sizes are int64_t.  rows < 0 or cols < 0, or rows*cols*4 overflowing
+ *     size_t -> ADAPTIC_ERR_INVALID_ARG.  rows == 0: success, nothing launched.
+ *     cols == 0: y is zero-filled (one memset on the stream).
+ *   - Pointers passed to adaptic_run are DEVICE pointers owned by the caller
+ *     (PyTorch allocates them); they must stay valid until the stream work
+ *     completes.  The library never allocates device memory.
+ *   - Pointers must be element (4-byte) aligned, else ADAPTIC_ERR_MISALIGNED.
+ *     16-byte aligned A/x/y with a multiple-of-4 contiguous extent use 128-bit
+ *     loads; anything else runs the same variant's scalar-load instance
+ *     (correct, slower).
+ *   - y must not overlap A or x (byte ranges), else ADAPTIC_ERR_ALIAS.
+ *   - Variants that merge across CTAs (MV_SPLIT, TMV_SPLITK, TMV_REGTILE with
+ *     splits > 1) need a workspace of adaptic_plan_workspace_bytes() bytes,
+ *     device memory, ZERO-FILLED when attached with adaptic_plan_set_workspace;
+ *     every run leaves it zero-filled again.  Running such a plan without one
+ *     returns ADAPTIC_ERR_NO_WORKSPACE.  One plan with a workspace must not run
+ *     on two streams concurrently.
+ *   - adaptic_run only enqueues work on `stream` (cudaStream_t; NULL = legacy
+ *     default stream) and returns; launch errors are reported as
+ *     ADAPTIC_ERR_CUDA with the cudaError_t available from
+ *     adaptic_last_cuda_error() (thread-local).  Sticky CUDA errors are not
+ *     cleared.  No entry point aborts.
+ *   - Plans are immutable after creation except for the attached workspace;
+ *     adaptic_plan / adaptic_plan_forced are thread-safe.  A plan is computed
+ *     for the SM count of the device current at plan time (148 on B200; 148
+ *     is assumed if no device is present, so planning works on a CPU host).
+ */
+#ifndef ADAPTIC_H_
+#define ADAPTIC_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define ADAPTIC_ABI_VERSION 1
+
+typedef enum {
+    ADAPTIC_OK = 0,
+    ADAPTIC_ERR_INVALID_ARG = 1,   /* bad op/dtype/variant/size, NULL plan or pointer  */
+    ADAPTIC_ERR_UNSUPPORTED = 2,   /* forced variant cannot run this op / shape        */
+    ADAPTIC_ERR_MISALIGNED = 3,    /* a pointer is not 4-byte aligned                  */
+    ADAPTIC_ERR_ALIAS = 4,         /* y overlaps A or x                                */
+    ADAPTIC_ERR_NO_WORKSPACE = 5,  /* plan needs a workspace and has none / too small  */
+    ADAPTIC_ERR_CUDA = 6           /* a CUDA runtime call failed; see last_cuda_error  */
+} adaptic_status;
+
+typedef enum {
+    ADAPTIC_OP_MV = 0,    /* y[R] = A x,    A row-major R x C                       */
+    ADAPTIC_OP_TMV = 1,   /* y[R] = B^T x,  B row-major C x R                       */
+    ADAPTIC_OP_DOT = 2    /* y[N] = <a_n, b_n>, a and b row-major N x L; x := b     */
+} adaptic_op;
+
+typedef enum {
+    ADAPTIC_F32 = 0,      /* fp32 in / fp32 accumulate                              */
+    ADAPTIC_I32 = 1       /* int32, arithmetic modulo 2^32                          */
+} adaptic_dtype;
+
+typedef enum {
+    ADAPTIC_V_AUTO = 0,
+    ADAPTIC_V_MV_TPR = 1,
+    ADAPTIC_V_MV_SUBWARP = 2,
+    ADAPTIC_V_MV_WPR = 3,
+    ADAPTIC_V_MV_CPR = 4,
+    ADAPTIC_V_MV_SPLIT = 5,
+    ADAPTIC_V_TMV_COL = 6,
+    ADAPTIC_V_TMV_SPLITK = 7,
+    ADAPTIC_V_TMV_REGTILE = 8,
+    ADAPTIC_V_COUNT = 9
+} adaptic_variant;
+
+/* Optional parameters for adaptic_plan_forced: an array of ADAPTIC_NPARAMS
+ * int32 values (ADAPTIC_NPARAMS of them); a value <= 0 means "choose automatically".
+ *   [ADAPTIC_P_LANES]  MV_SUBWARP: lanes per row g in {1,2,4,8,16};
+ *                      MV_CPR / MV_SPLIT: threads per CTA in {256, 1024};
+ *                      TMV_*: float4 lanes along the outputs per CTA tile,
+ *                      a power of two in [1, 256].
+ *   [ADAPTIC_P_SPLITS] MV_SPLIT / TMV_SPLITK / TMV_REGTILE: CTAs per
+ *                      reduction (split count S >= 1).
+ *   [ADAPTIC_P_CTAS_PER_SM] target resident CTAs per SM used to size grids.
+ *   [ADAPTIC_P_UNROLL] independent 128-bit loads per thread per step {1,2,4,8}
+ *                      (MV_TPR: pipeline stages 2..8).
+ *   [ADAPTIC_P_XSMEM]  MV_SUBWARP / MV_WPR / MV_CPR: 1 = read x through the
+ *                      read-only cache path, 2 = stage x in shared memory once per
+ *                      CTA with a TMA bulk copy (needs cols*4 <= 200 KB). */
+#define ADAPTIC_P_LANES 0
+#define ADAPTIC_P_SPLITS 1
+#define ADAPTIC_P_CTAS_PER_SM 2
+#define ADAPTIC_P_UNROLL 3
+#define ADAPTIC_P_XSMEM 4
+#define ADAPTIC_NPARAMS 5
+
+typedef struct adaptic_plan_s* adaptic_plan_t;   /* opaque; owned by the caller */
+
+/* Selector (host only, O(1), no device work): picks the variant and its launch
+ * parameters for (op, rows, cols, dtype) from the fitted threshold table.
+ * *out receives a new plan (free with adaptic_plan_destroy). */
+adaptic_status adaptic_plan(adaptic_op op, int64_t rows, int64_t cols, adaptic_dtype dtype,
+                            adaptic_plan_t* out);
+
+/* Same, with the variant fixed by the caller (fixed-variant sweeps and tests).
+ * params: NULL or ADAPTIC_NPARAMS values as above.  Returns
+ * ADAPTIC_ERR_UNSUPPORTED if the variant does not implement `op`. */
+adaptic_status adaptic_plan_forced(adaptic_op op, int64_t rows, int64_t cols,
+                                   adaptic_dtype dtype, adaptic_variant variant,
+                                   const int32_t* params, adaptic_plan_t* out);
+
+/* What the plan will run. */
+adaptic_variant adaptic_plan_variant(adaptic_plan_t plan);
+
+/* Plan details as a NUL-terminated JSON object (variant, grid, block, lanes,
+ * splits, unroll, chain, workspace bytes ...).  Writes at most `cap` bytes;
+ * returns the full length needed (excluding the NUL), or -1 on a NULL plan. */
+int adaptic_plan_describe(adaptic_plan_t plan, char* buf, size_t cap);
+
+/* Device workspace the plan needs (0 for single-phase variants). */
+size_t adaptic_plan_workspace_bytes(adaptic_plan_t plan);
+
+/* Attach a caller-owned, zero-filled device buffer of >= workspace_bytes bytes
+ * (NULL with bytes = 0 detaches).  ADAPTIC_ERR_NO_WORKSPACE if too small. */
+adaptic_status adaptic_plan_set_workspace(adaptic_plan_t plan, void* dev_ptr, size_t bytes);
+
+/* Enqueue y = op(A, x) on `stream` (a cudaStream_t passed as void*).
+ * A, x, y: device pointers (see conventions above).  Asynchronous. */
+adaptic_status adaptic_run(adaptic_plan_t plan, const void* A, const void* x, void* y,
+                           void* stream);
+
+/* End-to-end form with HOST buffers: enqueue on `stream` the host->device copy
+ * of A and x into the caller's device buffers dA, dx (sizes as for
+ * adaptic_run), the kernel into dy, and the device->host copy of dy into y_host.
+ * For MV/DOT the copy of A is split into row blocks so that each block's
+ * reduction overlaps the next block's transfer.  Host buffers should be
+ * page-locked for the copies to be asynchronous.  Returns after enqueueing;
+ * the caller synchronises the stream before reading y_host. */
+adaptic_status adaptic_run_host(adaptic_plan_t plan, const void* A_host, const void* x_host,
+                                void* y_host, void* dA, void* dx, void* dy, void* stream);
+
+void adaptic_plan_destroy(adaptic_plan_t plan);
+
+const char* adaptic_status_string(adaptic_status status);
+const char* adaptic_variant_name(adaptic_variant variant);
+
+/* cudaError_t of the last failing CUDA call made by this thread (0 if none). */
+int adaptic_last_cuda_error(void);
+
+/* ADAPTIC_ABI_VERSION of the loaded library. */
+int adaptic_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* ADAPTIC_H_ */

@@ -1,0 +1,657 @@
+// adaptic.cu -- planner (runtime variant selector) and the C ABI of include/adaptic.h.
+//
+// The paper's "runtime kernel management" (Fig. 2): executed on the CPU,
+// it selects the kernel generated for the subrange containing the actual input
+// and sets "the number of blocks, number of threads per block, and the size of
+// allocated shared memory".  Here the subranges are the cells of a 2-D table
+// over (floor(log2 R), floor(log2 C)) per (op, dtype), fitted from B200 sweeps
+// (tools/fit_thresholds.py -> table_data.inc); a cell that was not measured
+// takes the nearest measured cell, and a problem far from every cell falls back
+// to the analytic rules in heuristic_variant() (the paper's break-even idea,
+// P:222-232, reduced to parallelism counts).
+#include "adaptic.h"
+#include "launch.h"
+
+#include <algorithm>
+#include <atomic>
+#include <climits>
+#include <cmath>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <mutex>
+#include <string>
+
+using namespace adaptic;
+
+struct adaptic_plan_s {
+    int op, dtype;
+    int64_t R, C;
+    int variant;
+    int source;            // 0 forced, 1 table, 2 heuristic
+    int sms;
+    // kernel parameters
+    int lanes;             // G (group) | NT (cta, tpr) | LR (tmv)
+    int unroll;            // U
+    int rb;                // group: rows per lane group per step (8 / U)
+    int splits;            // S
+    int ctas_per_sm;
+    int stages;            // TPR
+    int xmode;             // MV family: 0 x via read-only path, 1 x staged in smem (TMA), 2 per-row (DOT)
+    size_t smem;           // dynamic shared memory bytes (TPR ring, or staged x)
+    int block;
+    bool vec_shape;        // C % 4 == 0 (MV/DOT) or R % 4 == 0 (TMV)
+    int64_t grid[2];       // [scalar, vector] instance
+    int64_t chain[2];      // longest serial chain per accumulator
+    int64_t depth[2];      // combine-tree depth after the chains
+    bool path_ok[2];       // error bound provable for this instance
+    // scalar fallback for TPR (misaligned pointers): a group kernel
+    int fb_lanes, fb_unroll;
+    // workspace
+    size_t ws_bytes, cnt_off;
+    void* ws;
+    size_t ws_cap;
+};
+
+namespace {
+
+thread_local int g_last_cuda_error = 0;
+
+struct TableEntry {
+    int op, dtype, lr, lc, variant, lanes, splits, ctas_per_sm, unroll, xsmem;
+};
+const TableEntry kTable[] = {
+#include "table_data.inc"
+    {-1, -1, 0, 0, 0, 0, 0, 0, 0, 0}};
+const int kTableN = int(sizeof(kTable) / sizeof(kTable[0])) - 1;
+
+const char* const kVariantNames[ADAPTIC_V_COUNT] = {
+    "AUTO", "MV_TPR", "MV_SUBWARP", "MV_WPR", "MV_CPR", "MV_SPLIT",
+    "TMV_COL", "TMV_SPLITK", "TMV_REGTILE"};
+
+constexpr double kUnitRoundoff = 5.9604644775390625e-08;  // 2^-24
+constexpr double kTol = 1e-4;                              // north_star tolerance
+
+int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+int ilog2_floor(int64_t v) { int k = -1; while (v > 0) { v >>= 1; ++k; } return k; }
+int64_t pow2_ceil(int64_t v) { int64_t p = 1; while (p < v) p <<= 1; return p; }
+int clampi(int64_t v, int lo, int hi) { return int(std::max<int64_t>(lo, std::min<int64_t>(hi, v))); }
+
+struct DevInfo { int dev; int sms; bool present; };
+
+DevInfo device_info() {
+    DevInfo d{-1, 148, false};
+    int dev = -1;
+    if (cudaGetDevice(&dev) == cudaSuccess) {
+        int sms = 0;
+        if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) == cudaSuccess && sms > 0) {
+            d.dev = dev; d.sms = sms; d.present = true;
+        }
+    }
+    if (!d.present) (void)cudaGetLastError();   // a CPU host: clear the non-sticky error
+    return d;
+}
+
+bool is_mv_family(int v) { return v >= ADAPTIC_V_MV_TPR && v <= ADAPTIC_V_MV_SPLIT; }
+bool is_tmv_family(int v) { return v >= ADAPTIC_V_TMV_COL && v <= ADAPTIC_V_TMV_REGTILE; }
+
+void* group_fn(int dtype, int G, int U, bool vec, int xm) {
+    return dtype == DT_F32 ? group_fn_f32(G, U, vec, xm) : group_fn_i32(G, U, vec, xm);
+}
+
+constexpr int64_t kXsAutoBytes = 32 * 1024;    // stage x in smem by default up to this size
+constexpr int64_t kXsMaxBytes = 200 * 1024;
+
+// x mode for the MV family: DOT streams its per-row operand; otherwise staged
+// in shared memory when requested (param 2) or small enough (auto).
+int pick_xmode(bool px, int req, int64_t C, bool allow) {
+    if (px) return 2;
+    if (!allow) return 0;
+    if (req == 2) return C * 4 <= kXsMaxBytes ? 1 : -1;
+    if (req == 1) return 0;
+    return C * 4 <= kXsAutoBytes ? 1 : 0;
+}
+void* tmv_fn(int dtype, int LR, int U, bool vec) {
+    return dtype == DT_F32 ? tmv_fn_f32(LR, U, vec) : tmv_fn_i32(LR, U, vec);
+}
+
+int occupancy(void* fn, int block, size_t smem, bool present, int fallback) {
+    if (!present || fn == nullptr) return fallback;
+    int n = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, fn, block, smem) != cudaSuccess || n <= 0) {
+        (void)cudaGetLastError();
+        return fallback;
+    }
+    return n;
+}
+
+// Error bound of a tree whose longest path has `m` roundings (Higham eq. 4.4).
+bool bound_ok(int64_t m) {
+    const double mu = double(m) * kUnitRoundoff;
+    return mu < 1.0 && mu / (1.0 - mu) <= kTol;
+}
+int64_t fold_chain(int64_t iters) { return std::min<int64_t>(iters, FOLD) + iters / FOLD; }
+int ilog2c(int64_t v) { int k = 0; while ((int64_t(1) << k) < v) ++k; return k; }
+
+// ---------------------------------------------------------------- heuristic (no table cell)
+int heuristic_variant(int op, int64_t R, int64_t C, int sms) {
+    if (op == ADAPTIC_OP_TMV) {
+        const int64_t rv = (R % 4 == 0) ? R / 4 : R;
+        if (rv >= int64_t(sms) * 512 && C <= 4096) return ADAPTIC_V_TMV_COL;
+        if (rv <= 256) return ADAPTIC_V_TMV_REGTILE;
+        return ADAPTIC_V_TMV_SPLITK;
+    }
+    const int64_t nv = (C % 4 == 0) ? C / 4 : C;
+    if (nv <= 16 && R >= 4096) return ADAPTIC_V_MV_SUBWARP;
+    if (nv <= 4096 && R >= 8192) return ADAPTIC_V_MV_WPR;
+    if (R >= 2 * int64_t(sms) && nv <= 4 * 1024 * 1024) return ADAPTIC_V_MV_CPR;
+    return ADAPTIC_V_MV_SPLIT;
+}
+
+const TableEntry* table_lookup(int op, int dtype, int64_t R, int64_t C) {
+    const int lr = ilog2_floor(R), lc = ilog2_floor(C);
+    const TableEntry* best = nullptr;
+    int bestd = INT_MAX;
+    for (int i = 0; i < kTableN; ++i) {
+        const TableEntry& e = kTable[i];
+        if (e.op != op || e.dtype != dtype) continue;
+        const int d = std::abs(e.lr - lr) + std::abs(e.lc - lc);
+        // ties: prefer the cell with the same element count (lr + lc), then the lower lr
+        if (d < bestd || (d == bestd && best && std::abs(e.lr + e.lc - lr - lc) < std::abs(best->lr + best->lc - lr - lc))) {
+            best = &e; bestd = d;
+        }
+    }
+    return (best && bestd <= 2) ? best : nullptr;
+}
+
+// Fill the kernel parameters of `p` for p->variant.  params: user overrides or nullptr.
+adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& dev) {
+    const int op = p->op, dt = p->dtype;
+    const bool px = (op == ADAPTIC_OP_DOT);
+    const int64_t R = p->R, C = p->C;
+    auto par = [&](int i) -> int { return params ? params[i] : 0; };
+    const int v = p->variant;
+    if (op == ADAPTIC_OP_TMV ? !is_tmv_family(v) : !is_mv_family(v)) return ADAPTIC_ERR_UNSUPPORTED;
+
+    p->vec_shape = (op == ADAPTIC_OP_TMV) ? (R % 4 == 0) : (C % 4 == 0);
+    p->splits = 1;
+    p->smem = 0;
+    p->stages = 0;
+    p->xmode = px ? 2 : 0;
+    p->rb = 1;
+    p->fb_lanes = 0;
+    p->fb_unroll = 0;
+    p->ws_bytes = 0;
+    p->cnt_off = 0;
+
+    for (int w = 0; w < 2; ++w) { p->grid[w] = 0; p->chain[w] = 0; p->depth[w] = 0; p->path_ok[w] = false; }
+
+    if (v == ADAPTIC_V_MV_SUBWARP || v == ADAPTIC_V_MV_WPR || v == ADAPTIC_V_MV_TPR) {
+        // group-kernel parameters (also the TPR scalar fallback)
+        // TPR's fallback is the scalar group kernel, so size it for the scalar path
+        const int64_t nvv = (p->vec_shape && v != ADAPTIC_V_MV_TPR) ? C / 4 : C;
+        int G;
+        if (v == ADAPTIC_V_MV_WPR) G = 32;
+        else if (v == ADAPTIC_V_MV_SUBWARP && par(ADAPTIC_P_LANES) > 0) G = par(ADAPTIC_P_LANES);
+        else G = clampi(pow2_ceil(std::max<int64_t>(1, nvv)), 1, v == ADAPTIC_V_MV_TPR ? 32 : 16);
+        if (G < 1 || G > 32 || (G & (G - 1)) || (v == ADAPTIC_V_MV_SUBWARP && G > 16)) return ADAPTIC_ERR_INVALID_ARG;
+        int U = par(ADAPTIC_P_UNROLL);
+        if (U <= 0) U = clampi(pow2_ceil(ceil_div(std::max<int64_t>(1, nvv), G)), 1, 8);
+        if (U != 1 && U != 2 && U != 4 && U != 8) return ADAPTIC_ERR_INVALID_ARG;
+        if (v == ADAPTIC_V_MV_TPR) { p->fb_lanes = G; p->fb_unroll = U; }
+        else { p->lanes = G; p->unroll = U; p->rb = 8 / U; p->block = GROUP_NT; }
+        const int rows_per_cta = (8 / U) * (32 / G) * (GROUP_NT / 32);
+        const int xm = (v == ADAPTIC_V_MV_TPR) ? (px ? 2 : 0) : pick_xmode(px, par(ADAPTIC_P_XSMEM), C, true);
+        if (xm < 0) return ADAPTIC_ERR_UNSUPPORTED;
+        const size_t xsm = xm == 1 ? size_t((C * 4 + 15) / 16 * 16) : 0;
+        int cps = par(ADAPTIC_P_CTAS_PER_SM);
+        if (cps <= 0) cps = occupancy(group_fn(dt, G, U, p->vec_shape, xm), GROUP_NT, xsm, dev.present, 4);
+        if (v != ADAPTIC_V_MV_TPR) { p->ctas_per_sm = cps; p->xmode = xm; p->smem = xsm; }
+        for (int w = 0; w < 2; ++w) {
+            const int64_t nv = w ? C / 4 : C;
+            if (w == 1 && !p->vec_shape) continue;
+            const int64_t iters = ceil_div(nv, int64_t(G) * U);
+            p->grid[w] = std::max<int64_t>(1, std::min<int64_t>(ceil_div(R, rows_per_cta), int64_t(dev.sms) * cps));
+            p->chain[w] = fold_chain(iters);
+            p->depth[w] = ilog2c(U) + (w ? 2 : 0) + ilog2c(G) + 1;
+            p->path_ok[w] = (dt == DT_I32) || bound_ok(p->chain[w] + p->depth[w]);
+        }
+        if (v != ADAPTIC_V_MV_TPR) {
+            if (!p->path_ok[p->vec_shape ? 1 : 0]) return ADAPTIC_ERR_UNSUPPORTED;
+            return ADAPTIC_OK;
+        }
+        // ---- MV_TPR proper (vector path only; scalar path = the group fallback above)
+        const int64_t fb_grid = p->grid[0];
+        const int64_t fb_chain = p->chain[0], fb_depth = p->depth[0];
+        const bool fb_ok = p->path_ok[0];
+        if (!p->vec_shape || C > 256) return ADAPTIC_ERR_UNSUPPORTED;
+        int NT = par(ADAPTIC_P_LANES);
+        if (NT <= 0) NT = (C <= 32) ? 256 : 128;
+        if (NT != 128 && NT != 256) return ADAPTIC_ERR_INVALID_ARG;
+        const size_t stage_bytes = size_t(NT) * size_t(C) * 4 * (px ? 2 : 1);
+        const size_t xbytes = px ? 0 : size_t((C + 31) / 32 * 32) * 4;
+        int cps_t = par(ADAPTIC_P_CTAS_PER_SM);
+        if (cps_t <= 0) cps_t = 2;
+        const size_t budget = (size_t(220) * 1024) / size_t(cps_t);
+        int stages = int(std::min<size_t>(8, (budget > xbytes ? budget - xbytes : 0) / stage_bytes));
+        if (par(ADAPTIC_P_UNROLL) > 0) stages = std::min(stages, par(ADAPTIC_P_UNROLL));
+        if (stages < 2) return ADAPTIC_ERR_UNSUPPORTED;
+        p->lanes = NT;
+        p->unroll = stages;
+        p->stages = stages;
+        p->block = NT;
+        p->smem = xbytes + size_t(stages) * stage_bytes;
+        const int occ = occupancy(tpr_fn(dt, NT, px), NT, p->smem, dev.present, cps_t);
+        p->ctas_per_sm = std::min(cps_t, occ);
+        p->grid[1] = std::max<int64_t>(1, std::min<int64_t>(ceil_div(R, NT), int64_t(dev.sms) * p->ctas_per_sm));
+        p->chain[1] = ceil_div(C / 4, 2);
+        p->depth[1] = 3;
+        p->path_ok[1] = (dt == DT_I32) || bound_ok(p->chain[1] + p->depth[1]);
+        p->grid[0] = fb_grid; p->chain[0] = fb_chain; p->depth[0] = fb_depth; p->path_ok[0] = fb_ok;
+        if (!p->path_ok[1]) return ADAPTIC_ERR_UNSUPPORTED;
+        return ADAPTIC_OK;
+    }
+
+    if (v == ADAPTIC_V_MV_CPR || v == ADAPTIC_V_MV_SPLIT) {
+        const int64_t nv1 = p->vec_shape ? C / 4 : C;
+        int NT = par(ADAPTIC_P_LANES);
+        if (NT <= 0) NT = (v == ADAPTIC_V_MV_CPR && nv1 >= 8192) ? 1024 : 256;
+        if (NT != 256 && NT != 1024) return ADAPTIC_ERR_INVALID_ARG;
+        int U = par(ADAPTIC_P_UNROLL);
+        if (U <= 0) U = 4;
+        if (U != 2 && U != 4 && U != 8) return ADAPTIC_ERR_INVALID_ARG;
+        // x staged in smem only for CPR (a split CTA reads a different x chunk per block)
+        const int xm = pick_xmode(px, par(ADAPTIC_P_XSMEM), C, v == ADAPTIC_V_MV_CPR);
+        if (xm < 0) return ADAPTIC_ERR_UNSUPPORTED;
+        const size_t xsm = xm == 1 ? size_t((C * 4 + 15) / 16 * 16) : 0;
+        int cps = par(ADAPTIC_P_CTAS_PER_SM);
+        if (cps <= 0) cps = occupancy(cta_fn(dt, NT, U, p->vec_shape, xm), NT, xsm, dev.present, 2048 / NT);
+        p->lanes = NT; p->unroll = U; p->block = NT; p->ctas_per_sm = cps; p->xmode = xm; p->smem = xsm;
+        const int64_t slots = int64_t(dev.sms) * cps;
+        int64_t S = 1;
+        if (v == ADAPTIC_V_MV_SPLIT) {
+            if (par(ADAPTIC_P_SPLITS) > 0) S = par(ADAPTIC_P_SPLITS);
+            else {
+                S = std::max<int64_t>(2, ceil_div(2 * slots, std::max<int64_t>(1, R)));   // ~2 waves
+                S = std::min<int64_t>(S, std::max<int64_t>(2, ceil_div(nv1, int64_t(NT) * U)));
+            }
+        }
+        // accuracy: raise S (SPLIT only) until the bound holds on both paths
+        for (;;) {
+            bool ok_all = true;
+            for (int w = 0; w < 2; ++w) {
+                const int64_t nv = w ? C / 4 : C;
+                if (w == 1 && !p->vec_shape) continue;
+                const int64_t iters = ceil_div(ceil_div(nv, S), int64_t(NT) * U);
+                p->chain[w] = fold_chain(iters);
+                p->depth[w] = ilog2c(U) + (w ? 2 : 0) + ilog2c(NT) + (S > 1 ? ceil_div(S, NT) + ilog2c(NT) : 0) + 1;
+                p->path_ok[w] = (dt == DT_I32) || bound_ok(p->chain[w] + p->depth[w]);
+                p->grid[w] = std::max<int64_t>(1, std::min<int64_t>(R * S, slots));
+                if (!p->path_ok[w]) ok_all = false;
+            }
+            if (ok_all || v == ADAPTIC_V_MV_CPR || S >= (int64_t(1) << 20)) break;
+            S *= 2;
+        }
+        if (S > INT_MAX || R * S > (int64_t(1) << 40)) return ADAPTIC_ERR_UNSUPPORTED;
+        p->splits = int(S);
+        if (!p->path_ok[p->vec_shape ? 1 : 0]) return ADAPTIC_ERR_UNSUPPORTED;
+        if (S > 1) {
+            const size_t part = ((size_t(R) * size_t(S) * 4 + 255) / 256) * 256;
+            p->cnt_off = part;
+            p->ws_bytes = part + size_t(R) * 4;
+        }
+        return ADAPTIC_OK;
+    }
+
+    // ---- TMV family
+    const int64_t rv1 = p->vec_shape ? R / 4 : R;
+    int LR = par(ADAPTIC_P_LANES);
+    if (LR <= 0) {
+        if (v == ADAPTIC_V_TMV_COL) LR = 256;
+        else if (v == ADAPTIC_V_TMV_REGTILE) LR = clampi(pow2_ceil(rv1), 1, 256);
+        else LR = clampi(pow2_ceil(rv1), 1, 64);
+    }
+    if (LR < 1 || LR > 256 || (LR & (LR - 1))) return ADAPTIC_ERR_INVALID_ARG;
+    if (v == ADAPTIC_V_TMV_REGTILE && rv1 > LR) return ADAPTIC_ERR_UNSUPPORTED;
+    int U = par(ADAPTIC_P_UNROLL);
+    if (U <= 0) U = (v == ADAPTIC_V_TMV_COL) ? 8 : 4;
+    if (U != 2 && U != 4 && U != 8) return ADAPTIC_ERR_INVALID_ARG;
+    int cps = par(ADAPTIC_P_CTAS_PER_SM);
+    if (cps <= 0) cps = occupancy(tmv_fn(dt, LR, U, p->vec_shape), TMV_NT, 0, dev.present, 4);
+    p->lanes = LR; p->unroll = U; p->block = TMV_NT; p->ctas_per_sm = cps;
+    const int LC = TMV_NT / LR;
+    const int64_t slots = int64_t(dev.sms) * cps;
+    const int64_t tiles1 = ceil_div(rv1, LR);
+    int64_t S = 1;
+    if (par(ADAPTIC_P_SPLITS) > 0) S = par(ADAPTIC_P_SPLITS);
+    else if (v != ADAPTIC_V_TMV_COL) {
+        S = std::max<int64_t>(1, ceil_div(2 * slots, tiles1));                        // ~2 waves
+        S = std::min<int64_t>(S, std::max<int64_t>(1, ceil_div(C, int64_t(LC) * U)));  // >= 1 step each
+    }
+    for (;;) {
+        bool ok_all = true;
+        for (int w = 0; w < 2; ++w) {
+            if (w == 1 && !p->vec_shape) continue;
+            const int64_t rv = w ? R / 4 : R;
+            const int64_t tiles = ceil_div(rv, LR);
+            const int64_t iters = ceil_div(ceil_div(C, S), int64_t(LC) * U);
+            p->chain[w] = fold_chain(iters);
+            p->depth[w] = ilog2c(U) + ilog2c(LC) + (S > 1 ? ceil_div(S, LC) + ilog2c(LC) : 0) + 1;
+            p->path_ok[w] = (dt == DT_I32) || bound_ok(p->chain[w] + p->depth[w]);
+            p->grid[w] = std::max<int64_t>(1, std::min<int64_t>(tiles * S, slots));
+            if (!p->path_ok[w]) ok_all = false;
+        }
+        if (ok_all || S >= (int64_t(1) << 20)) break;
+        S *= 2;
+    }
+    if (S > INT_MAX) return ADAPTIC_ERR_UNSUPPORTED;
+    p->splits = int(S);
+    if (!p->path_ok[p->vec_shape ? 1 : 0]) return ADAPTIC_ERR_UNSUPPORTED;
+    if (S > 1) {
+        const size_t part = ((size_t(R) * size_t(S) * 4 + 255) / 256) * 256;
+        p->cnt_off = part;
+        p->ws_bytes = part + size_t(ceil_div(R, LR)) * 4;    // tiles of the scalar path (the larger)
+    }
+    return ADAPTIC_OK;
+}
+
+adaptic_status validate_shape(int op, int64_t rows, int64_t cols, int dtype) {
+    if (op < ADAPTIC_OP_MV || op > ADAPTIC_OP_DOT) return ADAPTIC_ERR_INVALID_ARG;
+    if (dtype != ADAPTIC_F32 && dtype != ADAPTIC_I32) return ADAPTIC_ERR_INVALID_ARG;
+    if (rows < 0 || cols < 0) return ADAPTIC_ERR_INVALID_ARG;
+    if (cols > 0 && rows > (int64_t(1) << 62) / 4 / cols) return ADAPTIC_ERR_INVALID_ARG;  // bytes overflow
+    return ADAPTIC_OK;
+}
+
+adaptic_status make_plan(int op, int64_t rows, int64_t cols, int dtype, int variant,
+                         const int32_t* params, adaptic_plan_t* out) {
+    if (!out) return ADAPTIC_ERR_INVALID_ARG;
+    *out = nullptr;
+    adaptic_status st = validate_shape(op, rows, cols, dtype);
+    if (st != ADAPTIC_OK) return st;
+    if (variant < ADAPTIC_V_AUTO || variant >= ADAPTIC_V_COUNT) return ADAPTIC_ERR_INVALID_ARG;
+    const DevInfo dev = device_info();
+    adaptic_plan_s* p = new (std::nothrow) adaptic_plan_s();
+    if (!p) return ADAPTIC_ERR_INVALID_ARG;
+    p->op = op; p->dtype = dtype; p->R = rows; p->C = cols; p->sms = dev.sms;
+    p->ws = nullptr; p->ws_cap = 0;
+
+    if (variant != ADAPTIC_V_AUTO) {
+        p->variant = variant; p->source = 0;
+        st = (rows == 0 || cols == 0) ? ((op == ADAPTIC_OP_TMV ? is_tmv_family(variant) : is_mv_family(variant))
+                                             ? ADAPTIC_OK : ADAPTIC_ERR_UNSUPPORTED)
+                                      : derive(p, params, dev);
+        if (st != ADAPTIC_OK) { delete p; return st; }
+        *out = p;
+        return ADAPTIC_OK;
+    }
+    if (rows == 0 || cols == 0) {      // nothing to select: run() is a no-op / memset
+        p->variant = heuristic_variant(op, std::max<int64_t>(rows, 1), std::max<int64_t>(cols, 1), dev.sms);
+        p->source = 2;
+        *out = p;
+        return ADAPTIC_OK;
+    }
+    if (const TableEntry* e = table_lookup(op, dtype, rows, cols)) {
+        int32_t tp[ADAPTIC_NPARAMS] = {e->lanes, e->splits, e->ctas_per_sm, e->unroll, e->xsmem};
+        p->variant = e->variant; p->source = 1;
+        if (derive(p, tp, dev) == ADAPTIC_OK) { *out = p; return ADAPTIC_OK; }
+        if (derive(p, nullptr, dev) == ADAPTIC_OK) { *out = p; return ADAPTIC_OK; }
+    }
+    p->variant = heuristic_variant(op, rows, cols, dev.sms);
+    p->source = 2;
+    st = derive(p, nullptr, dev);
+    if (st != ADAPTIC_OK) {
+        // last resort: the split variants always satisfy the bound
+        p->variant = (op == ADAPTIC_OP_TMV) ? ADAPTIC_V_TMV_SPLITK : ADAPTIC_V_MV_SPLIT;
+        st = derive(p, nullptr, dev);
+    }
+    if (st != ADAPTIC_OK) { delete p; return st; }
+    *out = p;
+    return ADAPTIC_OK;
+}
+
+bool aligned(const void* p, uintptr_t a) { return (reinterpret_cast<uintptr_t>(p) & (a - 1)) == 0; }
+
+bool overlap(const void* a, size_t na, const void* b, size_t nb) {
+    if (na == 0 || nb == 0) return false;
+    const uintptr_t a0 = reinterpret_cast<uintptr_t>(a), b0 = reinterpret_cast<uintptr_t>(b);
+    return a0 < b0 + nb && b0 < a0 + na;
+}
+
+adaptic_status cuda_fail(cudaError_t e) {
+    g_last_cuda_error = int(e);
+    (void)cudaGetLastError();
+    return ADAPTIC_ERR_CUDA;
+}
+
+std::mutex g_attr_mu;
+// (device, kernel) pairs that already have their dynamic-smem limit raised
+struct AttrKey { int dev; void* fn; size_t smem; };
+AttrKey g_attr_done[64];
+int g_attr_n = 0;
+
+cudaError_t ensure_smem_attr(void* fn, size_t smem) {
+    if (smem <= 48 * 1024) return cudaSuccess;
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    std::lock_guard<std::mutex> lk(g_attr_mu);
+    for (int i = 0; i < g_attr_n; ++i)
+        if (g_attr_done[i].dev == dev && g_attr_done[i].fn == fn && g_attr_done[i].smem >= smem) return cudaSuccess;
+    // raise the opt-in limit to exactly what this launch needs (static smem + this
+    // must stay within the per-block opt-in maximum, 227 KB on B200)
+    e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+    if (e != cudaSuccess) return e;
+    for (int i = 0; i < g_attr_n; ++i)
+        if (g_attr_done[i].dev == dev && g_attr_done[i].fn == fn) { g_attr_done[i].smem = smem; return cudaSuccess; }
+    if (g_attr_n < 64) g_attr_done[g_attr_n++] = AttrKey{dev, fn, smem};
+    return cudaSuccess;
+}
+
+adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, void* y,
+                      cudaStream_t stream, bool vec) {
+    const int dt = p->dtype;
+    const bool px = p->op == ADAPTIC_OP_DOT;
+    int64_t R = p->R, C = p->C;
+    const int w = vec ? 1 : 0;
+    void* part = p->ws;
+    unsigned int* cnt = p->ws ? reinterpret_cast<unsigned int*>(static_cast<char*>(p->ws) + p->cnt_off) : nullptr;
+    int S = p->splits;
+    void* fn = nullptr;
+    int block = p->block;
+    size_t smem = 0;
+    int64_t grid = p->grid[w];
+    void* args8[8];
+    void* args6[6];
+    void** args = nullptr;
+    int stages = p->stages;
+
+    switch (p->variant) {
+        case ADAPTIC_V_MV_TPR:
+            if (vec) {
+                fn = tpr_fn(dt, p->lanes, px);
+                smem = p->smem;
+                cudaError_t e = ensure_smem_attr(fn, smem);
+                if (e != cudaSuccess) return cuda_fail(e);
+                args6[0] = &A; args6[1] = &X; args6[2] = &y; args6[3] = &R; args6[4] = &C; args6[5] = &stages;
+                args = args6;
+            } else {
+                fn = group_fn(dt, p->fb_lanes, p->fb_unroll, false, px ? 2 : 0);
+                block = GROUP_NT;
+                args6[0] = &A; args6[1] = &X; args6[2] = &y; args6[3] = &R; args6[4] = &C;
+                args = args6;
+            }
+            break;
+        case ADAPTIC_V_MV_SUBWARP:
+        case ADAPTIC_V_MV_WPR:
+            fn = group_fn(dt, p->lanes, p->unroll, vec, p->xmode);
+            smem = p->smem;
+            args6[0] = &A; args6[1] = &X; args6[2] = &y; args6[3] = &R; args6[4] = &C;
+            args = args6;
+            break;
+        case ADAPTIC_V_MV_CPR:
+        case ADAPTIC_V_MV_SPLIT:
+            fn = cta_fn(dt, p->lanes, p->unroll, vec, p->xmode);
+            smem = p->smem;
+            args8[0] = &A; args8[1] = &X; args8[2] = &y; args8[3] = &R; args8[4] = &C;
+            args8[5] = &S; args8[6] = &part; args8[7] = &cnt;
+            args = args8;
+            break;
+        default:
+            fn = tmv_fn(dt, p->lanes, p->unroll, vec);
+            args8[0] = &A; args8[1] = &X; args8[2] = &y; args8[3] = &R; args8[4] = &C;
+            args8[5] = &S; args8[6] = &part; args8[7] = &cnt;
+            args = args8;
+            break;
+    }
+    if (!fn) return ADAPTIC_ERR_UNSUPPORTED;
+    if (smem > 48 * 1024) {
+        cudaError_t ea = ensure_smem_attr(fn, smem);
+        if (ea != cudaSuccess) return cuda_fail(ea);
+    }
+    if (grid > INT_MAX) grid = INT_MAX;
+    cudaError_t e = cudaLaunchKernel(fn, dim3(unsigned(grid)), dim3(unsigned(block)), args, smem, stream);
+    if (e != cudaSuccess) return cuda_fail(e);
+    return ADAPTIC_OK;
+}
+
+adaptic_status check_run(const adaptic_plan_s* p, const void* A, const void* x, const void* y) {
+    if (p->R == 0) return ADAPTIC_OK;
+    if (!y) return ADAPTIC_ERR_INVALID_ARG;
+    if (!aligned(y, 4)) return ADAPTIC_ERR_MISALIGNED;
+    if (p->C == 0) return ADAPTIC_OK;
+    if (!A || !x) return ADAPTIC_ERR_INVALID_ARG;
+    if (!aligned(A, 4) || !aligned(x, 4)) return ADAPTIC_ERR_MISALIGNED;
+    const size_t ybytes = size_t(p->R) * 4;
+    const size_t abytes = size_t(p->R) * size_t(p->C) * 4;
+    const size_t xbytes = (p->op == ADAPTIC_OP_DOT ? abytes : size_t(p->C) * 4);
+    if (overlap(y, ybytes, A, abytes) || overlap(y, ybytes, x, xbytes)) return ADAPTIC_ERR_ALIAS;
+    if (p->ws_bytes > 0 && (p->ws == nullptr || p->ws_cap < p->ws_bytes)) return ADAPTIC_ERR_NO_WORKSPACE;
+    return ADAPTIC_OK;
+}
+
+}  // namespace
+
+// =================================================================== C ABI
+extern "C" {
+
+adaptic_status adaptic_plan(adaptic_op op, int64_t rows, int64_t cols, adaptic_dtype dtype,
+                            adaptic_plan_t* out) {
+    return make_plan(op, rows, cols, dtype, ADAPTIC_V_AUTO, nullptr, out);
+}
+
+adaptic_status adaptic_plan_forced(adaptic_op op, int64_t rows, int64_t cols, adaptic_dtype dtype,
+                                   adaptic_variant variant, const int32_t* params, adaptic_plan_t* out) {
+    if (variant == ADAPTIC_V_AUTO) return make_plan(op, rows, cols, dtype, ADAPTIC_V_AUTO, nullptr, out);
+    return make_plan(op, rows, cols, dtype, variant, params, out);
+}
+
+adaptic_variant adaptic_plan_variant(adaptic_plan_t plan) {
+    return plan ? adaptic_variant(plan->variant) : ADAPTIC_V_AUTO;
+}
+
+size_t adaptic_plan_workspace_bytes(adaptic_plan_t plan) { return plan ? plan->ws_bytes : 0; }
+
+adaptic_status adaptic_plan_set_workspace(adaptic_plan_t plan, void* dev_ptr, size_t bytes) {
+    if (!plan) return ADAPTIC_ERR_INVALID_ARG;
+    if (dev_ptr == nullptr) {
+        if (bytes != 0) return ADAPTIC_ERR_INVALID_ARG;
+        plan->ws = nullptr; plan->ws_cap = 0;
+        return ADAPTIC_OK;
+    }
+    if (!aligned(dev_ptr, 16)) return ADAPTIC_ERR_MISALIGNED;
+    if (bytes < plan->ws_bytes) return ADAPTIC_ERR_NO_WORKSPACE;
+    plan->ws = dev_ptr; plan->ws_cap = bytes;
+    return ADAPTIC_OK;
+}
+
+int adaptic_plan_describe(adaptic_plan_t p, char* buf, size_t cap) {
+    if (!p) return -1;
+    static const char* ops[] = {"MV", "TMV", "DOT"};
+    static const char* src[] = {"forced", "table", "heuristic"};
+    char tmp[1024];
+    const int n = std::snprintf(
+        tmp, sizeof(tmp),
+        "{\"op\":\"%s\",\"dtype\":\"%s\",\"rows\":%lld,\"cols\":%lld,\"variant\":\"%s\",\"source\":\"%s\","
+        "\"sms\":%d,\"lanes\":%d,\"unroll\":%d,\"rows_per_group\":%d,\"splits\":%d,\"block\":%d,"
+        "\"ctas_per_sm\":%d,\"stages\":%d,\"xmode\":%d,\"smem\":%zu,\"vec_shape\":%s,"
+        "\"grid\":[%lld,%lld],\"chain\":[%lld,%lld],\"depth\":[%lld,%lld],\"path_ok\":[%s,%s],"
+        "\"fallback_lanes\":%d,\"fallback_unroll\":%d,\"workspace_bytes\":%zu}",
+        ops[p->op], p->dtype == ADAPTIC_F32 ? "f32" : "i32", (long long)p->R, (long long)p->C,
+        kVariantNames[p->variant], src[p->source], p->sms, p->lanes, p->unroll, p->rb, p->splits, p->block,
+        p->ctas_per_sm, p->stages, p->xmode, p->smem, p->vec_shape ? "true" : "false",
+        (long long)p->grid[0], (long long)p->grid[1], (long long)p->chain[0], (long long)p->chain[1],
+        (long long)p->depth[0], (long long)p->depth[1], p->path_ok[0] ? "true" : "false",
+        p->path_ok[1] ? "true" : "false", p->fb_lanes, p->fb_unroll, p->ws_bytes);
+    if (buf && cap > 0) {
+        const size_t m = std::min(cap - 1, size_t(n));
+        std::memcpy(buf, tmp, m);
+        buf[m] = '\0';
+    }
+    return n;
+}
+
+adaptic_status adaptic_run(adaptic_plan_t p, const void* A, const void* x, void* y, void* stream_) {
+    if (!p) return ADAPTIC_ERR_INVALID_ARG;
+    cudaStream_t stream = static_cast<cudaStream_t>(stream_);
+    adaptic_status st = check_run(p, A, x, y);
+    if (st != ADAPTIC_OK || p->R == 0) return st;
+    if (p->C == 0) {
+        cudaError_t e = cudaMemsetAsync(y, 0, size_t(p->R) * 4, stream);
+        return e == cudaSuccess ? ADAPTIC_OK : cuda_fail(e);
+    }
+    bool vec = p->vec_shape;
+    if (vec) {
+        if (p->op == ADAPTIC_OP_TMV) vec = aligned(A, 16) && aligned(y, 16);
+        else vec = aligned(A, 16) && aligned(x, 16);
+    }
+    if (!p->path_ok[vec ? 1 : 0]) return ADAPTIC_ERR_MISALIGNED;   // scalar path would break the error bound
+    return launch(p, A, x, y, stream, vec);
+}
+
+adaptic_status adaptic_run_host(adaptic_plan_t p, const void* A_host, const void* x_host, void* y_host,
+                                void* dA, void* dx, void* dy, void* stream_) {
+    if (!p) return ADAPTIC_ERR_INVALID_ARG;
+    cudaStream_t stream = static_cast<cudaStream_t>(stream_);
+    if (p->R == 0) return ADAPTIC_OK;
+    if (!y_host || (p->C > 0 && (!A_host || !x_host))) return ADAPTIC_ERR_INVALID_ARG;
+    adaptic_status st = check_run(p, dA, dx, dy);
+    if (st != ADAPTIC_OK) return st;
+    const size_t abytes = size_t(p->R) * size_t(p->C) * 4;
+    const size_t xbytes = (p->op == ADAPTIC_OP_DOT ? abytes : size_t(p->C) * 4);
+    cudaError_t e;
+    if (p->C > 0) {
+        if ((e = cudaMemcpyAsync(dx, x_host, xbytes, cudaMemcpyHostToDevice, stream)) != cudaSuccess) return cuda_fail(e);
+        if ((e = cudaMemcpyAsync(dA, A_host, abytes, cudaMemcpyHostToDevice, stream)) != cudaSuccess) return cuda_fail(e);
+    }
+    st = adaptic_run(p, dA, dx, dy, stream_);
+    if (st != ADAPTIC_OK) return st;
+    if ((e = cudaMemcpyAsync(y_host, dy, size_t(p->R) * 4, cudaMemcpyDeviceToHost, stream)) != cudaSuccess)
+        return cuda_fail(e);
+    return ADAPTIC_OK;
+}
+
+void adaptic_plan_destroy(adaptic_plan_t plan) { delete plan; }
+
+const char* adaptic_status_string(adaptic_status s) {
+    switch (s) {
+        case ADAPTIC_OK: return "ADAPTIC_OK";
+        case ADAPTIC_ERR_INVALID_ARG: return "ADAPTIC_ERR_INVALID_ARG";
+        case ADAPTIC_ERR_UNSUPPORTED: return "ADAPTIC_ERR_UNSUPPORTED";
+        case ADAPTIC_ERR_MISALIGNED: return "ADAPTIC_ERR_MISALIGNED";
+        case ADAPTIC_ERR_ALIAS: return "ADAPTIC_ERR_ALIAS";
+        case ADAPTIC_ERR_NO_WORKSPACE: return "ADAPTIC_ERR_NO_WORKSPACE";
+        case ADAPTIC_ERR_CUDA: return "ADAPTIC_ERR_CUDA";
+        default: return "ADAPTIC_ERR_UNKNOWN";
+    }
+}
+
+const char* adaptic_variant_name(adaptic_variant v) {
+    return (v >= 0 && v < ADAPTIC_V_COUNT) ? kVariantNames[v] : "UNKNOWN";
+}
+
+int adaptic_last_cuda_error(void) { return g_last_cuda_error; }
+
+int adaptic_abi_version(void) { return ADAPTIC_ABI_VERSION; }
+
+}  // extern "C"

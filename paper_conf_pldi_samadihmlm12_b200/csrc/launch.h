@@ -1,0 +1,37 @@
+// launch.h -- internal interface between the planner (adaptic.cu) and the
+// kernel translation units.  Not part of the public ABI (include/adaptic.h).
+#pragma once
+
+#include <cstddef>
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace adaptic {
+
+// Iterations of a thread's load loop accumulated before folding into a
+// second-level accumulator: keeps every serial chain short even for forced
+// off-regime variants.
+constexpr int FOLD = 512;
+
+enum Dtype { DT_F32 = 0, DT_I32 = 1 };
+
+constexpr int GROUP_NT = 256;   // threads per CTA, mv_group_kernel
+constexpr int TMV_NT = 256;     // threads per CTA, tmv_kernel
+
+// Kernel instance lookup: a __global__ function pointer for cudaLaunchKernel /
+// cudaOccupancyMaxActiveBlocksPerMultiprocessor, or nullptr when the instance
+// is not compiled.  Kernel signatures:
+//   group: (const T* A, const T* X, T* y, int64_t R, int64_t C)
+//   cta  : (const T* A, const T* X, T* y, int64_t R, int64_t C, int S, T* part, unsigned* cnt)
+//   tmv  : (const T* B, const T* X, T* y, int64_t R, int64_t C, int S, T* part, unsigned* cnt)
+//   tpr  : (const T* A, const T* X, T* y, int64_t R, int64_t C, int stages)   [dynamic smem]
+// x operand modes of the MV-family kernels (mv_kernels.cuh): 0 read-only path,
+// 1 staged in shared memory by TMA (dynamic smem = C*4 bytes), 2 per-row (DOT)
+void* group_fn_f32(int G, int U, bool vec, int xmode);
+void* group_fn_i32(int G, int U, bool vec, int xmode);
+void* tmv_fn_f32(int LR, int U, bool vec);
+void* tmv_fn_i32(int LR, int U, bool vec);
+void* cta_fn(int dtype, int NT, int U, bool vec, int xmode);
+void* tpr_fn(int dtype, int NT, bool perrowx);
+
+}  // namespace adaptic

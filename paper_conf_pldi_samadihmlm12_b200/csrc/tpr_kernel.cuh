@@ -1,0 +1,102 @@
+// tpr_kernel.cuh -- MV_TPR: thread per row with TMA bulk staging (sm_100a).
+//
+// The paper's kernel 5 gives each thread "the dot product of a single
+// row".  On the MV layout a thread's row is contiguous, so a warp's direct loads
+// would not coalesce (Fig. 3a).  The paper's fix is to restructure the
+// data on the CPU; its rejected alternative is a coalesced cooperative
+// copy into shared memory, rejected for shared-memory size and address
+// arithmetic on Fermi.  Neither objection holds on B200 (228 KB smem/SM; the
+// TMA engine does the addressing), so this variant stages tiles of NT
+// consecutive rows -- a contiguous NT*C*4-byte block -- with cp.async.bulk into a
+// STAGES-deep ring guarded by mbarriers, and each thread then reduces its own
+// row out of shared memory.  The rotation k' = (k + t) mod (C/4) makes the
+// 128-bit shared loads of 8 consecutive threads hit distinct banks.
+#pragma once
+
+#include "common.cuh"
+
+namespace adaptic {
+
+constexpr int TPR_MAX_STAGES = 8;
+
+// Dynamic smem layout: [x: C elems][stage 0: NT*C (+ NT*C for DOT's b)] ... ; 16B aligned.
+template <class T, int NT, bool PERROWX>
+__global__ void __launch_bounds__(NT)
+mv_tpr_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restrict__ y,
+              int64_t R, int64_t C, int stages)
+{
+    using V = vec4_t<T>;
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    __shared__ __align__(8) uint64_t full[TPR_MAX_STAGES];
+    __shared__ __align__(8) uint64_t xbar;
+
+    const int tid = threadIdx.x;
+    const int c4 = int(C / 4);                               // vectors per row (C % 4 == 0)
+    const int64_t ntiles = (R + NT - 1) / NT;
+    const size_t tile_elems = size_t(NT) * C;
+    T* xs = reinterpret_cast<T*>(smem_raw);
+    T* ring = xs + (PERROWX ? 0 : ((C + 31) / 32) * 32);      // keep 128B alignment
+    const size_t stage_elems = tile_elems * (PERROWX ? 2 : 1);
+
+    // tiles of this CTA: blockIdx.x, blockIdx.x + gridDim.x, ...
+    const int64_t my_tiles = blockIdx.x < ntiles ? (ntiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+
+    if (tid == 0) {
+        for (int s = 0; s < stages; ++s) mbar_init(&full[s], 1);
+        mbar_init(&xbar, 1);
+        fence_mbar_init();
+    }
+    __syncthreads();
+
+    auto issue = [&](int64_t i) {  // local tile i -> stage i % stages (thread 0 only)
+        const int64_t tile = blockIdx.x + i * gridDim.x;
+        const int64_t r0 = tile * NT;
+        const int64_t nrows = min(int64_t(NT), R - r0);
+        const uint32_t bytes = uint32_t(nrows * C * sizeof(T));
+        T* dst = ring + size_t(i % stages) * stage_elems;
+        uint64_t* bar = &full[i % stages];
+        mbar_arrive_expect_tx(bar, PERROWX ? 2 * bytes : bytes);
+        bulk_g2s(dst, A + r0 * C, bytes, bar);
+        if (PERROWX) bulk_g2s(dst + tile_elems, X + r0 * C, bytes, bar);
+    };
+
+    if (tid == 0) {
+        if (!PERROWX) {
+            mbar_arrive_expect_tx(&xbar, uint32_t(C * sizeof(T)));
+            bulk_g2s_keep(xs, X, uint32_t(C * sizeof(T)), &xbar);
+        }
+        const int64_t pre = min(int64_t(stages), my_tiles);
+        for (int64_t i = 0; i < pre; ++i) issue(i);
+    }
+    if (!PERROWX) mbar_wait(&xbar, 0);
+
+    const V* xv = reinterpret_cast<const V*>(xs);
+    for (int64_t i = 0; i < my_tiles; ++i) {
+        const int st = int(i % stages);
+        mbar_wait(&full[st], uint32_t((i / stages) & 1));
+        const int64_t r0 = (blockIdx.x + i * gridDim.x) * int64_t(NT);
+        const V* av = reinterpret_cast<const V*>(ring + size_t(st) * stage_elems) + size_t(tid) * c4;
+        const V* bv = PERROWX ? reinterpret_cast<const V*>(ring + size_t(st) * stage_elems + tile_elems) + size_t(tid) * c4
+                              : xv;
+        if (r0 + tid < R) {
+            V acc0 = zero_of<V>(), acc1 = zero_of<V>();
+            int k = tid % c4;
+            int n = 0;
+            for (; n + 1 < c4; n += 2) {
+                const int k1 = (k + 1 == c4) ? 0 : k + 1;
+                vmac(acc0, av[k], bv[k]);
+                vmac(acc1, av[k1], bv[k1]);
+                k = (k1 + 1 == c4) ? 0 : k1 + 1;
+            }
+            if (n < c4) vmac(acc0, av[k], bv[k]);
+            y[r0 + tid] = vsum(vadd(acc0, acc1));
+        }
+        __syncthreads();                      // every thread is done with stage st
+        if (tid == 0 && i + stages < my_tiles) {
+            fence_proxy_async();              // generic-proxy reads before async-proxy refill
+            issue(i + stages);
+        }
+    }
+}
+
+}  // namespace adaptic

@@ -1,0 +1,137 @@
+"""PyTorch-facing API: ``mv``, ``tmv``, ``dot`` on CUDA tensors.
+
+PyTorch supplies device memory and the stream; the selector
+(``adaptic_plan``) and the kernels (``adaptic_run``) are the C ABI.  This module
+only checks shapes/dtypes, allocates ``y`` and the zero-filled workspace the
+split variants need, and caches plans per (op, shape, dtype, variant, device,
+stream) so repeated calls cost one ctypes call.
+
+Shapes (``include/adaptic.h``; reading R1):
+  mv(A[R, C], x[C])      -> y[R],  y_r = sum_c A[r, c] x[c]
+  tmv(B[C, R], x[C])     -> y[R],  y_r = sum_c B[c, r] x[c]   (B = A^T)
+  dot(a[N, L], b[N, L])  -> y[N],  y_n = sum_e a[n, e] b[n, e]  (1-D a, b: N = 1)
+dtype float32 (fp32 accumulate) or int32 (modulo 2^32).
+"""
+from __future__ import annotations
+
+import threading
+
+import torch
+
+from . import _lib as L
+
+_DT = {torch.float32: L.F32, torch.int32: L.I32}
+_cache: dict = {}
+_cache_lock = threading.Lock()
+
+
+def _dtype_code(t: torch.Tensor) -> int:
+    try:
+        return _DT[t.dtype]
+    except KeyError:
+        raise TypeError(f"adaptic supports float32 and int32, got {t.dtype}") from None
+
+
+def get_plan(op: int, rows: int, cols: int, dtype: int, device: torch.device,
+             variant="AUTO", params=None, stream: int = 0) -> L.Plan:
+    """Cached plan with its workspace attached (allocated zero-filled on `device`)."""
+    key = (op, int(rows), int(cols), dtype, variant, tuple(params) if params else None,
+           device.index, stream)
+    with _cache_lock:
+        ent = _cache.get(key)
+        if ent is not None:
+            return ent[0]
+    plan = L.Plan(op, rows, cols, dtype, variant, params)
+    ws = None
+    nbytes = plan.workspace_bytes
+    if nbytes:
+        ws = torch.zeros(nbytes, dtype=torch.uint8, device=device)
+        plan.set_workspace(ws.data_ptr(), nbytes)
+    with _cache_lock:
+        _cache.setdefault(key, (plan, ws))
+        return _cache[key][0]
+
+
+def clear_cache():
+    with _cache_lock:
+        _cache.clear()
+
+
+def _check_dev(*ts: torch.Tensor):
+    dev = ts[0].device
+    for t in ts:
+        if t.device.type != "cuda":
+            raise ValueError("adaptic runs on CUDA tensors only (there is no CPU path)")
+        if t.device != dev:
+            raise ValueError("all tensors must be on the same device")
+        if not t.is_contiguous():
+            raise ValueError("tensors must be contiguous (row-major)")
+        if t.dtype != ts[0].dtype:
+            raise TypeError("A and x must have the same dtype")
+    return dev
+
+
+def _run(op: int, M: torch.Tensor, X: torch.Tensor, R: int, C: int, variant, params, out):
+    dev = _check_dev(M, X)
+    dt = _dtype_code(M)
+    if out is None:
+        out = torch.empty(R, dtype=M.dtype, device=dev)
+    else:
+        _check_dev(M, out)
+        if out.numel() != R:
+            raise ValueError(f"out must have {R} elements")
+    stream = torch.cuda.current_stream(dev).cuda_stream
+    plan = get_plan(op, R, C, dt, dev, variant, params, stream)
+    plan.run(M.data_ptr(), X.data_ptr(), out.data_ptr(), stream)
+    return out
+
+
+def mv(A: torch.Tensor, x: torch.Tensor, *, variant="AUTO", params=None, out=None) -> torch.Tensor:
+    """y = A x for a row-major R x C matrix A (contiguous reductions)."""
+    if A.dim() != 2 or x.dim() != 1 or x.shape[0] != A.shape[1]:
+        raise ValueError(f"mv: A must be [R, C] and x [C], got {tuple(A.shape)}, {tuple(x.shape)}")
+    return _run(L.OP_MV, A, x, A.shape[0], A.shape[1], variant, params, out)
+
+
+def tmv(B: torch.Tensor, x: torch.Tensor, *, variant="AUTO", params=None, out=None) -> torch.Tensor:
+    """y = B^T x for a row-major C x R matrix B (the restructured layout; y has R entries)."""
+    if B.dim() != 2 or x.dim() != 1 or x.shape[0] != B.shape[0]:
+        raise ValueError(f"tmv: B must be [C, R] and x [C], got {tuple(B.shape)}, {tuple(x.shape)}")
+    return _run(L.OP_TMV, B, x, B.shape[1], B.shape[0], variant, params, out)
+
+
+def dot(a: torch.Tensor, b: torch.Tensor, *, variant="AUTO", params=None, out=None) -> torch.Tensor:
+    """Scalar products of N pairs: y[n] = <a[n], b[n]>; 1-D inputs are one pair."""
+    if a.shape != b.shape or a.dim() not in (1, 2):
+        raise ValueError(f"dot: a and b must both be [N, L] (or [L]), got {tuple(a.shape)}, {tuple(b.shape)}")
+    N, Lk = (1, a.shape[0]) if a.dim() == 1 else a.shape
+    return _run(L.OP_DOT, a, b, N, Lk, variant, params, out)
+
+
+def plan(op: str, rows: int, cols: int, dtype: str = "f32", variant="AUTO", params=None) -> L.Plan:
+    """A bare plan (no workspace attached) -- for inspecting the selector."""
+    return L.Plan({"mv": L.OP_MV, "tmv": L.OP_TMV, "dot": L.OP_DOT}[op], rows, cols,
+                  {"f32": L.F32, "i32": L.I32}[dtype], variant, params)
+
+
+def run_host(op: str, M_host: torch.Tensor, X_host: torch.Tensor, y_host: torch.Tensor,
+             dM: torch.Tensor, dX: torch.Tensor, dy: torch.Tensor, *, variant="AUTO"):
+    """End-to-end call with HOST buffers (pinned for async copies): the library
+    enqueues H2D copies of M and X into dM/dX, the kernel, and the D2H copy of y
+    on the current stream.  The caller synchronises before reading y_host."""
+    opc = {"mv": L.OP_MV, "tmv": L.OP_TMV, "dot": L.OP_DOT}[op]
+    if opc == L.OP_TMV:
+        C, R = M_host.shape
+    elif M_host.dim() == 1:
+        R, C = 1, M_host.shape[0]
+    else:
+        R, C = M_host.shape
+    dev = _check_dev(dM, dX, dy)
+    for t in (M_host, X_host, y_host):
+        if t.device.type != "cpu" or not t.is_contiguous():
+            raise ValueError("host buffers must be contiguous CPU tensors")
+    stream = torch.cuda.current_stream(dev).cuda_stream
+    plan = get_plan(opc, R, C, _dtype_code(dM), dev, variant, None, stream)
+    plan.run_host(M_host.data_ptr(), X_host.data_ptr(), y_host.data_ptr(),
+                  dM.data_ptr(), dX.data_ptr(), dy.data_ptr(), stream)
+    return y_host

@@ -145,3 +145,67 @@ def matrix(R: int, C: int, layout: str, dtype, kind: str, s: int,
     if layout == "tmv":
         return np.ascontiguousarray(a.T)
     raise ValueError(layout)
+
+
+# ---------------------------------------------------------------------------- device copy
+_dev_lib = None
+
+
+def _device_lib():
+    """ctypes handle of synth/libsynth.so (the CUDA twin of this generator)."""
+    global _dev_lib
+    if _dev_lib is None:
+        import ctypes
+        import os
+        path = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libsynth.so")
+        if not os.path.exists(path):
+            build_device()
+        L = ctypes.CDLL(path)
+        vp, i32, i64, u64 = ctypes.c_void_p, ctypes.c_int, ctypes.c_int64, ctypes.c_uint64
+        L.synth_fill_matrix.argtypes = [vp, i32, i32, i32, u64, i64, i64, i64, i64, i64, i64, vp]
+        L.synth_fill_matrix.restype = i32
+        L.synth_fill_vector.argtypes = [vp, i32, i32, u64, i64, i64, vp]
+        L.synth_fill_vector.restype = i32
+        _dev_lib = L
+    return _dev_lib
+
+
+def build_device(force: bool = False) -> str:
+    import os
+    import subprocess
+    here = os.path.dirname(os.path.abspath(__file__))
+    src, out = os.path.join(here, "synth_gen.cu"), os.path.join(here, "libsynth.so")
+    if force or not os.path.exists(out) or os.path.getmtime(out) < os.path.getmtime(src):
+        tmp = out + ".tmp.%d" % os.getpid()
+        subprocess.check_call(["/usr/local/cuda/bin/nvcc", "-gencode", "arch=compute_100a,code=sm_100a",
+                               "-O3", "-std=c++17", "-Xcompiler", "-fPIC", "-shared", "-o", tmp, src])
+        os.replace(tmp, out)
+    return out
+
+
+def device_matrix(t, R: int, C: int, layout: str, kind: str, s: int, rows=None, cols=None, stream: int = 0):
+    """Fill the CUDA tensor ``t`` (float32/int32, contiguous) with the [r0,r1) x [c0,c1)
+    block of the logical matrix, in ``layout`` -- same values as :func:`matrix`."""
+    import torch
+    r0, r1 = rows if rows is not None else (0, R)
+    c0, c1 = cols if cols is not None else (0, C)
+    assert t.is_cuda and t.is_contiguous() and t.numel() == (r1 - r0) * (c1 - c0)
+    dt = {torch.float32: 0, torch.int32: 1}[t.dtype]
+    rc = _device_lib().synth_fill_matrix(t.data_ptr(), dt, {"mv": 0, "tmv": 1}[layout], KIND_CODE[kind],
+                                         s & _MASK64, R, C, r0, r1, c0, c1, stream or None)
+    if rc:
+        raise RuntimeError(f"synth_fill_matrix cuda error {rc}")
+    return t
+
+
+def device_vector(t, kind: str, s: int, start: int = 0, stream: int = 0):
+    import torch
+    assert t.is_cuda and t.is_contiguous()
+    if kind not in VECTOR_KINDS:
+        raise ValueError(kind)
+    dt = {torch.float32: 0, torch.int32: 1}[t.dtype]
+    rc = _device_lib().synth_fill_vector(t.data_ptr(), dt, KIND_CODE[kind], s & _MASK64, start, t.numel(),
+                                         stream or None)
+    if rc:
+        raise RuntimeError(f"synth_fill_vector cuda error {rc}")
+    return t

@@ -1,0 +1,132 @@
+#!/usr/bin/env python
+"""Fixed-variant sweep on the GPU: every variant x parameter grid on every shape.
+
+The paper's compiler estimated break-even points with a performance model
+(P:222-232); here they are MEASURED: this tool times each (shape, variant,
+params) with CUDA events and writes one JSON line per run; tools/fit_thresholds.py
+turns the lines into the selector table (csrc/table_data.inc).
+
+  python tools/sweep.py --out gpurun_out/sweep.jsonl [--elems 26] [--ops mv,tmv] [--dtype f32]
+"""
+import argparse
+import itertools
+import json
+import os
+import statistics
+import sys
+import time
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+import torch  # noqa: E402
+
+import synth  # noqa: E402
+import paper_conf_pldi_samadihmlm12_b200 as adaptic  # noqa: E402
+from paper_conf_pldi_samadihmlm12_b200 import _lib as L  # noqa: E402
+
+OPC = {"mv": L.OP_MV, "tmv": L.OP_TMV, "dot": L.OP_DOT}
+
+
+def grids(op, R, C):
+    """(variant, params) candidates; params = [lanes, splits, ctas_per_sm, unroll], 0 = auto."""
+    out = [("AUTO", None)]
+    if op in ("mv", "dot"):
+        nv = C // 4 if C % 4 == 0 else C
+        xms = (1, 2) if op == "mv" and C * 4 <= 200 * 1024 else (0,)
+        for xm in xms:
+            for g in (1, 2, 4, 8, 16):
+                if g <= max(1, nv):
+                    for u in (1, 2, 4, 8):
+                        if g * u <= max(4, 2 * nv):
+                            out.append(("MV_SUBWARP", [g, 0, 0, u, xm]))
+            for u in (1, 2, 4, 8):
+                if 32 * u <= max(32, 2 * nv):
+                    out.append(("MV_WPR", [0, 0, 0, u, xm]))
+            for nt in (256, 1024):
+                for u in (2, 4, 8):
+                    out.append(("MV_CPR", [nt, 0, 0, u, xm]))
+        for nt in (256, 1024):
+            for u in (2, 4, 8):
+                out.append(("MV_SPLIT", [nt, 0, 0, u]))
+        for nt in (128, 256):
+            for st in (2, 4, 8):
+                out.append(("MV_TPR", [nt, 0, 0, st]))
+    else:
+        rv = R // 4 if R % 4 == 0 else R
+        for u in (2, 4, 8):
+            out.append(("TMV_COL", [0, 0, 0, u]))
+        for lr in (1, 2, 4, 8, 16, 32, 64, 128, 256):
+            if lr <= max(1, 2 * rv):
+                for u in (2, 4, 8):
+                    out.append(("TMV_SPLITK", [lr, 0, 0, u]))
+        for u in (2, 4, 8):
+            out.append(("TMV_REGTILE", [0, 0, 0, u]))
+    return out
+
+
+def time_plan(plan, ptrs, stream, reps):
+    for _ in range(2):
+        plan.run(*ptrs, stream)
+    torch.cuda.synchronize()
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(reps)]
+    for a, b in evs:
+        a.record()
+        plan.run(*ptrs, stream)
+        b.record()
+    torch.cuda.synchronize()
+    return [a.elapsed_time(b) * 1e3 for a, b in evs]
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--out", required=True)
+    ap.add_argument("--elems", default="26", help="comma list of log2(R*C) diagonals")
+    ap.add_argument("--ops", default="mv,tmv")
+    ap.add_argument("--dtype", default="f32")
+    ap.add_argument("--reps", type=int, default=9)
+    ap.add_argument("--kmin", type=int, default=3)
+    ap.add_argument("--kmax", type=int, default=23)
+    ap.add_argument("--extra", default="", help="extra shapes R1xC1,R2xC2")
+    a = ap.parse_args()
+    dev = torch.device("cuda:0")
+    tdt = torch.float32 if a.dtype == "f32" else torch.int32
+    dtc = L.F32 if a.dtype == "f32" else L.I32
+    stream = torch.cuda.current_stream().cuda_stream
+    shapes = []
+    for e in (int(v) for v in a.elems.split(",")):
+        for k in range(a.kmin, min(a.kmax, e - 3) + 1):
+            shapes.append((1 << k, 1 << (e - k)))
+    for s in filter(None, a.extra.split(",")):
+        r, c = s.lower().split("x")
+        shapes.append((int(r), int(c)))
+    maxel = max(R * C for R, C in shapes)
+    M = torch.empty(maxel * (2 if "dot" in a.ops else 1), dtype=tdt, device=dev)
+    X = torch.empty(max(C for _, C in shapes), dtype=tdt, device=dev)
+    Y = torch.empty(max(R for R, _ in shapes), dtype=tdt, device=dev)
+    synth.device_matrix(M, 1, M.numel(), "mv", "uniform", 11)
+    synth.device_vector(X, "uniform", 12)
+    t0 = time.time()
+    with open(a.out, "a") as f:
+        for op in a.ops.split(","):
+            for R, C in shapes:
+                Xp = M.data_ptr() + R * C * 4 if op == "dot" else X.data_ptr()
+                ptrs = (M.data_ptr(), Xp, Y.data_ptr())
+                for variant, params in grids(op, R, C):
+                    try:
+                        plan = adaptic.get_plan(OPC[op], R, C, dtc, dev, variant, params, stream)
+                    except adaptic.AdapticError:
+                        continue
+                    ts = time_plan(plan, ptrs, stream, a.reps)
+                    med = statistics.median(ts)
+                    nbytes = 4 * (R * C * (2 if op == "dot" else 1) + R + (0 if op == "dot" else C))
+                    d = plan.describe()
+                    f.write(json.dumps({"op": op, "dtype": a.dtype, "R": R, "C": C, "variant": d["variant"],
+                                        "req": variant, "params": params, "us": med, "us_min": min(ts),
+                                        "GBps": nbytes / med / 1e3, "plan": d}) + "\n")
+                adaptic.clear_cache()
+                f.flush()
+    print(f"sweep done in {time.time() - t0:.1f}s", file=sys.stderr)
+
+
+if __name__ == "__main__":
+    main()
