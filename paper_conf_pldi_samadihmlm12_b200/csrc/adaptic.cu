@@ -58,11 +58,11 @@ namespace {
 thread_local int g_last_cuda_error = 0;
 
 struct TableEntry {
-    int op, dtype, lr, lc, variant, lanes, splits, ctas_per_sm, unroll, xsmem;
+    int op, dtype, lr, lc, variant, lanes, splits, ctas_per_sm, unroll, xsmem, block;
 };
 const TableEntry kTable[] = {
 #include "table_data.inc"
-    {-1, -1, 0, 0, 0, 0, 0, 0, 0, 0}};
+    {-1, -1, 0, 0, 0, 0, 0, 0, 0, 0, 0}};
 const int kTableN = int(sizeof(kTable) / sizeof(kTable[0])) - 1;
 
 const char* const kVariantNames[ADAPTIC_V_COUNT] = {
@@ -111,8 +111,8 @@ int pick_xmode(bool px, int req, int64_t C, bool allow) {
     if (req == 1) return 0;
     return C * 4 <= kXsAutoBytes ? 1 : 0;
 }
-void* tmv_fn(int dtype, int LR, int U, bool vec) {
-    return dtype == DT_F32 ? tmv_fn_f32(LR, U, vec) : tmv_fn_i32(LR, U, vec);
+void* tmv_fn(int dtype, int LR, int U, bool vec, int NT) {
+    return dtype == DT_F32 ? tmv_fn_f32(LR, U, vec, NT) : tmv_fn_i32(LR, U, vec, NT);
 }
 
 int occupancy(void* fn, int block, size_t smem, bool present, int fallback) {
@@ -132,6 +132,26 @@ bool bound_ok(int64_t m) {
 }
 int64_t fold_chain(int64_t iters) { return std::min<int64_t>(iters, FOLD) + iters / FOLD; }
 int ilog2c(int64_t v) { int k = 0; while ((int64_t(1) << k) < v) ++k; return k; }
+
+// Split count for `units` independent reductions on `slots` resident CTAs: the
+// grid-stride kernels take ceil(units*S / slots) rounds, so pick the smallest S
+// in [smin, smax] whose last round is >= 90 % full and that fills >= 1 round
+// (more splits only add partials to merge); else the best-filled S up to 4 rounds.
+int64_t pick_splits(int64_t units, int64_t slots, int64_t smax, int64_t smin) {
+    units = std::max<int64_t>(1, units);
+    smax = std::max(smin, smax);
+    const int64_t hi = std::min(smax, std::max(smin, ceil_div(4 * slots, units)));
+    int64_t best = smin;
+    double best_eff = -1.0;
+    for (int64_t S = smin; S <= hi; ++S) {
+        const int64_t nblk = units * S;
+        const int64_t rounds = ceil_div(nblk, slots);
+        const double eff = double(nblk) / double(rounds * slots);
+        if (nblk >= slots && eff >= 0.9) return S;
+        if (eff > best_eff + 1e-9) { best_eff = eff; best = S; }
+    }
+    return best;
+}
 
 // ---------------------------------------------------------------- heuristic (no table cell)
 int heuristic_variant(int op, int64_t R, int64_t C, int sms) {
@@ -161,7 +181,10 @@ const TableEntry* table_lookup(int op, int dtype, int64_t R, int64_t C) {
             best = &e; bestd = d;
         }
     }
-    return (best && bestd <= 2) ? best : nullptr;
+    if (best && bestd <= 2) return best;
+    // int32 moves the same bytes as fp32: use the fp32 cells when int32 was not swept
+    if (dtype != ADAPTIC_F32) return table_lookup(op, ADAPTIC_F32, R, C);
+    return nullptr;
 }
 
 // Fill the kernel parameters of `p` for p->variant.  params: user overrides or nullptr.
@@ -272,8 +295,7 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
         if (v == ADAPTIC_V_MV_SPLIT) {
             if (par(ADAPTIC_P_SPLITS) > 0) S = par(ADAPTIC_P_SPLITS);
             else {
-                S = std::max<int64_t>(2, ceil_div(2 * slots, std::max<int64_t>(1, R)));   // ~2 waves
-                S = std::min<int64_t>(S, std::max<int64_t>(2, ceil_div(nv1, int64_t(NT) * U)));
+                S = pick_splits(R, slots, std::max<int64_t>(2, ceil_div(nv1, int64_t(NT) * U)), 2);
             }
         }
         // accuracy: raise S (SPLIT only) until the bound holds on both paths
@@ -316,17 +338,19 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
     int U = par(ADAPTIC_P_UNROLL);
     if (U <= 0) U = (v == ADAPTIC_V_TMV_COL) ? 8 : 4;
     if (U != 2 && U != 4 && U != 8) return ADAPTIC_ERR_INVALID_ARG;
+    int NT = par(ADAPTIC_P_BLOCK);
+    if (NT <= 0) NT = TMV_NT;
+    if ((NT != 256 && NT != 1024) || (NT == 1024 && U > 4)) return ADAPTIC_ERR_INVALID_ARG;
     int cps = par(ADAPTIC_P_CTAS_PER_SM);
-    if (cps <= 0) cps = occupancy(tmv_fn(dt, LR, U, p->vec_shape), TMV_NT, 0, dev.present, 4);
-    p->lanes = LR; p->unroll = U; p->block = TMV_NT; p->ctas_per_sm = cps;
-    const int LC = TMV_NT / LR;
+    if (cps <= 0) cps = occupancy(tmv_fn(dt, LR, U, p->vec_shape, NT), NT, 0, dev.present, 2048 / NT);
+    p->lanes = LR; p->unroll = U; p->block = NT; p->ctas_per_sm = cps;
+    const int LC = NT / LR;
     const int64_t slots = int64_t(dev.sms) * cps;
     const int64_t tiles1 = ceil_div(rv1, LR);
     int64_t S = 1;
     if (par(ADAPTIC_P_SPLITS) > 0) S = par(ADAPTIC_P_SPLITS);
     else if (v != ADAPTIC_V_TMV_COL) {
-        S = std::max<int64_t>(1, ceil_div(2 * slots, tiles1));                        // ~2 waves
-        S = std::min<int64_t>(S, std::max<int64_t>(1, ceil_div(C, int64_t(LC) * U)));  // >= 1 step each
+        S = pick_splits(tiles1, slots, std::max<int64_t>(1, ceil_div(C, int64_t(LC) * U)), 1);
     }
     for (;;) {
         bool ok_all = true;
@@ -392,7 +416,7 @@ adaptic_status make_plan(int op, int64_t rows, int64_t cols, int dtype, int vari
         return ADAPTIC_OK;
     }
     if (const TableEntry* e = table_lookup(op, dtype, rows, cols)) {
-        int32_t tp[ADAPTIC_NPARAMS] = {e->lanes, e->splits, e->ctas_per_sm, e->unroll, e->xsmem};
+        int32_t tp[ADAPTIC_NPARAMS] = {e->lanes, e->splits, e->ctas_per_sm, e->unroll, e->xsmem, e->block};
         p->variant = e->variant; p->source = 1;
         if (derive(p, tp, dev) == ADAPTIC_OK) { *out = p; return ADAPTIC_OK; }
         if (derive(p, nullptr, dev) == ADAPTIC_OK) { *out = p; return ADAPTIC_OK; }
@@ -498,7 +522,7 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
             args = args8;
             break;
         default:
-            fn = tmv_fn(dt, p->lanes, p->unroll, vec);
+            fn = tmv_fn(dt, p->lanes, p->unroll, vec, p->block);
             args8[0] = &A; args8[1] = &X; args8[2] = &y; args8[3] = &R; args8[4] = &C;
             args8[5] = &S; args8[6] = &part; args8[7] = &cnt;
             args = args8;

@@ -16,7 +16,7 @@ constexpr int FOLD = 512;
 enum Dtype { DT_F32 = 0, DT_I32 = 1 };
 
 constexpr int GROUP_NT = 256;   // threads per CTA, mv_group_kernel
-constexpr int TMV_NT = 256;     // threads per CTA, tmv_kernel
+constexpr int TMV_NT = 256;     // default threads per CTA, tmv_kernel (256 or 1024)
 
 // Kernel instance lookup: a __global__ function pointer for cudaLaunchKernel /
 // cudaOccupancyMaxActiveBlocksPerMultiprocessor, or nullptr when the instance
@@ -29,8 +29,8 @@ constexpr int TMV_NT = 256;     // threads per CTA, tmv_kernel
 // 1 staged in shared memory by TMA (dynamic smem = C*4 bytes), 2 per-row (DOT)
 void* group_fn_f32(int G, int U, bool vec, int xmode);
 void* group_fn_i32(int G, int U, bool vec, int xmode);
-void* tmv_fn_f32(int LR, int U, bool vec);
-void* tmv_fn_i32(int LR, int U, bool vec);
+void* tmv_fn_f32(int LR, int U, bool vec, int NT);
+void* tmv_fn_i32(int LR, int U, bool vec, int NT);
 void* cta_fn(int dtype, int NT, int U, bool vec, int xmode);
 void* tpr_fn(int dtype, int NT, bool perrowx);
 

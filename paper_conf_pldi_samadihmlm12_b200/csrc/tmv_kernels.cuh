@@ -70,8 +70,26 @@ __device__ __forceinline__ E lc_combine(E v, E* red) {
     }
 }
 
+// Sum of partials p[k*stride] for k = k0, k0+STEP, ... < S: two independent
+// loads in flight per round into two accumulators (kept register-light: the
+// kernel's register count -- and so its occupancy -- is set by its largest
+// section), then a fixed combine, so the result does not depend on timing.
+template <int STEP, class E>
+__device__ __forceinline__ E merge_partials(const E* p, int64_t stride, int k0, int S) {
+    E m0 = zero_of<E>(), m1 = zero_of<E>();
+    int k = k0;
+    for (; k + STEP < S; k += 2 * STEP) {
+        const E t0 = ld_partial(p + int64_t(k) * stride);
+        const E t1 = ld_partial(p + int64_t(k + STEP) * stride);
+        m0 = eadd(m0, t0);
+        m1 = eadd(m1, t1);
+    }
+    if (k < S) m0 = eadd(m0, ld_partial(p + int64_t(k) * stride));
+    return eadd(m0, m1);
+}
+
 template <class T, int LR, int U, bool VEC, int NT>
-__global__ void __launch_bounds__(NT)
+__global__ void __launch_bounds__(NT, NT <= 256 ? (U <= 2 ? 6 : 4) : 1)
 tmv_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restrict__ y,
            int64_t R, int64_t C, int S, T* __restrict__ ws_part, unsigned int* __restrict__ ws_cnt)
 {
@@ -135,7 +153,7 @@ tmv_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restrict__ y,
             if (ticket_is_last(ws_cnt + tile, unsigned(S), &flag)) {
                 E m = zero_of<E>();
                 if (rok)
-                    for (int k = lc; k < S; k += LC) m = eadd(m, ld_partial(pv + int64_t(k) * rv + r4));
+                    m = merge_partials<LC>(pv + r4, rv, lc, S);
                 __syncthreads();  // red[] reuse
                 m = lc_combine<NT, LR>(m, red);
                 if (tid < LR && rok) yv[r4] = m;

@@ -56,9 +56,12 @@ def mv_rowshard(A_local: torch.Tensor, x: torch.Tensor, *, group=None, gather: b
     G, _ = _world(group)
     sizes = [None] * G
     dist.all_gather_object(sizes, int(y_local.numel()), group=group)
-    parts = [torch.empty(s, dtype=y_local.dtype, device=y_local.device) for s in sizes]
-    dist.all_gather(parts, y_local.contiguous(), group=group)
-    return torch.cat(parts)
+    width = max(sizes)                  # collectives need equal sizes: pad, gather, trim
+    padded = torch.zeros(width, dtype=y_local.dtype, device=y_local.device)
+    padded[: y_local.numel()] = y_local
+    parts = [torch.empty(width, dtype=y_local.dtype, device=y_local.device) for _ in sizes]
+    dist.all_gather(parts, padded, group=group)
+    return torch.cat([p[:s] for p, s in zip(parts, sizes)])
 
 
 def combine_splitk(y_part: torch.Tensor, *, group=None,
@@ -72,7 +75,7 @@ def combine_splitk(y_part: torch.Tensor, *, group=None,
         raise TypeError("split-K combine supports float32 and int32")
     G, _ = _world(group)
     P = torch.empty(G, y_part.numel(), dtype=torch.int32, device=y_part.device)
-    dist.all_gather_into_tensor(P, y_part.contiguous(), group=group)
+    dist.all_gather(list(P.unbind(0)), y_part.contiguous().view(-1), group=group)
     if merge_fn is not None:
         return merge_fn(P)
     ones = torch.ones(G, dtype=torch.int32, device=P.device)

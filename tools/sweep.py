@@ -28,7 +28,7 @@ OPC = {"mv": L.OP_MV, "tmv": L.OP_TMV, "dot": L.OP_DOT}
 
 
 def grids(op, R, C):
-    """(variant, params) candidates; params = [lanes, splits, ctas_per_sm, unroll], 0 = auto."""
+    """(variant, params) candidates; params = [lanes, splits, ctas_per_sm, unroll, xsmem, block], 0 = auto."""
     out = [("AUTO", None)]
     if op in ("mv", "dot"):
         nv = C // 4 if C % 4 == 0 else C
@@ -55,10 +55,17 @@ def grids(op, R, C):
         rv = R // 4 if R % 4 == 0 else R
         for u in (2, 4, 8):
             out.append(("TMV_COL", [0, 0, 0, u]))
-        for lr in (1, 2, 4, 8, 16, 32, 64, 128, 256):
-            if lr <= max(1, 2 * rv):
-                for u in (2, 4, 8):
-                    out.append(("TMV_SPLITK", [lr, 0, 0, u]))
+        for nt in (256, 1024):
+            for lr in (1, 2, 4, 8, 16, 32, 64, 128, 256):
+                if lr > max(1, 2 * rv) or (rv >= 4096 and lr < 8):
+                    continue
+                tiles = -(-rv // lr)
+                splits = sorted({0} | {max(1, -(-148 * k // tiles)) for k in (1, 2, 4, 8)})
+                for u in ((2, 4, 8) if nt == 256 else (2, 4)):
+                    for sp in splits:
+                        if sp > C:
+                            continue
+                        out.append(("TMV_SPLITK", [lr, sp, 0, u, 0, nt]))
         for u in (2, 4, 8):
             out.append(("TMV_REGTILE", [0, 0, 0, u]))
     return out
