@@ -146,14 +146,17 @@ typedef enum {
  *   [ADAPTIC_P_XSMEM]  MV_SUBWARP / MV_WPR / MV_CPR: 1 = read x through the
  *                      read-only cache path, 2 = stage x in shared memory once per
  *                      CTA with a TMA bulk copy (needs cols*4 <= 200 KB).
- *   [ADAPTIC_P_BLOCK]  TMV_*: threads per CTA, 256 or 1024 (unroll <= 4 at 1024). */
+ *   [ADAPTIC_P_BLOCK]  TMV_*: threads per CTA, 256 or 1024 (unroll <= 4 at 1024).
+ *   [ADAPTIC_P_ROWS]   MV_CPR / MV_SPLIT: rows per CTA step sharing each x load,
+ *                      (rows, unroll) in {(1,2),(1,4),(1,8),(2,2),(2,4),(4,2)}. */
 #define ADAPTIC_P_LANES 0
 #define ADAPTIC_P_SPLITS 1
 #define ADAPTIC_P_CTAS_PER_SM 2
 #define ADAPTIC_P_UNROLL 3
 #define ADAPTIC_P_XSMEM 4
 #define ADAPTIC_P_BLOCK 5
-#define ADAPTIC_NPARAMS 6
+#define ADAPTIC_P_ROWS 6
+#define ADAPTIC_NPARAMS 7
 
 typedef struct adaptic_plan_s* adaptic_plan_t;   /* opaque; owned by the caller */
 

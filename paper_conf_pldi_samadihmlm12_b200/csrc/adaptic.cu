@@ -58,11 +58,11 @@ namespace {
 thread_local int g_last_cuda_error = 0;
 
 struct TableEntry {
-    int op, dtype, lr, lc, variant, lanes, splits, ctas_per_sm, unroll, xsmem, block;
+    int op, dtype, lr, lc, variant, lanes, splits, ctas_per_sm, unroll, xsmem, block, rows;
 };
 const TableEntry kTable[] = {
 #include "table_data.inc"
-    {-1, -1, 0, 0, 0, 0, 0, 0, 0, 0, 0}};
+    {-1, -1, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0}};
 const int kTableN = int(sizeof(kTable) / sizeof(kTable[0])) - 1;
 
 const char* const kVariantNames[ADAPTIC_V_COUNT] = {
@@ -280,22 +280,27 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
         int NT = par(ADAPTIC_P_LANES);
         if (NT <= 0) NT = (v == ADAPTIC_V_MV_CPR && nv1 >= 8192) ? 1024 : 256;
         if (NT != 256 && NT != 1024) return ADAPTIC_ERR_INVALID_ARG;
+        int RB = par(ADAPTIC_P_ROWS);
+        if (RB <= 0) RB = 1;
         int U = par(ADAPTIC_P_UNROLL);
-        if (U <= 0) U = 4;
-        if (U != 2 && U != 4 && U != 8) return ADAPTIC_ERR_INVALID_ARG;
+        if (U <= 0) U = RB == 4 ? 2 : 4;
+        const bool combo_ok = (RB == 1 && (U == 2 || U == 4 || U == 8)) || (RB == 2 && (U == 2 || U == 4)) ||
+                              (RB == 4 && U == 2);
+        if (!combo_ok || (NT == 1024 && RB * U > 4)) return ADAPTIC_ERR_INVALID_ARG;
         // x staged in smem only for CPR (a split CTA reads a different x chunk per block)
         const int xm = pick_xmode(px, par(ADAPTIC_P_XSMEM), C, v == ADAPTIC_V_MV_CPR);
         if (xm < 0) return ADAPTIC_ERR_UNSUPPORTED;
         const size_t xsm = xm == 1 ? size_t((C * 4 + 15) / 16 * 16) : 0;
         int cps = par(ADAPTIC_P_CTAS_PER_SM);
-        if (cps <= 0) cps = occupancy(cta_fn(dt, NT, U, p->vec_shape, xm), NT, xsm, dev.present, 2048 / NT);
-        p->lanes = NT; p->unroll = U; p->block = NT; p->ctas_per_sm = cps; p->xmode = xm; p->smem = xsm;
+        if (cps <= 0) cps = occupancy(cta_fn(dt, NT, RB, U, p->vec_shape, xm), NT, xsm, dev.present, 2048 / NT);
+        p->lanes = NT; p->unroll = U; p->rb = RB; p->block = NT; p->ctas_per_sm = cps; p->xmode = xm; p->smem = xsm;
         const int64_t slots = int64_t(dev.sms) * cps;
+        const int64_t groups = ceil_div(R, RB);
         int64_t S = 1;
         if (v == ADAPTIC_V_MV_SPLIT) {
             if (par(ADAPTIC_P_SPLITS) > 0) S = par(ADAPTIC_P_SPLITS);
             else {
-                S = pick_splits(R, slots, std::max<int64_t>(2, ceil_div(nv1, int64_t(NT) * U)), 2);
+                S = pick_splits(groups, slots, std::max<int64_t>(2, ceil_div(nv1, int64_t(NT) * U)), 2);
             }
         }
         // accuracy: raise S (SPLIT only) until the bound holds on both paths
@@ -308,7 +313,7 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
                 p->chain[w] = fold_chain(iters);
                 p->depth[w] = ilog2c(U) + (w ? 2 : 0) + ilog2c(NT) + (S > 1 ? ceil_div(S, NT) + ilog2c(NT) : 0) + 1;
                 p->path_ok[w] = (dt == DT_I32) || bound_ok(p->chain[w] + p->depth[w]);
-                p->grid[w] = std::max<int64_t>(1, std::min<int64_t>(R * S, slots));
+                p->grid[w] = std::max<int64_t>(1, std::min<int64_t>(groups * S, slots));
                 if (!p->path_ok[w]) ok_all = false;
             }
             if (ok_all || v == ADAPTIC_V_MV_CPR || S >= (int64_t(1) << 20)) break;
@@ -320,7 +325,7 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
         if (S > 1) {
             const size_t part = ((size_t(R) * size_t(S) * 4 + 255) / 256) * 256;
             p->cnt_off = part;
-            p->ws_bytes = part + size_t(R) * 4;
+            p->ws_bytes = part + size_t(groups) * 4;
         }
         return ADAPTIC_OK;
     }
@@ -416,7 +421,7 @@ adaptic_status make_plan(int op, int64_t rows, int64_t cols, int dtype, int vari
         return ADAPTIC_OK;
     }
     if (const TableEntry* e = table_lookup(op, dtype, rows, cols)) {
-        int32_t tp[ADAPTIC_NPARAMS] = {e->lanes, e->splits, e->ctas_per_sm, e->unroll, e->xsmem, e->block};
+        int32_t tp[ADAPTIC_NPARAMS] = {e->lanes, e->splits, e->ctas_per_sm, e->unroll, e->xsmem, e->block, e->rows};
         p->variant = e->variant; p->source = 1;
         if (derive(p, tp, dev) == ADAPTIC_OK) { *out = p; return ADAPTIC_OK; }
         if (derive(p, nullptr, dev) == ADAPTIC_OK) { *out = p; return ADAPTIC_OK; }
@@ -446,6 +451,15 @@ adaptic_status cuda_fail(cudaError_t e) {
     g_last_cuda_error = int(e);
     (void)cudaGetLastError();
     return ADAPTIC_ERR_CUDA;
+}
+
+// ADAPTIC_PDL=0 disables programmatic dependent launch (read once).
+bool pdl_enabled() {
+    static const bool on = [] {
+        const char* v = std::getenv("ADAPTIC_PDL");
+        return !(v && v[0] == '0');
+    }();
+    return on;
 }
 
 std::mutex g_attr_mu;
@@ -515,7 +529,7 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
             break;
         case ADAPTIC_V_MV_CPR:
         case ADAPTIC_V_MV_SPLIT:
-            fn = cta_fn(dt, p->lanes, p->unroll, vec, p->xmode);
+            fn = cta_fn(dt, p->lanes, p->rb, p->unroll, vec, p->xmode);
             smem = p->smem;
             args8[0] = &A; args8[1] = &X; args8[2] = &y; args8[3] = &R; args8[4] = &C;
             args8[5] = &S; args8[6] = &part; args8[7] = &cnt;
@@ -534,7 +548,20 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
         if (ea != cudaSuccess) return cuda_fail(ea);
     }
     if (grid > INT_MAX) grid = INT_MAX;
-    cudaError_t e = cudaLaunchKernel(fn, dim3(unsigned(grid)), dim3(unsigned(block)), args, smem, stream);
+    // Programmatic dependent launch: the kernel may be scheduled while the previous
+    // grid on the stream drains; every kernel begins with griddepcontrol.wait, so it
+    // still observes all of that grid's writes (common.cuh pdl_prologue).
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(unsigned(grid));
+    cfg.blockDim = dim3(unsigned(block));
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = stream;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = pdl_enabled() ? 1 : 0;
+    cudaError_t e = cudaLaunchKernelExC(&cfg, fn, args);
     if (e != cudaSuccess) return cuda_fail(e);
     return ADAPTIC_OK;
 }

@@ -83,6 +83,17 @@ __device__ __forceinline__ uint32_t ld_partial(const uint32_t* p) { return __ldc
 __device__ __forceinline__ float4 ld_partial(const float4* p) { return __ldcg(p); }
 __device__ __forceinline__ uint4 ld_partial(const uint4* p) { return __ldcg(p); }
 
+// ---------------------------------------------------------------- programmatic dependent launch
+// Every kernel is launched with cudaLaunchAttributeProgrammaticStreamSerialization,
+// so it may be scheduled while the previous kernel on the stream drains.  It must
+// therefore wait for that grid (and its memory) before touching inputs, and it
+// immediately allows the NEXT kernel to be scheduled into SMs its own CTAs free.
+// Without PDL both instructions are no-ops.
+__device__ __forceinline__ void pdl_prologue() {
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    asm volatile("griddepcontrol.launch_dependents;" :::);
+}
+
 // ---------------------------------------------------------------- TMA bulk copy + mbarrier
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));

@@ -100,6 +100,7 @@ __global__ void __launch_bounds__(NT)
 mv_group_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restrict__ y,
                 int64_t R, int64_t C)
 {
+    pdl_prologue();
     using E = typename ElemOf<T, VEC>::type;
     constexpr int W = ElemOf<T, VEC>::W;
     constexpr int NG = 32 / G;
@@ -179,73 +180,128 @@ mv_group_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restrict_
 }
 
 // ------------------------------------------------------------------ MV_CPR / MV_SPLIT
-// One CTA per (row, split).  The row's vector range is cut into S contiguous
-// chunks; thread t reads vectors t, t+NT, ... of its chunk (U loads in flight,
-// unpredicated main loop + predicated tail).  S == 1: the CTA writes y[row].
-// S > 1: the CTA writes its partial to ws_part[row*S + s]; the last CTA of the
-// row (ticket) sums the S partials in a fixed order and writes y[row].
-template <class T, int NT, int U, bool VEC, int XM>
+// One CTA per (group of RB consecutive rows, split).  The rows' vector range is
+// cut into S contiguous chunks; thread t reads vectors t, t+NT, ... of its chunk
+// for all RB rows at once (RB*U loads in flight, unpredicated main loop +
+// predicated tail), so each x vector is fetched once per RB rows -- without
+// that, x (C*4 bytes) is re-read from L2 for every row and doubles the
+// on-chip traffic of long rows.  RB > 1 is the paper's horizontal thread
+// integration applied to the block-per-row kernel.
+// S == 1: the CTA writes y for its rows.  S > 1: it writes partials
+// ws_part[row*S + s]; the last CTA of the row group (ticket) sums the S partials
+// of each row in a fixed order and writes y.
+//
+// Block combine of RB values: warp butterfly, one smem stage, fixed order.
+template <int NT, int RB, class T>
+__device__ __forceinline__ void cta_sum_rows(T (&v)[RB], T* red /* RB*(NT/32) */) {
+    constexpr int NW = NT / 32;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+#pragma unroll
+    for (int i = 0; i < RB; ++i) v[i] = group_sum<32>(v[i]);
+    if (lane == 0) {
+#pragma unroll
+        for (int i = 0; i < RB; ++i) red[i * NW + warp] = v[i];
+    }
+    __syncthreads();
+    if (threadIdx.x < RB) {
+        T t = T(0);
+#pragma unroll
+        for (int w = 0; w < NW; ++w) t += red[threadIdx.x * NW + w];
+        v[0] = t;                         // thread i < RB holds row i's total in v[0]
+    }
+}
+
+template <class T, int NT, int RB, int U, bool VEC, int XM>
 __global__ void __launch_bounds__(NT)
 mv_cta_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restrict__ y,
               int64_t R, int64_t C, int S, T* __restrict__ ws_part, unsigned int* __restrict__ ws_cnt)
 {
+    pdl_prologue();
     using E = typename ElemOf<T, VEC>::type;
     constexpr int W = ElemOf<T, VEC>::W;
     constexpr bool PERROWX = (XM == XM_ROW);
-    __shared__ T red[NT / 32];
+    __shared__ T red[RB * (NT / 32)];
     __shared__ unsigned int flag;
     const int64_t nv = C / W;
     const int64_t chunk = (nv + S - 1) / S;
     const E* __restrict__ Av = reinterpret_cast<const E*>(A);
     const E* __restrict__ Xv = stage_x<T, VEC, XM, NT>(X, nv);   // XM_SMEM only with S == 1
     const int tid = threadIdx.x;
-    const int64_t nblk = R * S;
+    const int64_t ngroups = (R + RB - 1) / RB;
+    const int64_t nblk = ngroups * S;
 
     for (int64_t blk = blockIdx.x; blk < nblk; blk += gridDim.x) {
-        const int64_t row = blk / S;
-        const int s = int(blk - row * S);
+        const int64_t grp = blk / S;
+        const int s = int(blk - grp * S);
+        const int64_t row0 = grp * RB;
         const int64_t v0 = int64_t(s) * chunk;
         const int64_t v1 = min(nv, v0 + chunk);
-        const E* __restrict__ Ar = Av + row * nv;
-        const E* __restrict__ Xr = PERROWX ? Xv + row * nv : Xv;
-
-        E acc[U];
+        int64_t off[RB];                   // rows past R read row 0 (discarded)
 #pragma unroll
-        for (int u = 0; u < U; ++u) acc[u] = zero_of<E>();
-        T outer = T(0);
+        for (int i = 0; i < RB; ++i) off[i] = (row0 + i < R ? row0 + i : 0) * nv;
+
+        E acc[RB][U];
+#pragma unroll
+        for (int i = 0; i < RB; ++i)
+#pragma unroll
+            for (int u = 0; u < U; ++u) acc[i][u] = zero_of<E>();
+        T outer[RB];
+#pragma unroll
+        for (int i = 0; i < RB; ++i) outer[i] = T(0);
         int it = 0;
         int64_t v = v0 + tid;
         for (; v + int64_t(NT) * (U - 1) < v1; v += int64_t(NT) * U) {
-            E a[U], b[U];
+            E a[RB][U], b[PERROWX ? RB : 1][U];
 #pragma unroll
             for (int u = 0; u < U; ++u) {
-                a[u] = ld_stream(Ar + v + int64_t(NT) * u);
-                b[u] = PERROWX ? ld_stream(Xr + v + int64_t(NT) * u) : ld_xm<XM>(Xr + v + int64_t(NT) * u);
+                const int64_t vv = v + int64_t(NT) * u;
+                if (!PERROWX) b[0][u] = ld_xm<XM>(Xv + vv);
+#pragma unroll
+                for (int i = 0; i < RB; ++i) {
+                    a[i][u] = ld_stream(Av + off[i] + vv);
+                    if (PERROWX) b[PERROWX ? i : 0][u] = ld_stream(Xv + off[i] + vv);
+                }
             }
 #pragma unroll
-            for (int u = 0; u < U; ++u) emac(acc[u], a[u], b[u]);
+            for (int i = 0; i < RB; ++i)
+#pragma unroll
+                for (int u = 0; u < U; ++u) emac(acc[i][u], a[i][u], b[PERROWX ? i : 0][u]);
             if (++it == FOLD) {
                 it = 0;
-                outer += esum(tree_sum<U>(acc));
 #pragma unroll
-                for (int u = 0; u < U; ++u) acc[u] = zero_of<E>();
+                for (int i = 0; i < RB; ++i) {
+                    outer[i] += esum(tree_sum<U>(acc[i]));
+#pragma unroll
+                    for (int u = 0; u < U; ++u) acc[i][u] = zero_of<E>();
+                }
             }
         }
-        for (; v < v1; v += NT)            // tail: fewer than U vectors left for this thread
-            emac(acc[0], ld_stream(Ar + v), PERROWX ? ld_stream(Xr + v) : ld_xm<XM>(Xr + v));
-        T val = outer + esum(tree_sum<U>(acc));
-        val = cta_sum<NT>(val, red);
+        for (; v < v1; v += NT) {          // tail: fewer than U vectors left for this thread
+            const E bx = PERROWX ? zero_of<E>() : ld_xm<XM>(Xv + v);
+#pragma unroll
+            for (int i = 0; i < RB; ++i)
+                emac(acc[i][0], ld_stream(Av + off[i] + v), PERROWX ? ld_stream(Xv + off[i] + v) : bx);
+        }
+        T val[RB];
+#pragma unroll
+        for (int i = 0; i < RB; ++i) val[i] = outer[i] + esum(tree_sum<U>(acc[i]));
+        cta_sum_rows<NT, RB>(val, red);
 
         if (S == 1) {
-            if (tid == 0) y[row] = val;
+            if (tid < RB && row0 + tid < R) y[row0 + tid] = val[0];
         } else {
-            if (tid == 0) ws_part[row * S + s] = val;
-            if (ticket_is_last(ws_cnt + row, unsigned(S), &flag)) {
+            if (tid < RB && row0 + tid < R) ws_part[(row0 + tid) * S + s] = val[0];
+            if (ticket_is_last(ws_cnt + grp, unsigned(S), &flag)) {
                 __syncthreads();  // red[] reuse
-                T m = T(0);
-                for (int k = tid; k < S; k += NT) m += ld_partial(ws_part + row * S + k);
-                m = cta_sum<NT>(m, red);
-                if (tid == 0) y[row] = m;
+                T m[RB];
+#pragma unroll
+                for (int i = 0; i < RB; ++i) {
+                    m[i] = T(0);
+                    if (row0 + i < R)
+                        for (int k = tid; k < S; k += NT) m[i] += ld_partial(ws_part + (row0 + i) * S + k);
+                }
+                cta_sum_rows<NT, RB>(m, red);
+                if (tid < RB && row0 + tid < R) y[row0 + tid] = m[0];
             }
         }
         __syncthreads();  // red[] / flag reuse in the next grid-stride step

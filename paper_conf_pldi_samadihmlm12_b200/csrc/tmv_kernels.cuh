@@ -93,6 +93,7 @@ __global__ void __launch_bounds__(NT, NT <= 256 ? (U <= 2 ? 6 : 4) : 1)
 tmv_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restrict__ y,
            int64_t R, int64_t C, int S, T* __restrict__ ws_part, unsigned int* __restrict__ ws_cnt)
 {
+    pdl_prologue();
     using E = typename ElemOf<T, VEC>::type;
     constexpr int W = ElemOf<T, VEC>::W;
     constexpr int LC = NT / LR;

@@ -25,6 +25,7 @@ __global__ void __launch_bounds__(NT)
 mv_tpr_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restrict__ y,
               int64_t R, int64_t C, int stages)
 {
+    pdl_prologue();
     using V = vec4_t<T>;
     extern __shared__ __align__(128) unsigned char smem_raw[];
     __shared__ __align__(8) uint64_t full[TPR_MAX_STAGES];

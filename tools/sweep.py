@@ -28,29 +28,34 @@ OPC = {"mv": L.OP_MV, "tmv": L.OP_TMV, "dot": L.OP_DOT}
 
 
 def grids(op, R, C):
-    """(variant, params) candidates; params = [lanes, splits, ctas_per_sm, unroll, xsmem, block], 0 = auto."""
+    """(variant, params) candidates; params = [lanes, splits, ctas_per_sm, unroll, xsmem, block, rows], 0 = auto."""
     out = [("AUTO", None)]
     if op in ("mv", "dot"):
         nv = C // 4 if C % 4 == 0 else C
         xms = (1, 2) if op == "mv" and C * 4 <= 200 * 1024 else (0,)
         for xm in xms:
-            for g in (1, 2, 4, 8, 16):
-                if g <= max(1, nv):
-                    for u in (1, 2, 4, 8):
-                        if g * u <= max(4, 2 * nv):
-                            out.append(("MV_SUBWARP", [g, 0, 0, u, xm]))
-            for u in (1, 2, 4, 8):
-                if 32 * u <= max(32, 2 * nv):
-                    out.append(("MV_WPR", [0, 0, 0, u, xm]))
-            for nt in (256, 1024):
-                for u in (2, 4, 8):
-                    out.append(("MV_CPR", [nt, 0, 0, u, xm]))
-        for nt in (256, 1024):
-            for u in (2, 4, 8):
-                out.append(("MV_SPLIT", [nt, 0, 0, u]))
-        for nt in (128, 256):
-            for st in (2, 4, 8):
-                out.append(("MV_TPR", [nt, 0, 0, st]))
+            if nv <= 64:
+                for g in (1, 2, 4, 8, 16):
+                    if g <= max(1, nv):
+                        for u in (1, 2, 4, 8):
+                            if g * u <= max(4, 2 * nv):
+                                out.append(("MV_SUBWARP", [g, 0, 0, u, xm]))
+            if nv <= 8192:
+                for u in (1, 2, 4, 8):
+                    if 32 * u <= max(32, 2 * nv):
+                        out.append(("MV_WPR", [0, 0, 0, u, xm]))
+            if C >= 512:
+                for nt, rb, u in ((256, 1, 2), (256, 1, 4), (256, 1, 8), (256, 2, 2), (256, 2, 4), (256, 4, 2),
+                                  (1024, 1, 2), (1024, 1, 4), (1024, 2, 2)):
+                    out.append(("MV_CPR", [nt, 0, 0, u, xm, 0, rb]))
+        if R <= 8192:
+            for nt, rb, u in ((256, 1, 2), (256, 1, 4), (256, 1, 8), (256, 2, 2), (256, 2, 4), (256, 4, 2),
+                              (1024, 1, 2), (1024, 1, 4), (1024, 2, 2)):
+                out.append(("MV_SPLIT", [nt, 0, 0, u, 0, 0, rb]))
+        if C <= 256:
+            for nt in (128, 256):
+                for st in (2, 4, 8):
+                    out.append(("MV_TPR", [nt, 0, 0, st]))
     else:
         rv = R // 4 if R % 4 == 0 else R
         for u in (2, 4, 8):
@@ -71,17 +76,20 @@ def grids(op, R, C):
     return out
 
 
-def time_plan(plan, ptrs, stream, reps):
+def time_plan(plan, ptrs, stream, reps, batch=5):
+    """Per-launch time of back-to-back launches (the way bench.py and a stream of
+    calls see it): `reps` samples, each = CUDA-event time of `batch` launches / batch."""
     for _ in range(2):
         plan.run(*ptrs, stream)
     torch.cuda.synchronize()
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(reps)]
     for a, b in evs:
         a.record()
-        plan.run(*ptrs, stream)
+        for _ in range(batch):
+            plan.run(*ptrs, stream)
         b.record()
     torch.cuda.synchronize()
-    return [a.elapsed_time(b) * 1e3 for a, b in evs]
+    return [a.elapsed_time(b) * 1e3 / batch for a, b in evs]
 
 
 def main():
