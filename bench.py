@@ -46,6 +46,8 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--detail", default=None, help="write per-problem JSONL here")
+    ap.add_argument("--kernel-events-in-timed", action="store_true",
+                    help="record per-launch events inside the timed region (default: separate pass)")
     return ap.parse_args()
 
 
@@ -225,7 +227,11 @@ def run_adaptic(args):
         one_step()
     torch.cuda.synchronize()
 
-    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(n + 1)] for _ in range(args.steps)]
+    # Timed region: K steps back to back, CUDA events only at its two ends (events
+    # between launches would cut the programmatic-dependent-launch overlap).
+    inner = args.kernel_events_in_timed
+    kev_steps = args.steps if inner else min(args.steps, 20)
+    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(n + 1)] for _ in range(kev_steps)]
     t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     clocks = Clocks(torch.cuda.current_device())
     clocks.start()
@@ -233,7 +239,7 @@ def run_adaptic(args):
     torch.cuda.synchronize()
     t0.record()
     for s in range(args.steps):
-        one_step(evs[s])
+        one_step(evs[s] if inner else None)
     t1.record()
     torch.cuda.synchronize()
     barrier(world)
@@ -241,9 +247,31 @@ def run_adaptic(args):
     elapsed_ms = max_over_ranks(t0.elapsed_time(t1), world)
     value = world * step_bytes * args.steps / (elapsed_ms / 1e3) / 1e9
 
-    # per-kernel durations (CUDA events on the launching stream)
-    dur = [[evs[s][i].elapsed_time(evs[s][i + 1]) for s in range(args.steps)] for i in range(n)]
+    # per-kernel durations: CUDA events on the launching stream around every launch,
+    # in a separate pass of kev_steps steps right after the timed region
+    if inner:
+        dur = [[evs[s][i].elapsed_time(evs[s][i + 1]) for s in range(kev_steps)] for i in range(n)]
+    else:
+        # per-kernel pass: each problem's kernel BATCH times back to back between two
+        # events, kev_steps samples -> the duration it sustains inside a stream of calls
+        # (an event between every launch would add its launch latency to each sample
+        # and cut the programmatic-dependent-launch overlap)
+        batch = 5
+        torch.cuda.synchronize()
+        dur = []
+        for i, p in enumerate(probs):
+            ds = []
+            for s in range(kev_steps):
+                evs[s][0].record()
+                for _ in range(batch):
+                    p.launch()
+                evs[s][1].record()
+            torch.cuda.synchronize()
+            for s in range(kev_steps):
+                ds.append(evs[s][0].elapsed_time(evs[s][1]) / batch)
+            dur.append(ds)
     mean_ms = [statistics.mean(d) for d in dur]
+    kernel_sum_ms = sum(mean_ms)
     peak, peak_src = peaks()
     per = []
     for i, p in enumerate(probs):
@@ -285,6 +313,10 @@ def run_adaptic(args):
                                l2="every input >= 256 MiB > 126 MB L2 and problems alternate; no flush needed"
                                if args.workload == "sweep" else "inputs > L2; no flush needed"),
                 "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
+                "kernel_timing": ("per-launch CUDA events inside the timed region" if inner else
+                                  f"per-kernel CUDA events after the timed region: each kernel 5x back to back, "
+                                  f"{kev_steps} samples (the timed region itself has events only at its ends)"),
+                "kernel_sum_ms": kernel_sum_ms,
                 "gpu_launches": n * args.steps, "clocks": clk,
                 "selected": {q["op"] + f" {q['R']}x{q['C']}": [q["variant"], round(q["frac"], 3)] for q in per}}
         print(json.dumps(line), flush=True)

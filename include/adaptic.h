@@ -148,7 +148,12 @@ typedef enum {
  *                      CTA with a TMA bulk copy (needs cols*4 <= 200 KB).
  *   [ADAPTIC_P_BLOCK]  TMV_*: threads per CTA, 256 or 1024 (unroll <= 4 at 1024).
  *   [ADAPTIC_P_ROWS]   MV_CPR / MV_SPLIT: rows per CTA step sharing each x load,
- *                      (rows, unroll) in {(1,2),(1,4),(1,8),(2,2),(2,4),(4,2)}. */
+ *                      (rows, unroll) in {(1,2),(1,4),(1,8),(2,2),(2,4),(4,2)}.
+ *   [ADAPTIC_P_ORDER]  MV_SPLIT: 1 = each split reads one contiguous chunk of
+ *                      the row, 2 = the splits interleave in steps of
+ *                      threads*unroll vectors (default when splits > 1).
+ *   [ADAPTIC_P_PIPE]   MV_CPR / MV_SPLIT with 256 threads: 1 = single-buffered
+ *                      loads (default), 2 = register double-buffered main loop. */
 #define ADAPTIC_P_LANES 0
 #define ADAPTIC_P_SPLITS 1
 #define ADAPTIC_P_CTAS_PER_SM 2
@@ -156,7 +161,9 @@ typedef enum {
 #define ADAPTIC_P_XSMEM 4
 #define ADAPTIC_P_BLOCK 5
 #define ADAPTIC_P_ROWS 6
-#define ADAPTIC_NPARAMS 7
+#define ADAPTIC_P_ORDER 7
+#define ADAPTIC_P_PIPE 8
+#define ADAPTIC_NPARAMS 9
 
 typedef struct adaptic_plan_s* adaptic_plan_t;   /* opaque; owned by the caller */
 

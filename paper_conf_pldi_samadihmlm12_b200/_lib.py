@@ -23,7 +23,7 @@ VARIANTS = ("AUTO", "MV_TPR", "MV_SUBWARP", "MV_WPR", "MV_CPR", "MV_SPLIT",
 V = {name: i for i, name in enumerate(VARIANTS)}
 MV_VARIANTS = ("MV_TPR", "MV_SUBWARP", "MV_WPR", "MV_CPR", "MV_SPLIT")
 TMV_VARIANTS = ("TMV_COL", "TMV_SPLITK", "TMV_REGTILE")
-P_LANES, P_SPLITS, P_CTAS_PER_SM, P_UNROLL, P_XSMEM, P_BLOCK, P_ROWS, NPARAMS = 0, 1, 2, 3, 4, 5, 6, 7
+P_LANES, P_SPLITS, P_CTAS_PER_SM, P_UNROLL, P_XSMEM, P_BLOCK, P_ROWS, P_ORDER, P_PIPE, NPARAMS = 0, 1, 2, 3, 4, 5, 6, 7, 8, 9
 
 # every symbol the header declares (tests check they are all exported)
 SYMBOLS = ("adaptic_plan", "adaptic_plan_forced", "adaptic_plan_variant", "adaptic_plan_describe",

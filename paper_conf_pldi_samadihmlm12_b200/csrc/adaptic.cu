@@ -38,6 +38,8 @@ struct adaptic_plan_s {
     int ctas_per_sm;
     int stages;            // TPR
     int xmode;             // MV family: 0 x via read-only path, 1 x staged in smem (TMA), 2 per-row (DOT)
+    int ilv;               // MV_SPLIT: 1 = splits interleave in steps of NT*U vectors, 0 = contiguous chunks
+    int pipe;              // MV_CPR / MV_SPLIT: register double-buffered main loop
     size_t smem;           // dynamic shared memory bytes (TPR ring, or staged x)
     int block;
     bool vec_shape;        // C % 4 == 0 (MV/DOT) or R % 4 == 0 (TMV)
@@ -58,11 +60,11 @@ namespace {
 thread_local int g_last_cuda_error = 0;
 
 struct TableEntry {
-    int op, dtype, lr, lc, variant, lanes, splits, ctas_per_sm, unroll, xsmem, block, rows;
+    int op, dtype, lr, lc, variant, lanes, splits, ctas_per_sm, unroll, xsmem, block, rows, order, pipe;
 };
 const TableEntry kTable[] = {
 #include "table_data.inc"
-    {-1, -1, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0}};
+    {-1, -1, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0}};
 const int kTableN = int(sizeof(kTable) / sizeof(kTable[0])) - 1;
 
 const char* const kVariantNames[ADAPTIC_V_COUNT] = {
@@ -201,6 +203,8 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
     p->smem = 0;
     p->stages = 0;
     p->xmode = px ? 2 : 0;
+    p->ilv = 0;
+    p->pipe = 0;
     p->rb = 1;
     p->fb_lanes = 0;
     p->fb_unroll = 0;
@@ -292,8 +296,15 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
         if (xm < 0) return ADAPTIC_ERR_UNSUPPORTED;
         const size_t xsm = xm == 1 ? size_t((C * 4 + 15) / 16 * 16) : 0;
         int cps = par(ADAPTIC_P_CTAS_PER_SM);
-        if (cps <= 0) cps = occupancy(cta_fn(dt, NT, RB, U, p->vec_shape, xm), NT, xsm, dev.present, 2048 / NT);
+        // register double buffering (NT 256 only): 1 off, 2 on; default off
+        const int pipe_req = par(ADAPTIC_P_PIPE);
+        if (pipe_req < 0 || pipe_req > 2 || (pipe_req == 2 && NT != 256)) return ADAPTIC_ERR_INVALID_ARG;
+        p->pipe = pipe_req == 2 ? 1 : 0;
+        if (cps <= 0) cps = occupancy(cta_fn(dt, NT, RB, U, p->vec_shape, xm, p->pipe), NT, xsm, dev.present, 2048 / NT);
         p->lanes = NT; p->unroll = U; p->rb = RB; p->block = NT; p->ctas_per_sm = cps; p->xmode = xm; p->smem = xsm;
+        // split order: 1 contiguous chunks, 2 interleaved steps (default for S > 1)
+        const int order = par(ADAPTIC_P_ORDER);
+        if (order < 0 || order > 2) return ADAPTIC_ERR_INVALID_ARG;
         const int64_t slots = int64_t(dev.sms) * cps;
         const int64_t groups = ceil_div(R, RB);
         int64_t S = 1;
@@ -321,6 +332,7 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
         }
         if (S > INT_MAX || R * S > (int64_t(1) << 40)) return ADAPTIC_ERR_UNSUPPORTED;
         p->splits = int(S);
+        p->ilv = (S > 1 && order != 1) ? 1 : 0;
         if (!p->path_ok[p->vec_shape ? 1 : 0]) return ADAPTIC_ERR_UNSUPPORTED;
         if (S > 1) {
             const size_t part = ((size_t(R) * size_t(S) * 4 + 255) / 256) * 256;
@@ -421,7 +433,8 @@ adaptic_status make_plan(int op, int64_t rows, int64_t cols, int dtype, int vari
         return ADAPTIC_OK;
     }
     if (const TableEntry* e = table_lookup(op, dtype, rows, cols)) {
-        int32_t tp[ADAPTIC_NPARAMS] = {e->lanes, e->splits, e->ctas_per_sm, e->unroll, e->xsmem, e->block, e->rows};
+        int32_t tp[ADAPTIC_NPARAMS] = {e->lanes, e->splits, e->ctas_per_sm, e->unroll, e->xsmem, e->block, e->rows,
+                                       e->order, e->pipe};
         p->variant = e->variant; p->source = 1;
         if (derive(p, tp, dev) == ADAPTIC_OK) { *out = p; return ADAPTIC_OK; }
         if (derive(p, nullptr, dev) == ADAPTIC_OK) { *out = p; return ADAPTIC_OK; }
@@ -500,6 +513,8 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
     size_t smem = 0;
     int64_t grid = p->grid[w];
     void* args8[8];
+    void* args9[9];
+    int ilv = p->ilv;
     void* args6[6];
     void** args = nullptr;
     int stages = p->stages;
@@ -529,11 +544,11 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
             break;
         case ADAPTIC_V_MV_CPR:
         case ADAPTIC_V_MV_SPLIT:
-            fn = cta_fn(dt, p->lanes, p->rb, p->unroll, vec, p->xmode);
+            fn = cta_fn(dt, p->lanes, p->rb, p->unroll, vec, p->xmode, p->pipe != 0);
             smem = p->smem;
-            args8[0] = &A; args8[1] = &X; args8[2] = &y; args8[3] = &R; args8[4] = &C;
-            args8[5] = &S; args8[6] = &part; args8[7] = &cnt;
-            args = args8;
+            args9[0] = &A; args9[1] = &X; args9[2] = &y; args9[3] = &R; args9[4] = &C;
+            args9[5] = &S; args9[6] = &ilv; args9[7] = &part; args9[8] = &cnt;
+            args = args9;
             break;
         default:
             fn = tmv_fn(dt, p->lanes, p->unroll, vec, p->block);
@@ -625,12 +640,12 @@ int adaptic_plan_describe(adaptic_plan_t p, char* buf, size_t cap) {
         tmp, sizeof(tmp),
         "{\"op\":\"%s\",\"dtype\":\"%s\",\"rows\":%lld,\"cols\":%lld,\"variant\":\"%s\",\"source\":\"%s\","
         "\"sms\":%d,\"lanes\":%d,\"unroll\":%d,\"rows_per_group\":%d,\"splits\":%d,\"block\":%d,"
-        "\"ctas_per_sm\":%d,\"stages\":%d,\"xmode\":%d,\"smem\":%zu,\"vec_shape\":%s,"
+        "\"ctas_per_sm\":%d,\"stages\":%d,\"xmode\":%d,\"ilv\":%d,\"pipe\":%d,\"smem\":%zu,\"vec_shape\":%s,"
         "\"grid\":[%lld,%lld],\"chain\":[%lld,%lld],\"depth\":[%lld,%lld],\"path_ok\":[%s,%s],"
         "\"fallback_lanes\":%d,\"fallback_unroll\":%d,\"workspace_bytes\":%zu}",
         ops[p->op], p->dtype == ADAPTIC_F32 ? "f32" : "i32", (long long)p->R, (long long)p->C,
         kVariantNames[p->variant], src[p->source], p->sms, p->lanes, p->unroll, p->rb, p->splits, p->block,
-        p->ctas_per_sm, p->stages, p->xmode, p->smem, p->vec_shape ? "true" : "false",
+        p->ctas_per_sm, p->stages, p->xmode, p->ilv, p->pipe, p->smem, p->vec_shape ? "true" : "false",
         (long long)p->grid[0], (long long)p->grid[1], (long long)p->chain[0], (long long)p->chain[1],
         (long long)p->depth[0], (long long)p->depth[1], p->path_ok[0] ? "true" : "false",
         p->path_ok[1] ? "true" : "false", p->fb_lanes, p->fb_unroll, p->ws_bytes);

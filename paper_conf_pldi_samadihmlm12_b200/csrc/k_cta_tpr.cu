@@ -5,47 +5,48 @@
 namespace adaptic {
 
 // (RB, U) combinations: RB rows per CTA step x U loads per row.
-template <class T, int NT, int RB, int U, bool VEC, int XM>
+template <class T, int NT, int RB, int U, bool VEC, int XM, bool PIPE>
 static void* cfn() {
-    // 1024-thread CTAs have 64 registers per thread: at most 4 vector loads per step
-    if constexpr (NT == 1024 && RB * U > 4) return nullptr;
-    else return reinterpret_cast<void*>(&mv_cta_kernel<T, NT, RB, U, VEC, XM>);
+    // 1024-thread CTAs have 64 registers per thread: at most 4 vector loads per
+    // step and no register double buffering
+    if constexpr (NT == 1024 && (RB * U > 4 || PIPE)) return nullptr;
+    else return reinterpret_cast<void*>(&mv_cta_kernel<T, NT, RB, U, VEC, XM, PIPE>);
 }
 
-template <class T, bool VEC, int XM, int NT>
+template <class T, bool VEC, int XM, int NT, bool PIPE>
 static void* cpick_nt(int RB, int U) {
     switch (RB * 16 + U) {
-        case 1 * 16 + 2: return cfn<T, NT, 1, 2, VEC, XM>();
-        case 1 * 16 + 4: return cfn<T, NT, 1, 4, VEC, XM>();
-        case 1 * 16 + 8: return cfn<T, NT, 1, 8, VEC, XM>();
-        case 2 * 16 + 2: return cfn<T, NT, 2, 2, VEC, XM>();
-        case 2 * 16 + 4: return cfn<T, NT, 2, 4, VEC, XM>();
-        case 4 * 16 + 2: return cfn<T, NT, 4, 2, VEC, XM>();
+        case 1 * 16 + 2: return cfn<T, NT, 1, 2, VEC, XM, PIPE>();
+        case 1 * 16 + 4: return cfn<T, NT, 1, 4, VEC, XM, PIPE>();
+        case 1 * 16 + 8: return cfn<T, NT, 1, 8, VEC, XM, PIPE>();
+        case 2 * 16 + 2: return cfn<T, NT, 2, 2, VEC, XM, PIPE>();
+        case 2 * 16 + 4: return cfn<T, NT, 2, 4, VEC, XM, PIPE>();
+        case 4 * 16 + 2: return cfn<T, NT, 4, 2, VEC, XM, PIPE>();
         default: return nullptr;
     }
 }
 
 template <class T, bool VEC, int XM>
-static void* cpick(int NT, int RB, int U) {
+static void* cpick(int NT, int RB, int U, bool pipe) {
     switch (NT) {
-        case 256: return cpick_nt<T, VEC, XM, 256>(RB, U);
-        case 1024: return cpick_nt<T, VEC, XM, 1024>(RB, U);
+        case 256: return pipe ? cpick_nt<T, VEC, XM, 256, true>(RB, U) : cpick_nt<T, VEC, XM, 256, false>(RB, U);
+        case 1024: return pipe ? nullptr : cpick_nt<T, VEC, XM, 1024, false>(RB, U);
         default: return nullptr;
     }
 }
 
 template <class T>
-static void* cta_fn_t(int NT, int RB, int U, bool vec, int xm) {
+static void* cta_fn_t(int NT, int RB, int U, bool vec, int xm, bool pipe) {
     switch (xm) {
-        case XM_LDG: return vec ? cpick<T, true, XM_LDG>(NT, RB, U) : cpick<T, false, XM_LDG>(NT, RB, U);
-        case XM_SMEM: return vec ? cpick<T, true, XM_SMEM>(NT, RB, U) : cpick<T, false, XM_SMEM>(NT, RB, U);
-        case XM_ROW: return vec ? cpick<T, true, XM_ROW>(NT, RB, U) : cpick<T, false, XM_ROW>(NT, RB, U);
+        case XM_LDG: return vec ? cpick<T, true, XM_LDG>(NT, RB, U, pipe) : cpick<T, false, XM_LDG>(NT, RB, U, pipe);
+        case XM_SMEM: return vec ? cpick<T, true, XM_SMEM>(NT, RB, U, pipe) : cpick<T, false, XM_SMEM>(NT, RB, U, pipe);
+        case XM_ROW: return vec ? cpick<T, true, XM_ROW>(NT, RB, U, pipe) : cpick<T, false, XM_ROW>(NT, RB, U, pipe);
         default: return nullptr;
     }
 }
 
-void* cta_fn(int dtype, int NT, int RB, int U, bool vec, int xm) {
-    return dtype == DT_F32 ? cta_fn_t<float>(NT, RB, U, vec, xm) : cta_fn_t<uint32_t>(NT, RB, U, vec, xm);
+void* cta_fn(int dtype, int NT, int RB, int U, bool vec, int xm, bool pipe) {
+    return dtype == DT_F32 ? cta_fn_t<float>(NT, RB, U, vec, xm, pipe) : cta_fn_t<uint32_t>(NT, RB, U, vec, xm, pipe);
 }
 
 template <class T>

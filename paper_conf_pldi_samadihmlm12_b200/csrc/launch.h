@@ -22,7 +22,7 @@ constexpr int TMV_NT = 256;     // default threads per CTA, tmv_kernel (256 or 1
 // cudaOccupancyMaxActiveBlocksPerMultiprocessor, or nullptr when the instance
 // is not compiled.  Kernel signatures:
 //   group: (const T* A, const T* X, T* y, int64_t R, int64_t C)
-//   cta  : (const T* A, const T* X, T* y, int64_t R, int64_t C, int S, T* part, unsigned* cnt)
+//   cta  : (const T* A, const T* X, T* y, int64_t R, int64_t C, int S, int ilv, T* part, unsigned* cnt)
 //          (RB rows per CTA step; (RB, U) in {(1,2),(1,4),(1,8),(2,2),(2,4),(4,2)})
 //   tmv  : (const T* B, const T* X, T* y, int64_t R, int64_t C, int S, T* part, unsigned* cnt)
 //   tpr  : (const T* A, const T* X, T* y, int64_t R, int64_t C, int stages)   [dynamic smem]
@@ -32,7 +32,7 @@ void* group_fn_f32(int G, int U, bool vec, int xmode);
 void* group_fn_i32(int G, int U, bool vec, int xmode);
 void* tmv_fn_f32(int LR, int U, bool vec, int NT);
 void* tmv_fn_i32(int LR, int U, bool vec, int NT);
-void* cta_fn(int dtype, int NT, int RB, int U, bool vec, int xmode);
+void* cta_fn(int dtype, int NT, int RB, int U, bool vec, int xmode, bool pipe);
 void* tpr_fn(int dtype, int NT, bool perrowx);
 
 }  // namespace adaptic

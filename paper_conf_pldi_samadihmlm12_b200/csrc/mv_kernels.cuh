@@ -211,15 +211,16 @@ __device__ __forceinline__ void cta_sum_rows(T (&v)[RB], T* red /* RB*(NT/32) */
     }
 }
 
-template <class T, int NT, int RB, int U, bool VEC, int XM>
+template <class T, int NT, int RB, int U, bool VEC, int XM, bool PIPE>
 __global__ void __launch_bounds__(NT)
 mv_cta_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restrict__ y,
-              int64_t R, int64_t C, int S, T* __restrict__ ws_part, unsigned int* __restrict__ ws_cnt)
+              int64_t R, int64_t C, int S, int ilv, T* __restrict__ ws_part, unsigned int* __restrict__ ws_cnt)
 {
     pdl_prologue();
     using E = typename ElemOf<T, VEC>::type;
     constexpr int W = ElemOf<T, VEC>::W;
     constexpr bool PERROWX = (XM == XM_ROW);
+    constexpr int64_t BV = int64_t(NT) * U;       // vectors per CTA step
     __shared__ T red[RB * (NT / 32)];
     __shared__ unsigned int flag;
     const int64_t nv = C / W;
@@ -234,8 +235,12 @@ mv_cta_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restrict__ 
         const int64_t grp = blk / S;
         const int s = int(blk - grp * S);
         const int64_t row0 = grp * RB;
-        const int64_t v0 = int64_t(s) * chunk;
-        const int64_t v1 = min(nv, v0 + chunk);
+        // split s covers either one contiguous chunk of the row (ilv == 0) or every
+        // S-th step of BV vectors (ilv == 1: the S CTAs of a row sweep it together,
+        // which keeps the in-flight addresses in one window, like a linear stream)
+        const int64_t start = ilv ? int64_t(s) * BV : int64_t(s) * chunk;
+        const int64_t stride = ilv ? int64_t(S) * BV : BV;
+        const int64_t end = ilv ? nv : min(nv, start + chunk);
         int64_t off[RB];                   // rows past R read row 0 (discarded)
 #pragma unroll
         for (int i = 0; i < RB; ++i) off[i] = (row0 + i < R ? row0 + i : 0) * nv;
@@ -249,19 +254,51 @@ mv_cta_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restrict__ 
 #pragma unroll
         for (int i = 0; i < RB; ++i) outer[i] = T(0);
         int it = 0;
-        int64_t v = v0 + tid;
-        for (; v + int64_t(NT) * (U - 1) < v1; v += int64_t(NT) * U) {
-            E a[RB][U], b[PERROWX ? RB : 1][U];
+        int64_t base = start;
+        // PIPE: register double buffering -- the loads of step k+1 are issued before
+        // the FMAs of step k, so RB*U loads stay in flight whatever order ptxas
+        // chooses inside a step (measured: it rescues instances where ptxas
+        // interleaved loads and FMAs, and costs occupancy elsewhere; the selector
+        // table records which one wins per shape).
+        E a[RB][U], b[PERROWX ? RB : 1][U];
+        auto load_step = [&](int64_t bs, E (&aa)[RB][U], E (&bb)[PERROWX ? RB : 1][U]) {
 #pragma unroll
             for (int u = 0; u < U; ++u) {
-                const int64_t vv = v + int64_t(NT) * u;
-                if (!PERROWX) b[0][u] = ld_xm<XM>(Xv + vv);
+                const int64_t vv = bs + tid + int64_t(NT) * u;
+                if (!PERROWX) bb[0][u] = ld_xm<XM>(Xv + vv);
 #pragma unroll
                 for (int i = 0; i < RB; ++i) {
-                    a[i][u] = ld_stream(Av + off[i] + vv);
-                    if (PERROWX) b[PERROWX ? i : 0][u] = ld_stream(Xv + off[i] + vv);
+                    aa[i][u] = ld_stream(Av + off[i] + vv);
+                    if (PERROWX) bb[PERROWX ? i : 0][u] = ld_stream(Xv + off[i] + vv);
                 }
             }
+        };
+        bool have = base + tid + int64_t(NT) * (U - 1) < end;
+        if constexpr (!PIPE) {
+            // single buffer (1024-thread CTAs have 64 registers/thread: no room for two)
+            for (; have; base += stride, have = base + tid + int64_t(NT) * (U - 1) < end) {
+                load_step(base, a, b);
+#pragma unroll
+                for (int i = 0; i < RB; ++i)
+#pragma unroll
+                    for (int u = 0; u < U; ++u) emac(acc[i][u], a[i][u], b[PERROWX ? i : 0][u]);
+                if (++it == FOLD) {
+                    it = 0;
+#pragma unroll
+                    for (int i = 0; i < RB; ++i) {
+                        outer[i] += esum(tree_sum<U>(acc[i]));
+#pragma unroll
+                        for (int u = 0; u < U; ++u) acc[i][u] = zero_of<E>();
+                    }
+                }
+            }
+        }
+        if (have) load_step(base, a, b);
+        while (have) {
+            const int64_t nbase = base + stride;
+            const bool more = nbase + tid + int64_t(NT) * (U - 1) < end;
+            E an[RB][U], bn[PERROWX ? RB : 1][U];
+            if (more) load_step(nbase, an, bn);
 #pragma unroll
             for (int i = 0; i < RB; ++i)
 #pragma unroll
@@ -275,8 +312,20 @@ mv_cta_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restrict__ 
                     for (int u = 0; u < U; ++u) acc[i][u] = zero_of<E>();
                 }
             }
+            base = nbase;
+            have = more;
+            if (more) {
+#pragma unroll
+                for (int u = 0; u < U; ++u) {
+#pragma unroll
+                    for (int i = 0; i < RB; ++i) a[i][u] = an[i][u];
+#pragma unroll
+                    for (int i = 0; i < (PERROWX ? RB : 1); ++i) b[i][u] = bn[i][u];
+                }
+            }
         }
-        for (; v < v1; v += NT) {          // tail: fewer than U vectors left for this thread
+        const int64_t tail_end = min(end, base + BV);
+        for (int64_t v = base + tid; v < tail_end; v += NT) {   // tail: < U vectors left for this thread
             const E bx = PERROWX ? zero_of<E>() : ld_xm<XM>(Xv + v);
 #pragma unroll
             for (int i = 0; i < RB; ++i)

@@ -135,20 +135,33 @@ def test_variant_parameter_grid(op):
     if op == "mv":
         grid = [("MV_SUBWARP", [g, 0, 0, u]) for g in (1, 2, 4, 8, 16) for u in (1, 2, 4, 8)]
         grid += [("MV_WPR", [0, 0, 0, u]) for u in (1, 2, 4, 8)]
-        grid += [("MV_CPR", [nt, 0, 0, u]) for nt in (256, 1024) for u in (2, 4, 8)]
-        grid += [("MV_SPLIT", [nt, s, 0, u]) for nt in (256, 1024) for s in (2, 7) for u in (2, 4, 8)]
+        rbu = [(1, 2), (1, 4), (1, 8), (2, 2), (2, 4), (4, 2)]
+        grid += [("MV_CPR", [nt, 0, 0, u, xs, 0, rb, 0, pp]) for nt in (256, 1024) for rb, u in rbu
+                 for xs in (1, 2) for pp in (1, 2)]
+        grid += [("MV_SPLIT", [nt, s, 0, u, 0, 0, rb, order, pp]) for nt in (256, 1024) for s in (2, 7)
+                 for rb, u in rbu for order in (1, 2) for pp in (1, 2)]
         grid += [("MV_TPR", [nt, 0, 0, st]) for nt in (128, 256) for st in (2, 3)]
     else:
-        grid = [("TMV_SPLITK", [lr, s, 0, u]) for lr in (1, 2, 4, 8, 16, 32, 64, 128, 256)
-                for s in (1, 5) for u in (2, 4, 8)]
+        grid = [("TMV_SPLITK", [lr, s, 0, u, 0, nt]) for lr in (1, 2, 4, 8, 16, 32, 64, 128, 256)
+                for s in (1, 5) for u in (2, 4, 8) for nt in (256, 1024)]
+    cache = {}
+
+    def case(R, C, v, params, dti):
+        if (R, C, dti) not in cache:
+            M, X = make_inputs(op, R, C, dti)
+            cache[(R, C, dti)] = (M, X, run_oracle(op, M, X))
+        M, X, ref = cache[(R, C, dti)]
+        check(run_gpu(op, M, X, v, params), ref, dti, f"{op} {R}x{C} {v} {params}")
+
+    cases = []
     for (R, C), (v, params) in itertools.product(shapes, grid):
         for dti in ("f32", "i32"):
             try:
                 adaptic.plan(op, R, C, dti, variant=v, params=params)
             except adaptic.AdapticError:
                 continue
-            M, X = make_inputs(op, R, C, dti)
-            check(run_gpu(op, M, X, v, params), run_oracle(op, M, X), dti, f"{op} {R}x{C} {v} {params}")
+            cases.append((f"{v} {params} {R}x{C} {dti}", lambda a=(R, C, v, params, dti): case(*a)))
+    _collect(cases)
 
 
 # ------------------------------------------------------------------------ closed forms

@@ -27,6 +27,10 @@ from paper_conf_pldi_samadihmlm12_b200 import _lib as L  # noqa: E402
 OPC = {"mv": L.OP_MV, "tmv": L.OP_TMV, "dot": L.OP_DOT}
 
 
+CTA_GRID = [(256, rb, u, pp) for rb, u in ((1, 2), (1, 4), (1, 8), (2, 2), (2, 4), (4, 2)) for pp in (1, 2)] + \
+           [(1024, 1, 2, 1), (1024, 1, 4, 1), (1024, 2, 2, 1)]
+
+
 def grids(op, R, C):
     """(variant, params) candidates; params = [lanes, splits, ctas_per_sm, unroll, xsmem, block, rows], 0 = auto."""
     out = [("AUTO", None)]
@@ -45,13 +49,12 @@ def grids(op, R, C):
                     if 32 * u <= max(32, 2 * nv):
                         out.append(("MV_WPR", [0, 0, 0, u, xm]))
             if C >= 512:
-                for nt, rb, u in ((256, 1, 2), (256, 1, 4), (256, 1, 8), (256, 2, 2), (256, 2, 4), (256, 4, 2),
-                                  (1024, 1, 2), (1024, 1, 4), (1024, 2, 2)):
-                    out.append(("MV_CPR", [nt, 0, 0, u, xm, 0, rb]))
+                for nt, rb, u, pp in CTA_GRID:
+                    out.append(("MV_CPR", [nt, 0, 0, u, xm, 0, rb, 0, pp]))
         if R <= 8192:
-            for nt, rb, u in ((256, 1, 2), (256, 1, 4), (256, 1, 8), (256, 2, 2), (256, 2, 4), (256, 4, 2),
-                              (1024, 1, 2), (1024, 1, 4), (1024, 2, 2)):
-                out.append(("MV_SPLIT", [nt, 0, 0, u, 0, 0, rb]))
+            for nt, rb, u, pp in CTA_GRID:
+                for order in (1, 2):
+                    out.append(("MV_SPLIT", [nt, 0, 0, u, 0, 0, rb, order, pp]))
         if C <= 256:
             for nt in (128, 256):
                 for st in (2, 4, 8):
