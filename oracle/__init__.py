@@ -160,3 +160,56 @@ def restructure(buf: np.ndarray, T: int, P: int) -> np.ndarray:
     if rc:
         raise ValueError("oracle_restructure_f32 failed")
     return out
+
+
+# ---------------------------------------------------------------- BLAS-1
+def _blas1_lib():
+    lib = _load()
+    if not getattr(lib, "_blas1_ready", False):
+        P, I = ctypes.c_void_p, ctypes.c_int64
+        lib.oracle_asum_f64.argtypes = [P, I, I, P]
+        lib.oracle_asum_f64.restype = ctypes.c_int
+        lib.oracle_nrm2_f64.argtypes = [P, I, I, P, P]
+        lib.oracle_nrm2_f64.restype = ctypes.c_int
+        lib.oracle_iamaxmin.argtypes = [P, I, I, ctypes.c_int, P]
+        lib.oracle_iamaxmin.restype = ctypes.c_int
+        lib._blas1_ready = True
+    return lib
+
+
+def _rows2d(a):
+    a = _c(a, np.float32)
+    return a.reshape(1, -1) if a.ndim == 1 else a
+
+
+def asum(a: np.ndarray) -> np.ndarray:
+    """y_n = sum_e |a[n, e]| (float64)."""
+    a = _rows2d(a)
+    y = np.empty(a.shape[0], np.float64)
+    assert _blas1_lib().oracle_asum_f64(_ptr(a), a.shape[0], a.shape[1], _ptr(y)) == 0
+    return y
+
+
+def nrm2(a: np.ndarray):
+    """(y, ssq): y_n = sqrt(sum_e a[n, e]^2), ssq_n the sum of squares (float64)."""
+    a = _rows2d(a)
+    y = np.empty(a.shape[0], np.float64)
+    s = np.empty(a.shape[0], np.float64)
+    assert _blas1_lib().oracle_nrm2_f64(_ptr(a), a.shape[0], a.shape[1], _ptr(y), _ptr(s)) == 0
+    return y, s
+
+
+def iamax(a: np.ndarray) -> np.ndarray:
+    """1-based first index of max |a[n, :]| (0 for empty rows), int64."""
+    a = _rows2d(a)
+    y = np.empty(a.shape[0], np.int64)
+    assert _blas1_lib().oracle_iamaxmin(_ptr(a), a.shape[0], a.shape[1], 1, _ptr(y)) == 0
+    return y
+
+
+def iamin(a: np.ndarray) -> np.ndarray:
+    """1-based first index of min |a[n, :]| (0 for empty rows), int64."""
+    a = _rows2d(a)
+    y = np.empty(a.shape[0], np.int64)
+    assert _blas1_lib().oracle_iamaxmin(_ptr(a), a.shape[0], a.shape[1], -1, _ptr(y)) == 0
+    return y

@@ -183,3 +183,56 @@ int oracle_restructure_f32(const float* in, int64_t T, int64_t P, float* out)
             out[T * k + t] = in[P * t + k];
     return 0;
 }
+
+/* ---- BLAS-1 reductions ------------------------------------
+ * The paper's Fig. 9 input-portability benchmarks include the CUBLAS routines
+ * Isamax/Isamin, Snrm2 and Sasum, sped up by "actor segmentation and actor
+ * integration" (Sec. 5.1) -- the same one-output-per-array stream
+ * reduction as above with a different operator.  Definitions (BLAS):
+ *   asum : y_n = sum_e |a[n,e]|
+ *   nrm2 : y_n = sqrt(sum_e a[n,e]^2)        (squares of fp32 are exact in double)
+ *   iamax: smallest 1-based e with |a[n,e]| = max_k |a[n,k]|   (0 when L == 0)
+ *   iamin: smallest 1-based e with |a[n,e]| = min_k |a[n,k]|   (0 when L == 0)
+ * N vectors of length L, row-major (rows = N outputs, cols = L). */
+int oracle_asum_f64(const float* a, int64_t N, int64_t L, double* y)
+{
+    if (N < 0 || L < 0) return 1;
+    for (int64_t n = 0; n < N; ++n) {
+        double acc = 0.0;
+        for (int64_t e = 0; e < L; ++e) acc += fabs((double)a[n * L + e]);
+        y[n] = acc;
+    }
+    return 0;
+}
+
+int oracle_nrm2_f64(const float* a, int64_t N, int64_t L, double* y, double* ssq)
+{
+    if (N < 0 || L < 0) return 1;
+    for (int64_t n = 0; n < N; ++n) {
+        double acc = 0.0;
+        for (int64_t e = 0; e < L; ++e) {
+            double v = (double)a[n * L + e];
+            acc += v * v;
+        }
+        if (ssq) ssq[n] = acc;
+        y[n] = sqrt(acc);
+    }
+    return 0;
+}
+
+/* which = +1: iamax, -1: iamin.  |a| of an fp32 value is exact in fp32, so the
+ * comparison (and so the index) is exact; ties keep the first index. */
+int oracle_iamaxmin(const float* a, int64_t N, int64_t L, int which, int64_t* idx)
+{
+    if (N < 0 || L < 0 || (which != 1 && which != -1)) return 1;
+    for (int64_t n = 0; n < N; ++n) {
+        int64_t best = 0;
+        float bv = 0.0f;
+        for (int64_t e = 0; e < L; ++e) {
+            float v = fabsf(a[n * L + e]);
+            if (e == 0 || (which == 1 ? v > bv : v < bv)) { bv = v; best = e + 1; }
+        }
+        idx[n] = best;
+    }
+    return 0;
+}
