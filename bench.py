@@ -9,6 +9,8 @@ Workloads (``--workload``):
   rowshard (BJ:configs[3]) MV 131072 x 32768 fp32, rows sharded over ranks.
   splitk   (BJ:configs[4]) TMV 1024 x 16M fp32, C split over ranks + NCCL all-reduce.
   dot      (BJ:configs[2]) scalar product N = 1, L = 2^10..2^30 (fp32).
+  blas1 Sasum / Snrm2 / Isamax / Isamin (the paper's Fig. 9
+           CUBLAS benchmarks) on 256 MiB inputs: N x L = 1 x 2^26 .. 2^22 x 16.
 Multi-GPU: one process per GPU (torchrun), barrier + synchronize around the
 timed region, max elapsed over ranks; ``value`` = bytes of all ranks / that time.
 
@@ -40,7 +42,7 @@ def parse():
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", choices=["adaptic", "reference"], default="adaptic")
-    ap.add_argument("--workload", choices=["sweep", "rowshard", "splitk", "dot"], default="sweep")
+    ap.add_argument("--workload", choices=["sweep", "rowshard", "splitk", "dot", "blas1"], default="sweep")
     ap.add_argument("--variant", default="AUTO", help="force one variant (fixed-variant sweeps)")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-e2e", action="store_true")
@@ -145,6 +147,20 @@ def max_over_ranks(v: float, world: int) -> float:
 
 
 # ------------------------------------------------------------------------------ problems
+B1_OPS = ("asum", "nrm2", "iamax", "iamin")
+B1_SHAPES = [(1, 1 << 26), (64, 1 << 20), (4096, 1 << 14), (1 << 16, 1024), (1 << 20, 64), (1 << 22, 16)]
+
+
+def algo_bytes(op, R, C):
+    """What the method must move (SURVEY 8(d)): MV/TMV A + x + y; DOT a + b + y;
+    BLAS-1 a + y."""
+    if op == "dot":
+        return 4 * (2 * R * C + R)
+    if op in B1_OPS:
+        return 4 * (R * C + R)
+    return 4 * (R * C + C + R)
+
+
 class Problem:
     """One (op, R, C) instance, resident in HBM, with its selected plan."""
 
@@ -160,18 +176,20 @@ class Problem:
         self.M = torch.empty(R * C, dtype=torch.float32, device=dev)
         layout = "tmv" if op == "tmv" else "mv"
         synth.device_matrix(self.M, Rf, Cf, layout, "uniform", synth.seed(cfg, "A"), rows=rows, cols=cols)
-        if op == "dot":
+        if op in B1_OPS:
+            self.X = torch.empty(0, dtype=torch.float32, device=dev)      # unused
+        elif op == "dot":
             self.X = torch.empty(R * C, dtype=torch.float32, device=dev)
             synth.device_matrix(self.X, Rf, Cf, "mv", "uniform", synth.seed(cfg, "b"), rows=rows, cols=cols)
         else:
             self.X = torch.empty(C, dtype=torch.float32, device=dev)
             synth.device_vector(self.X, "uniform", synth.seed(cfg, "x"), start=cols[0])
-        self.y = torch.empty(R, dtype=torch.float32, device=dev)
-        opc = {"mv": L.OP_MV, "tmv": L.OP_TMV, "dot": L.OP_DOT}[op]
+        self.y = torch.empty(R, dtype=torch.int32 if op in ("iamax", "iamin") else torch.float32, device=dev)
+        opc = L.OPS[op]
         self.stream = torch.cuda.current_stream().cuda_stream
         self.plan = adaptic.get_plan(opc, R, C, L.F32, dev, variant, None, self.stream)
         self.desc = self.plan.describe()
-        self.bytes = 4 * (R * C + C + R) if op != "dot" else 4 * (2 * R * C + R)   # algorithmic
+        self.bytes = algo_bytes(op, R, C)
         self.ptrs = (self.M.data_ptr(), self.X.data_ptr(), self.y.data_ptr())
 
     def launch(self):
@@ -187,6 +205,10 @@ def build_problems(args, world, rank):
                 for k in range(3, 24) for op in ("mv", "tmv")], \
             {"workload": "configs[1]: TMV/MV fp32 shape sweep at 256 MiB, 8Mx8 .. 8192x8192 .. 8x8M, "
                          "both layouts, variant selector", "shapes": 42, "per_gpu": "full sweep (weak)"}
+    if args.workload == "blas1":
+        return [Problem(op, R, C, 7, args.variant) for R, C in B1_SHAPES for op in B1_OPS], \
+            {"workload": "SURVEY 8(f)#1: BLAS-1 Sasum/Snrm2/Isamax/Isamin fp32 at 256 MiB, N x L = 1x2^26 .. 2^22x16",
+             "shapes": len(B1_SHAPES) * len(B1_OPS)}
     if args.workload == "dot":
         return [Problem("dot", 1, 1 << k, 2, args.variant) for k in range(10, 31)], \
             {"workload": "configs[2]: scalar product fp32 N=1, L=2^10..2^30", "shapes": 21}
@@ -340,7 +362,7 @@ def measure_e2e(args, probs, world):
         Xh = torch.empty(p.X.numel(), dtype=torch.float32, pin_memory=True)
         Mh.copy_(p.M)
         Xh.copy_(p.X)
-        yh = torch.empty(p.R, dtype=torch.float32, pin_memory=True)
+        yh = torch.empty(p.R, dtype=p.y.dtype, pin_memory=True)
         hosts.append((Mh.data_ptr(), Xh.data_ptr(), yh.data_ptr(), Mh, Xh, yh))
     torch.cuda.synchronize()
 
@@ -384,6 +406,8 @@ def cpu_baseline(probs, args, budget_s: float = 20.0):
             oracle.mv(M.reshape(p.R, p.C), X)
         elif p.op == "tmv":
             oracle.tmv(M.reshape(p.C, p.R), X)
+        elif p.op in B1_OPS:
+            getattr(oracle, p.op)(M.reshape(p.R, p.C))
         else:
             oracle.dot(M.reshape(p.R, p.C), X.reshape(p.R, p.C))
         t_total += time.perf_counter() - t
@@ -416,6 +440,9 @@ def run_reference(args):
     elif args.workload == "rowshard":
         pool = [("mv", 2048, 32768)]
         cfg = 3
+    elif args.workload == "blas1":
+        pool = [(op, 1, 1 << 24) for op in B1_OPS] + [(op, 1 << 16, 256) for op in B1_OPS]
+        cfg = 7
     else:
         pool = [("tmv", 1024, 1 << 16)]
         cfg = 4
@@ -425,11 +452,15 @@ def run_reference(args):
             a = synth.matrix(R, C, "mv", np.float32, "uniform", synth.seed(cfg, "A"))
             b = synth.matrix(R, C, "mv", np.float32, "uniform", synth.seed(cfg, "b"))
             data.append((op, R, C, a, b, 4 * (2 * R * C + R)))
+        elif op in B1_OPS:
+            a = synth.matrix(R, C, "mv", np.float32, "uniform", synth.seed(cfg, "A"))
+            data.append((op, R, C, a, None, algo_bytes(op, R, C)))
         else:
             M = synth.matrix(R, C, op, np.float32, "uniform", synth.seed(cfg, "A"))
             x = synth.vector(C, np.float32, "uniform", synth.seed(cfg, "x"))
             data.append((op, R, C, M, x, 4 * (R * C + R + C)))
     fns = {"mv": oracle.mv, "tmv": oracle.tmv, "dot": oracle.dot}
+    fns.update({op: (lambda M, X, f=getattr(oracle, op): f(M)) for op in B1_OPS})
     for s in range(args.warmup):
         op, R, C, M, X, _ = data[s % len(data)]
         fns[op](M, X)

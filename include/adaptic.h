@@ -24,6 +24,26 @@
  *   For every op, `rows` (R) is the number of outputs and `cols` (C) is the
  *   reduction length (reading R1).
  *
+ *   BLAS-1 reductions on the same engine: the paper's Fig. 9
+ *   input-portability benchmarks include the CUBLAS routines Sasum, Snrm2 and
+ *   Isamax/Isamin (Sec. 5.1) -- the same one-output-per-array reduction
+ *    with another associative/commutative operator.  For N
+ *   vectors of length L (a row-major N x L; rows = N, cols = L; x unused):
+ *     ADAPTIC_OP_ASUM   y[n] = sum_e |a[n*L + e]|                  (float y)
+ *     ADAPTIC_OP_NRM2   y[n] = sqrt(sum_e a[n*L + e]^2)            (float y)
+ *     ADAPTIC_OP_IAMAX  y[n] = smallest 1-based e with |a[n*L+e-1]| maximal
+ *     ADAPTIC_OP_IAMIN  y[n] = smallest 1-based e with |a[n*L+e-1]| minimal
+ *                       (int32 y; 0 when L == 0; BLAS NaN rule: a NaN never
+ *                       replaces the running extreme, so only a leading NaN
+ *                       yields 1.  L must be <= 2^31 - 1, else UNSUPPORTED.)
+ *   Arithmetic: ASUM accumulates in fp32 like MV (same 1e-4 * sum|a| bound);
+ *   NRM2 accumulates the exact fp64 squares in fp64 (no overflow / underflow for
+ *   any finite fp32 input) and rounds sqrt once to fp32; IAMAX/IAMIN compare
+ *   |a| exactly, so the index is exact.  dtype must be ADAPTIC_F32
+ *   (else UNSUPPORTED).  Variants: MV_SUBWARP, MV_WPR, MV_CPR, MV_SPLIT
+ *   (MV_TPR and the TMV family -> UNSUPPORTED).  Workspace (MV_SPLIT): 8-byte
+ *   partials per (row, split) plus one counter per row.
+ *
  * The input-adaptive part (Fig. 2): adaptic_plan() is the paper's
  * "runtime kernel management" -- on the CPU, from the actual input dimensions,
  * it selects one of several hand-written kernels and fixes its launch
@@ -96,7 +116,7 @@
 extern "C" {
 #endif
 
-#define ADAPTIC_ABI_VERSION 1
+#define ADAPTIC_ABI_VERSION 2
 
 typedef enum {
     ADAPTIC_OK = 0,
@@ -111,7 +131,13 @@ typedef enum {
 typedef enum {
     ADAPTIC_OP_MV = 0,    /* y[R] = A x,    A row-major R x C                       */
     ADAPTIC_OP_TMV = 1,   /* y[R] = B^T x,  B row-major C x R                       */
-    ADAPTIC_OP_DOT = 2    /* y[N] = <a_n, b_n>, a and b row-major N x L; x := b     */
+    ADAPTIC_OP_DOT = 2,   /* y[N] = <a_n, b_n>, a and b row-major N x L; x := b     */
+    /* BLAS-1 reductions of N vectors a_n of length L (a row-major N x L, rows = N,
+     * cols = L; x is unused and may be NULL).  fp32 only (ADAPTIC_F32).        */
+    ADAPTIC_OP_ASUM = 3,  /* float y[N] = sum_e |a_n[e]|                            */
+    ADAPTIC_OP_NRM2 = 4,  /* float y[N] = sqrt(sum_e a_n[e]^2)                      */
+    ADAPTIC_OP_IAMAX = 5, /* int32 y[N] = smallest 1-based e maximising |a_n[e]|    */
+    ADAPTIC_OP_IAMIN = 6  /* int32 y[N] = smallest 1-based e minimising |a_n[e]|    */
 } adaptic_op;
 
 typedef enum {

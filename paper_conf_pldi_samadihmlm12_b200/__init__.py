@@ -4,13 +4,15 @@ Public API (thin marshalling over the C ABI in ``include/adaptic.h``):
 
 * :func:`mv`, :func:`tmv`, :func:`dot` -- run on CUDA tensors; the runtime
   selector picks the kernel variant from the actual (rows, cols).
+* :func:`asum`, :func:`nrm2`, :func:`iamax`, :func:`iamin` -- BLAS-1 reductions
+  (the paper's Fig. 9 CUBLAS benchmarks) on the same engine.
 * :func:`plan` -- inspect what the selector picks (``Plan.describe()``).
 * :mod:`.dist` -- multi-GPU row sharding and split-K over ``torch.distributed``.
 
 There is no CPU fallback: without ``libadaptic.so`` every call raises.
 """
 from ._lib import VARIANTS, MV_VARIANTS, TMV_VARIANTS, AdapticError, Plan, lib  # noqa: F401
-from .ops import clear_cache, dot, get_plan, mv, plan, run_host, tmv  # noqa: F401
+from .ops import asum, clear_cache, dot, get_plan, iamax, iamin, mv, nrm2, plan, run_host, tmv  # noqa: F401
 
-__all__ = ["mv", "tmv", "dot", "plan", "run_host", "Plan", "AdapticError", "lib",
+__all__ = ["mv", "tmv", "dot", "asum", "nrm2", "iamax", "iamin", "plan", "run_host", "Plan", "AdapticError", "lib",
            "VARIANTS", "MV_VARIANTS", "TMV_VARIANTS", "get_plan", "clear_cache"]

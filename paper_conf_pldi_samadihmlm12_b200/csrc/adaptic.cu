@@ -64,6 +64,7 @@ struct TableEntry {
 };
 const TableEntry kTable[] = {
 #include "table_data.inc"
+#include "table_b1.inc"
     {-1, -1, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0}};
 const int kTableN = int(sizeof(kTable) / sizeof(kTable[0])) - 1;
 
@@ -94,8 +95,15 @@ DevInfo device_info() {
     return d;
 }
 
-bool is_mv_family(int v) { return v >= ADAPTIC_V_MV_TPR && v <= ADAPTIC_V_MV_SPLIT; }
 bool is_tmv_family(int v) { return v >= ADAPTIC_V_TMV_COL && v <= ADAPTIC_V_TMV_REGTILE; }
+bool is_mv_family(int v) { return v >= ADAPTIC_V_MV_TPR && v <= ADAPTIC_V_MV_SPLIT; }
+bool is_b1_op(int op) { return op >= ADAPTIC_OP_ASUM && op <= ADAPTIC_OP_IAMIN; }
+bool is_b1_variant(int v) { return v >= ADAPTIC_V_MV_SUBWARP && v <= ADAPTIC_V_MV_SPLIT; }
+bool op_has_variant(int op, int v) {
+    if (op == ADAPTIC_OP_TMV) return is_tmv_family(v);
+    if (is_b1_op(op)) return is_b1_variant(v);
+    return is_mv_family(v);
+}
 
 void* group_fn(int dtype, int G, int U, bool vec, int xm) {
     return dtype == DT_F32 ? group_fn_f32(G, U, vec, xm) : group_fn_i32(G, U, vec, xm);
@@ -112,6 +120,24 @@ int pick_xmode(bool px, int req, int64_t C, bool allow) {
     if (req == 2) return C * 4 <= kXsMaxBytes ? 1 : -1;
     if (req == 1) return 0;
     return C * 4 <= kXsAutoBytes ? 1 : 0;
+}
+void* b1_group_fn(int op, int G, int rbu, bool vec) {
+    switch (op) {
+        case ADAPTIC_OP_ASUM: return b1_group_fn_asum(G, rbu, vec);
+        case ADAPTIC_OP_NRM2: return b1_group_fn_nrm2(G, rbu, vec);
+        case ADAPTIC_OP_IAMAX: return b1_group_fn_iamax(G, rbu, vec);
+        case ADAPTIC_OP_IAMIN: return b1_group_fn_iamin(G, rbu, vec);
+        default: return nullptr;
+    }
+}
+void* b1_cta_fn(int op, bool vec) {
+    switch (op) {
+        case ADAPTIC_OP_ASUM: return b1_cta_fn_asum(vec);
+        case ADAPTIC_OP_NRM2: return b1_cta_fn_nrm2(vec);
+        case ADAPTIC_OP_IAMAX: return b1_cta_fn_iamax(vec);
+        case ADAPTIC_OP_IAMIN: return b1_cta_fn_iamin(vec);
+        default: return nullptr;
+    }
 }
 void* tmv_fn(int dtype, int LR, int U, bool vec, int NT) {
     return dtype == DT_F32 ? tmv_fn_f32(LR, U, vec, NT) : tmv_fn_i32(LR, U, vec, NT);
@@ -157,6 +183,17 @@ int64_t pick_splits(int64_t units, int64_t slots, int64_t smax, int64_t smin) {
 
 // ---------------------------------------------------------------- heuristic (no table cell)
 int heuristic_variant(int op, int64_t R, int64_t C, int sms) {
+    if (is_b1_op(op)) {
+        // the paper's regimes (Fig. 1) for a unary reduction: lane groups
+        // for many short rows, a CTA per row once rows are long and numerous
+        // enough to fill the GPU, split rows (K1) when there are too few rows
+        const int64_t nv = (C % 4 == 0) ? C / 4 : C;
+        if (nv <= 32) return ADAPTIC_V_MV_SUBWARP;
+        if (nv <= 2048 && R >= 4096) return ADAPTIC_V_MV_WPR;
+        if (R >= 4 * int64_t(sms)) return ADAPTIC_V_MV_CPR;
+        if (nv <= 1024) return ADAPTIC_V_MV_WPR;      // tiny: one launch, no merge
+        return ADAPTIC_V_MV_SPLIT;
+    }
     if (op == ADAPTIC_OP_TMV) {
         const int64_t rv = (R % 4 == 0) ? R / 4 : R;
         if (rv >= int64_t(sms) * 512 && C <= 4096) return ADAPTIC_V_TMV_COL;
@@ -189,6 +226,85 @@ const TableEntry* table_lookup(int op, int dtype, int64_t R, int64_t C) {
     return nullptr;
 }
 
+// BLAS-1 reductions (ASUM/NRM2/IAMAX/IAMIN): the MV-family thread shapes with an
+// operator policy (blas1_kernels.cuh).  Only ASUM has fp32 chains to bound; NRM2
+// accumulates in fp64 and IAMAX/IAMIN are exact.
+adaptic_status derive_b1(adaptic_plan_s* p, const int32_t* params, const DevInfo& dev) {
+    const int op = p->op, v = p->variant;
+    const int64_t R = p->R, C = p->C;
+    auto par = [&](int i) -> int { return params ? params[i] : 0; };
+    const bool fp32_chain = (op == ADAPTIC_OP_ASUM);
+    p->vec_shape = (C % 4 == 0);
+    p->splits = 1; p->smem = 0; p->stages = 0; p->xmode = 0; p->ilv = 0; p->pipe = 0; p->rb = 1;
+    p->fb_lanes = 0; p->fb_unroll = 0; p->ws_bytes = 0; p->cnt_off = 0;
+    for (int w = 0; w < 2; ++w) { p->grid[w] = 0; p->chain[w] = 0; p->depth[w] = 0; p->path_ok[w] = false; }
+    const int64_t nv1 = p->vec_shape ? C / 4 : C;
+
+    if (v == ADAPTIC_V_MV_SUBWARP || v == ADAPTIC_V_MV_WPR) {
+        int G;
+        if (v == ADAPTIC_V_MV_WPR) G = 32;
+        else if (par(ADAPTIC_P_LANES) > 0) G = par(ADAPTIC_P_LANES);
+        else G = clampi(pow2_ceil(ceil_div(std::max<int64_t>(1, nv1), 2)), 1, 16);
+        if (G < 1 || G > 32 || (G & (G - 1)) || (v == ADAPTIC_V_MV_SUBWARP && G > 16)) return ADAPTIC_ERR_INVALID_ARG;
+        // (RB, U): 4 rows x 2 loads (short rows) or 1 row x 8 loads (long rows)
+        int rb = par(ADAPTIC_P_ROWS);
+        if (rb <= 0) rb = (v == ADAPTIC_V_MV_WPR && nv1 >= 512) ? 1 : 4;
+        if (rb != 1 && rb != 4) return ADAPTIC_ERR_INVALID_ARG;
+        const int U = rb == 1 ? 8 : 2;
+        p->lanes = G; p->unroll = U; p->rb = rb; p->block = GROUP_NT;
+        const int rows_per_cta = rb * (32 / G) * (GROUP_NT / 32);
+        int cps = par(ADAPTIC_P_CTAS_PER_SM);
+        if (cps <= 0) cps = occupancy(b1_group_fn(op, G, rb == 1 ? 1 : 0, p->vec_shape), GROUP_NT, 0, dev.present, 4);
+        p->ctas_per_sm = cps;
+        for (int w = 0; w < 2; ++w) {
+            if (w == 1 && !p->vec_shape) continue;
+            const int64_t nv = w ? C / 4 : C;
+            const int64_t iters = ceil_div(nv, int64_t(G) * U);
+            p->grid[w] = std::max<int64_t>(1, std::min<int64_t>(ceil_div(R, rows_per_cta), int64_t(dev.sms) * cps));
+            p->chain[w] = fp32_chain ? fold_chain(iters) : 0;
+            p->depth[w] = ilog2c(U) + (w ? 2 : 0) + ilog2c(G) + 1;
+            p->path_ok[w] = !fp32_chain || bound_ok(p->chain[w] + p->depth[w]);
+        }
+        return p->path_ok[p->vec_shape ? 1 : 0] ? ADAPTIC_OK : ADAPTIC_ERR_UNSUPPORTED;
+    }
+    // MV_CPR / MV_SPLIT: B1_CTA_NT threads, 4 loads per thread per step
+    const int NT = B1_CTA_NT, U = 4;
+    int cps = par(ADAPTIC_P_CTAS_PER_SM);
+    if (cps <= 0) cps = occupancy(b1_cta_fn(op, p->vec_shape), NT, 0, dev.present, 2048 / NT);
+    p->lanes = NT; p->unroll = U; p->block = NT; p->ctas_per_sm = cps;
+    const int64_t slots = int64_t(dev.sms) * cps;
+    int64_t S = 1;
+    if (v == ADAPTIC_V_MV_SPLIT) {
+        S = par(ADAPTIC_P_SPLITS) > 0 ? par(ADAPTIC_P_SPLITS)
+                                      : pick_splits(R, slots, std::max<int64_t>(2, ceil_div(nv1, int64_t(NT) * U)), 2);
+    }
+    for (;;) {
+        bool ok_all = true;
+        for (int w = 0; w < 2; ++w) {
+            if (w == 1 && !p->vec_shape) continue;
+            const int64_t nv = w ? C / 4 : C;
+            const int64_t iters = ceil_div(nv, int64_t(S) * NT * U);   // interleaved splits
+            p->chain[w] = fp32_chain ? fold_chain(iters) : 0;
+            p->depth[w] = ilog2c(U) + (w ? 2 : 0) + 10 + (S > 1 ? ceil_div(S, NT) + 10 : 0) + 1;
+            p->path_ok[w] = !fp32_chain || bound_ok(p->chain[w] + p->depth[w]);
+            p->grid[w] = std::max<int64_t>(1, std::min<int64_t>(R * S, slots));
+            if (!p->path_ok[w]) ok_all = false;
+        }
+        if (ok_all || v == ADAPTIC_V_MV_CPR || S >= (int64_t(1) << 20)) break;
+        S *= 2;
+    }
+    if (S > INT_MAX || R * S > (int64_t(1) << 40)) return ADAPTIC_ERR_UNSUPPORTED;
+    p->splits = int(S);
+    p->ilv = S > 1 ? 1 : 0;
+    if (!p->path_ok[p->vec_shape ? 1 : 0]) return ADAPTIC_ERR_UNSUPPORTED;
+    if (S > 1) {
+        const size_t part = ((size_t(R) * size_t(S) * 8 + 255) / 256) * 256;
+        p->cnt_off = part;
+        p->ws_bytes = part + size_t(R) * 4;
+    }
+    return ADAPTIC_OK;
+}
+
 // Fill the kernel parameters of `p` for p->variant.  params: user overrides or nullptr.
 adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& dev) {
     const int op = p->op, dt = p->dtype;
@@ -196,7 +312,8 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
     const int64_t R = p->R, C = p->C;
     auto par = [&](int i) -> int { return params ? params[i] : 0; };
     const int v = p->variant;
-    if (op == ADAPTIC_OP_TMV ? !is_tmv_family(v) : !is_mv_family(v)) return ADAPTIC_ERR_UNSUPPORTED;
+    if (!op_has_variant(op, v)) return ADAPTIC_ERR_UNSUPPORTED;
+    if (is_b1_op(op)) return derive_b1(p, params, dev);
 
     p->vec_shape = (op == ADAPTIC_OP_TMV) ? (R % 4 == 0) : (C % 4 == 0);
     p->splits = 1;
@@ -397,9 +514,11 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
 }
 
 adaptic_status validate_shape(int op, int64_t rows, int64_t cols, int dtype) {
-    if (op < ADAPTIC_OP_MV || op > ADAPTIC_OP_DOT) return ADAPTIC_ERR_INVALID_ARG;
+    if (op < ADAPTIC_OP_MV || op > ADAPTIC_OP_IAMIN) return ADAPTIC_ERR_INVALID_ARG;
     if (dtype != ADAPTIC_F32 && dtype != ADAPTIC_I32) return ADAPTIC_ERR_INVALID_ARG;
     if (rows < 0 || cols < 0) return ADAPTIC_ERR_INVALID_ARG;
+    if (is_b1_op(op) && dtype != ADAPTIC_F32) return ADAPTIC_ERR_UNSUPPORTED;
+    if ((op == ADAPTIC_OP_IAMAX || op == ADAPTIC_OP_IAMIN) && cols > int64_t(INT_MAX)) return ADAPTIC_ERR_UNSUPPORTED;
     if (cols > 0 && rows > (int64_t(1) << 62) / 4 / cols) return ADAPTIC_ERR_INVALID_ARG;  // bytes overflow
     return ADAPTIC_OK;
 }
@@ -419,8 +538,7 @@ adaptic_status make_plan(int op, int64_t rows, int64_t cols, int dtype, int vari
 
     if (variant != ADAPTIC_V_AUTO) {
         p->variant = variant; p->source = 0;
-        st = (rows == 0 || cols == 0) ? ((op == ADAPTIC_OP_TMV ? is_tmv_family(variant) : is_mv_family(variant))
-                                             ? ADAPTIC_OK : ADAPTIC_ERR_UNSUPPORTED)
+        st = (rows == 0 || cols == 0) ? (op_has_variant(op, variant) ? ADAPTIC_OK : ADAPTIC_ERR_UNSUPPORTED)
                                       : derive(p, params, dev);
         if (st != ADAPTIC_OK) { delete p; return st; }
         *out = p;
@@ -444,7 +562,7 @@ adaptic_status make_plan(int op, int64_t rows, int64_t cols, int dtype, int vari
     st = derive(p, nullptr, dev);
     if (st != ADAPTIC_OK) {
         // last resort: the split variants always satisfy the bound
-        p->variant = (op == ADAPTIC_OP_TMV) ? ADAPTIC_V_TMV_SPLITK : ADAPTIC_V_MV_SPLIT;
+        p->variant = (op == ADAPTIC_OP_TMV) ? ADAPTIC_V_TMV_SPLITK : ADAPTIC_V_MV_SPLIT;   // b1 too
         st = derive(p, nullptr, dev);
     }
     if (st != ADAPTIC_OK) { delete p; return st; }
@@ -519,7 +637,19 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
     void** args = nullptr;
     int stages = p->stages;
 
-    switch (p->variant) {
+    void* args7[7];
+    if (is_b1_op(p->op)) {
+        if (p->variant == ADAPTIC_V_MV_SUBWARP || p->variant == ADAPTIC_V_MV_WPR) {
+            fn = b1_group_fn(p->op, p->lanes, p->rb == 1 ? 1 : 0, vec);
+            args6[0] = &A; args6[1] = &y; args6[2] = &R; args6[3] = &C;
+            args = args6;
+        } else {
+            fn = b1_cta_fn(p->op, vec);
+            args7[0] = &A; args7[1] = &y; args7[2] = &R; args7[3] = &C; args7[4] = &S;
+            args7[5] = &part; args7[6] = &cnt;
+            args = args7;
+        }
+    } else switch (p->variant) {
         case ADAPTIC_V_MV_TPR:
             if (vec) {
                 fn = tpr_fn(dt, p->lanes, px);
@@ -586,12 +716,13 @@ adaptic_status check_run(const adaptic_plan_s* p, const void* A, const void* x, 
     if (!y) return ADAPTIC_ERR_INVALID_ARG;
     if (!aligned(y, 4)) return ADAPTIC_ERR_MISALIGNED;
     if (p->C == 0) return ADAPTIC_OK;
-    if (!A || !x) return ADAPTIC_ERR_INVALID_ARG;
-    if (!aligned(A, 4) || !aligned(x, 4)) return ADAPTIC_ERR_MISALIGNED;
+    const bool b1 = is_b1_op(p->op);          // BLAS-1: x is unused (may be NULL)
+    if (!A || (!x && !b1)) return ADAPTIC_ERR_INVALID_ARG;
+    if (!aligned(A, 4) || (!b1 && !aligned(x, 4))) return ADAPTIC_ERR_MISALIGNED;
     const size_t ybytes = size_t(p->R) * 4;
     const size_t abytes = size_t(p->R) * size_t(p->C) * 4;
-    const size_t xbytes = (p->op == ADAPTIC_OP_DOT ? abytes : size_t(p->C) * 4);
-    if (overlap(y, ybytes, A, abytes) || overlap(y, ybytes, x, xbytes)) return ADAPTIC_ERR_ALIAS;
+    const size_t xbytes = b1 ? 0 : (p->op == ADAPTIC_OP_DOT ? abytes : size_t(p->C) * 4);
+    if (overlap(y, ybytes, A, abytes) || (!b1 && overlap(y, ybytes, x, xbytes))) return ADAPTIC_ERR_ALIAS;
     if (p->ws_bytes > 0 && (p->ws == nullptr || p->ws_cap < p->ws_bytes)) return ADAPTIC_ERR_NO_WORKSPACE;
     return ADAPTIC_OK;
 }
@@ -633,7 +764,7 @@ adaptic_status adaptic_plan_set_workspace(adaptic_plan_t plan, void* dev_ptr, si
 
 int adaptic_plan_describe(adaptic_plan_t p, char* buf, size_t cap) {
     if (!p) return -1;
-    static const char* ops[] = {"MV", "TMV", "DOT"};
+    static const char* ops[] = {"MV", "TMV", "DOT", "ASUM", "NRM2", "IAMAX", "IAMIN"};
     static const char* src[] = {"forced", "table", "heuristic"};
     char tmp[1024];
     const int n = std::snprintf(
@@ -669,6 +800,7 @@ adaptic_status adaptic_run(adaptic_plan_t p, const void* A, const void* x, void*
     bool vec = p->vec_shape;
     if (vec) {
         if (p->op == ADAPTIC_OP_TMV) vec = aligned(A, 16) && aligned(y, 16);
+        else if (is_b1_op(p->op)) vec = aligned(A, 16);
         else vec = aligned(A, 16) && aligned(x, 16);
     }
     if (!p->path_ok[vec ? 1 : 0]) return ADAPTIC_ERR_MISALIGNED;   // scalar path would break the error bound
@@ -680,14 +812,16 @@ adaptic_status adaptic_run_host(adaptic_plan_t p, const void* A_host, const void
     if (!p) return ADAPTIC_ERR_INVALID_ARG;
     cudaStream_t stream = static_cast<cudaStream_t>(stream_);
     if (p->R == 0) return ADAPTIC_OK;
-    if (!y_host || (p->C > 0 && (!A_host || !x_host))) return ADAPTIC_ERR_INVALID_ARG;
+    const bool b1 = is_b1_op(p->op);
+    if (!y_host || (p->C > 0 && (!A_host || (!x_host && !b1)))) return ADAPTIC_ERR_INVALID_ARG;
     adaptic_status st = check_run(p, dA, dx, dy);
     if (st != ADAPTIC_OK) return st;
     const size_t abytes = size_t(p->R) * size_t(p->C) * 4;
     const size_t xbytes = (p->op == ADAPTIC_OP_DOT ? abytes : size_t(p->C) * 4);
     cudaError_t e;
     if (p->C > 0) {
-        if ((e = cudaMemcpyAsync(dx, x_host, xbytes, cudaMemcpyHostToDevice, stream)) != cudaSuccess) return cuda_fail(e);
+        if (!b1 && (e = cudaMemcpyAsync(dx, x_host, xbytes, cudaMemcpyHostToDevice, stream)) != cudaSuccess)
+            return cuda_fail(e);
         if ((e = cudaMemcpyAsync(dA, A_host, abytes, cudaMemcpyHostToDevice, stream)) != cudaSuccess) return cuda_fail(e);
     }
     st = adaptic_run(p, dA, dx, dy, stream_);

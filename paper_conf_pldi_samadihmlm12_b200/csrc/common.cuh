@@ -82,6 +82,7 @@ __device__ __forceinline__ float ld_partial(const float* p) { return __ldcg(p); 
 __device__ __forceinline__ uint32_t ld_partial(const uint32_t* p) { return __ldcg(p); }
 __device__ __forceinline__ float4 ld_partial(const float4* p) { return __ldcg(p); }
 __device__ __forceinline__ uint4 ld_partial(const uint4* p) { return __ldcg(p); }
+template <class T> __device__ __forceinline__ T ld_partial_any(const T* p) { return __ldcg(p); }
 
 // ---------------------------------------------------------------- programmatic dependent launch
 // Every kernel is launched with cudaLaunchAttributeProgrammaticStreamSerialization,

@@ -35,4 +35,17 @@ void* tmv_fn_i32(int LR, int U, bool vec, int NT);
 void* cta_fn(int dtype, int NT, int RB, int U, bool vec, int xmode, bool pipe);
 void* tpr_fn(int dtype, int NT, bool perrowx);
 
+// BLAS-1 reductions (blas1_kernels.cuh), fp32 input, one translation unit per operator:
+//   b1 group: (const float* A, void* y, int64_t R, int64_t C); rbu 0 = (RB 4, U 2), 1 = (RB 1, U 8)
+//   b1 cta  : (const float* A, void* y, int64_t R, int64_t C, int S, P* part, unsigned* cnt)
+constexpr int B1_CTA_NT = 256;
+void* b1_group_fn_asum(int G, int rbu, bool vec);
+void* b1_group_fn_nrm2(int G, int rbu, bool vec);
+void* b1_group_fn_iamax(int G, int rbu, bool vec);
+void* b1_group_fn_iamin(int G, int rbu, bool vec);
+void* b1_cta_fn_asum(bool vec);
+void* b1_cta_fn_nrm2(bool vec);
+void* b1_cta_fn_iamax(bool vec);
+void* b1_cta_fn_iamin(bool vec);
+
 }  // namespace adaptic

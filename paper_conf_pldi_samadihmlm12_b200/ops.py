@@ -1,4 +1,5 @@
-"""PyTorch-facing API: ``mv``, ``tmv``, ``dot`` on CUDA tensors.
+"""PyTorch-facing API: ``mv``, ``tmv``, ``dot`` and the BLAS-1 reductions
+``asum``, ``nrm2``, ``iamax``, ``iamin`` on CUDA tensors.
 
 PyTorch supplies device memory and the stream; the selector
 (``adaptic_plan``) and the kernels (``adaptic_run``) are the C ABI.  This module
@@ -108,10 +109,46 @@ def dot(a: torch.Tensor, b: torch.Tensor, *, variant="AUTO", params=None, out=No
     return _run(L.OP_DOT, a, b, N, Lk, variant, params, out)
 
 
+def _blas1(op: int, a: torch.Tensor, variant, params, out, ydtype) -> torch.Tensor:
+    if a.dim() not in (1, 2):
+        raise ValueError(f"expected [N, L] (or [L]) input, got {tuple(a.shape)}")
+    if a.dtype != torch.float32:
+        raise TypeError(f"BLAS-1 reductions take float32, got {a.dtype}")
+    N, Lk = (1, a.shape[0]) if a.dim() == 1 else a.shape
+    dev = _check_dev(a)
+    if out is None:
+        out = torch.empty(N, dtype=ydtype, device=dev)
+    elif out.numel() != N or out.dtype != ydtype or out.device != dev or not out.is_contiguous():
+        raise ValueError(f"out must be a contiguous {ydtype} tensor of {N} elements on {dev}")
+    stream = torch.cuda.current_stream(dev).cuda_stream
+    plan = get_plan(op, N, Lk, L.F32, dev, variant, params, stream)
+    plan.run(a.data_ptr(), 0, out.data_ptr(), stream)
+    return out
+
+
+def asum(a: torch.Tensor, *, variant="AUTO", params=None, out=None) -> torch.Tensor:
+    """Sasum per row: y[n] = sum_e |a[n, e]| (float32)."""
+    return _blas1(L.OP_ASUM, a, variant, params, out, torch.float32)
+
+
+def nrm2(a: torch.Tensor, *, variant="AUTO", params=None, out=None) -> torch.Tensor:
+    """Snrm2 per row: y[n] = sqrt(sum_e a[n, e]^2) (float32; fp64 accumulation)."""
+    return _blas1(L.OP_NRM2, a, variant, params, out, torch.float32)
+
+
+def iamax(a: torch.Tensor, *, variant="AUTO", params=None, out=None) -> torch.Tensor:
+    """Isamax per row: smallest 1-based index of max |a[n, e]| (int32; 0 for empty rows)."""
+    return _blas1(L.OP_IAMAX, a, variant, params, out, torch.int32)
+
+
+def iamin(a: torch.Tensor, *, variant="AUTO", params=None, out=None) -> torch.Tensor:
+    """Isamin per row: smallest 1-based index of min |a[n, e]| (int32; 0 for empty rows)."""
+    return _blas1(L.OP_IAMIN, a, variant, params, out, torch.int32)
+
+
 def plan(op: str, rows: int, cols: int, dtype: str = "f32", variant="AUTO", params=None) -> L.Plan:
     """A bare plan (no workspace attached) -- for inspecting the selector."""
-    return L.Plan({"mv": L.OP_MV, "tmv": L.OP_TMV, "dot": L.OP_DOT}[op], rows, cols,
-                  {"f32": L.F32, "i32": L.I32}[dtype], variant, params)
+    return L.Plan(L.OPS[op], rows, cols, {"f32": L.F32, "i32": L.I32}[dtype], variant, params)
 
 
 def run_host(op: str, M_host: torch.Tensor, X_host: torch.Tensor, y_host: torch.Tensor,
@@ -119,7 +156,7 @@ def run_host(op: str, M_host: torch.Tensor, X_host: torch.Tensor, y_host: torch.
     """End-to-end call with HOST buffers (pinned for async copies): the library
     enqueues H2D copies of M and X into dM/dX, the kernel, and the D2H copy of y
     on the current stream.  The caller synchronises before reading y_host."""
-    opc = {"mv": L.OP_MV, "tmv": L.OP_TMV, "dot": L.OP_DOT}[op]
+    opc = L.OPS[op]
     if opc == L.OP_TMV:
         C, R = M_host.shape
     elif M_host.dim() == 1:

@@ -24,7 +24,8 @@ import synth  # noqa: E402
 import paper_conf_pldi_samadihmlm12_b200 as adaptic  # noqa: E402
 from paper_conf_pldi_samadihmlm12_b200 import _lib as L  # noqa: E402
 
-OPC = {"mv": L.OP_MV, "tmv": L.OP_TMV, "dot": L.OP_DOT}
+OPC = L.OPS
+B1 = ("asum", "nrm2", "iamax", "iamin")
 
 
 CTA_GRID = [(256, rb, u, pp) for rb, u in ((1, 2), (1, 4), (1, 8), (2, 2), (2, 4), (4, 2)) for pp in (1, 2)] + \
@@ -34,6 +35,22 @@ CTA_GRID = [(256, rb, u, pp) for rb, u in ((1, 2), (1, 4), (1, 8), (2, 2), (2, 4
 def grids(op, R, C):
     """(variant, params) candidates; params = [lanes, splits, ctas_per_sm, unroll, xsmem, block, rows], 0 = auto."""
     out = [("AUTO", None)]
+    if op in B1:
+        nv = C // 4 if C % 4 == 0 else C
+        if nv <= 64:
+            for g in (1, 2, 4, 8, 16):
+                if g <= max(1, nv):
+                    for rb in (1, 4):
+                        out.append(("MV_SUBWARP", [g, 0, 0, 0, 0, 0, rb]))
+        if nv <= 16384:
+            for rb in (1, 4):
+                out.append(("MV_WPR", [0, 0, 0, 0, 0, 0, rb]))
+        if C >= 256:
+            out.append(("MV_CPR", None))
+        if R <= 16384:
+            for sp in sorted({0} | {max(2, -(-148 * k // R)) for k in (2, 4, 6, 8)}):
+                out.append(("MV_SPLIT", [0, sp]))
+        return out
     if op in ("mv", "dot"):
         nv = C // 4 if C % 4 == 0 else C
         xms = (1, 2) if op == "mv" and C * 4 <= 200 * 1024 else (0,)
@@ -120,7 +137,7 @@ def main():
     maxel = max(R * C for R, C in shapes)
     M = torch.empty(maxel * (2 if "dot" in a.ops else 1), dtype=tdt, device=dev)
     X = torch.empty(max(C for _, C in shapes), dtype=tdt, device=dev)
-    Y = torch.empty(max(R for R, _ in shapes), dtype=tdt, device=dev)
+    Y = torch.empty(max(R for R, _ in shapes), dtype=tdt, device=dev)   # 4-byte y (int32 for IAMAX/IAMIN)
     synth.device_matrix(M, 1, M.numel(), "mv", "uniform", 11)
     synth.device_vector(X, "uniform", 12)
     t0 = time.time()
@@ -136,7 +153,7 @@ def main():
                         continue
                     ts = time_plan(plan, ptrs, stream, a.reps)
                     med = statistics.median(ts)
-                    nbytes = 4 * (R * C * (2 if op == "dot" else 1) + R + (0 if op == "dot" else C))
+                    nbytes = 4 * (R * C * (2 if op == "dot" else 1) + R + (0 if op in ("dot",) + B1 else C))
                     d = plan.describe()
                     f.write(json.dumps({"op": op, "dtype": a.dtype, "R": R, "C": C, "variant": d["variant"],
                                         "req": variant, "params": params, "us": med, "us_min": min(ts),
