@@ -147,7 +147,7 @@ def max_over_ranks(v: float, world: int) -> float:
 
 
 # ------------------------------------------------------------------------------ problems
-B1_OPS = ("asum", "nrm2", "iamax", "iamin")
+B1_OPS = ("asum", "nrm2", "iamax", "iamin", "b1all")
 B1_SHAPES = [(1, 1 << 26), (64, 1 << 20), (4096, 1 << 14), (1 << 16, 1024), (1 << 20, 64), (1 << 22, 16)]
 
 
@@ -157,7 +157,7 @@ def algo_bytes(op, R, C):
     if op == "dot":
         return 4 * (2 * R * C + R)
     if op in B1_OPS:
-        return 4 * (R * C + R)
+        return 4 * (R * C + (4 if op == "b1all" else 1) * R)
     return 4 * (R * C + C + R)
 
 
@@ -184,7 +184,8 @@ class Problem:
         else:
             self.X = torch.empty(C, dtype=torch.float32, device=dev)
             synth.device_vector(self.X, "uniform", synth.seed(cfg, "x"), start=cols[0])
-        self.y = torch.empty(R, dtype=torch.int32 if op in ("iamax", "iamin") else torch.float32, device=dev)
+        self.y = torch.empty(R * (4 if op == "b1all" else 1),
+                             dtype=torch.int32 if op in ("iamax", "iamin") else torch.float32, device=dev)
         opc = L.OPS[op]
         self.stream = torch.cuda.current_stream().cuda_stream
         self.plan = adaptic.get_plan(opc, R, C, L.F32, dev, variant, None, self.stream)
@@ -207,7 +208,8 @@ def build_problems(args, world, rank):
                          "both layouts, variant selector", "shapes": 42, "per_gpu": "full sweep (weak)"}
     if args.workload == "blas1":
         return [Problem(op, R, C, 7, args.variant) for R, C in B1_SHAPES for op in B1_OPS], \
-            {"workload": "SURVEY 8(f)#1: BLAS-1 Sasum/Snrm2/Isamax/Isamin fp32 at 256 MiB, N x L = 1x2^26 .. 2^22x16",
+            {"workload": "SURVEY 8(f)#1-2: BLAS-1 Sasum/Snrm2/Isamax/Isamin + the four fused in one pass "
+                         "(B1ALL, horizontal actor integration) fp32 at 256 MiB, N x L = 1x2^26 .. 2^22x16",
              "shapes": len(B1_SHAPES) * len(B1_OPS)}
     if args.workload == "dot":
         return [Problem("dot", 1, 1 << k, 2, args.variant) for k in range(10, 31)], \
@@ -362,7 +364,7 @@ def measure_e2e(args, probs, world):
         Xh = torch.empty(p.X.numel(), dtype=torch.float32, pin_memory=True)
         Mh.copy_(p.M)
         Xh.copy_(p.X)
-        yh = torch.empty(p.R, dtype=p.y.dtype, pin_memory=True)
+        yh = torch.empty(p.y.numel(), dtype=p.y.dtype, pin_memory=True)
         hosts.append((Mh.data_ptr(), Xh.data_ptr(), yh.data_ptr(), Mh, Xh, yh))
     torch.cuda.synchronize()
 
@@ -384,7 +386,7 @@ def measure_e2e(args, probs, world):
     ms = max_over_ranks(t0.elapsed_time(t1), world)
     b = sum(p.bytes for p in sel)
     h2d = sum(p.M.numel() * 4 + p.X.numel() * 4 for p in sel)
-    d2h = sum(p.R * 4 for p in sel)
+    d2h = sum(p.y.numel() * 4 for p in sel)
     return {"value": world * b * args.e2e_steps / (ms / 1e3) / 1e9, "unit": UNIT,
             "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h, "steps": args.e2e_steps,
             "problems": len(sel), "api": "adaptic_run_host (C ABI, pinned host buffers)"}
@@ -407,7 +409,8 @@ def cpu_baseline(probs, args, budget_s: float = 20.0):
         elif p.op == "tmv":
             oracle.tmv(M.reshape(p.C, p.R), X)
         elif p.op in B1_OPS:
-            getattr(oracle, p.op)(M.reshape(p.R, p.C))
+            for f in (("asum", "nrm2", "iamax", "iamin") if p.op == "b1all" else (p.op,)):
+                getattr(oracle, f)(M.reshape(p.R, p.C))
         else:
             oracle.dot(M.reshape(p.R, p.C), X.reshape(p.R, p.C))
         t_total += time.perf_counter() - t
@@ -441,7 +444,7 @@ def run_reference(args):
         pool = [("mv", 2048, 32768)]
         cfg = 3
     elif args.workload == "blas1":
-        pool = [(op, 1, 1 << 24) for op in B1_OPS] + [(op, 1 << 16, 256) for op in B1_OPS]
+        pool = [(op, 1, 1 << 24) for op in B1_OPS[:4]] + [(op, 1 << 16, 256) for op in B1_OPS[:4]]
         cfg = 7
     else:
         pool = [("tmv", 1024, 1 << 16)]
@@ -460,7 +463,7 @@ def run_reference(args):
             x = synth.vector(C, np.float32, "uniform", synth.seed(cfg, "x"))
             data.append((op, R, C, M, x, 4 * (R * C + R + C)))
     fns = {"mv": oracle.mv, "tmv": oracle.tmv, "dot": oracle.dot}
-    fns.update({op: (lambda M, X, f=getattr(oracle, op): f(M)) for op in B1_OPS})
+    fns.update({op: (lambda M, X, f=getattr(oracle, op): f(M)) for op in B1_OPS if op != "b1all"})
     for s in range(args.warmup):
         op, R, C, M, X, _ = data[s % len(data)]
         fns[op](M, X)

@@ -43,6 +43,12 @@
  *   (else UNSUPPORTED).  Variants: MV_SUBWARP, MV_WPR, MV_CPR, MV_SPLIT
  *   (MV_TPR and the TMV family -> UNSUPPORTED).  Workspace (MV_SPLIT): 8-byte
  *   partials per (row, split) plus one counter per row.
+ *   ADAPTIC_OP_B1ALL is the paper's horizontal actor integration ("a
+ *   program that needs maximum and summation of all elements in an array ...
+ *   Adaptic launches one kernel to compute both"): the four reductions above from
+ *   one read of a, written as four N-vectors back to back in y (16*N bytes: asum,
+ *   nrm2 as float, then iamax, iamin as int32); same arithmetic and results as the
+ *   four separate ops; workspace partials are 32 bytes.
  *
  * The input-adaptive part (Fig. 2): adaptic_plan() is the paper's
  * "runtime kernel management" -- on the CPU, from the actual input dimensions,
@@ -137,7 +143,10 @@ typedef enum {
     ADAPTIC_OP_ASUM = 3,  /* float y[N] = sum_e |a_n[e]|                            */
     ADAPTIC_OP_NRM2 = 4,  /* float y[N] = sqrt(sum_e a_n[e]^2)                      */
     ADAPTIC_OP_IAMAX = 5, /* int32 y[N] = smallest 1-based e maximising |a_n[e]|    */
-    ADAPTIC_OP_IAMIN = 6  /* int32 y[N] = smallest 1-based e minimising |a_n[e]|    */
+    ADAPTIC_OP_IAMIN = 6, /* int32 y[N] = smallest 1-based e minimising |a_n[e]|    */
+    ADAPTIC_OP_B1ALL = 7  /* all four in ONE pass over a (horizontal actor integration,
+                           * P:600): y = [asum N floats | nrm2 N floats | iamax N int32 |
+                           * iamin N int32], 16*N bytes                               */
 } adaptic_op;
 
 typedef enum {

@@ -43,6 +43,8 @@ struct adaptic_plan_s {
     size_t smem;           // dynamic shared memory bytes (TPR ring, or staged x)
     int block;
     bool vec_shape;        // C % 4 == 0 (MV/DOT) or R % 4 == 0 (TMV)
+    bool mis;              // MV/DOT with C % 4 != 0: index 1 describes the misaligned-row
+                           // kernels (128-bit body + scalar head/tail, mv_mis_kernels.cuh)
     int64_t grid[2];       // [scalar, vector] instance
     int64_t chain[2];      // longest serial chain per accumulator
     int64_t depth[2];      // combine-tree depth after the chains
@@ -60,12 +62,12 @@ namespace {
 thread_local int g_last_cuda_error = 0;
 
 struct TableEntry {
-    int op, dtype, lr, lc, variant, lanes, splits, ctas_per_sm, unroll, xsmem, block, rows, order, pipe;
+    int op, dtype, vec, lr, lc, variant, lanes, splits, ctas_per_sm, unroll, xsmem, block, rows, order, pipe;
 };
 const TableEntry kTable[] = {
 #include "table_data.inc"
 #include "table_b1.inc"
-    {-1, -1, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0}};
+    {-1, -1, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0}};
 const int kTableN = int(sizeof(kTable) / sizeof(kTable[0])) - 1;
 
 const char* const kVariantNames[ADAPTIC_V_COUNT] = {
@@ -97,7 +99,9 @@ DevInfo device_info() {
 
 bool is_tmv_family(int v) { return v >= ADAPTIC_V_TMV_COL && v <= ADAPTIC_V_TMV_REGTILE; }
 bool is_mv_family(int v) { return v >= ADAPTIC_V_MV_TPR && v <= ADAPTIC_V_MV_SPLIT; }
-bool is_b1_op(int op) { return op >= ADAPTIC_OP_ASUM && op <= ADAPTIC_OP_IAMIN; }
+bool is_b1_op(int op) { return op >= ADAPTIC_OP_ASUM && op <= ADAPTIC_OP_B1ALL; }
+// bytes of y per output row (B1ALL writes four N-vectors)
+size_t y_bytes_per_row(int op) { return op == ADAPTIC_OP_B1ALL ? 16 : 4; }
 bool is_b1_variant(int v) { return v >= ADAPTIC_V_MV_SUBWARP && v <= ADAPTIC_V_MV_SPLIT; }
 bool op_has_variant(int op, int v) {
     if (op == ADAPTIC_OP_TMV) return is_tmv_family(v);
@@ -127,6 +131,7 @@ void* b1_group_fn(int op, int G, int rbu, bool vec) {
         case ADAPTIC_OP_NRM2: return b1_group_fn_nrm2(G, rbu, vec);
         case ADAPTIC_OP_IAMAX: return b1_group_fn_iamax(G, rbu, vec);
         case ADAPTIC_OP_IAMIN: return b1_group_fn_iamin(G, rbu, vec);
+        case ADAPTIC_OP_B1ALL: return b1_group_fn_all(G, rbu, vec);
         default: return nullptr;
     }
 }
@@ -136,9 +141,17 @@ void* b1_cta_fn(int op, bool vec) {
         case ADAPTIC_OP_NRM2: return b1_cta_fn_nrm2(vec);
         case ADAPTIC_OP_IAMAX: return b1_cta_fn_iamax(vec);
         case ADAPTIC_OP_IAMIN: return b1_cta_fn_iamin(vec);
+        case ADAPTIC_OP_B1ALL: return b1_cta_fn_all(vec);
         default: return nullptr;
     }
 }
+void* mis_group_fn(int dtype, int G, int U, int xm) {
+    return dtype == DT_F32 ? mis_group_fn_f32(G, U, xm) : mis_group_fn_i32(G, U, xm);
+}
+void* mis_cta_fn(int dtype, int NT, int U, int xm) {
+    return dtype == DT_F32 ? mis_cta_fn_f32(NT, U, xm) : mis_cta_fn_i32(NT, U, xm);
+}
+constexpr int64_t kMisMinCols = 16;   // below this a row is one or two vectors: scalar path
 void* tmv_fn(int dtype, int LR, int U, bool vec, int NT) {
     return dtype == DT_F32 ? tmv_fn_f32(LR, U, vec, NT) : tmv_fn_i32(LR, U, vec, NT);
 }
@@ -207,13 +220,19 @@ int heuristic_variant(int op, int64_t R, int64_t C, int sms) {
     return ADAPTIC_V_MV_SPLIT;
 }
 
-const TableEntry* table_lookup(int op, int dtype, int64_t R, int64_t C) {
+// Nearest measured cell of the same (op, dtype) and load-path shape (vec: the 128-bit
+// path needs C % 4 == 0, for TMV R % 4 == 0 -- the two paths have different optima).
+constexpr int kBeyondL2Log2 = 26;   // 2^26 elements = 256 MiB of fp32, 2x the 126 MB L2
+
+const TableEntry* table_lookup(int op, int dtype, int64_t R, int64_t C, bool* projected) {
     const int lr = ilog2_floor(R), lc = ilog2_floor(C);
+    *projected = false;
+    const int vec = (op == ADAPTIC_OP_TMV) ? (R % 4 == 0) : (C % 4 == 0);
     const TableEntry* best = nullptr;
     int bestd = INT_MAX;
     for (int i = 0; i < kTableN; ++i) {
         const TableEntry& e = kTable[i];
-        if (e.op != op || e.dtype != dtype) continue;
+        if (e.op != op || e.dtype != dtype || e.vec != vec) continue;
         const int d = std::abs(e.lr - lr) + std::abs(e.lc - lc);
         // ties: prefer the cell with the same element count (lr + lc), then the lower lr
         if (d < bestd || (d == bestd && best && std::abs(e.lr + e.lc - lr - lc) < std::abs(best->lr + best->lc - lr - lc))) {
@@ -221,8 +240,28 @@ const TableEntry* table_lookup(int op, int dtype, int64_t R, int64_t C) {
         }
     }
     if (best && bestd <= 2) return best;
+    // Larger than every measured cell nearby: once the input is well beyond L2 the
+    // streaming behaviour depends on the aspect ratio, not on the size, so project onto
+    // the largest measured diagonal (>= 2^26 elements, not above this problem) at the
+    // same rows:cols ratio; absolute counts (splits, CTAs per SM) are then re-derived.
+    int diag = -1;
+    for (int i = 0; i < kTableN; ++i) {
+        const TableEntry& e = kTable[i];
+        if (e.op == op && e.dtype == dtype && e.vec == vec && e.lr + e.lc <= lr + lc) diag = std::max(diag, e.lr + e.lc);
+    }
+    if (diag >= kBeyondL2Log2) {
+        const TableEntry* pb = nullptr;
+        int pd = INT_MAX;
+        for (int i = 0; i < kTableN; ++i) {
+            const TableEntry& e = kTable[i];
+            if (e.op != op || e.dtype != dtype || e.vec != vec || e.lr + e.lc != diag) continue;
+            const int d = std::abs((e.lr - e.lc) - (lr - lc));
+            if (d < pd) { pb = &e; pd = d; }
+        }
+        if (pb && pd <= 2) { *projected = true; return pb; }
+    }
     // int32 moves the same bytes as fp32: use the fp32 cells when int32 was not swept
-    if (dtype != ADAPTIC_F32) return table_lookup(op, ADAPTIC_F32, R, C);
+    if (dtype != ADAPTIC_F32) return table_lookup(op, ADAPTIC_F32, R, C, projected);
     return nullptr;
 }
 
@@ -233,7 +272,15 @@ adaptic_status derive_b1(adaptic_plan_s* p, const int32_t* params, const DevInfo
     const int op = p->op, v = p->variant;
     const int64_t R = p->R, C = p->C;
     auto par = [&](int i) -> int { return params ? params[i] : 0; };
-    const bool fp32_chain = (op == ADAPTIC_OP_ASUM);
+    const bool fp32_chain = (op == ADAPTIC_OP_ASUM || op == ADAPTIC_OP_B1ALL);
+    // B1ALL keeps one accumulator per row (U loads per step feed it) and folds every FOLD/U steps
+    const bool one_slot = (op == ADAPTIC_OP_B1ALL);
+    auto chain_of = [&](int64_t iters, int U) -> int64_t {
+        if (!one_slot) return fold_chain(iters);
+        const int64_t f = FOLD / U;
+        return int64_t(U) * std::min<int64_t>(iters, f) + iters / f;
+    };
+    const size_t part_bytes = (op == ADAPTIC_OP_B1ALL) ? 32 : 8;
     p->vec_shape = (C % 4 == 0);
     p->splits = 1; p->smem = 0; p->stages = 0; p->xmode = 0; p->ilv = 0; p->pipe = 0; p->rb = 1;
     p->fb_lanes = 0; p->fb_unroll = 0; p->ws_bytes = 0; p->cnt_off = 0;
@@ -261,7 +308,7 @@ adaptic_status derive_b1(adaptic_plan_s* p, const int32_t* params, const DevInfo
             const int64_t nv = w ? C / 4 : C;
             const int64_t iters = ceil_div(nv, int64_t(G) * U);
             p->grid[w] = std::max<int64_t>(1, std::min<int64_t>(ceil_div(R, rows_per_cta), int64_t(dev.sms) * cps));
-            p->chain[w] = fp32_chain ? fold_chain(iters) : 0;
+            p->chain[w] = fp32_chain ? chain_of(iters, U) : 0;
             p->depth[w] = ilog2c(U) + (w ? 2 : 0) + ilog2c(G) + 1;
             p->path_ok[w] = !fp32_chain || bound_ok(p->chain[w] + p->depth[w]);
         }
@@ -284,7 +331,7 @@ adaptic_status derive_b1(adaptic_plan_s* p, const int32_t* params, const DevInfo
             if (w == 1 && !p->vec_shape) continue;
             const int64_t nv = w ? C / 4 : C;
             const int64_t iters = ceil_div(nv, int64_t(S) * NT * U);   // interleaved splits
-            p->chain[w] = fp32_chain ? fold_chain(iters) : 0;
+            p->chain[w] = fp32_chain ? chain_of(iters, U) : 0;
             p->depth[w] = ilog2c(U) + (w ? 2 : 0) + 10 + (S > 1 ? ceil_div(S, NT) + 10 : 0) + 1;
             p->path_ok[w] = !fp32_chain || bound_ok(p->chain[w] + p->depth[w]);
             p->grid[w] = std::max<int64_t>(1, std::min<int64_t>(R * S, slots));
@@ -298,7 +345,7 @@ adaptic_status derive_b1(adaptic_plan_s* p, const int32_t* params, const DevInfo
     p->ilv = S > 1 ? 1 : 0;
     if (!p->path_ok[p->vec_shape ? 1 : 0]) return ADAPTIC_ERR_UNSUPPORTED;
     if (S > 1) {
-        const size_t part = ((size_t(R) * size_t(S) * 8 + 255) / 256) * 256;
+        const size_t part = ((size_t(R) * size_t(S) * part_bytes + 255) / 256) * 256;
         p->cnt_off = part;
         p->ws_bytes = part + size_t(R) * 4;
     }
@@ -316,6 +363,7 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
     if (is_b1_op(op)) return derive_b1(p, params, dev);
 
     p->vec_shape = (op == ADAPTIC_OP_TMV) ? (R % 4 == 0) : (C % 4 == 0);
+    p->mis = false;
     p->splits = 1;
     p->smem = 0;
     p->stages = 0;
@@ -330,10 +378,14 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
 
     for (int w = 0; w < 2; ++w) { p->grid[w] = 0; p->chain[w] = 0; p->depth[w] = 0; p->path_ok[w] = false; }
 
+    // rows not 16-byte aligned (C % 4 != 0): the misaligned-row kernels keep the matrix
+    // stream 128-bit; the plain scalar kernels (index 0) remain for DOT operands whose
+    // addresses differ modulo 16
+    const bool mis = !p->vec_shape && op != ADAPTIC_OP_TMV && v != ADAPTIC_V_MV_TPR && C >= kMisMinCols;
     if (v == ADAPTIC_V_MV_SUBWARP || v == ADAPTIC_V_MV_WPR || v == ADAPTIC_V_MV_TPR) {
         // group-kernel parameters (also the TPR scalar fallback)
         // TPR's fallback is the scalar group kernel, so size it for the scalar path
-        const int64_t nvv = (p->vec_shape && v != ADAPTIC_V_MV_TPR) ? C / 4 : C;
+        const int64_t nvv = ((p->vec_shape || mis) && v != ADAPTIC_V_MV_TPR) ? C / 4 : C;
         int G;
         if (v == ADAPTIC_V_MV_WPR) G = 32;
         else if (v == ADAPTIC_V_MV_SUBWARP && par(ADAPTIC_P_LANES) > 0) G = par(ADAPTIC_P_LANES);
@@ -349,19 +401,23 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
         if (xm < 0) return ADAPTIC_ERR_UNSUPPORTED;
         const size_t xsm = xm == 1 ? size_t((C * 4 + 15) / 16 * 16) : 0;
         int cps = par(ADAPTIC_P_CTAS_PER_SM);
-        if (cps <= 0) cps = occupancy(group_fn(dt, G, U, p->vec_shape, xm), GROUP_NT, xsm, dev.present, 4);
-        if (v != ADAPTIC_V_MV_TPR) { p->ctas_per_sm = cps; p->xmode = xm; p->smem = xsm; }
+        if (cps <= 0) cps = occupancy(mis ? mis_group_fn(dt, G, U, xm) : group_fn(dt, G, U, p->vec_shape, xm),
+                                      GROUP_NT, xsm, dev.present, 4);
+        if (v != ADAPTIC_V_MV_TPR) { p->ctas_per_sm = cps; p->xmode = xm; p->smem = xsm; p->mis = mis; }
+        const int rows_per_cta_mis = std::max(1, 4 / U) * (32 / G) * (GROUP_NT / 32);
         for (int w = 0; w < 2; ++w) {
             const int64_t nv = w ? C / 4 : C;
-            if (w == 1 && !p->vec_shape) continue;
+            if (w == 1 && !p->vec_shape && !mis) continue;
+            const bool wm = (w == 1 && mis);
             const int64_t iters = ceil_div(nv, int64_t(G) * U);
-            p->grid[w] = std::max<int64_t>(1, std::min<int64_t>(ceil_div(R, rows_per_cta), int64_t(dev.sms) * cps));
+            p->grid[w] = std::max<int64_t>(1, std::min<int64_t>(ceil_div(R, wm ? rows_per_cta_mis : rows_per_cta),
+                                                                int64_t(dev.sms) * cps));
             p->chain[w] = fold_chain(iters);
-            p->depth[w] = ilog2c(U) + (w ? 2 : 0) + ilog2c(G) + 1;
+            p->depth[w] = ilog2c(U) + (w ? 2 : 0) + ilog2c(G) + 1 + (wm ? 1 : 0);   // + head/tail term
             p->path_ok[w] = (dt == DT_I32) || bound_ok(p->chain[w] + p->depth[w]);
         }
         if (v != ADAPTIC_V_MV_TPR) {
-            if (!p->path_ok[p->vec_shape ? 1 : 0]) return ADAPTIC_ERR_UNSUPPORTED;
+            if (!p->path_ok[(p->vec_shape || mis) ? 1 : 0]) return ADAPTIC_ERR_UNSUPPORTED;
             return ADAPTIC_OK;
         }
         // ---- MV_TPR proper (vector path only; scalar path = the group fallback above)
@@ -402,7 +458,7 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
         if (NT <= 0) NT = (v == ADAPTIC_V_MV_CPR && nv1 >= 8192) ? 1024 : 256;
         if (NT != 256 && NT != 1024) return ADAPTIC_ERR_INVALID_ARG;
         int RB = par(ADAPTIC_P_ROWS);
-        if (RB <= 0) RB = 1;
+        if (RB <= 0 || mis) RB = 1;                        // misaligned kernels: one row per CTA step
         int U = par(ADAPTIC_P_UNROLL);
         if (U <= 0) U = RB == 4 ? 2 : 4;
         const bool combo_ok = (RB == 1 && (U == 2 || U == 4 || U == 8)) || (RB == 2 && (U == 2 || U == 4)) ||
@@ -416,8 +472,10 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
         // register double buffering (NT 256 only): 1 off, 2 on; default off
         const int pipe_req = par(ADAPTIC_P_PIPE);
         if (pipe_req < 0 || pipe_req > 2 || (pipe_req == 2 && NT != 256)) return ADAPTIC_ERR_INVALID_ARG;
-        p->pipe = pipe_req == 2 ? 1 : 0;
-        if (cps <= 0) cps = occupancy(cta_fn(dt, NT, RB, U, p->vec_shape, xm, p->pipe), NT, xsm, dev.present, 2048 / NT);
+        p->pipe = (pipe_req == 2 && !mis) ? 1 : 0;
+        p->mis = mis;
+        if (cps <= 0) cps = occupancy(mis ? mis_cta_fn(dt, NT, U, xm) : cta_fn(dt, NT, RB, U, p->vec_shape, xm, p->pipe),
+                                      NT, xsm, dev.present, 2048 / NT);
         p->lanes = NT; p->unroll = U; p->rb = RB; p->block = NT; p->ctas_per_sm = cps; p->xmode = xm; p->smem = xsm;
         // split order: 1 contiguous chunks, 2 interleaved steps (default for S > 1)
         const int order = par(ADAPTIC_P_ORDER);
@@ -436,10 +494,11 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
             bool ok_all = true;
             for (int w = 0; w < 2; ++w) {
                 const int64_t nv = w ? C / 4 : C;
-                if (w == 1 && !p->vec_shape) continue;
+                if (w == 1 && !p->vec_shape && !mis) continue;
                 const int64_t iters = ceil_div(ceil_div(nv, S), int64_t(NT) * U);
                 p->chain[w] = fold_chain(iters);
-                p->depth[w] = ilog2c(U) + (w ? 2 : 0) + ilog2c(NT) + (S > 1 ? ceil_div(S, NT) + ilog2c(NT) : 0) + 1;
+                p->depth[w] = ilog2c(U) + (w ? 2 : 0) + ilog2c(NT) + (S > 1 ? ceil_div(S, NT) + ilog2c(NT) : 0) + 1 +
+                              ((w == 1 && mis) ? 1 : 0);
                 p->path_ok[w] = (dt == DT_I32) || bound_ok(p->chain[w] + p->depth[w]);
                 p->grid[w] = std::max<int64_t>(1, std::min<int64_t>(groups * S, slots));
                 if (!p->path_ok[w]) ok_all = false;
@@ -450,7 +509,7 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
         if (S > INT_MAX || R * S > (int64_t(1) << 40)) return ADAPTIC_ERR_UNSUPPORTED;
         p->splits = int(S);
         p->ilv = (S > 1 && order != 1) ? 1 : 0;
-        if (!p->path_ok[p->vec_shape ? 1 : 0]) return ADAPTIC_ERR_UNSUPPORTED;
+        if (!p->path_ok[(p->vec_shape || mis) ? 1 : 0]) return ADAPTIC_ERR_UNSUPPORTED;
         if (S > 1) {
             const size_t part = ((size_t(R) * size_t(S) * 4 + 255) / 256) * 256;
             p->cnt_off = part;
@@ -514,11 +573,12 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
 }
 
 adaptic_status validate_shape(int op, int64_t rows, int64_t cols, int dtype) {
-    if (op < ADAPTIC_OP_MV || op > ADAPTIC_OP_IAMIN) return ADAPTIC_ERR_INVALID_ARG;
+    if (op < ADAPTIC_OP_MV || op > ADAPTIC_OP_B1ALL) return ADAPTIC_ERR_INVALID_ARG;
     if (dtype != ADAPTIC_F32 && dtype != ADAPTIC_I32) return ADAPTIC_ERR_INVALID_ARG;
     if (rows < 0 || cols < 0) return ADAPTIC_ERR_INVALID_ARG;
     if (is_b1_op(op) && dtype != ADAPTIC_F32) return ADAPTIC_ERR_UNSUPPORTED;
-    if ((op == ADAPTIC_OP_IAMAX || op == ADAPTIC_OP_IAMIN) && cols > int64_t(INT_MAX)) return ADAPTIC_ERR_UNSUPPORTED;
+    if ((op == ADAPTIC_OP_IAMAX || op == ADAPTIC_OP_IAMIN || op == ADAPTIC_OP_B1ALL) && cols > int64_t(INT_MAX))
+        return ADAPTIC_ERR_UNSUPPORTED;
     if (cols > 0 && rows > (int64_t(1) << 62) / 4 / cols) return ADAPTIC_ERR_INVALID_ARG;  // bytes overflow
     return ADAPTIC_OK;
 }
@@ -550,9 +610,10 @@ adaptic_status make_plan(int op, int64_t rows, int64_t cols, int dtype, int vari
         *out = p;
         return ADAPTIC_OK;
     }
-    if (const TableEntry* e = table_lookup(op, dtype, rows, cols)) {
-        int32_t tp[ADAPTIC_NPARAMS] = {e->lanes, e->splits, e->ctas_per_sm, e->unroll, e->xsmem, e->block, e->rows,
-                                       e->order, e->pipe};
+    bool projected = false;
+    if (const TableEntry* e = table_lookup(op, dtype, rows, cols, &projected)) {
+        int32_t tp[ADAPTIC_NPARAMS] = {e->lanes, projected ? 0 : e->splits, projected ? 0 : e->ctas_per_sm, e->unroll,
+                                       e->xsmem, e->block, e->rows, e->order, e->pipe};
         p->variant = e->variant; p->source = 1;
         if (derive(p, tp, dev) == ADAPTIC_OK) { *out = p; return ADAPTIC_OK; }
         if (derive(p, nullptr, dev) == ADAPTIC_OK) { *out = p; return ADAPTIC_OK; }
@@ -618,11 +679,11 @@ cudaError_t ensure_smem_attr(void* fn, size_t smem) {
 }
 
 adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, void* y,
-                      cudaStream_t stream, bool vec) {
+                      cudaStream_t stream, bool vec, bool mis) {
     const int dt = p->dtype;
     const bool px = p->op == ADAPTIC_OP_DOT;
     int64_t R = p->R, C = p->C;
-    const int w = vec ? 1 : 0;
+    const int w = (vec || mis) ? 1 : 0;
     void* part = p->ws;
     unsigned int* cnt = p->ws ? reinterpret_cast<unsigned int*>(static_cast<char*>(p->ws) + p->cnt_off) : nullptr;
     int S = p->splits;
@@ -667,14 +728,15 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
             break;
         case ADAPTIC_V_MV_SUBWARP:
         case ADAPTIC_V_MV_WPR:
-            fn = group_fn(dt, p->lanes, p->unroll, vec, p->xmode);
+            fn = mis ? mis_group_fn(dt, p->lanes, p->unroll, p->xmode) : group_fn(dt, p->lanes, p->unroll, vec, p->xmode);
             smem = p->smem;
             args6[0] = &A; args6[1] = &X; args6[2] = &y; args6[3] = &R; args6[4] = &C;
             args = args6;
             break;
         case ADAPTIC_V_MV_CPR:
         case ADAPTIC_V_MV_SPLIT:
-            fn = cta_fn(dt, p->lanes, p->rb, p->unroll, vec, p->xmode, p->pipe != 0);
+            fn = mis ? mis_cta_fn(dt, p->lanes, p->unroll, p->xmode)
+                     : cta_fn(dt, p->lanes, p->rb, p->unroll, vec, p->xmode, p->pipe != 0);
             smem = p->smem;
             args9[0] = &A; args9[1] = &X; args9[2] = &y; args9[3] = &R; args9[4] = &C;
             args9[5] = &S; args9[6] = &ilv; args9[7] = &part; args9[8] = &cnt;
@@ -719,7 +781,7 @@ adaptic_status check_run(const adaptic_plan_s* p, const void* A, const void* x, 
     const bool b1 = is_b1_op(p->op);          // BLAS-1: x is unused (may be NULL)
     if (!A || (!x && !b1)) return ADAPTIC_ERR_INVALID_ARG;
     if (!aligned(A, 4) || (!b1 && !aligned(x, 4))) return ADAPTIC_ERR_MISALIGNED;
-    const size_t ybytes = size_t(p->R) * 4;
+    const size_t ybytes = size_t(p->R) * y_bytes_per_row(p->op);
     const size_t abytes = size_t(p->R) * size_t(p->C) * 4;
     const size_t xbytes = b1 ? 0 : (p->op == ADAPTIC_OP_DOT ? abytes : size_t(p->C) * 4);
     if (overlap(y, ybytes, A, abytes) || (!b1 && overlap(y, ybytes, x, xbytes))) return ADAPTIC_ERR_ALIAS;
@@ -764,19 +826,20 @@ adaptic_status adaptic_plan_set_workspace(adaptic_plan_t plan, void* dev_ptr, si
 
 int adaptic_plan_describe(adaptic_plan_t p, char* buf, size_t cap) {
     if (!p) return -1;
-    static const char* ops[] = {"MV", "TMV", "DOT", "ASUM", "NRM2", "IAMAX", "IAMIN"};
+    static const char* ops[] = {"MV", "TMV", "DOT", "ASUM", "NRM2", "IAMAX", "IAMIN", "B1ALL"};
     static const char* src[] = {"forced", "table", "heuristic"};
     char tmp[1024];
     const int n = std::snprintf(
         tmp, sizeof(tmp),
         "{\"op\":\"%s\",\"dtype\":\"%s\",\"rows\":%lld,\"cols\":%lld,\"variant\":\"%s\",\"source\":\"%s\","
         "\"sms\":%d,\"lanes\":%d,\"unroll\":%d,\"rows_per_group\":%d,\"splits\":%d,\"block\":%d,"
-        "\"ctas_per_sm\":%d,\"stages\":%d,\"xmode\":%d,\"ilv\":%d,\"pipe\":%d,\"smem\":%zu,\"vec_shape\":%s,"
+        "\"ctas_per_sm\":%d,\"stages\":%d,\"xmode\":%d,\"ilv\":%d,\"pipe\":%d,\"smem\":%zu,\"vec_shape\":%s,\"mis\":%s,"
         "\"grid\":[%lld,%lld],\"chain\":[%lld,%lld],\"depth\":[%lld,%lld],\"path_ok\":[%s,%s],"
         "\"fallback_lanes\":%d,\"fallback_unroll\":%d,\"workspace_bytes\":%zu}",
         ops[p->op], p->dtype == ADAPTIC_F32 ? "f32" : "i32", (long long)p->R, (long long)p->C,
         kVariantNames[p->variant], src[p->source], p->sms, p->lanes, p->unroll, p->rb, p->splits, p->block,
         p->ctas_per_sm, p->stages, p->xmode, p->ilv, p->pipe, p->smem, p->vec_shape ? "true" : "false",
+        p->mis ? "true" : "false",
         (long long)p->grid[0], (long long)p->grid[1], (long long)p->chain[0], (long long)p->chain[1],
         (long long)p->depth[0], (long long)p->depth[1], p->path_ok[0] ? "true" : "false",
         p->path_ok[1] ? "true" : "false", p->fb_lanes, p->fb_unroll, p->ws_bytes);
@@ -794,7 +857,7 @@ adaptic_status adaptic_run(adaptic_plan_t p, const void* A, const void* x, void*
     adaptic_status st = check_run(p, A, x, y);
     if (st != ADAPTIC_OK || p->R == 0) return st;
     if (p->C == 0) {
-        cudaError_t e = cudaMemsetAsync(y, 0, size_t(p->R) * 4, stream);
+        cudaError_t e = cudaMemsetAsync(y, 0, size_t(p->R) * y_bytes_per_row(p->op), stream);
         return e == cudaSuccess ? ADAPTIC_OK : cuda_fail(e);
     }
     bool vec = p->vec_shape;
@@ -803,8 +866,12 @@ adaptic_status adaptic_run(adaptic_plan_t p, const void* A, const void* x, void*
         else if (is_b1_op(p->op)) vec = aligned(A, 16);
         else vec = aligned(A, 16) && aligned(x, 16);
     }
-    if (!p->path_ok[vec ? 1 : 0]) return ADAPTIC_ERR_MISALIGNED;   // scalar path would break the error bound
-    return launch(p, A, x, y, stream, vec);
+    // misaligned-row kernels: any 4-byte aligned A; DOT's b must share A's address modulo 16
+    const bool mis = !vec && p->mis &&
+                     (p->op != ADAPTIC_OP_DOT ||
+                      ((reinterpret_cast<uintptr_t>(A) - reinterpret_cast<uintptr_t>(x)) & 15u) == 0);
+    if (!p->path_ok[(vec || mis) ? 1 : 0]) return ADAPTIC_ERR_MISALIGNED;   // scalar path would break the error bound
+    return launch(p, A, x, y, stream, vec, mis);
 }
 
 adaptic_status adaptic_run_host(adaptic_plan_t p, const void* A_host, const void* x_host, void* y_host,
@@ -826,7 +893,8 @@ adaptic_status adaptic_run_host(adaptic_plan_t p, const void* A_host, const void
     }
     st = adaptic_run(p, dA, dx, dy, stream_);
     if (st != ADAPTIC_OK) return st;
-    if ((e = cudaMemcpyAsync(y_host, dy, size_t(p->R) * 4, cudaMemcpyDeviceToHost, stream)) != cudaSuccess)
+    if ((e = cudaMemcpyAsync(y_host, dy, size_t(p->R) * y_bytes_per_row(p->op), cudaMemcpyDeviceToHost, stream)) !=
+        cudaSuccess)
         return cuda_fail(e);
     return ADAPTIC_OK;
 }

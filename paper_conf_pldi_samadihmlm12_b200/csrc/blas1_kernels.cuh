@@ -37,7 +37,7 @@
 
 namespace adaptic {
 
-enum B1Op { B1_ASUM = 0, B1_NRM2 = 1, B1_IAMAX = 2, B1_IAMIN = 3 };
+enum B1Op { B1_ASUM = 0, B1_NRM2 = 1, B1_IAMAX = 2, B1_IAMIN = 3, B1_ALL = 4 };
 
 // Per-op policy.  Acc<VEC> is a load slot's accumulator; P is what crosses
 // lanes, warps and CTAs; comb() is the associative/commutative operator.
@@ -60,7 +60,7 @@ template <> struct B1<B1_ASUM> {
     __device__ static P comb(P a, P b) { return a + b; }
     __device__ static void add(float& a, const float& b) { a += b; }
     __device__ static void add(float4& a, const float4& b) { a.x += b.x; a.y += b.y; a.z += b.z; a.w += b.w; }
-    __device__ static void store(void* y, int64_t r, P v, const float*) { static_cast<float*>(y)[r] = v; }
+    __device__ static void store(void* y, int64_t r, P v, int64_t) { static_cast<float*>(y)[r] = v; }
 };
 
 template <> struct B1<B1_NRM2> {
@@ -78,7 +78,7 @@ template <> struct B1<B1_NRM2> {
     __device__ static P fin(const double& a) { return a; }
     __device__ static P comb(P a, P b) { return a + b; }
     __device__ static void add(double& a, const double& b) { a += b; }
-    __device__ static void store(void* y, int64_t r, P v, const float*) {
+    __device__ static void store(void* y, int64_t r, P v, int64_t) {
         static_cast<float*>(y)[r] = float(sqrt(v));   // one rounding to fp32
     }
 };
@@ -148,7 +148,7 @@ template <int OP> struct B1Arg {
         return (static_cast<P>(key) << 32) | (kMax ? 0xffffffffu - a.e : a.e);
     }
     __device__ static P comb(P a, P b) { return kMax ? (a > b ? a : b) : (a < b ? a : b); }
-    __device__ static void store(void* y, int64_t r, P v, const float*) {
+    __device__ static void store(void* y, int64_t r, P v, int64_t) {
         const uint32_t lo = uint32_t(v & 0xffffffffull);
         static_cast<int32_t*>(y)[r] = int32_t((kMax ? 0xffffffffu - lo : lo) + 1u);
     }
@@ -156,9 +156,73 @@ template <int OP> struct B1Arg {
 template <> struct B1<B1_IAMAX> : B1Arg<B1_IAMAX> {};
 template <> struct B1<B1_IAMIN> : B1Arg<B1_IAMIN> {};
 
+// ALL: horizontal actor integration ("assume there is a program that needs
+// maximum and summation of all elements in an array. Instead of running two kernels
+// ... Adaptic launches one kernel to compute both") -- the four BLAS-1 actors above
+// share one pass over a.  y holds four N-vectors back to back:
+// [asum (float) | nrm2 (float) | iamax (int32) | iamin (int32)].
+// One accumulator per row (kOneSlot; 10 registers instead of 10 per load slot), so
+// the fp32 asum chain takes U terms per step: it folds every FOLD/U steps.
+struct B1AllP { double ssq; unsigned long long mx, mn; float asum; };
+template <> struct B1<B1_ALL> {
+    using MX = B1Arg<B1_IAMAX>;
+    using MN = B1Arg<B1_IAMIN>;
+    using P = B1AllP;
+    template <bool VEC> struct Acc_ {
+        typename B1<B1_ASUM>::template Acc<VEC> asum;
+        double ssq;
+        MX::Acc_ mx;
+        MN::Acc_ mn;
+    };
+    template <bool VEC> using Acc = Acc_<VEC>;
+    static constexpr bool kFold = true;
+    static constexpr bool kOneSlot = true;
+    __device__ static P ident() { P p; p.ssq = 0.0; p.mx = MX::ident(); p.mn = MN::ident(); p.asum = 0.f; return p; }
+    template <bool VEC> __device__ static void zero(Acc_<VEC>& a) {
+        B1<B1_ASUM>::zero(a.asum); a.ssq = 0.0; MX::zero(a.mx); MN::zero(a.mn);
+    }
+    template <bool VEC, class E> __device__ static void elem(Acc_<VEC>& a, const E& v, int64_t i) {
+        B1<B1_ASUM>::elem(a.asum, v, i); B1<B1_NRM2>::elem(a.ssq, v, i); MX::elem(a.mx, v, i); MN::elem(a.mn, v, i);
+    }
+    template <bool VEC> __device__ static void add(Acc_<VEC>& a, const Acc_<VEC>& b) {
+        B1<B1_ASUM>::add(a.asum, b.asum); a.ssq += b.ssq; MX::add(a.mx, b.mx); MN::add(a.mn, b.mn);
+    }
+    template <bool VEC> __device__ static P fin(const Acc_<VEC>& a) {
+        P p; p.asum = B1<B1_ASUM>::fin(a.asum); p.ssq = a.ssq; p.mx = MX::fin(a.mx); p.mn = MN::fin(a.mn); return p;
+    }
+    __device__ static P comb(P a, const P& b) {
+        a.asum += b.asum; a.ssq += b.ssq; a.mx = MX::comb(a.mx, b.mx); a.mn = MN::comb(a.mn, b.mn); return a;
+    }
+    __device__ static P shfl(P v, int o) {
+        v.asum = __shfl_xor_sync(0xffffffffu, v.asum, o); v.ssq = __shfl_xor_sync(0xffffffffu, v.ssq, o);
+        v.mx = __shfl_xor_sync(0xffffffffu, v.mx, o); v.mn = __shfl_xor_sync(0xffffffffu, v.mn, o);
+        return v;
+    }
+    __device__ static void store(void* y, int64_t r, const P& v, int64_t R) {
+        float* yf = static_cast<float*>(y);
+        B1<B1_ASUM>::store(yf, r, v.asum, R);
+        B1<B1_NRM2>::store(yf + R, r, v.ssq, R);
+        MX::store(yf + 2 * R, r, v.mx, R);
+        MN::store(yf + 3 * R, r, v.mn, R);
+    }
+};
+
+// workspace partials of the fused op, read back by the merging CTA (bypass L1)
+__device__ __forceinline__ B1AllP ld_partial_any(const B1AllP* p) {
+    B1AllP v;
+    v.ssq = __ldcg(&p->ssq); v.mx = __ldcg(&p->mx); v.mn = __ldcg(&p->mn); v.asum = __ldcg(&p->asum);
+    return v;
+}
+
+// lane exchange: plain shuffle for scalar partials, the policy's own for structs
+template <int OP, class P> __device__ __forceinline__ P b1_shfl(const P& v, int o) {
+    if constexpr (std::is_arithmetic<P>::value) return __shfl_xor_sync(0xffffffffu, v, o);
+    else return B1<OP>::shfl(v, o);
+}
+
 template <int OP, int G> __device__ __forceinline__ typename B1<OP>::P b1_group_comb(typename B1<OP>::P v) {
 #pragma unroll
-    for (int o = G / 2; o >= 1; o >>= 1) v = B1<OP>::comb(v, __shfl_xor_sync(0xffffffffu, v, o));
+    for (int o = G / 2; o >= 1; o >>= 1) v = B1<OP>::comb(v, b1_shfl<OP>(v, o));
     return v;
 }
 
@@ -219,7 +283,7 @@ b1_group_kernel(const float* __restrict__ A, void* __restrict__ y, int64_t R, in
             for (int i = 0; i < RB; ++i)
 #pragma unroll
                 for (int u = 0; u < U; ++u) Pol::elem(acc[i][Pol::kOneSlot ? 0 : u], a[i][u], j0 + int64_t(G) * u);
-            if (Pol::kFold && ++it == FOLD) {
+            if (Pol::kFold && ++it == (Pol::kOneSlot ? FOLD / U : FOLD)) {
                 it = 0;
 #pragma unroll
                 for (int i = 0; i < RB; ++i) {
@@ -238,7 +302,7 @@ b1_group_kernel(const float* __restrict__ A, void* __restrict__ y, int64_t R, in
             P s = Pol::comb(outer[i], b1_slots<OP, U>(acc[i]));
             s = b1_group_comb<OP, G>(s);
             const int64_t row = base + i * NG + g;
-            if (li == 0 && row < R) Pol::store(y, row, s, A + row * C);
+            if (li == 0 && row < R) Pol::store(y, row, s, R);
         }
     }
 }
@@ -298,7 +362,7 @@ b1_cta_kernel(const float* __restrict__ A, void* __restrict__ y, int64_t R, int6
             for (int u = 0; u < U; ++u) a[u] = ld_stream(Ar + b + tid + int64_t(NT) * u);
 #pragma unroll
             for (int u = 0; u < U; ++u) Pol::elem(acc[Pol::kOneSlot ? 0 : u], a[u], b + tid + int64_t(NT) * u);
-            if (Pol::kFold && ++it == FOLD) {
+            if (Pol::kFold && ++it == (Pol::kOneSlot ? FOLD / U : FOLD)) {
                 it = 0;
                 outer = Pol::comb(outer, b1_slots<OP, U>(acc));
 #pragma unroll
@@ -310,7 +374,7 @@ b1_cta_kernel(const float* __restrict__ A, void* __restrict__ y, int64_t R, int6
         P val = b1_cta_comb<OP, NT>(Pol::comb(outer, b1_slots<OP, U>(acc)), red);
 
         if (S == 1) {
-            if (tid == 0) Pol::store(y, row, val, A + row * C);
+            if (tid == 0) Pol::store(y, row, val, R);
         } else {
             if (tid == 0) ws_part[row * S + s] = val;
             if (ticket_is_last(ws_cnt + row, unsigned(S), &flag)) {
@@ -318,7 +382,7 @@ b1_cta_kernel(const float* __restrict__ A, void* __restrict__ y, int64_t R, int6
                 P m = Pol::ident();
                 for (int k = tid; k < S; k += NT) m = Pol::comb(m, ld_partial_any(ws_part + row * S + k));
                 m = b1_cta_comb<OP, NT>(m, red);
-                if (tid == 0) Pol::store(y, row, m, A + row * C);
+                if (tid == 0) Pol::store(y, row, m, R);
             }
         }
         __syncthreads();

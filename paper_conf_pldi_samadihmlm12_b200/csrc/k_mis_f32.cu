@@ -1,0 +1,4 @@
+#define KT float
+#define MIS_GROUP_FN mis_group_fn_f32
+#define MIS_CTA_FN mis_cta_fn_f32
+#include "k_mis.inc"

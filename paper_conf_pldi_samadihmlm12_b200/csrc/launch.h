@@ -35,6 +35,14 @@ void* tmv_fn_i32(int LR, int U, bool vec, int NT);
 void* cta_fn(int dtype, int NT, int RB, int U, bool vec, int xmode, bool pipe);
 void* tpr_fn(int dtype, int NT, bool perrowx);
 
+// Misaligned-row MV/DOT (mv_mis_kernels.cuh; C % 4 != 0, 128-bit body + scalar head/tail):
+//   group: (const T* A, const T* X, T* y, int64_t R, int64_t C), RB = max(1, 4/U)
+//   cta  : (const T* A, const T* X, T* y, int64_t R, int64_t C, int S, int ilv, T* part, unsigned* cnt)
+void* mis_group_fn_f32(int G, int U, int xmode);
+void* mis_group_fn_i32(int G, int U, int xmode);
+void* mis_cta_fn_f32(int NT, int U, int xmode);
+void* mis_cta_fn_i32(int NT, int U, int xmode);
+
 // BLAS-1 reductions (blas1_kernels.cuh), fp32 input, one translation unit per operator:
 //   b1 group: (const float* A, void* y, int64_t R, int64_t C); rbu 0 = (RB 4, U 2), 1 = (RB 1, U 8)
 //   b1 cta  : (const float* A, void* y, int64_t R, int64_t C, int S, P* part, unsigned* cnt)
@@ -47,5 +55,7 @@ void* b1_cta_fn_asum(bool vec);
 void* b1_cta_fn_nrm2(bool vec);
 void* b1_cta_fn_iamax(bool vec);
 void* b1_cta_fn_iamin(bool vec);
+void* b1_group_fn_all(int G, int rbu, bool vec);
+void* b1_cta_fn_all(bool vec);
 
 }  // namespace adaptic

@@ -146,6 +146,28 @@ def iamin(a: torch.Tensor, *, variant="AUTO", params=None, out=None) -> torch.Te
     return _blas1(L.OP_IAMIN, a, variant, params, out, torch.int32)
 
 
+def b1all(a: torch.Tensor, *, variant="AUTO", params=None, out=None):
+    """All four BLAS-1 reductions of every row from ONE pass over ``a`` (the paper's
+    horizontal actor integration).  Returns (asum, nrm2, iamax, iamin): two
+    float32 and two int32 tensors of N elements, views of one 16*N-byte buffer."""
+    if a.dim() not in (1, 2):
+        raise ValueError(f"expected [N, L] (or [L]) input, got {tuple(a.shape)}")
+    if a.dtype != torch.float32:
+        raise TypeError(f"BLAS-1 reductions take float32, got {a.dtype}")
+    N, Lk = (1, a.shape[0]) if a.dim() == 1 else a.shape
+    dev = _check_dev(a)
+    if out is None:
+        out = torch.empty(4 * N, dtype=torch.float32, device=dev)
+    elif out.numel() != 4 * N or out.element_size() != 4 or out.device != dev or not out.is_contiguous():
+        raise ValueError(f"out must be a contiguous 4-byte tensor of {4 * N} elements on {dev}")
+    stream = torch.cuda.current_stream(dev).cuda_stream
+    plan = get_plan(L.OP_B1ALL, N, Lk, L.F32, dev, variant, params, stream)
+    plan.run(a.data_ptr(), 0, out.data_ptr(), stream)
+    f = out.view(torch.float32)
+    i = out.view(torch.int32)
+    return f[:N], f[N:2 * N], i[2 * N:3 * N], i[3 * N:]
+
+
 def plan(op: str, rows: int, cols: int, dtype: str = "f32", variant="AUTO", params=None) -> L.Plan:
     """A bare plan (no workspace attached) -- for inspecting the selector."""
     return L.Plan(L.OPS[op], rows, cols, {"f32": L.F32, "i32": L.I32}[dtype], variant, params)

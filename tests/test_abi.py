@@ -106,7 +106,7 @@ def test_invalid_args():
     h = ctypes.c_void_p()
     assert lib.adaptic_plan(0, -1, 5, 0, ctypes.byref(h)) == L.ERR_INVALID_ARG
     assert lib.adaptic_plan(0, 5, -1, 0, ctypes.byref(h)) == L.ERR_INVALID_ARG
-    assert lib.adaptic_plan(7, 5, 5, 0, ctypes.byref(h)) == L.ERR_INVALID_ARG
+    assert lib.adaptic_plan(8, 5, 5, 0, ctypes.byref(h)) == L.ERR_INVALID_ARG
     assert lib.adaptic_plan(0, 5, 5, 9, ctypes.byref(h)) == L.ERR_INVALID_ARG
     assert lib.adaptic_plan(0, 1 << 40, 1 << 40, 0, ctypes.byref(h)) == L.ERR_INVALID_ARG  # byte overflow
     assert lib.adaptic_plan(0, 5, 5, 0, None) == L.ERR_INVALID_ARG

@@ -97,3 +97,21 @@ def test_run_contract_x_unused():
     q = adaptic.plan("nrm2", 4, 1 << 22, variant="MV_SPLIT")
     assert q.run_ptrs(A, 0, 0x30000000) == L.ERR_NO_WORKSPACE
     assert adaptic.plan("iamax", 0, 5).run_ptrs(0, 0, 0) == L.OK
+
+
+def test_b1all_plan_and_contract():
+    """B1ALL (horizontal actor integration): four N-vectors in y, 32-byte
+    partials, the asum chain bound with one accumulator per row."""
+    src = open(os.path.join(ROOT, "include", "adaptic.h")).read()
+    assert re.search(r"ADAPTIC_OP_B1ALL\s*=\s*7\b", src)
+    for R, C in SHAPES:
+        d = adaptic.plan("b1all", R, C).describe()
+        w = 1 if d["vec_shape"] else 0
+        assert d["path_ok"][w] and d["chain"][w] + d["depth"][w] <= 1677, d
+    p = adaptic.plan("b1all", 4, 1 << 22, variant="MV_SPLIT")
+    d = p.describe()
+    assert p.workspace_bytes >= 4 * d["splits"] * 32 + 4 * 4
+    A = 0x10000000
+    assert p.run_ptrs(A, 0, A + 4 * (1 << 22) * 4 - 8) == L.ERR_ALIAS      # y spans 16*N bytes
+    with pytest.raises(adaptic.AdapticError):
+        adaptic.plan("b1all", 1, 1 << 31)

@@ -199,3 +199,47 @@ def test_device_generated_256MiB_batch():
     t = t.view(R, C)
     for op in OPS:
         check(op, gpu(op, None, dev_tensor=t), ref(op, a), f"{op} 64x2^20")
+
+
+# ------------------------------------------------------------------ horizontal actor integration
+def check_all(a, outs, what):
+    for op, y in zip(OPS, outs):
+        check(op, y.cpu().numpy(), ref(op, a), f"b1all/{op} {what}")
+
+
+@pytest.mark.parametrize("kind", ["uniform", "smallint"])
+def test_b1all_matches_the_four_oracles(kind):
+    """One pass computes asum, nrm2, iamax, iamin -- each equal to its own
+    oracle (same tolerances / bit-exactness as the separate ops), every variant."""
+    shapes = [(1, 1), (3, 5), (7, 33), (33, 257), (129, 1025), (5, 4099), (1, 100003), (1000, 12), (2, 1 << 20)]
+
+    def case(R, C, v, p):
+        a = synth.matrix(R, C, "mv", np.float32, kind, synth.seed(8, "A") + R + C)
+        try:
+            outs = adaptic.b1all(torch.from_numpy(a).to(DEV), variant=v, params=p)
+        except adaptic.AdapticError as e:
+            assert e.status == L.ERR_UNSUPPORTED, str(e)
+            return
+        check_all(a, outs, f"{kind} {R}x{C} {v} {p}")
+    _collect([(f"{R}x{C} {v} {p}", lambda R=R, C=C, v=v, p=p: case(R, C, v, p))
+              for (R, C), (v, p) in itertools.product(shapes, [("AUTO", None)] + FORCED)])
+
+
+def test_b1all_special_values_and_degenerate():
+    rows = [[np.nan, 1, 5, 2], [1, np.nan, 5, 2], [2, -np.inf, np.inf, 3], [7, 7, 7, 7], [0, 0, 0, 0]]
+    a = np.tile(np.array(rows, np.float32), (1, 257))
+    for v in ("AUTO", "MV_SUBWARP", "MV_WPR", "MV_CPR", "MV_SPLIT"):
+        asum, nrm2, imax, imin = adaptic.b1all(torch.from_numpy(a).to(DEV), variant=v)
+        check("iamax", imax.cpu().numpy(), ref("iamax", a), f"b1all special {v}")
+        check("iamin", imin.cpu().numpy(), ref("iamin", a), f"b1all special {v}")
+        assert np.isnan(asum.cpu().numpy()[:2]).all() and np.isinf(nrm2.cpu().numpy()[2])
+    outs = adaptic.b1all(torch.empty(3, 0, device=DEV))
+    assert all(o.cpu().tolist() == [0, 0, 0] for o in outs)
+
+
+def test_b1all_256MiB_batch_and_single_vector():
+    for R, C in [(64, 1 << 20), (1, 1 << 26)]:
+        t = torch.empty(R * C, dtype=torch.float32, device=DEV)
+        synth.device_matrix(t, R, C, "mv", "uniform", synth.seed(9, "A"))
+        a = t.cpu().numpy().reshape(R, C)
+        check_all(a, adaptic.b1all(t.view(R, C)), f"{R}x{C}")

@@ -1,0 +1,122 @@
+"""Misaligned-row MV/DOT kernels (C % 4 != 0: 128-bit body + scalar head/tail,
+csrc/mv_mis_kernels.cuh) against the oracle -- needs a GPU.
+
+fp32 within 1e-4 * S_r (north_star), int32 bit-exact.  Covers every head length
+h = 0..3 (rows start at every alignment), every forced variant, base pointers that
+are not 16-byte aligned, and DOT operands whose addresses differ modulo 16 (which
+take the scalar kernels)."""
+import itertools
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import synth
+
+pytestmark = pytest.mark.gpu
+
+if torch.cuda.is_available():
+    import paper_conf_pldi_samadihmlm12_b200 as adaptic
+    from paper_conf_pldi_samadihmlm12_b200 import _lib as L
+
+DEV = "cuda:0"
+TOL = 1e-4
+FORCED = [("AUTO", None)] + [("MV_SUBWARP", [g, 0, 0, u]) for g in (1, 4, 16) for u in (1, 2, 4, 8)] + \
+         [("MV_WPR", [0, 0, 0, u, xm]) for u in (1, 2, 4, 8) for xm in (1, 2)] + \
+         [("MV_CPR", [nt, 0, 0, u, xm]) for nt, u in ((256, 2), (256, 4), (256, 8), (1024, 2), (1024, 4))
+          for xm in (1, 2)] + \
+         [("MV_SPLIT", [nt, s, 0, u, 0, 0, 0, o]) for nt, u in ((256, 4), (1024, 2)) for s in (2, 5) for o in (1, 2)]
+
+
+def check(y, ref, dt, what):
+    if dt == "i32":
+        assert np.array_equal(y, ref), f"{what}: int32 mismatch at {np.nonzero(y != ref)[0][:8]}"
+    else:
+        yr, S = ref
+        err = np.abs(y.astype(np.float64) - yr)
+        bad = ~(err <= TOL * S)
+        assert not bad.any(), f"{what}: {bad.sum()} out of tolerance, worst {np.max(err - TOL * S)}"
+
+
+def _collect(cases):
+    fails = []
+    for what, fn in cases:
+        try:
+            fn()
+        except Exception as e:  # noqa: BLE001 -- report every failing case at once
+            fails.append(f"{what}: {type(e).__name__}: {str(e)[:200]}")
+    assert not fails, f"{len(fails)} failures:\n" + "\n".join(fails[:40])
+
+
+@pytest.mark.parametrize("op", ["mv", "dot"])
+@pytest.mark.parametrize("dt", ["f32", "i32"])
+def test_every_variant_every_head_length(op, dt):
+    npdt = np.float32 if dt == "f32" else np.int32
+    shapes = [(7, 17), (9, 18), (33, 19), (65, 127), (130, 1001), (3, 4099), (257, 66), (5, 100003), (1000, 21)]
+
+    def case(R, C, v, p):
+        A = synth.matrix(R, C, "mv", npdt, "uniform", synth.seed(11, "A") + R + C)
+        X = (synth.matrix(R, C, "mv", npdt, "uniform", synth.seed(11, "b") + R) if op == "dot"
+             else synth.vector(C, npdt, "uniform", synth.seed(11, "x") + C))
+        try:
+            plan = adaptic.plan(op, R, C, dt, variant=v, params=p)
+        except adaptic.AdapticError as e:
+            assert e.status == L.ERR_UNSUPPORTED, str(e)
+            return
+        if C >= 16 and v != "AUTO":
+            assert plan.describe()["mis"], plan.describe()
+        fn = adaptic.mv if op == "mv" else adaptic.dot
+        y = fn(torch.from_numpy(A).to(DEV), torch.from_numpy(X).to(DEV), variant=v, params=p).cpu().numpy()
+        ref = oracle.mv(A, X) if op == "mv" else oracle.dot(A, X)
+        check(y, ref, dt, f"{op} {dt} {R}x{C} {v} {p}")
+    _collect([(f"{R}x{C} {v} {p}", lambda R=R, C=C, v=v, p=p: case(R, C, v, p))
+              for (R, C), (v, p) in itertools.product(shapes, FORCED)])
+
+
+def test_unaligned_base_pointer_any_C():
+    """The head length is computed from the actual row address, so a matrix whose
+    base is only 4-byte aligned runs the same kernels."""
+    for R, C, off in [(31, 37, 1), (64, 1001, 2), (9, 5000, 3), (100, 16, 1)]:
+        A = synth.matrix(R, C, "mv", np.float32, "uniform", 5 + C)
+        x = synth.vector(C, np.float32, "uniform", 6 + C)
+        big = torch.zeros(R * C + 8, dtype=torch.float32, device=DEV)
+        big[off:off + R * C] = torch.from_numpy(A.reshape(-1)).to(DEV)
+        Ad = big[off:off + R * C].view(R, C)
+        for v in ("AUTO", "MV_SUBWARP", "MV_WPR", "MV_CPR", "MV_SPLIT"):
+            try:
+                y = adaptic.mv(Ad, torch.from_numpy(x).to(DEV), variant=v).cpu().numpy()
+            except adaptic.AdapticError as e:
+                assert e.status == L.ERR_UNSUPPORTED
+                continue
+            check(y, oracle.mv(A, x), "f32", f"off {off} {R}x{C} {v}")
+
+
+def test_dot_operands_with_different_alignment():
+    """a and b differing modulo 16 bytes: the scalar kernels (still exact/in tolerance)."""
+    R, C = 17, 1003
+    a = synth.matrix(R, C, "mv", np.int32, "uniform", 71)
+    b = synth.matrix(R, C, "mv", np.int32, "uniform", 72)
+    bb = torch.zeros(R * C + 4, dtype=torch.int32, device=DEV)
+    bb[1:1 + R * C] = torch.from_numpy(b.reshape(-1)).to(DEV)
+    for v in ("AUTO", "MV_WPR", "MV_CPR", "MV_SPLIT"):
+        y = adaptic.dot(torch.from_numpy(a).to(DEV), bb[1:1 + R * C].view(R, C), variant=v).cpu().numpy()
+        check(y, oracle.dot(a, b), "i32", f"dot mismatched {v}")
+
+
+@pytest.mark.parametrize("k", [2, 5, 8, 11, 14, 17, 20])
+def test_held_out_shapes_3x2k(k):
+    """The selector's held-out grid (SURVEY 8(d) configs[1]): R = 3*2^k, C = 2^26/R
+    (not a multiple of 4), scaled to 2^22 elements for the oracle, exact on smallint."""
+    R = 3 << (k - 2) if k >= 2 else 3
+    C = (1 << 22) // R
+    for kind, dt in (("uniform", "f32"), ("smallint", "f32"), ("uniform", "i32")):
+        npdt = np.float32 if dt == "f32" else np.int32
+        A = synth.matrix(R, C, "mv", npdt, kind, synth.seed(1, "A"))
+        x = synth.vector(C, npdt, kind, synth.seed(1, "x"))
+        y = adaptic.mv(torch.from_numpy(A).to(DEV), torch.from_numpy(x).to(DEV)).cpu().numpy()
+        ref = oracle.mv(A, x)
+        if kind == "smallint" and dt == "f32":
+            assert np.array_equal(y.astype(np.float64), ref[0]), f"P5 exact {R}x{C}"
+        else:
+            check(y, ref, dt, f"held-out {R}x{C} {kind} {dt}")

@@ -122,6 +122,9 @@ def main():
     ap.add_argument("--kmin", type=int, default=3)
     ap.add_argument("--kmax", type=int, default=23)
     ap.add_argument("--extra", default="", help="extra shapes R1xC1,R2xC2")
+    ap.add_argument("--perturb", action="store_true",
+                    help="also time each diagonal shape with the reduction length (MV/DOT: C+1) or the "
+                         "output count (TMV: R+1) off the 128-bit path, for the scalar-shape table cells")
     a = ap.parse_args()
     dev = torch.device("cuda:0")
     tdt = torch.float32 if a.dtype == "f32" else torch.int32
@@ -134,16 +137,21 @@ def main():
     for s in filter(None, a.extra.split(",")):
         r, c = s.lower().split("x")
         shapes.append((int(r), int(c)))
-    maxel = max(R * C for R, C in shapes)
+    if a.perturb:
+        shapes = [(R, C, p) for R, C in shapes for p in (0, 1)]
+    else:
+        shapes = [(R, C, 0) for R, C in shapes]
+    maxel = max(R * C for R, C, _ in shapes) + max(R + C for R, C, _ in shapes)
     M = torch.empty(maxel * (2 if "dot" in a.ops else 1), dtype=tdt, device=dev)
-    X = torch.empty(max(C for _, C in shapes), dtype=tdt, device=dev)
-    Y = torch.empty(max(R for R, _ in shapes), dtype=tdt, device=dev)   # 4-byte y (int32 for IAMAX/IAMIN)
+    X = torch.empty(max(C for _, C, _ in shapes) + 1, dtype=tdt, device=dev)
+    Y = torch.empty(max(R for R, _, _ in shapes) + 1, dtype=tdt, device=dev)   # 4-byte y (int32 for IAMAX/IAMIN)
     synth.device_matrix(M, 1, M.numel(), "mv", "uniform", 11)
     synth.device_vector(X, "uniform", 12)
     t0 = time.time()
     with open(a.out, "a") as f:
         for op in a.ops.split(","):
-            for R, C in shapes:
+            for R0, C0, pert in shapes:
+                R, C = (R0 + pert, C0) if op == "tmv" else (R0, C0 + pert)
                 Xp = M.data_ptr() + R * C * 4 if op == "dot" else X.data_ptr()
                 ptrs = (M.data_ptr(), Xp, Y.data_ptr())
                 for variant, params in grids(op, R, C):
