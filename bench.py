@@ -9,6 +9,8 @@ Workloads (``--workload``):
   rowshard (BJ:configs[3]) MV 131072 x 32768 fp32, rows sharded over ranks.
   splitk   (BJ:configs[4]) TMV 1024 x 16M fp32, C split over ranks + NCCL all-reduce.
   dot      (BJ:configs[2]) scalar product N = 1, L = 2^10..2^30 (fp32).
+  config0  (BJ:configs[0]) TMV fp32 256 x 256 (L2-resident, launch-latency bound): the
+           line adds single-launch and CUDA-graph-amortized latency in microseconds.
   blas1 Sasum / Snrm2 / Isamax / Isamin (the paper's Fig. 9
            CUBLAS benchmarks) on 256 MiB inputs: N x L = 1 x 2^26 .. 2^22 x 16.
 Multi-GPU: one process per GPU (torchrun), barrier + synchronize around the
@@ -42,7 +44,7 @@ def parse():
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", choices=["adaptic", "reference"], default="adaptic")
-    ap.add_argument("--workload", choices=["sweep", "rowshard", "splitk", "dot", "blas1"], default="sweep")
+    ap.add_argument("--workload", choices=["sweep", "rowshard", "splitk", "dot", "blas1", "config0"], default="sweep")
     ap.add_argument("--variant", default="AUTO", help="force one variant (fixed-variant sweeps)")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-e2e", action="store_true")
@@ -206,6 +208,9 @@ def build_problems(args, world, rank):
                 for k in range(3, 24) for op in ("mv", "tmv")], \
             {"workload": "configs[1]: TMV/MV fp32 shape sweep at 256 MiB, 8Mx8 .. 8192x8192 .. 8x8M, "
                          "both layouts, variant selector", "shapes": 42, "per_gpu": "full sweep (weak)"}
+    if args.workload == "config0":
+        return [Problem("tmv", 256, 256, 0, args.variant)], \
+            {"workload": "configs[0]: TMV fp32 256x256 (L2-resident; latency-bound)", "shapes": 1}
     if args.workload == "blas1":
         return [Problem(op, R, C, 7, args.variant) for R, C in B1_SHAPES for op in B1_OPS], \
             {"workload": "SURVEY 8(f)#1-2: BLAS-1 Sasum/Snrm2/Isamax/Isamin + the four fused in one pass "
@@ -318,6 +323,9 @@ def run_adaptic(args):
                 f"{min(per, key=lambda q: q['frac'])['C']}",
                 "median_frac": statistics.median(q["frac"] for q in per)}
 
+    latency = None
+    if args.workload == "config0" and rank == 0:
+        latency = measure_latency(probs[0])
     e2e = None
     if not args.no_e2e and args.e2e_steps > 0:
         e2e = measure_e2e(args, probs, world)
@@ -334,18 +342,57 @@ def run_adaptic(args):
                 "scaling": "weak" if args.workload in ("sweep", "dot") else "strong",
                 "vs_baseline": None, "dtype": "f32", "data": "synthetic (seeded splitmix64, U[-1,1))",
                 "config": dict(config, bytes_per_step_per_gpu=step_bytes, variant=args.variant,
-                               l2="every input >= 256 MiB > 126 MB L2 and problems alternate; no flush needed"
-                               if args.workload == "sweep" else "inputs > L2; no flush needed"),
+                               l2=("every input >= 256 MiB > 126 MB L2 and problems alternate; no flush needed"
+                                   if args.workload in ("sweep", "blas1") else
+                                   "L2-resident by design (256 KiB): latency-bound, see latency_us"
+                                   if args.workload == "config0" else
+                                   "dot: lengths 2^10..2^30 back to back; the >= 2^25 ones exceed L2"
+                                   if args.workload == "dot" else "inputs > L2; no flush needed")),
                 "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
                 "kernel_timing": ("per-launch CUDA events inside the timed region" if inner else
                                   f"per-kernel CUDA events after the timed region: each kernel 5x back to back, "
                                   f"{kev_steps} samples (the timed region itself has events only at its ends)"),
-                "kernel_sum_ms": kernel_sum_ms,
+                "kernel_sum_ms": kernel_sum_ms, "latency_us": latency,
                 "gpu_launches": n * args.steps, "clocks": clk,
                 "selected": {q["op"] + f" {q['R']}x{q['C']}": [q["variant"], round(q["frac"], 3)] for q in per}}
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()
+
+
+def measure_latency(p, reps=200):
+    """configs[0]: one launch between two events (single-launch latency as a caller of
+    adaptic_run sees it, host enqueue included) and a CUDA graph of `reps` launches
+    (graph-amortized per-launch time)."""
+    import torch
+    stream = torch.cuda.Stream()
+    evs = [torch.cuda.Event(enable_timing=True) for _ in range(2)]
+    single = []
+    with torch.cuda.stream(stream):
+        s = stream.cuda_stream
+        for _ in range(20):
+            p.plan.run(*p.ptrs, s)
+        torch.cuda.synchronize()
+        for _ in range(50):
+            evs[0].record(stream)
+            p.plan.run(*p.ptrs, s)
+            evs[1].record(stream)
+            evs[1].synchronize()
+            single.append(evs[0].elapsed_time(evs[1]) * 1e3)
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=stream):
+            for _ in range(reps):
+                p.plan.run(*p.ptrs, torch.cuda.current_stream().cuda_stream)
+        g.replay()
+        torch.cuda.synchronize()
+        evs[0].record(stream)
+        for _ in range(5):
+            g.replay()
+        evs[1].record(stream)
+        torch.cuda.synchronize()
+        amort = evs[0].elapsed_time(evs[1]) * 1e3 / (5 * reps)
+    return {"single_launch_median": statistics.median(single), "single_launch_min": min(single),
+            "graph_amortized": amort, "graph_launches": reps, "variant": p.desc["variant"]}
 
 
 def measure_e2e(args, probs, world):

@@ -152,6 +152,9 @@ void* mis_cta_fn(int dtype, int NT, int U, int xm) {
     return dtype == DT_F32 ? mis_cta_fn_f32(NT, U, xm) : mis_cta_fn_i32(NT, U, xm);
 }
 constexpr int64_t kMisMinCols = 16;   // below this a row is one or two vectors: scalar path
+void* tmv_mis_fn(int dtype, int LR, int U) {
+    return dtype == DT_F32 ? tmv_mis_fn_f32(LR, U) : tmv_mis_fn_i32(LR, U);
+}
 void* tmv_fn(int dtype, int LR, int U, bool vec, int NT) {
     return dtype == DT_F32 ? tmv_fn_f32(LR, U, vec, NT) : tmv_fn_i32(LR, U, vec, NT);
 }
@@ -519,7 +522,12 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
     }
 
     // ---- TMV family
-    const int64_t rv1 = p->vec_shape ? R / 4 : R;
+    // R % 4 != 0: the misaligned-row kernel (two aligned loads + funnel shift) keeps the
+    // stream 128-bit over ceil(R/4) output vectors; it handles any B / y alignment, so no
+    // scalar path is planned for these shapes
+    const bool tmis = !p->vec_shape && R >= 8;
+    p->mis = tmis;
+    const int64_t rv1 = p->vec_shape ? R / 4 : tmis ? ceil_div(R, 4) : R;
     int LR = par(ADAPTIC_P_LANES);
     if (LR <= 0) {
         if (v == ADAPTIC_V_TMV_COL) LR = 256;
@@ -532,10 +540,11 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
     if (U <= 0) U = (v == ADAPTIC_V_TMV_COL) ? 8 : 4;
     if (U != 2 && U != 4 && U != 8) return ADAPTIC_ERR_INVALID_ARG;
     int NT = par(ADAPTIC_P_BLOCK);
-    if (NT <= 0) NT = TMV_NT;
+    if (NT <= 0 || tmis) NT = TMV_NT;                      // misaligned kernel: 256 threads
     if ((NT != 256 && NT != 1024) || (NT == 1024 && U > 4)) return ADAPTIC_ERR_INVALID_ARG;
     int cps = par(ADAPTIC_P_CTAS_PER_SM);
-    if (cps <= 0) cps = occupancy(tmv_fn(dt, LR, U, p->vec_shape, NT), NT, 0, dev.present, 2048 / NT);
+    if (cps <= 0) cps = occupancy(tmis ? tmv_mis_fn(dt, LR, U) : tmv_fn(dt, LR, U, p->vec_shape, NT), NT, 0,
+                                  dev.present, 2048 / NT);
     p->lanes = LR; p->unroll = U; p->block = NT; p->ctas_per_sm = cps;
     const int LC = NT / LR;
     const int64_t slots = int64_t(dev.sms) * cps;
@@ -548,8 +557,9 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
     for (;;) {
         bool ok_all = true;
         for (int w = 0; w < 2; ++w) {
-            if (w == 1 && !p->vec_shape) continue;
-            const int64_t rv = w ? R / 4 : R;
+            if (w == 1 && !p->vec_shape && !tmis) continue;
+            if (w == 0 && tmis) continue;
+            const int64_t rv = w ? (tmis ? ceil_div(R, 4) : R / 4) : R;
             const int64_t tiles = ceil_div(rv, LR);
             const int64_t iters = ceil_div(ceil_div(C, S), int64_t(LC) * U);
             p->chain[w] = fold_chain(iters);
@@ -563,9 +573,10 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
     }
     if (S > INT_MAX) return ADAPTIC_ERR_UNSUPPORTED;
     p->splits = int(S);
-    if (!p->path_ok[p->vec_shape ? 1 : 0]) return ADAPTIC_ERR_UNSUPPORTED;
+    if (!p->path_ok[(p->vec_shape || tmis) ? 1 : 0]) return ADAPTIC_ERR_UNSUPPORTED;
     if (S > 1) {
-        const size_t part = ((size_t(R) * size_t(S) * 4 + 255) / 256) * 256;
+        // partials: S x (R, or 4*ceil(R/4) for the misaligned kernel's whole vectors)
+        const size_t part = ((size_t(tmis ? 4 * ceil_div(R, 4) : R) * size_t(S) * 4 + 255) / 256) * 256;
         p->cnt_off = part;
         p->ws_bytes = part + size_t(ceil_div(R, LR)) * 4;    // tiles of the scalar path (the larger)
     }
@@ -743,7 +754,7 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
             args = args9;
             break;
         default:
-            fn = tmv_fn(dt, p->lanes, p->unroll, vec, p->block);
+            fn = mis ? tmv_mis_fn(dt, p->lanes, p->unroll) : tmv_fn(dt, p->lanes, p->unroll, vec, p->block);
             args8[0] = &A; args8[1] = &X; args8[2] = &y; args8[3] = &R; args8[4] = &C;
             args8[5] = &S; args8[6] = &part; args8[7] = &cnt;
             args = args8;
@@ -868,7 +879,7 @@ adaptic_status adaptic_run(adaptic_plan_t p, const void* A, const void* x, void*
     }
     // misaligned-row kernels: any 4-byte aligned A; DOT's b must share A's address modulo 16
     const bool mis = !vec && p->mis &&
-                     (p->op != ADAPTIC_OP_DOT ||
+                     (p->op != ADAPTIC_OP_DOT ||   // TMV / MV: any 4-byte alignment
                       ((reinterpret_cast<uintptr_t>(A) - reinterpret_cast<uintptr_t>(x)) & 15u) == 0);
     if (!p->path_ok[(vec || mis) ? 1 : 0]) return ADAPTIC_ERR_MISALIGNED;   // scalar path would break the error bound
     return launch(p, A, x, y, stream, vec, mis);

@@ -42,6 +42,10 @@ void* mis_group_fn_f32(int G, int U, int xmode);
 void* mis_group_fn_i32(int G, int U, int xmode);
 void* mis_cta_fn_f32(int NT, int U, int xmode);
 void* mis_cta_fn_i32(int NT, int U, int xmode);
+// Misaligned-row TMV (tmv_mis_kernel.cuh; R % 4 != 0, two aligned loads + funnel shift), NT = 256:
+//   (const T* B, const T* X, T* y, int64_t R, int64_t C, int S, T* part, unsigned* cnt)
+void* tmv_mis_fn_f32(int LR, int U);
+void* tmv_mis_fn_i32(int LR, int U);
 
 // BLAS-1 reductions (blas1_kernels.cuh), fp32 input, one translation unit per operator:
 //   b1 group: (const float* A, void* y, int64_t R, int64_t C); rbu 0 = (RB 4, U 2), 1 = (RB 1, U 8)

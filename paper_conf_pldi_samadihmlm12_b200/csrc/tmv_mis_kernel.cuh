@@ -1,0 +1,122 @@
+// tmv_mis_kernel.cuh -- TMV when B's rows are not 16-byte aligned (R % 4 != 0), sm_100a.
+//
+// B is C x R row-major; row c starts at element c*R, so with R % 4 != 0 the
+// 16-byte alignment of a thread's four outputs 4*r4 .. 4*r4+3 shifts from row to
+// row by s_c = (b0 + c*R) mod 4 (b0 = B's own element offset mod 4).  The
+// aligned tmv_kernel cannot be used; the scalar one moves 4 bytes per load and
+// reached only 2.6-5.2 TB/s (profiles/, perturbed sweep).  Here a thread loads
+// the two aligned 128-bit vectors that cover its four elements of row c and
+// selects them by s_c (a funnel shift in registers), so the stream stays 128-bit;
+// the second vector is the neighbouring thread's first, so HBM traffic is
+// unchanged and only L2 sees it twice.  Tiling, splits and the merge are those of
+// tmv_kernel (TMV_COL / TMV_SPLITK / TMV_REGTILE; the paper's restructured-layout
+// kernels).  y and the partials are written per element (y is not
+// 16-byte aligned in general), the last vector of a tile row masked to R.
+#pragma once
+
+#include "tmv_kernels.cuh"
+
+namespace adaptic {
+
+// elements s .. s+3 of the 8-element concatenation (lo, hi), s in 0..3
+template <class V> __device__ __forceinline__ V funnel4(const V& lo, const V& hi, int s) {
+    V r;
+    r.x = s == 0 ? lo.x : s == 1 ? lo.y : s == 2 ? lo.z : lo.w;
+    r.y = s == 0 ? lo.y : s == 1 ? lo.z : s == 2 ? lo.w : hi.x;
+    r.z = s == 0 ? lo.z : s == 1 ? lo.w : s == 2 ? hi.x : hi.y;
+    r.w = s == 0 ? lo.w : s == 1 ? hi.x : s == 2 ? hi.y : hi.z;
+    return r;
+}
+
+template <class T, int LR, int U, int NT>
+__global__ void __launch_bounds__(NT, U <= 2 ? 4 : U <= 4 ? 3 : 2)
+tmv_mis_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restrict__ y,
+               int64_t R, int64_t C, int S, T* __restrict__ ws_part, unsigned int* __restrict__ ws_cnt)
+{
+    pdl_prologue();
+    using E = vec4_t<T>;
+    constexpr int LC = NT / LR;
+    __shared__ E red[LC > 1 ? NT : 1];
+    __shared__ unsigned int flag;
+    const int64_t rv = (R + 3) / 4;                   // output vectors (last one partial)
+    const int64_t ntiles = (rv + LR - 1) / LR;
+    const int64_t chunk = (C + S - 1) / S;
+    // aligned view of B: element e of B is element b0 + e of Ba
+    const int b0 = int((reinterpret_cast<uintptr_t>(B) >> 2) & 3u);
+    const E* __restrict__ Ba = reinterpret_cast<const E*>(B - b0);
+    const int64_t qmax = (b0 + R * C - 1) >> 2;       // last aligned vector holding B data
+    E* __restrict__ pv = reinterpret_cast<E*>(ws_part);
+    const int tid = threadIdx.x;
+    const int lr = tid % LR, lc = tid / LR;
+    const int64_t nblk = ntiles * S;
+
+    for (int64_t blk = blockIdx.x; blk < nblk; blk += gridDim.x) {
+        const int64_t tile = blk % ntiles;
+        const int s = int(blk / ntiles);
+        const int64_t r4 = tile * LR + lr;
+        const bool rok = r4 < rv;
+        const int64_t c0 = int64_t(s) * chunk;
+        const int64_t c1 = min(C, c0 + chunk);
+        const int64_t col = 4 * (rok ? r4 : 0);       // ragged tile: read column 0, discard
+
+        E acc[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) acc[u] = zero_of<E>();
+        E outer = zero_of<E>();
+        int it = 0;
+        int64_t c = c0 + lc;
+        for (; c + int64_t(LC) * (U - 1) < c1; c += int64_t(LC) * U) {
+            E lo[U], hi[U];
+            T xs[U];
+            int sh[U];
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                const int64_t cc = c + int64_t(LC) * u;
+                const int64_t f = b0 + cc * R + col;             // aligned-view element index
+                const int64_t q = f >> 2;
+                sh[u] = int(f & 3);
+                lo[u] = ld_stream(Ba + q);
+                hi[u] = ld_stream(Ba + min(q + 1, qmax));
+                xs[u] = ld_x(X + cc);
+            }
+#pragma unroll
+            for (int u = 0; u < U; ++u) esmac(acc[u], funnel4(lo[u], hi[u], sh[u]), xs[u]);
+            if (++it == FOLD) {
+                it = 0;
+                outer = eadd(outer, tree_sum<U>(acc));
+#pragma unroll
+                for (int u = 0; u < U; ++u) acc[u] = zero_of<E>();
+            }
+        }
+        for (; c < c1; c += LC) {
+            const int64_t f = b0 + c * R + col;
+            const int64_t q = f >> 2;
+            esmac(acc[0], funnel4(ld_stream(Ba + q), ld_stream(Ba + min(q + 1, qmax)), int(f & 3)), ld_x(X + c));
+        }
+        E tot = eadd(outer, tree_sum<U>(acc));
+        tot = lc_combine<NT, LR>(tot, red);
+
+        auto store4 = [&](T* dst, const E& v) {       // the outputs of vector r4 that exist
+            const int64_t r = 4 * r4;
+            dst[r] = v.x;
+            if (r + 1 < R) dst[r + 1] = v.y;
+            if (r + 2 < R) dst[r + 2] = v.z;
+            if (r + 3 < R) dst[r + 3] = v.w;
+        };
+        if (S == 1) {
+            if (tid < LR && rok) store4(y, tot);
+        } else {
+            if (tid < LR && rok) pv[int64_t(s) * rv + r4] = tot;
+            if (ticket_is_last(ws_cnt + tile, unsigned(S), &flag)) {
+                E m = zero_of<E>();
+                if (rok) m = merge_partials<LC>(pv + r4, rv, lc, S);
+                __syncthreads();
+                m = lc_combine<NT, LR>(m, red);
+                if (tid < LR && rok) store4(y, m);
+            }
+        }
+        __syncthreads();
+    }
+}
+
+}  // namespace adaptic

@@ -120,3 +120,46 @@ def test_held_out_shapes_3x2k(k):
             assert np.array_equal(y.astype(np.float64), ref[0]), f"P5 exact {R}x{C}"
         else:
             check(y, ref, dt, f"held-out {R}x{C} {kind} {dt}")
+
+
+TMV_FORCED = [("AUTO", None), ("TMV_COL", [0, 0, 0, 4]), ("TMV_COL", [0, 0, 0, 8])] + \
+             [("TMV_SPLITK", [lr, s, 0, u]) for lr in (1, 4, 32, 256) for s in (0, 3) for u in (2, 8)] + \
+             [("TMV_REGTILE", [0, 0, 0, u]) for u in (2, 4)]
+
+
+@pytest.mark.parametrize("dt", ["f32", "i32"])
+def test_tmv_misaligned_rows_every_variant(dt):
+    """R % 4 != 0: B's rows start at every alignment; two aligned loads + funnel shift."""
+    npdt = np.float32 if dt == "f32" else np.int32
+    shapes = [(9, 33), (13, 1000), (63, 257), (129, 4099), (1023, 65), (5, 100003), (1001, 1001), (30, 7)]
+
+    def case(R, C, v, p):
+        B = synth.matrix(R, C, "tmv", npdt, "uniform", synth.seed(12, "A") + R + C)
+        x = synth.vector(C, npdt, "uniform", synth.seed(12, "x") + C)
+        try:
+            y = adaptic.tmv(torch.from_numpy(B).to(DEV), torch.from_numpy(x).to(DEV), variant=v, params=p)
+        except adaptic.AdapticError as e:
+            assert e.status == L.ERR_UNSUPPORTED, str(e)
+            return
+        check(y.cpu().numpy(), oracle.tmv(B, x), dt, f"tmv {dt} {R}x{C} {v} {p}")
+    _collect([(f"{R}x{C} {v} {p}", lambda R=R, C=C, v=v, p=p: case(R, C, v, p))
+              for (R, C), (v, p) in itertools.product(shapes, TMV_FORCED)])
+
+
+def test_tmv_misaligned_base_and_output():
+    """B and y at every 4-byte offset (the kernel computes B's own offset b0)."""
+    for R, C in [(9, 1000), (61, 333), (1027, 64)]:
+        B = synth.matrix(R, C, "tmv", np.float32, "uniform", 91 + R)
+        x = synth.vector(C, np.float32, "uniform", 92 + C)
+        for off in (1, 2, 3):
+            big = torch.zeros(R * C + 8, dtype=torch.float32, device=DEV)
+            big[off:off + R * C] = torch.from_numpy(B.reshape(-1)).to(DEV)
+            yb = torch.zeros(R + 8, dtype=torch.float32, device=DEV)
+            for v in ("AUTO", "TMV_COL", "TMV_SPLITK", "TMV_REGTILE"):
+                try:
+                    adaptic.tmv(big[off:off + R * C].view(C, R), torch.from_numpy(x).to(DEV), variant=v,
+                                out=yb[off:off + R])
+                except adaptic.AdapticError as e:
+                    assert e.status == L.ERR_UNSUPPORTED
+                    continue
+                check(yb[off:off + R].cpu().numpy(), oracle.tmv(B, x), "f32", f"tmv off {off} {R}x{C} {v}")

@@ -125,6 +125,8 @@ def main():
     ap.add_argument("--perturb", action="store_true",
                     help="also time each diagonal shape with the reduction length (MV/DOT: C+1) or the "
                          "output count (TMV: R+1) off the 128-bit path, for the scalar-shape table cells")
+    ap.add_argument("--perturb-only", action="store_true", help="only the perturbed (off-128-bit-path) shapes")
+    ap.add_argument("--auto-only", action="store_true", help="time only the selector's pick (validation runs)")
     a = ap.parse_args()
     dev = torch.device("cuda:0")
     tdt = torch.float32 if a.dtype == "f32" else torch.int32
@@ -137,7 +139,9 @@ def main():
     for s in filter(None, a.extra.split(",")):
         r, c = s.lower().split("x")
         shapes.append((int(r), int(c)))
-    if a.perturb:
+    if a.perturb_only:
+        shapes = [(R, C, 1) for R, C in shapes]
+    elif a.perturb:
         shapes = [(R, C, p) for R, C in shapes for p in (0, 1)]
     else:
         shapes = [(R, C, 0) for R, C in shapes]
@@ -154,7 +158,7 @@ def main():
                 R, C = (R0 + pert, C0) if op == "tmv" else (R0, C0 + pert)
                 Xp = M.data_ptr() + R * C * 4 if op == "dot" else X.data_ptr()
                 ptrs = (M.data_ptr(), Xp, Y.data_ptr())
-                for variant, params in grids(op, R, C):
+                for variant, params in (grids(op, R, C) if not a.auto_only else [("AUTO", None)]):
                     try:
                         plan = adaptic.get_plan(OPC[op], R, C, dtc, dev, variant, params, stream)
                     except adaptic.AdapticError:
