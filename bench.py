@@ -11,6 +11,8 @@ Workloads (``--workload``):
   dot      (BJ:configs[2]) scalar product N = 1, L = 2^10..2^30 (fp32).
   config0  (BJ:configs[0]) TMV fp32 256 x 256 (L2-resident, launch-latency bound): the
            line adds single-launch and CUDA-graph-amortized latency in microseconds.
+  multi multi-vector MV/TMV, K = 4 vectors per pass over a 256 MiB
+           matrix (horizontal actor integration, adaptic_plan_multi).
   blas1 Sasum / Snrm2 / Isamax / Isamin (the paper's Fig. 9
            CUBLAS benchmarks) on 256 MiB inputs: N x L = 1 x 2^26 .. 2^22 x 16.
 Multi-GPU: one process per GPU (torchrun), barrier + synchronize around the
@@ -44,8 +46,11 @@ def parse():
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", choices=["adaptic", "reference"], default="adaptic")
-    ap.add_argument("--workload", choices=["sweep", "rowshard", "splitk", "dot", "blas1", "config0"], default="sweep")
+    ap.add_argument("--workload", choices=["sweep", "rowshard", "splitk", "dot", "blas1", "config0", "multi"], default="sweep")
     ap.add_argument("--variant", default="AUTO", help="force one variant (fixed-variant sweeps)")
+    ap.add_argument("--streams", type=int, default=1,
+                    help="issue the step's independent problems round-robin on this many CUDA streams "
+                         "(joined by events at the end of every step)")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -153,25 +158,25 @@ B1_OPS = ("asum", "nrm2", "iamax", "iamin", "b1all")
 B1_SHAPES = [(1, 1 << 26), (64, 1 << 20), (4096, 1 << 14), (1 << 16, 1024), (1 << 20, 64), (1 << 22, 16)]
 
 
-def algo_bytes(op, R, C):
-    """What the method must move (SURVEY 8(d)): MV/TMV A + x + y; DOT a + b + y;
-    BLAS-1 a + y."""
+def algo_bytes(op, R, C, nvec=1):
+    """What the method must move: MV/TMV A + x + y (K vectors: A once,
+    K x's and K y's); DOT a + b + y; BLAS-1 a + y."""
     if op == "dot":
         return 4 * (2 * R * C + R)
     if op in B1_OPS:
         return 4 * (R * C + (4 if op == "b1all" else 1) * R)
-    return 4 * (R * C + C + R)
+    return 4 * (R * C + nvec * (C + R))
 
 
 class Problem:
     """One (op, R, C) instance, resident in HBM, with its selected plan."""
 
-    def __init__(self, op, R, C, cfg, variant="AUTO", shard=None, full=None):
+    def __init__(self, op, R, C, cfg, variant="AUTO", shard=None, full=None, nvec=1):
         import torch
         import synth
         import paper_conf_pldi_samadihmlm12_b200 as adaptic
         from paper_conf_pldi_samadihmlm12_b200 import _lib as L
-        self.op, self.R, self.C = op, R, C
+        self.op, self.R, self.C, self.nvec = op, R, C, nvec
         dev = torch.device("cuda", torch.cuda.current_device())
         Rf, Cf = full if full else (R, C)           # logical full problem (shards are slices)
         rows, cols = shard if shard else ((0, R), (0, C))
@@ -184,22 +189,22 @@ class Problem:
             self.X = torch.empty(R * C, dtype=torch.float32, device=dev)
             synth.device_matrix(self.X, Rf, Cf, "mv", "uniform", synth.seed(cfg, "b"), rows=rows, cols=cols)
         else:
-            self.X = torch.empty(C, dtype=torch.float32, device=dev)
+            self.X = torch.empty(C * nvec, dtype=torch.float32, device=dev)
             synth.device_vector(self.X, "uniform", synth.seed(cfg, "x"), start=cols[0])
-        self.y = torch.empty(R * (4 if op == "b1all" else 1),
+        self.y = torch.empty(R * (4 if op == "b1all" else nvec),
                              dtype=torch.int32 if op in ("iamax", "iamin") else torch.float32, device=dev)
         opc = L.OPS[op]
         self.stream = torch.cuda.current_stream().cuda_stream
-        self.plan = adaptic.get_plan(opc, R, C, L.F32, dev, variant, None, self.stream)
+        self.plan = adaptic.get_plan(opc, R, C, L.F32, dev, variant, None, self.stream, nvec)
         self.desc = self.plan.describe()
-        self.bytes = algo_bytes(op, R, C)
+        self.bytes = algo_bytes(op, R, C, nvec)
         self.ptrs = (self.M.data_ptr(), self.X.data_ptr(), self.y.data_ptr())
 
     def launch(self):
         self.plan.run(*self.ptrs, self.stream)
 
     def key(self):
-        return f"{self.op}:{self.R}x{self.C}:{self.desc['variant']}"
+        return f"{self.op}{'' if self.nvec == 1 else 'x%d' % self.nvec}:{self.R}x{self.C}:{self.desc['variant']}"
 
 
 def build_problems(args, world, rank):
@@ -208,6 +213,11 @@ def build_problems(args, world, rank):
                 for k in range(3, 24) for op in ("mv", "tmv")], \
             {"workload": "configs[1]: TMV/MV fp32 shape sweep at 256 MiB, 8Mx8 .. 8192x8192 .. 8x8M, "
                          "both layouts, variant selector", "shapes": 42, "per_gpu": "full sweep (weak)"}
+    if args.workload == "multi":
+        shapes = [(8192, 8192), (65536, 1024), (1 << 20, 64), (64, 1 << 20)]
+        return [Problem(op, R, C, 8, args.variant, nvec=4) for R, C in shapes for op in ("mv", "tmv")], \
+            {"workload": "SURVEY 8(f)#2: multi-vector MV/TMV fp32, K=4 vectors per pass, 256 MiB matrices "
+                         "(8192^2, 65536x1024, 1Mx64, 64x1M)", "shapes": 8, "nvec": 4}
     if args.workload == "config0":
         return [Problem("tmv", 256, 256, 0, args.variant)], \
             {"workload": "configs[0]: TMV fp32 256x256 (L2-resident; latency-bound)", "shapes": 1}
@@ -242,13 +252,37 @@ def run_adaptic(args):
     n = len(probs)
     step_bytes = sum(p.bytes for p in probs)
 
+    # optional multi-stream issue: problem i on stream i % streams; each side stream's
+    # problems get their own plan (and so their own workspace)
+    main = torch.cuda.current_stream()
+    side = [torch.cuda.Stream() for _ in range(max(1, args.streams) - 1)]
+    if side:
+        import paper_conf_pldi_samadihmlm12_b200 as adaptic
+        from paper_conf_pldi_samadihmlm12_b200 import _lib as L
+        for i, p in enumerate(probs):
+            k = i % (len(side) + 1)
+            if k:
+                p.stream = side[k - 1].cuda_stream
+                p.plan = adaptic.get_plan(L.OPS[p.op], p.R, p.C, L.F32, torch.device("cuda", torch.cuda.current_device()),
+                                          args.variant, None, p.stream)
+    fork = torch.cuda.Event()
+    joins = [torch.cuda.Event() for _ in side]
+
     def one_step(evs=None):
+        if side and evs is None:
+            fork.record(main)
+            for st in side:
+                st.wait_event(fork)
         for i, p in enumerate(probs):
             if evs is not None:
                 evs[i].record()
             p.launch()
         if evs is not None:
             evs[n].record()
+        if side and evs is None:
+            for st, ev in zip(side, joins):
+                ev.record(st)
+                main.wait_event(ev)
         if splitk:
             dist.all_reduce(probs[0].y, op=dist.ReduceOp.SUM)
 
@@ -292,8 +326,8 @@ def run_adaptic(args):
             ds = []
             for s in range(kev_steps):
                 evs[s][0].record()
-                for _ in range(batch):
-                    p.launch()
+                for _ in range(batch):       # on the events' (main) stream, whatever --streams says
+                    p.plan.run(*p.ptrs, main.cuda_stream)
                 evs[s][1].record()
             torch.cuda.synchronize()
             for s in range(kev_steps):
@@ -352,7 +386,7 @@ def run_adaptic(args):
                 "kernel_timing": ("per-launch CUDA events inside the timed region" if inner else
                                   f"per-kernel CUDA events after the timed region: each kernel 5x back to back, "
                                   f"{kev_steps} samples (the timed region itself has events only at its ends)"),
-                "kernel_sum_ms": kernel_sum_ms, "latency_us": latency,
+                "kernel_sum_ms": kernel_sum_ms, "latency_us": latency, "streams": max(1, args.streams),
                 "gpu_launches": n * args.steps, "clocks": clk,
                 "selected": {q["op"] + f" {q['R']}x{q['C']}": [q["variant"], round(q["frac"], 3)] for q in per}}
         print(json.dumps(line), flush=True)
@@ -452,9 +486,11 @@ def cpu_baseline(probs, args, budget_s: float = 20.0):
         X = p.X.cpu().numpy()
         t = time.perf_counter()
         if p.op == "mv":
-            oracle.mv(M.reshape(p.R, p.C), X)
+            for j in range(p.nvec):
+                oracle.mv(M.reshape(p.R, p.C), X[j * p.C:(j + 1) * p.C])
         elif p.op == "tmv":
-            oracle.tmv(M.reshape(p.C, p.R), X)
+            for j in range(p.nvec):
+                oracle.tmv(M.reshape(p.C, p.R), X[j * p.C:(j + 1) * p.C])
         elif p.op in B1_OPS:
             for f in (("asum", "nrm2", "iamax", "iamin") if p.op == "b1all" else (p.op,)):
                 getattr(oracle, f)(M.reshape(p.R, p.C))

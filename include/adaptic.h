@@ -122,7 +122,7 @@
 extern "C" {
 #endif
 
-#define ADAPTIC_ABI_VERSION 2
+#define ADAPTIC_ABI_VERSION 3
 
 typedef enum {
     ADAPTIC_OK = 0,
@@ -214,6 +214,24 @@ adaptic_status adaptic_plan(adaptic_op op, int64_t rows, int64_t cols, adaptic_d
 adaptic_status adaptic_plan_forced(adaptic_op op, int64_t rows, int64_t cols,
                                    adaptic_dtype dtype, adaptic_variant variant,
                                    const int32_t* params, adaptic_plan_t* out);
+
+/* Multi-vector form: Y = A [x_0 ... x_{K-1}] (op = ADAPTIC_OP_MV) or
+ * Y = B^T [x_0 ... x_{K-1}] (op = ADAPTIC_OP_TMV) with K = nvec vectors sharing ONE
+ * pass over the matrix -- the paper's horizontal actor integration (actors
+ * "working on the same data" run as one kernel, so "off-chip memory accesses and
+ * synchronizations only happen once").  nvec in {1, 2, 4, 8} (1 = adaptic_plan /
+ * adaptic_plan_forced; other counts -> UNSUPPORTED: split them into these sizes);
+ * fp32 only.  adaptic_run then takes x = X, a K x C row-major array (vector j at
+ * X + j*C), and y = Y, a K x R row-major array (Y + j*R = A x_j); results equal K
+ * separate calls up to rounding (same 1e-4 bound; one accumulator per vector folded
+ * every FOLD/U steps).  Variants: MV_SUBWARP / MV_WPR (rows of at most G*U loads,
+ * x held in registers), MV_CPR / MV_SPLIT (8/K rows per CTA share each x load),
+ * TMV_COL / TMV_SPLITK / TMV_REGTILE; variant = ADAPTIC_V_AUTO selects (params
+ * ignored).  A 128-bit-shape lane-group plan run on pointers that are not 16-byte
+ * aligned returns ADAPTIC_ERR_MISALIGNED. */
+adaptic_status adaptic_plan_multi(adaptic_op op, int64_t rows, int64_t cols, int32_t nvec,
+                                  adaptic_dtype dtype, adaptic_variant variant,
+                                  const int32_t* params, adaptic_plan_t* out);
 
 /* What the plan will run. */
 adaptic_variant adaptic_plan_variant(adaptic_plan_t plan);

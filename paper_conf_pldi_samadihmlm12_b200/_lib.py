@@ -30,7 +30,7 @@ TMV_VARIANTS = ("TMV_COL", "TMV_SPLITK", "TMV_REGTILE")
 P_LANES, P_SPLITS, P_CTAS_PER_SM, P_UNROLL, P_XSMEM, P_BLOCK, P_ROWS, P_ORDER, P_PIPE, NPARAMS = 0, 1, 2, 3, 4, 5, 6, 7, 8, 9
 
 # every symbol the header declares (tests check they are all exported)
-SYMBOLS = ("adaptic_plan", "adaptic_plan_forced", "adaptic_plan_variant", "adaptic_plan_describe",
+SYMBOLS = ("adaptic_plan", "adaptic_plan_forced", "adaptic_plan_multi", "adaptic_plan_variant", "adaptic_plan_describe",
            "adaptic_plan_workspace_bytes", "adaptic_plan_set_workspace", "adaptic_run",
            "adaptic_run_host", "adaptic_plan_destroy", "adaptic_status_string",
            "adaptic_variant_name", "adaptic_last_cuda_error", "adaptic_abi_version")
@@ -67,6 +67,9 @@ def lib():
         L.adaptic_plan_forced.argtypes = [i32, i64, i64, i32, i32, ctypes.POINTER(ctypes.c_int32),
                                           ctypes.POINTER(vp)]
         L.adaptic_plan_forced.restype = i32
+        L.adaptic_plan_multi.argtypes = [i32, i64, i64, ctypes.c_int32, i32, i32, ctypes.POINTER(ctypes.c_int32),
+                                         ctypes.POINTER(vp)]
+        L.adaptic_plan_multi.restype = i32
         L.adaptic_plan_variant.argtypes = [vp]
         L.adaptic_plan_variant.restype = i32
         L.adaptic_plan_describe.argtypes = [vp, ctypes.c_char_p, ctypes.c_size_t]
@@ -101,11 +104,17 @@ def _check(status: int, where: str):
 class Plan:
     """An ``adaptic_plan_t`` (selector output).  ``variant='AUTO'`` runs the selector."""
 
-    def __init__(self, op: int, rows: int, cols: int, dtype: int, variant="AUTO", params=None):
+    def __init__(self, op: int, rows: int, cols: int, dtype: int, variant="AUTO", params=None, nvec: int = 1):
         L = lib()
         h = ctypes.c_void_p()
         v = V[variant] if isinstance(variant, str) else int(variant)
-        if v == 0 and params is None:
+        if nvec != 1:
+            arr = None
+            if params is not None:
+                vals = list(params) + [0] * (NPARAMS - len(params))
+                arr = (ctypes.c_int32 * NPARAMS)(*vals)
+            st = L.adaptic_plan_multi(op, int(rows), int(cols), int(nvec), dtype, v, arr, ctypes.byref(h))
+        elif v == 0 and params is None:
             st = L.adaptic_plan(op, int(rows), int(cols), dtype, ctypes.byref(h))
         else:
             arr = None
@@ -115,7 +124,7 @@ class Plan:
             st = L.adaptic_plan_forced(op, int(rows), int(cols), dtype, v, arr, ctypes.byref(h))
         _check(st, f"adaptic_plan({op},{rows},{cols},{dtype},{variant})")
         self._h = h
-        self.op, self.rows, self.cols, self.dtype = op, int(rows), int(cols), dtype
+        self.op, self.rows, self.cols, self.dtype, self.nvec = op, int(rows), int(cols), dtype, int(nvec)
 
     @property
     def handle(self):

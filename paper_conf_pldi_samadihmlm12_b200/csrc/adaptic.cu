@@ -26,6 +26,7 @@ using namespace adaptic;
 
 struct adaptic_plan_s {
     int op, dtype;
+    int nvec;              // vectors per call: 1, or K in {2, 4, 8} (adaptic_plan_multi)
     int64_t R, C;
     int variant;
     int source;            // 0 forced, 1 table, 2 heuristic
@@ -268,6 +269,131 @@ const TableEntry* table_lookup(int op, int dtype, int64_t R, int64_t C, bool* pr
     return nullptr;
 }
 
+// Multi-vector MV / TMV (adaptic_plan_multi): K = nvec vectors share one pass over the
+// matrix (horizontal actor integration; mmv_kernels.cuh).  fp32, 128-bit path
+// shapes and scalar shapes alike (aligned pointers take the 128-bit instances).
+adaptic_status derive_multi(adaptic_plan_s* p, const int32_t* params, const DevInfo& dev) {
+    const int op = p->op, v = p->variant, K = p->nvec;
+    const int64_t R = p->R, C = p->C;
+    auto par = [&](int i) -> int { return params ? params[i] : 0; };
+    p->vec_shape = (op == ADAPTIC_OP_TMV) ? (R % 4 == 0) : (C % 4 == 0);
+    p->mis = false; p->splits = 1; p->smem = 0; p->stages = 0; p->xmode = 0; p->ilv = 0; p->pipe = 0; p->rb = 1;
+    p->fb_lanes = 0; p->fb_unroll = 0; p->ws_bytes = 0; p->cnt_off = 0;
+    for (int w = 0; w < 2; ++w) { p->grid[w] = 0; p->chain[w] = 0; p->depth[w] = 0; p->path_ok[w] = false; }
+    auto chain_of = [&](int64_t iters, int U) -> int64_t {
+        const int64_t f = FOLD / U;
+        return int64_t(U) * std::min<int64_t>(iters, f) + iters / f;
+    };
+    if (op == ADAPTIC_OP_MV && (v == ADAPTIC_V_MV_SUBWARP || v == ADAPTIC_V_MV_WPR)) {
+        // short rows, x in registers: each lane covers <= U vectors of a row.  Only the
+        // plan's own load path is planned (G and U depend on the row length in loads),
+        // so a 128-bit-shape plan run on misaligned pointers reports MISALIGNED.
+        {
+            const int w = p->vec_shape ? 1 : 0;
+            const int64_t nv = w ? C / 4 : C;
+            int U = par(ADAPTIC_P_UNROLL);
+            int G = (v == ADAPTIC_V_MV_WPR) ? 32 : par(ADAPTIC_P_LANES);
+            if (U <= 0) U = (K == 8 || nv > 64) ? 2 : 4;
+            if (G <= 0) G = clampi(pow2_ceil(ceil_div(std::max<int64_t>(1, nv), U)), 1, 32);
+            if (G < 1 || G > 32 || (G & (G - 1)) || (U != 1 && U != 2 && U != 4) || K * U > 16)
+                return ADAPTIC_ERR_INVALID_ARG;
+            if (nv > int64_t(G) * U) return ADAPTIC_ERR_UNSUPPORTED;       // row longer than one step
+            p->lanes = G; p->unroll = U; p->block = GROUP_NT; p->rb = MMV_GROUP_RB;
+            int cps = par(ADAPTIC_P_CTAS_PER_SM);
+            if (cps <= 0) cps = occupancy(mmv_group_fn(K, G, U, w == 1), GROUP_NT, 0, dev.present, 4);
+            p->ctas_per_sm = cps;
+            const int rows_per_cta = MMV_GROUP_RB * (32 / G) * (GROUP_NT / 32);
+            p->grid[w] = std::max<int64_t>(1, std::min<int64_t>(ceil_div(R, rows_per_cta), int64_t(dev.sms) * cps));
+            p->chain[w] = U;
+            p->depth[w] = (w ? 2 : 0) + ilog2c(G) + 1;
+            p->path_ok[w] = bound_ok(p->chain[w] + p->depth[w]);
+        }
+        return p->path_ok[p->vec_shape ? 1 : 0] ? ADAPTIC_OK : ADAPTIC_ERR_UNSUPPORTED;
+    }
+    if (op == ADAPTIC_OP_MV && (v == ADAPTIC_V_MV_CPR || v == ADAPTIC_V_MV_SPLIT)) {
+        const int NT = 256, RB = 8 / K;
+        int U = par(ADAPTIC_P_UNROLL);
+        if (U <= 0) U = 2;
+        if (U != 1 && U != 2) return ADAPTIC_ERR_INVALID_ARG;
+        int cps = par(ADAPTIC_P_CTAS_PER_SM);
+        if (cps <= 0) cps = occupancy(mmv_cta_fn(K, U, p->vec_shape), NT, 0, dev.present, 2048 / NT);
+        p->lanes = NT; p->unroll = U; p->block = NT; p->rb = RB; p->ctas_per_sm = cps;
+        const int64_t slots = int64_t(dev.sms) * cps;
+        const int64_t groups = ceil_div(R, RB);
+        const int64_t nv1 = p->vec_shape ? C / 4 : C;
+        int64_t S = 1;
+        if (v == ADAPTIC_V_MV_SPLIT)
+            S = par(ADAPTIC_P_SPLITS) > 0 ? par(ADAPTIC_P_SPLITS)
+                                          : pick_splits(groups, slots, std::max<int64_t>(2, ceil_div(nv1, int64_t(NT) * U)), 2);
+        for (;;) {
+            bool ok_all = true;
+            for (int w = 0; w < 2; ++w) {
+                if (w == 1 && !p->vec_shape) continue;
+                const int64_t nv = w ? C / 4 : C;
+                const int64_t iters = ceil_div(nv, int64_t(S) * NT * U);
+                p->chain[w] = chain_of(iters, U);
+                p->depth[w] = (w ? 2 : 0) + ilog2c(NT) + (S > 1 ? ceil_div(S, NT) + ilog2c(NT) : 0) + 1;
+                p->path_ok[w] = bound_ok(p->chain[w] + p->depth[w]);
+                p->grid[w] = std::max<int64_t>(1, std::min<int64_t>(groups * S, slots));
+                if (!p->path_ok[w]) ok_all = false;
+            }
+            if (ok_all || v == ADAPTIC_V_MV_CPR || S >= (int64_t(1) << 20)) break;
+            S *= 2;
+        }
+        if (S > INT_MAX) return ADAPTIC_ERR_UNSUPPORTED;
+        p->splits = int(S);
+        p->ilv = S > 1 ? 1 : 0;
+        if (!p->path_ok[p->vec_shape ? 1 : 0]) return ADAPTIC_ERR_UNSUPPORTED;
+        if (S > 1) {
+            const size_t part = ((size_t(R) * size_t(K) * size_t(S) * 4 + 255) / 256) * 256;
+            p->cnt_off = part;
+            p->ws_bytes = part + size_t(groups) * 4;
+        }
+        return ADAPTIC_OK;
+    }
+    if (op != ADAPTIC_OP_TMV || !is_tmv_family(v)) return ADAPTIC_ERR_UNSUPPORTED;
+    // TMV tiles: LR output vectors x (256 / LR) c-lanes, S c-ranges
+    const int NT = 256, U = 2;
+    const int64_t rv1 = p->vec_shape ? R / 4 : R;
+    int LR = par(ADAPTIC_P_LANES);
+    if (LR <= 0) LR = (v == ADAPTIC_V_TMV_COL) ? 256 : (v == ADAPTIC_V_TMV_REGTILE) ? clampi(pow2_ceil(rv1), 1, 256)
+                                                                                  : clampi(pow2_ceil(rv1), 1, 64);
+    if (LR < 1 || LR > 256 || (LR & (LR - 1))) return ADAPTIC_ERR_INVALID_ARG;
+    if (v == ADAPTIC_V_TMV_REGTILE && rv1 > LR) return ADAPTIC_ERR_UNSUPPORTED;
+    int cps = par(ADAPTIC_P_CTAS_PER_SM);
+    if (cps <= 0) cps = occupancy(tmmv_fn(K, LR, p->vec_shape), NT, 0, dev.present, 2048 / NT);
+    p->lanes = LR; p->unroll = U; p->block = NT; p->ctas_per_sm = cps;
+    const int LC = NT / LR;
+    const int64_t slots = int64_t(dev.sms) * cps;
+    int64_t S = 1;
+    if (par(ADAPTIC_P_SPLITS) > 0) S = par(ADAPTIC_P_SPLITS);
+    else if (v != ADAPTIC_V_TMV_COL) S = pick_splits(ceil_div(rv1, LR), slots, std::max<int64_t>(1, ceil_div(C, int64_t(LC) * U)), 1);
+    for (;;) {
+        bool ok_all = true;
+        for (int w = 0; w < 2; ++w) {
+            if (w == 1 && !p->vec_shape) continue;
+            const int64_t rv = w ? R / 4 : R;
+            const int64_t iters = ceil_div(ceil_div(C, S), int64_t(LC) * U);
+            p->chain[w] = chain_of(iters, U);
+            p->depth[w] = ilog2c(LC) + (S > 1 ? ceil_div(S, LC) + ilog2c(LC) : 0) + 1;
+            p->path_ok[w] = bound_ok(p->chain[w] + p->depth[w]);
+            p->grid[w] = std::max<int64_t>(1, std::min<int64_t>(ceil_div(rv, LR) * S, slots));
+            if (!p->path_ok[w]) ok_all = false;
+        }
+        if (ok_all || S >= (int64_t(1) << 20)) break;
+        S *= 2;
+    }
+    if (S > INT_MAX) return ADAPTIC_ERR_UNSUPPORTED;
+    p->splits = int(S);
+    if (!p->path_ok[p->vec_shape ? 1 : 0]) return ADAPTIC_ERR_UNSUPPORTED;
+    if (S > 1) {
+        const size_t part = ((size_t(R) * size_t(K) * size_t(S) * 4 + 255) / 256) * 256;
+        p->cnt_off = part;
+        p->ws_bytes = part + size_t(ceil_div(R, LR)) * 4;
+    }
+    return ADAPTIC_OK;
+}
+
 // BLAS-1 reductions (ASUM/NRM2/IAMAX/IAMIN): the MV-family thread shapes with an
 // operator policy (blas1_kernels.cuh).  Only ASUM has fp32 chains to bound; NRM2
 // accumulates in fp64 and IAMAX/IAMIN are exact.
@@ -363,6 +489,7 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
     auto par = [&](int i) -> int { return params ? params[i] : 0; };
     const int v = p->variant;
     if (!op_has_variant(op, v)) return ADAPTIC_ERR_UNSUPPORTED;
+    if (p->nvec > 1) return derive_multi(p, params, dev);
     if (is_b1_op(op)) return derive_b1(p, params, dev);
 
     p->vec_shape = (op == ADAPTIC_OP_TMV) ? (R % 4 == 0) : (C % 4 == 0);
@@ -595,16 +722,20 @@ adaptic_status validate_shape(int op, int64_t rows, int64_t cols, int dtype) {
 }
 
 adaptic_status make_plan(int op, int64_t rows, int64_t cols, int dtype, int variant,
-                         const int32_t* params, adaptic_plan_t* out) {
+                         const int32_t* params, adaptic_plan_t* out, int nvec = 1) {
     if (!out) return ADAPTIC_ERR_INVALID_ARG;
     *out = nullptr;
     adaptic_status st = validate_shape(op, rows, cols, dtype);
     if (st != ADAPTIC_OK) return st;
+    if (nvec != 1 && nvec != 2 && nvec != 4 && nvec != 8) return nvec < 1 ? ADAPTIC_ERR_INVALID_ARG : ADAPTIC_ERR_UNSUPPORTED;
+    if (nvec > 1 && (dtype != ADAPTIC_F32 || (op != ADAPTIC_OP_MV && op != ADAPTIC_OP_TMV))) return ADAPTIC_ERR_UNSUPPORTED;
+    if (nvec > 1 && (rows > (int64_t(1) << 62) / 4 / nvec || cols > (int64_t(1) << 62) / 4 / nvec))
+        return ADAPTIC_ERR_INVALID_ARG;
     if (variant < ADAPTIC_V_AUTO || variant >= ADAPTIC_V_COUNT) return ADAPTIC_ERR_INVALID_ARG;
     const DevInfo dev = device_info();
     adaptic_plan_s* p = new (std::nothrow) adaptic_plan_s();
     if (!p) return ADAPTIC_ERR_INVALID_ARG;
-    p->op = op; p->dtype = dtype; p->R = rows; p->C = cols; p->sms = dev.sms;
+    p->op = op; p->dtype = dtype; p->R = rows; p->C = cols; p->sms = dev.sms; p->nvec = nvec;
     p->ws = nullptr; p->ws_cap = 0;
 
     if (variant != ADAPTIC_V_AUTO) {
@@ -618,6 +749,22 @@ adaptic_status make_plan(int op, int64_t rows, int64_t cols, int dtype, int vari
     if (rows == 0 || cols == 0) {      // nothing to select: run() is a no-op / memset
         p->variant = heuristic_variant(op, std::max<int64_t>(rows, 1), std::max<int64_t>(cols, 1), dev.sms);
         p->source = 2;
+        *out = p;
+        return ADAPTIC_OK;
+    }
+    if (nvec > 1) {                    // multi-vector: the regime rules of the paper (Fig. 1)
+        const int64_t nv = (cols % 4 == 0) ? cols / 4 : cols;
+        if (op == ADAPTIC_OP_TMV) p->variant = heuristic_variant(op, rows, cols, dev.sms);
+        else if (nv <= 32 * (nvec == 8 ? 2 : 4)) p->variant = ADAPTIC_V_MV_SUBWARP;
+        else if (rows >= 4 * int64_t(dev.sms)) p->variant = ADAPTIC_V_MV_CPR;
+        else p->variant = ADAPTIC_V_MV_SPLIT;
+        p->source = 2;
+        st = derive(p, nullptr, dev);
+        if (st != ADAPTIC_OK) {
+            p->variant = (op == ADAPTIC_OP_TMV) ? ADAPTIC_V_TMV_SPLITK : ADAPTIC_V_MV_SPLIT;
+            st = derive(p, nullptr, dev);
+        }
+        if (st != ADAPTIC_OK) { delete p; return st; }
         *out = p;
         return ADAPTIC_OK;
     }
@@ -710,7 +857,20 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
     int stages = p->stages;
 
     void* args7[7];
-    if (is_b1_op(p->op)) {
+    if (p->nvec > 1) {
+        const int K = p->nvec;
+        if (p->op == ADAPTIC_OP_TMV) fn = tmmv_fn(K, p->lanes, vec);
+        else if (p->variant == ADAPTIC_V_MV_SUBWARP || p->variant == ADAPTIC_V_MV_WPR) fn = mmv_group_fn(K, p->lanes, p->unroll, vec);
+        else fn = mmv_cta_fn(K, p->unroll, vec);
+        if (p->op == ADAPTIC_OP_MV && (p->variant == ADAPTIC_V_MV_SUBWARP || p->variant == ADAPTIC_V_MV_WPR)) {
+            args6[0] = &A; args6[1] = &X; args6[2] = &y; args6[3] = &R; args6[4] = &C;
+            args = args6;
+        } else {
+            args8[0] = &A; args8[1] = &X; args8[2] = &y; args8[3] = &R; args8[4] = &C;
+            args8[5] = &S; args8[6] = &part; args8[7] = &cnt;
+            args = args8;
+        }
+    } else if (is_b1_op(p->op)) {
         if (p->variant == ADAPTIC_V_MV_SUBWARP || p->variant == ADAPTIC_V_MV_WPR) {
             fn = b1_group_fn(p->op, p->lanes, p->rb == 1 ? 1 : 0, vec);
             args6[0] = &A; args6[1] = &y; args6[2] = &R; args6[3] = &C;
@@ -792,9 +952,9 @@ adaptic_status check_run(const adaptic_plan_s* p, const void* A, const void* x, 
     const bool b1 = is_b1_op(p->op);          // BLAS-1: x is unused (may be NULL)
     if (!A || (!x && !b1)) return ADAPTIC_ERR_INVALID_ARG;
     if (!aligned(A, 4) || (!b1 && !aligned(x, 4))) return ADAPTIC_ERR_MISALIGNED;
-    const size_t ybytes = size_t(p->R) * y_bytes_per_row(p->op);
+    const size_t ybytes = size_t(p->R) * y_bytes_per_row(p->op) * size_t(p->nvec);
     const size_t abytes = size_t(p->R) * size_t(p->C) * 4;
-    const size_t xbytes = b1 ? 0 : (p->op == ADAPTIC_OP_DOT ? abytes : size_t(p->C) * 4);
+    const size_t xbytes = b1 ? 0 : (p->op == ADAPTIC_OP_DOT ? abytes : size_t(p->C) * 4 * size_t(p->nvec));
     if (overlap(y, ybytes, A, abytes) || (!b1 && overlap(y, ybytes, x, xbytes))) return ADAPTIC_ERR_ALIAS;
     if (p->ws_bytes > 0 && (p->ws == nullptr || p->ws_cap < p->ws_bytes)) return ADAPTIC_ERR_NO_WORKSPACE;
     return ADAPTIC_OK;
@@ -814,6 +974,11 @@ adaptic_status adaptic_plan_forced(adaptic_op op, int64_t rows, int64_t cols, ad
                                    adaptic_variant variant, const int32_t* params, adaptic_plan_t* out) {
     if (variant == ADAPTIC_V_AUTO) return make_plan(op, rows, cols, dtype, ADAPTIC_V_AUTO, nullptr, out);
     return make_plan(op, rows, cols, dtype, variant, params, out);
+}
+
+adaptic_status adaptic_plan_multi(adaptic_op op, int64_t rows, int64_t cols, int32_t nvec, adaptic_dtype dtype,
+                                  adaptic_variant variant, const int32_t* params, adaptic_plan_t* out) {
+    return make_plan(op, rows, cols, dtype, variant, variant == ADAPTIC_V_AUTO ? nullptr : params, out, nvec);
 }
 
 adaptic_variant adaptic_plan_variant(adaptic_plan_t plan) {
@@ -843,12 +1008,12 @@ int adaptic_plan_describe(adaptic_plan_t p, char* buf, size_t cap) {
     const int n = std::snprintf(
         tmp, sizeof(tmp),
         "{\"op\":\"%s\",\"dtype\":\"%s\",\"rows\":%lld,\"cols\":%lld,\"variant\":\"%s\",\"source\":\"%s\","
-        "\"sms\":%d,\"lanes\":%d,\"unroll\":%d,\"rows_per_group\":%d,\"splits\":%d,\"block\":%d,"
+        "\"nvec\":%d,\"sms\":%d,\"lanes\":%d,\"unroll\":%d,\"rows_per_group\":%d,\"splits\":%d,\"block\":%d,"
         "\"ctas_per_sm\":%d,\"stages\":%d,\"xmode\":%d,\"ilv\":%d,\"pipe\":%d,\"smem\":%zu,\"vec_shape\":%s,\"mis\":%s,"
         "\"grid\":[%lld,%lld],\"chain\":[%lld,%lld],\"depth\":[%lld,%lld],\"path_ok\":[%s,%s],"
         "\"fallback_lanes\":%d,\"fallback_unroll\":%d,\"workspace_bytes\":%zu}",
         ops[p->op], p->dtype == ADAPTIC_F32 ? "f32" : "i32", (long long)p->R, (long long)p->C,
-        kVariantNames[p->variant], src[p->source], p->sms, p->lanes, p->unroll, p->rb, p->splits, p->block,
+        kVariantNames[p->variant], src[p->source], p->nvec, p->sms, p->lanes, p->unroll, p->rb, p->splits, p->block,
         p->ctas_per_sm, p->stages, p->xmode, p->ilv, p->pipe, p->smem, p->vec_shape ? "true" : "false",
         p->mis ? "true" : "false",
         (long long)p->grid[0], (long long)p->grid[1], (long long)p->chain[0], (long long)p->chain[1],
@@ -868,11 +1033,13 @@ adaptic_status adaptic_run(adaptic_plan_t p, const void* A, const void* x, void*
     adaptic_status st = check_run(p, A, x, y);
     if (st != ADAPTIC_OK || p->R == 0) return st;
     if (p->C == 0) {
-        cudaError_t e = cudaMemsetAsync(y, 0, size_t(p->R) * y_bytes_per_row(p->op), stream);
+        cudaError_t e = cudaMemsetAsync(y, 0, size_t(p->R) * y_bytes_per_row(p->op) * size_t(p->nvec), stream);
         return e == cudaSuccess ? ADAPTIC_OK : cuda_fail(e);
     }
     bool vec = p->vec_shape;
-    if (vec) {
+    if (vec && p->nvec > 1) {
+        vec = aligned(A, 16) && aligned(x, 16) && aligned(y, 16);
+    } else if (vec) {
         if (p->op == ADAPTIC_OP_TMV) vec = aligned(A, 16) && aligned(y, 16);
         else if (is_b1_op(p->op)) vec = aligned(A, 16);
         else vec = aligned(A, 16) && aligned(x, 16);
@@ -895,7 +1062,7 @@ adaptic_status adaptic_run_host(adaptic_plan_t p, const void* A_host, const void
     adaptic_status st = check_run(p, dA, dx, dy);
     if (st != ADAPTIC_OK) return st;
     const size_t abytes = size_t(p->R) * size_t(p->C) * 4;
-    const size_t xbytes = (p->op == ADAPTIC_OP_DOT ? abytes : size_t(p->C) * 4);
+    const size_t xbytes = (p->op == ADAPTIC_OP_DOT ? abytes : size_t(p->C) * 4 * size_t(p->nvec));
     cudaError_t e;
     if (p->C > 0) {
         if (!b1 && (e = cudaMemcpyAsync(dx, x_host, xbytes, cudaMemcpyHostToDevice, stream)) != cudaSuccess)
@@ -904,7 +1071,8 @@ adaptic_status adaptic_run_host(adaptic_plan_t p, const void* A_host, const void
     }
     st = adaptic_run(p, dA, dx, dy, stream_);
     if (st != ADAPTIC_OK) return st;
-    if ((e = cudaMemcpyAsync(y_host, dy, size_t(p->R) * y_bytes_per_row(p->op), cudaMemcpyDeviceToHost, stream)) !=
+    if ((e = cudaMemcpyAsync(y_host, dy, size_t(p->R) * y_bytes_per_row(p->op) * size_t(p->nvec), cudaMemcpyDeviceToHost,
+                             stream)) !=
         cudaSuccess)
         return cuda_fail(e);
     return ADAPTIC_OK;

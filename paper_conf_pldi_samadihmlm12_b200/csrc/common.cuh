@@ -72,6 +72,20 @@ __device__ __forceinline__ uint32_t ld_stream(const uint32_t* p) {
     asm("ld.global.nc.L1::no_allocate.L2::128B.u32 %0, [%1];" : "=r"(v) : "l"(p));
     return v;
 }
+// Matrix stream whose 16-byte chunks are read twice by neighbouring lanes (the
+// misaligned TMV funnel): allocate in L1 so the second read is an L1 hit.
+__device__ __forceinline__ float4 ld_stream_l1(const float4* p) {
+    float4 v;
+    asm("ld.global.nc.L2::256B.v4.f32 {%0,%1,%2,%3}, [%4];"
+        : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p));
+    return v;
+}
+__device__ __forceinline__ uint4 ld_stream_l1(const uint4* p) {
+    uint4 v;
+    asm("ld.global.nc.L2::256B.v4.u32 {%0,%1,%2,%3}, [%4];"
+        : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
+    return v;
+}
 // x (re-read by many rows / CTAs): read-only path, cached in L1 and L2.
 __device__ __forceinline__ float4 ld_x(const float4* p) { return __ldg(p); }
 __device__ __forceinline__ uint4 ld_x(const uint4* p) { return __ldg(p); }

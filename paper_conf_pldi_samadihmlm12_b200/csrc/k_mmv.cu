@@ -1,0 +1,71 @@
+// Instances of the multi-vector kernels (mmv_kernels.cuh), fp32, K in {2, 4, 8}:
+//   group: G in {1,2,4,8,16,32} x U in {1,2,4} (K*U <= 16) x VEC, RB = 2
+//   cta  : NT = 256, U in {1, 2} x VEC
+//   tmmv : LR in {1,...,256} x VEC, U = 2, NT = 256
+#include "mmv_kernels.cuh"
+
+namespace adaptic {
+
+template <int K, int G, bool VEC>
+static void* mg_u(int U) {
+    switch (U) {
+        case 1: return reinterpret_cast<void*>(&mmv_group_kernel<K, G, 2, 1, VEC, GROUP_NT>);
+        case 2: return reinterpret_cast<void*>(&mmv_group_kernel<K, G, 2, 2, VEC, GROUP_NT>);
+        case 4: if constexpr (K * 4 <= 16) return reinterpret_cast<void*>(&mmv_group_kernel<K, G, 2, 4, VEC, GROUP_NT>);
+                else return nullptr;
+        default: return nullptr;
+    }
+}
+
+template <int K, bool VEC>
+static void* mg_g(int G, int U) {
+    switch (G) {
+        case 1: return mg_u<K, 1, VEC>(U);
+        case 2: return mg_u<K, 2, VEC>(U);
+        case 4: return mg_u<K, 4, VEC>(U);
+        case 8: return mg_u<K, 8, VEC>(U);
+        case 16: return mg_u<K, 16, VEC>(U);
+        case 32: return mg_u<K, 32, VEC>(U);
+        default: return nullptr;
+    }
+}
+
+template <int K, bool VEC>
+static void* mc_u(int U) {
+    switch (U) {
+        case 1: return reinterpret_cast<void*>(&mmv_cta_kernel<K, 256, 1, VEC>);
+        case 2: return reinterpret_cast<void*>(&mmv_cta_kernel<K, 256, 2, VEC>);
+        default: return nullptr;
+    }
+}
+
+template <int K, bool VEC>
+static void* mt_l(int LR) {
+    switch (LR) {
+        case 1: return reinterpret_cast<void*>(&tmmv_kernel<K, 1, 2, VEC, 256>);
+        case 2: return reinterpret_cast<void*>(&tmmv_kernel<K, 2, 2, VEC, 256>);
+        case 4: return reinterpret_cast<void*>(&tmmv_kernel<K, 4, 2, VEC, 256>);
+        case 8: return reinterpret_cast<void*>(&tmmv_kernel<K, 8, 2, VEC, 256>);
+        case 16: return reinterpret_cast<void*>(&tmmv_kernel<K, 16, 2, VEC, 256>);
+        case 32: return reinterpret_cast<void*>(&tmmv_kernel<K, 32, 2, VEC, 256>);
+        case 64: return reinterpret_cast<void*>(&tmmv_kernel<K, 64, 2, VEC, 256>);
+        case 128: return reinterpret_cast<void*>(&tmmv_kernel<K, 128, 2, VEC, 256>);
+        case 256: return reinterpret_cast<void*>(&tmmv_kernel<K, 256, 2, VEC, 256>);
+        default: return nullptr;
+    }
+}
+
+#define ADAPTIC_K(FN, ...)                                                       \
+    switch (K) {                                                                 \
+        case 2: return vec ? FN<2, true>(__VA_ARGS__) : FN<2, false>(__VA_ARGS__); \
+        case 4: return vec ? FN<4, true>(__VA_ARGS__) : FN<4, false>(__VA_ARGS__); \
+        case 8: return vec ? FN<8, true>(__VA_ARGS__) : FN<8, false>(__VA_ARGS__); \
+        default: return nullptr;                                                 \
+    }
+
+void* mmv_group_fn(int K, int G, int U, bool vec) { ADAPTIC_K(mg_g, G, U) }
+void* mmv_cta_fn(int K, int U, bool vec) { ADAPTIC_K(mc_u, U) }
+void* tmmv_fn(int K, int LR, bool vec) { ADAPTIC_K(mt_l, LR) }
+#undef ADAPTIC_K
+
+}  // namespace adaptic

@@ -34,15 +34,15 @@ def _dtype_code(t: torch.Tensor) -> int:
 
 
 def get_plan(op: int, rows: int, cols: int, dtype: int, device: torch.device,
-             variant="AUTO", params=None, stream: int = 0) -> L.Plan:
+             variant="AUTO", params=None, stream: int = 0, nvec: int = 1) -> L.Plan:
     """Cached plan with its workspace attached (allocated zero-filled on `device`)."""
     key = (op, int(rows), int(cols), dtype, variant, tuple(params) if params else None,
-           device.index, stream)
+           device.index, stream, int(nvec))
     with _cache_lock:
         ent = _cache.get(key)
         if ent is not None:
             return ent[0]
-    plan = L.Plan(op, rows, cols, dtype, variant, params)
+    plan = L.Plan(op, rows, cols, dtype, variant, params, nvec)
     ws = None
     nbytes = plan.workspace_bytes
     if nbytes:
@@ -146,6 +146,45 @@ def iamin(a: torch.Tensor, *, variant="AUTO", params=None, out=None) -> torch.Te
     return _blas1(L.OP_IAMIN, a, variant, params, out, torch.int32)
 
 
+MULTI_SIZES = (8, 4, 2, 1)
+
+
+def _multi(op: int, M: torch.Tensor, X: torch.Tensor, R: int, C: int, variant, params, out):
+    if X.dim() != 2 or X.shape[1] != C:
+        raise ValueError(f"X must be [K, {C}], got {tuple(X.shape)}")
+    dev = _check_dev(M, X)
+    if M.dtype != torch.float32:
+        raise TypeError("multi-vector forms take float32")
+    K = X.shape[0]
+    if out is None:
+        out = torch.empty(K, R, dtype=M.dtype, device=dev)
+    elif tuple(out.shape) != (K, R) or out.dtype != M.dtype or not out.is_contiguous():
+        raise ValueError(f"out must be a contiguous float32 [{K}, {R}] tensor")
+    stream = torch.cuda.current_stream(dev).cuda_stream
+    j = 0
+    while j < K:                       # the library runs K in {1, 2, 4, 8}: cover K greedily
+        k = next(m for m in MULTI_SIZES if m <= K - j)
+        plan = get_plan(op, R, C, L.F32, dev, variant if k > 1 else "AUTO", params if k > 1 else None, stream, k)
+        plan.run(M.data_ptr(), X[j:j + k].data_ptr(), out[j:j + k].data_ptr(), stream)
+        j += k
+    return out
+
+
+def mv_multi(A: torch.Tensor, X: torch.Tensor, *, variant="AUTO", params=None, out=None) -> torch.Tensor:
+    """Y[j] = A X[j] for K vectors in one pass over A (horizontal actor integration,
+    P:600).  A [R, C], X [K, C] -> Y [K, R], float32."""
+    if A.dim() != 2:
+        raise ValueError(f"mv_multi: A must be [R, C], got {tuple(A.shape)}")
+    return _multi(L.OP_MV, A, X, A.shape[0], A.shape[1], variant, params, out)
+
+
+def tmv_multi(B: torch.Tensor, X: torch.Tensor, *, variant="AUTO", params=None, out=None) -> torch.Tensor:
+    """Y[j] = B^T X[j] for K vectors in one pass over B.  B [C, R], X [K, C] -> Y [K, R]."""
+    if B.dim() != 2:
+        raise ValueError(f"tmv_multi: B must be [C, R], got {tuple(B.shape)}")
+    return _multi(L.OP_TMV, B, X, B.shape[1], B.shape[0], variant, params, out)
+
+
 def b1all(a: torch.Tensor, *, variant="AUTO", params=None, out=None):
     """All four BLAS-1 reductions of every row from ONE pass over ``a`` (the paper's
     horizontal actor integration).  Returns (asum, nrm2, iamax, iamin): two
@@ -168,9 +207,9 @@ def b1all(a: torch.Tensor, *, variant="AUTO", params=None, out=None):
     return f[:N], f[N:2 * N], i[2 * N:3 * N], i[3 * N:]
 
 
-def plan(op: str, rows: int, cols: int, dtype: str = "f32", variant="AUTO", params=None) -> L.Plan:
+def plan(op: str, rows: int, cols: int, dtype: str = "f32", variant="AUTO", params=None, nvec: int = 1) -> L.Plan:
     """A bare plan (no workspace attached) -- for inspecting the selector."""
-    return L.Plan(L.OPS[op], rows, cols, {"f32": L.F32, "i32": L.I32}[dtype], variant, params)
+    return L.Plan(L.OPS[op], rows, cols, {"f32": L.F32, "i32": L.I32}[dtype], variant, params, nvec)
 
 
 def run_host(op: str, M_host: torch.Tensor, X_host: torch.Tensor, y_host: torch.Tensor,

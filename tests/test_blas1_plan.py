@@ -115,3 +115,24 @@ def test_b1all_plan_and_contract():
     assert p.run_ptrs(A, 0, A + 4 * (1 << 22) * 4 - 8) == L.ERR_ALIAS      # y spans 16*N bytes
     with pytest.raises(adaptic.AdapticError):
         adaptic.plan("b1all", 1, 1 << 31)
+
+
+def test_multi_vector_plans():
+    """adaptic_plan_multi (K vectors, one pass): K in {1,2,4,8}, fp32, MV/TMV only."""
+    for op, R, C in (("mv", 1 << 16, 1024), ("mv", 1 << 20, 64), ("mv", 64, 1 << 20), ("tmv", 8192, 8192),
+                     ("tmv", 8, 1 << 23), ("mv", 100, 1001), ("tmv", 1001, 100)):
+        for K in (2, 4, 8):
+            d = adaptic.plan(op, R, C, nvec=K).describe()
+            w = 1 if d["vec_shape"] else 0
+            assert d["nvec"] == K and d["path_ok"][w] and d["chain"][w] + d["depth"][w] <= 1677, d
+    for bad in ((3, L.ERR_UNSUPPORTED), (0, L.ERR_INVALID_ARG), (16, L.ERR_UNSUPPORTED)):
+        with pytest.raises(adaptic.AdapticError) as e:
+            adaptic.plan("mv", 64, 64, nvec=bad[0])
+        assert e.value.status == bad[1]
+    for op, dt in (("dot", "f32"), ("asum", "f32"), ("mv", "i32")):
+        with pytest.raises(adaptic.AdapticError) as e:
+            adaptic.plan(op, 64, 64, dt, nvec=4)
+        assert e.value.status == L.ERR_UNSUPPORTED
+    p = adaptic.plan("mv", 16, 64, nvec=4)
+    A, X = 0x10000000, 0x20000000
+    assert p.run_ptrs(A, X, X + 4 * 64 * 4 - 4) == L.ERR_ALIAS      # X spans K*C elements
