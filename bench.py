@@ -13,6 +13,8 @@ Workloads (``--workload``):
            line adds single-launch and CUDA-graph-amortized latency in microseconds.
   multi multi-vector MV/TMV, K = 4 vectors per pass over a 256 MiB
            matrix (horizontal actor integration, adaptic_plan_multi).
+  bicgstab BiCGSTAB on the adaptive MV, n = 8192 (the paper's Fig. 11
+           largest system): one step = one iteration (3 fused step kernels + 2 MVs).
   blas1 Sasum / Snrm2 / Isamax / Isamin (the paper's Fig. 9
            CUBLAS benchmarks) on 256 MiB inputs: N x L = 1 x 2^26 .. 2^22 x 16.
 Multi-GPU: one process per GPU (torchrun), barrier + synchronize around the
@@ -46,7 +48,7 @@ def parse():
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", choices=["adaptic", "reference"], default="adaptic")
-    ap.add_argument("--workload", choices=["sweep", "rowshard", "splitk", "dot", "blas1", "config0", "multi"], default="sweep")
+    ap.add_argument("--workload", choices=["sweep", "rowshard", "splitk", "dot", "blas1", "config0", "multi", "bicgstab"], default="sweep")
     ap.add_argument("--variant", default="AUTO", help="force one variant (fixed-variant sweeps)")
     ap.add_argument("--streams", type=int, default=1,
                     help="issue the step's independent problems round-robin on this many CUDA streams "
@@ -570,9 +572,76 @@ def run_reference(args):
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}), flush=True)
 
 
+def run_bicgstab(args):
+    """One step = one BiCGSTAB iteration on an n x n diagonally dominant system (device
+    resident); value = algorithmic bytes / s (2 MVs of 4(n^2 + 2n) bytes plus the
+    step kernels' 17 n-vector reads/writes)."""
+    import torch
+    import synth
+    import paper_conf_pldi_samadihmlm12_b200 as adaptic
+    world, rank, local = dist_setup()
+    n = 8192
+    dev = torch.device("cuda", torch.cuda.current_device())
+    A = torch.empty(n * n, dtype=torch.float32, device=dev)
+    synth.device_matrix(A, n, n, "mv", "diagdom", synth.seed(22, "A"))
+    b = torch.empty(n, dtype=torch.float32, device=dev)
+    synth.device_vector(b, "uniform", synth.seed(22, "b"))
+    x = torch.empty(n, dtype=torch.float32, device=dev)
+    S = adaptic.bicgstab_solver(n, dev)
+    stream = torch.cuda.current_stream().cuda_stream
+    step_bytes = 2 * 4 * (n * n + 2 * n) + 17 * 4 * n
+    # convergence run (reported): iterations to 1e-6
+    it_conv, rel_conv = S.solve(A.data_ptr(), b.data_ptr(), x.data_ptr(), 200, 1e-6, 8, stream)
+    S.start(b.data_ptr(), x.data_ptr(), stream)
+    S.iterate(A.data_ptr(), x.data_ptr(), max(3, args.warmup), 0.0, stream)   # tol 0: every iteration runs
+    torch.cuda.synchronize()
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    clocks = Clocks(torch.cuda.current_device())
+    clocks.start()
+    barrier(world)
+    torch.cuda.synchronize()
+    t0.record()
+    S.iterate(A.data_ptr(), x.data_ptr(), args.steps, 0.0, stream)
+    t1.record()
+    torch.cuda.synchronize()
+    barrier(world)
+    clk = clocks.stop()
+    ms = max_over_ranks(t0.elapsed_time(t1), world)
+    it_done, rel, done = S.state(stream)
+    value = world * step_bytes * args.steps / (ms / 1e3) / 1e9
+    plan = adaptic.plan("mv", n, n).describe()
+    peak, peak_src = peaks()
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        import numpy as np
+        from oracle.bicgstab import bicgstab as obicg
+        Ah = A.view(n, n).cpu().numpy().astype(np.float64)
+        bh = b.cpu().numpy().astype(np.float64)
+        t = time.perf_counter()
+        obicg(Ah, bh, tol=0.0, max_iters=5)
+        el = time.perf_counter() - t
+        cpu = {"value": step_bytes * 5 / el / 1e9, "unit": UNIT, "cores": os.cpu_count(), "kind": "oracle",
+               "sample": f"5 fp64 iterations of the oracle (numpy; BLAS threads available: {os.cpu_count()}), n={n}"}
+    if rank == 0:
+        print(json.dumps({
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f32", "data": "synthetic (seeded splitmix64; diagonally dominant A)",
+            "config": {"workload": f"SURVEY 8(f)#3: BiCGSTAB n={n} (Fig. 11 largest), one iteration per step",
+                       "mv_plan": plan["variant"], "l2": "A is 256 MiB > L2; no flush needed"},
+            "roofline": {"bound": "hbm", "achieved": value / world, "peak": peak, "unit": "GB/s",
+                         "frac": value / world / peak, "traffic": None, "peak_source": peak_src,
+                         "kernel": "whole iteration (2 MVs dominate)"},
+            "iterations_per_s": world * args.steps / (ms / 1e3),
+            "converge": {"tol": 1e-6, "iterations": it_conv, "relres": rel_conv},
+            "cpu_baseline": cpu, "e2e": None, "gpu_launches": 5 * args.steps, "clocks": clk}), flush=True)
+
+
 if __name__ == "__main__":
     a = parse()
     if a.impl == "reference":
         run_reference(a)
+    elif a.workload == "bicgstab":
+        run_bicgstab(a)
     else:
         run_adaptic(a)

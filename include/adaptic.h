@@ -122,7 +122,7 @@
 extern "C" {
 #endif
 
-#define ADAPTIC_ABI_VERSION 3
+#define ADAPTIC_ABI_VERSION 4
 
 typedef enum {
     ADAPTIC_OK = 0,
@@ -264,6 +264,46 @@ adaptic_status adaptic_run_host(adaptic_plan_t plan, const void* A_host, const v
                                 void* y_host, void* dA, void* dx, void* dy, void* stream);
 
 void adaptic_plan_destroy(adaptic_plan_t plan);
+
+/* ---------------------------------------------------------------------------------
+ * BiCGSTAB on the adaptive MV (the paper's Sec. 5.2.2 case study,
+ * P:1252-1304).  Solves A x = b for a dense, row-major n x n fp32 A (nonsymmetric),
+ * x0 = 0, shadow residual r^ = b, the textbook unpreconditioned iteration (DESIGN.md
+ * lists its 11 steps).  The paper's point is vertical integration: the sub-steps that
+ * CUBLAS needs separate Sdot/Sscal/Saxpy calls for are merged into one kernel per step
+ * ("Adaptic merges all these sub-steps together and launches a single kernel for one
+ * step").  One iteration = 5 launches on `stream` (3 fused step kernels + 2 MVs
+ * from adaptic_plan(MV, n, n)); every scalar stays on the device.
+ *
+ * Ownership: the solver object is the library's (free with adaptic_bicgstab_destroy);
+ * it needs a caller-owned device workspace of adaptic_bicgstab_workspace_bytes() bytes,
+ * 256-byte aligned and ZERO-FILLED when attached (it holds the MV plan's workspace,
+ * six n-vectors and the scalar state).  A, b, x are caller-owned device pointers,
+ * 16-byte aligned for the 128-bit MV path (else the scalar kernels run).
+ *   create   : 1 <= n <= ADAPTIC_BICGSTAB_MAX_N, else INVALID_ARG / UNSUPPORTED.
+ *   start    : enqueue x = 0, r = r^ = b, p = v = 0 and the state (||b||, ...).
+ *   iterate  : enqueue `iters` iterations; after convergence (||r|| / ||b|| < tol, or
+ *              ||s|| / ||b|| < tol at step 7) or a breakdown ((r^, r) = 0, (r^, v) = 0,
+ *              omega = 0) the step kernels leave x untouched, so batches can be
+ *              enqueued without host checks.
+ *   state    : synchronises `stream` and reads back iterations done, the recurrence
+ *              residual ||r|| / ||b||, and done (0 running, 1 converged, 2 breakdown).
+ *   solve    : start + iterate in batches of check_every (<= 0: 8) + state, until done
+ *              or max_iters; blocking.  Outputs may be NULL. */
+#define ADAPTIC_BICGSTAB_MAX_N 65536
+typedef struct adaptic_bicgstab_s* adaptic_bicgstab_t;
+adaptic_status adaptic_bicgstab_create(int64_t n, adaptic_bicgstab_t* out);
+size_t adaptic_bicgstab_workspace_bytes(adaptic_bicgstab_t solver);
+adaptic_status adaptic_bicgstab_set_workspace(adaptic_bicgstab_t solver, void* dev_ptr, size_t bytes);
+adaptic_status adaptic_bicgstab_start(adaptic_bicgstab_t solver, const void* b, void* x, void* stream);
+adaptic_status adaptic_bicgstab_iterate(adaptic_bicgstab_t solver, const void* A, void* x, int32_t iters,
+                                        float tol, void* stream);
+adaptic_status adaptic_bicgstab_state(adaptic_bicgstab_t solver, int32_t* iters, float* relres,
+                                      int32_t* done, void* stream);
+adaptic_status adaptic_bicgstab_solve(adaptic_bicgstab_t solver, const void* A, const void* b, void* x,
+                                      int32_t max_iters, float tol, int32_t check_every,
+                                      int32_t* iters_out, float* relres_out, void* stream);
+void adaptic_bicgstab_destroy(adaptic_bicgstab_t solver);
 
 const char* adaptic_status_string(adaptic_status status);
 const char* adaptic_variant_name(adaptic_variant variant);

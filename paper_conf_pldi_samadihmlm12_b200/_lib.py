@@ -33,7 +33,10 @@ P_LANES, P_SPLITS, P_CTAS_PER_SM, P_UNROLL, P_XSMEM, P_BLOCK, P_ROWS, P_ORDER, P
 SYMBOLS = ("adaptic_plan", "adaptic_plan_forced", "adaptic_plan_multi", "adaptic_plan_variant", "adaptic_plan_describe",
            "adaptic_plan_workspace_bytes", "adaptic_plan_set_workspace", "adaptic_run",
            "adaptic_run_host", "adaptic_plan_destroy", "adaptic_status_string",
-           "adaptic_variant_name", "adaptic_last_cuda_error", "adaptic_abi_version")
+           "adaptic_variant_name", "adaptic_last_cuda_error", "adaptic_abi_version",
+           "adaptic_bicgstab_create", "adaptic_bicgstab_workspace_bytes", "adaptic_bicgstab_set_workspace",
+           "adaptic_bicgstab_start", "adaptic_bicgstab_iterate", "adaptic_bicgstab_state",
+           "adaptic_bicgstab_solve", "adaptic_bicgstab_destroy")
 
 _lib = None
 _lock = threading.Lock()
@@ -92,6 +95,23 @@ def lib():
         L.adaptic_last_cuda_error.restype = i32
         L.adaptic_abi_version.argtypes = []
         L.adaptic_abi_version.restype = i32
+        f32, pi32, pf32 = ctypes.c_float, ctypes.POINTER(ctypes.c_int32), ctypes.POINTER(ctypes.c_float)
+        L.adaptic_bicgstab_create.argtypes = [i64, ctypes.POINTER(vp)]
+        L.adaptic_bicgstab_create.restype = i32
+        L.adaptic_bicgstab_workspace_bytes.argtypes = [vp]
+        L.adaptic_bicgstab_workspace_bytes.restype = ctypes.c_size_t
+        L.adaptic_bicgstab_set_workspace.argtypes = [vp, vp, ctypes.c_size_t]
+        L.adaptic_bicgstab_set_workspace.restype = i32
+        L.adaptic_bicgstab_start.argtypes = [vp, vp, vp, vp]
+        L.adaptic_bicgstab_start.restype = i32
+        L.adaptic_bicgstab_iterate.argtypes = [vp, vp, vp, ctypes.c_int32, f32, vp]
+        L.adaptic_bicgstab_iterate.restype = i32
+        L.adaptic_bicgstab_state.argtypes = [vp, pi32, pf32, pi32, vp]
+        L.adaptic_bicgstab_state.restype = i32
+        L.adaptic_bicgstab_solve.argtypes = [vp, vp, vp, vp, ctypes.c_int32, f32, ctypes.c_int32, pi32, pf32, vp]
+        L.adaptic_bicgstab_solve.restype = i32
+        L.adaptic_bicgstab_destroy.argtypes = [vp]
+        L.adaptic_bicgstab_destroy.restype = None
         _lib = L
     return _lib
 
@@ -166,4 +186,51 @@ class Plan:
         h = getattr(self, "_h", None)
         if h is not None and h.value and _lib is not None:
             _lib.adaptic_plan_destroy(h)
+            self._h = None
+
+
+class BiCGSTAB:
+    """An ``adaptic_bicgstab_t`` (BiCGSTAB on the adaptive MV; include/adaptic.h)."""
+
+    def __init__(self, n: int):
+        h = ctypes.c_void_p()
+        _check(lib().adaptic_bicgstab_create(int(n), ctypes.byref(h)), f"adaptic_bicgstab_create({n})")
+        self._h = h
+        self.n = int(n)
+
+    @property
+    def workspace_bytes(self) -> int:
+        return int(lib().adaptic_bicgstab_workspace_bytes(self._h))
+
+    def set_workspace(self, ptr: int, nbytes: int):
+        _check(lib().adaptic_bicgstab_set_workspace(self._h, ctypes.c_void_p(ptr or None), nbytes),
+               "adaptic_bicgstab_set_workspace")
+
+    def start(self, b: int, x: int, stream: int = 0):
+        _check(lib().adaptic_bicgstab_start(self._h, ctypes.c_void_p(b or None), ctypes.c_void_p(x or None),
+                                            ctypes.c_void_p(stream or None)), "adaptic_bicgstab_start")
+
+    def iterate(self, A: int, x: int, iters: int, tol: float, stream: int = 0):
+        _check(lib().adaptic_bicgstab_iterate(self._h, ctypes.c_void_p(A or None), ctypes.c_void_p(x or None),
+                                              int(iters), float(tol), ctypes.c_void_p(stream or None)),
+               "adaptic_bicgstab_iterate")
+
+    def state(self, stream: int = 0):
+        it, rel, done = ctypes.c_int32(), ctypes.c_float(), ctypes.c_int32()
+        _check(lib().adaptic_bicgstab_state(self._h, ctypes.byref(it), ctypes.byref(rel), ctypes.byref(done),
+                                            ctypes.c_void_p(stream or None)), "adaptic_bicgstab_state")
+        return it.value, rel.value, done.value
+
+    def solve(self, A: int, b: int, x: int, max_iters: int, tol: float, check_every: int = 8, stream: int = 0):
+        it, rel = ctypes.c_int32(), ctypes.c_float()
+        _check(lib().adaptic_bicgstab_solve(self._h, *(ctypes.c_void_p(p or None) for p in (A, b, x)),
+                                            int(max_iters), float(tol), int(check_every), ctypes.byref(it),
+                                            ctypes.byref(rel), ctypes.c_void_p(stream or None)),
+               "adaptic_bicgstab_solve")
+        return it.value, rel.value
+
+    def __del__(self):
+        h = getattr(self, "_h", None)
+        if h is not None and h.value and _lib is not None:
+            _lib.adaptic_bicgstab_destroy(h)
             self._h = None

@@ -353,7 +353,10 @@ adaptic_status derive_multi(adaptic_plan_s* p, const int32_t* params, const DevI
     }
     if (op != ADAPTIC_OP_TMV || !is_tmv_family(v)) return ADAPTIC_ERR_UNSUPPORTED;
     // TMV tiles: LR output vectors x (256 / LR) c-lanes, S c-ranges
-    const int NT = 256, U = 2;
+    const int NT = 256;
+    int U = par(ADAPTIC_P_UNROLL);
+    if (U <= 0) U = K <= 4 ? 4 : 2;
+    if (U != 2 && !(U == 4 && K <= 4)) return ADAPTIC_ERR_INVALID_ARG;
     const int64_t rv1 = p->vec_shape ? R / 4 : R;
     int LR = par(ADAPTIC_P_LANES);
     if (LR <= 0) LR = (v == ADAPTIC_V_TMV_COL) ? 256 : (v == ADAPTIC_V_TMV_REGTILE) ? clampi(pow2_ceil(rv1), 1, 256)
@@ -361,7 +364,7 @@ adaptic_status derive_multi(adaptic_plan_s* p, const int32_t* params, const DevI
     if (LR < 1 || LR > 256 || (LR & (LR - 1))) return ADAPTIC_ERR_INVALID_ARG;
     if (v == ADAPTIC_V_TMV_REGTILE && rv1 > LR) return ADAPTIC_ERR_UNSUPPORTED;
     int cps = par(ADAPTIC_P_CTAS_PER_SM);
-    if (cps <= 0) cps = occupancy(tmmv_fn(K, LR, p->vec_shape), NT, 0, dev.present, 2048 / NT);
+    if (cps <= 0) cps = occupancy(tmmv_fn(K, LR, U, p->vec_shape), NT, 0, dev.present, 2048 / NT);
     p->lanes = LR; p->unroll = U; p->block = NT; p->ctas_per_sm = cps;
     const int LC = NT / LR;
     const int64_t slots = int64_t(dev.sms) * cps;
@@ -859,7 +862,7 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
     void* args7[7];
     if (p->nvec > 1) {
         const int K = p->nvec;
-        if (p->op == ADAPTIC_OP_TMV) fn = tmmv_fn(K, p->lanes, vec);
+        if (p->op == ADAPTIC_OP_TMV) fn = tmmv_fn(K, p->lanes, p->unroll, vec);
         else if (p->variant == ADAPTIC_V_MV_SUBWARP || p->variant == ADAPTIC_V_MV_WPR) fn = mmv_group_fn(K, p->lanes, p->unroll, vec);
         else fn = mmv_cta_fn(K, p->unroll, vec);
         if (p->op == ADAPTIC_OP_MV && (p->variant == ADAPTIC_V_MV_SUBWARP || p->variant == ADAPTIC_V_MV_WPR)) {

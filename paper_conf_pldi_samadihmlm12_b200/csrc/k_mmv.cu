@@ -1,7 +1,7 @@
 // Instances of the multi-vector kernels (mmv_kernels.cuh), fp32, K in {2, 4, 8}:
 //   group: G in {1,2,4,8,16,32} x U in {1,2,4} (K*U <= 16) x VEC, RB = 2
 //   cta  : NT = 256, U in {1, 2} x VEC
-//   tmmv : LR in {1,...,256} x VEC, U = 2, NT = 256
+//   tmmv : LR in {1,...,256} x VEC x U in {2, 4} (4 only for K <= 4), NT = 256
 #include "mmv_kernels.cuh"
 
 namespace adaptic {
@@ -39,20 +39,27 @@ static void* mc_u(int U) {
     }
 }
 
-template <int K, bool VEC>
-static void* mt_l(int LR) {
+template <int K, int U, bool VEC>
+static void* mt_lu(int LR) {
     switch (LR) {
-        case 1: return reinterpret_cast<void*>(&tmmv_kernel<K, 1, 2, VEC, 256>);
-        case 2: return reinterpret_cast<void*>(&tmmv_kernel<K, 2, 2, VEC, 256>);
-        case 4: return reinterpret_cast<void*>(&tmmv_kernel<K, 4, 2, VEC, 256>);
-        case 8: return reinterpret_cast<void*>(&tmmv_kernel<K, 8, 2, VEC, 256>);
-        case 16: return reinterpret_cast<void*>(&tmmv_kernel<K, 16, 2, VEC, 256>);
-        case 32: return reinterpret_cast<void*>(&tmmv_kernel<K, 32, 2, VEC, 256>);
-        case 64: return reinterpret_cast<void*>(&tmmv_kernel<K, 64, 2, VEC, 256>);
-        case 128: return reinterpret_cast<void*>(&tmmv_kernel<K, 128, 2, VEC, 256>);
-        case 256: return reinterpret_cast<void*>(&tmmv_kernel<K, 256, 2, VEC, 256>);
+        case 1: return reinterpret_cast<void*>(&tmmv_kernel<K, 1, U, VEC, 256>);
+        case 2: return reinterpret_cast<void*>(&tmmv_kernel<K, 2, U, VEC, 256>);
+        case 4: return reinterpret_cast<void*>(&tmmv_kernel<K, 4, U, VEC, 256>);
+        case 8: return reinterpret_cast<void*>(&tmmv_kernel<K, 8, U, VEC, 256>);
+        case 16: return reinterpret_cast<void*>(&tmmv_kernel<K, 16, U, VEC, 256>);
+        case 32: return reinterpret_cast<void*>(&tmmv_kernel<K, 32, U, VEC, 256>);
+        case 64: return reinterpret_cast<void*>(&tmmv_kernel<K, 64, U, VEC, 256>);
+        case 128: return reinterpret_cast<void*>(&tmmv_kernel<K, 128, U, VEC, 256>);
+        case 256: return reinterpret_cast<void*>(&tmmv_kernel<K, 256, U, VEC, 256>);
         default: return nullptr;
     }
+}
+
+template <int K, bool VEC>
+static void* mt_l(int LR, int U) {
+    if (U == 2) return mt_lu<K, 2, VEC>(LR);
+    if constexpr (K <= 4) { if (U == 4) return mt_lu<K, 4, VEC>(LR); }
+    return nullptr;
 }
 
 #define ADAPTIC_K(FN, ...)                                                       \
@@ -65,7 +72,7 @@ static void* mt_l(int LR) {
 
 void* mmv_group_fn(int K, int G, int U, bool vec) { ADAPTIC_K(mg_g, G, U) }
 void* mmv_cta_fn(int K, int U, bool vec) { ADAPTIC_K(mc_u, U) }
-void* tmmv_fn(int K, int LR, bool vec) { ADAPTIC_K(mt_l, LR) }
+void* tmmv_fn(int K, int LR, int U, bool vec) { ADAPTIC_K(mt_l, LR, U) }
 #undef ADAPTIC_K
 
 }  // namespace adaptic

@@ -50,11 +50,11 @@ void* tmv_mis_fn_i32(int LR, int U);
 // Multi-vector MV / TMV (mmv_kernels.cuh), fp32, K in {2, 4, 8}; X is K x C, Y is K x R:
 //   group: (const float* A, const float* X, float* Y, int64_t R, int64_t C), rows of <= G*U vectors
 //   cta  : (A, X, Y, R, C, int S, float* part, unsigned* cnt), RB = 8/K rows per CTA, NT = 256
-//   tmmv : (B, X, Y, R, C, int S, float* part, unsigned* cnt), NT = 256, U = 2
+//   tmmv : (B, X, Y, R, C, int S, float* part, unsigned* cnt), NT = 256, U in {2, 4}
 constexpr int MMV_GROUP_RB = 2;
 void* mmv_group_fn(int K, int G, int U, bool vec);
 void* mmv_cta_fn(int K, int U, bool vec);
-void* tmmv_fn(int K, int LR, bool vec);
+void* tmmv_fn(int K, int LR, int U, bool vec);
 
 // BLAS-1 reductions (blas1_kernels.cuh), fp32 input, one translation unit per operator:
 //   b1 group: (const float* A, void* y, int64_t R, int64_t C); rbu 0 = (RB 4, U 2), 1 = (RB 1, U 8)

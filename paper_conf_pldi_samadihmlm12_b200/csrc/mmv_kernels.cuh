@@ -146,11 +146,14 @@ mmv_cta_kernel(const float* __restrict__ A, const float* __restrict__ X, float* 
         }
         const int64_t tail_end = min(nv, b + BV);
         for (int64_t v = b + tid; v < tail_end; v += NT) {
+            E a[RB];
+#pragma unroll
+            for (int i = 0; i < RB; ++i) a[i] = ld_stream(Av + off[i] + v);
 #pragma unroll
             for (int j = 0; j < K; ++j) {
                 const E xv = ld_x(Xv + j * nv + v);
 #pragma unroll
-                for (int i = 0; i < RB; ++i) emac(acc[i][j], ld_stream(Av + off[i] + v), xv);
+                for (int i = 0; i < RB; ++i) emac(acc[i][j], a[i], xv);
             }
         }
         float val[KR];                                   // index i*K + j
@@ -187,7 +190,7 @@ mmv_cta_kernel(const float* __restrict__ A, const float* __restrict__ X, float* 
 // As tmv_kernel: CTA tile of LR output vectors x LC = NT/LR c-lanes, S c-ranges,
 // with K accumulators per thread (one per vector) and the lc-combine per vector.
 template <int K, int LR, int U, bool VEC, int NT>
-__global__ void __launch_bounds__(NT)
+__global__ void __launch_bounds__(NT, 2)
 tmmv_kernel(const float* __restrict__ B, const float* __restrict__ X, float* __restrict__ Y,
             int64_t R, int64_t C, int S, float* __restrict__ ws_part, unsigned int* __restrict__ ws_cnt)
 {

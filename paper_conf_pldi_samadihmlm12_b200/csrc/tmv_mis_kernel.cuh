@@ -8,7 +8,8 @@
 // the two aligned 128-bit vectors that cover its four elements of row c and
 // selects them by s_c (a funnel shift in registers), so the stream stays 128-bit;
 // the second vector is the neighbouring thread's first, so HBM traffic is
-// unchanged; both loads allocate in L1, where the second one hits.  Tiling, splits and the merge are those of
+// unchanged and only L2 sees it twice (L1-allocating loads for the pair were
+// measured no faster: profiles/, sweep_tmv_mis2).  Tiling, splits and the merge are those of
 // tmv_kernel (TMV_COL / TMV_SPLITK / TMV_REGTILE; the paper's restructured-layout
 // kernels).  y and the partials are written per element (y is not
 // 16-byte aligned in general), the last vector of a tile row masked to R.
@@ -75,8 +76,8 @@ tmv_mis_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restrict__
                 const int64_t f = b0 + cc * R + col;             // aligned-view element index
                 const int64_t q = f >> 2;
                 sh[u] = int(f & 3);
-                lo[u] = ld_stream_l1(Ba + q);
-                hi[u] = ld_stream_l1(Ba + min(q + 1, qmax));
+                lo[u] = ld_stream(Ba + q);
+                hi[u] = ld_stream(Ba + min(q + 1, qmax));
                 xs[u] = ld_x(X + cc);
             }
 #pragma unroll
@@ -91,7 +92,7 @@ tmv_mis_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restrict__
         for (; c < c1; c += LC) {
             const int64_t f = b0 + c * R + col;
             const int64_t q = f >> 2;
-            esmac(acc[0], funnel4(ld_stream_l1(Ba + q), ld_stream_l1(Ba + min(q + 1, qmax)), int(f & 3)), ld_x(X + c));
+            esmac(acc[0], funnel4(ld_stream(Ba + q), ld_stream(Ba + min(q + 1, qmax)), int(f & 3)), ld_x(X + c));
         }
         E tot = eadd(outer, tree_sum<U>(acc));
         tot = lc_combine<NT, LR>(tot, red);

@@ -233,3 +233,37 @@ def run_host(op: str, M_host: torch.Tensor, X_host: torch.Tensor, y_host: torch.
     plan.run_host(M_host.data_ptr(), X_host.data_ptr(), y_host.data_ptr(),
                   dM.data_ptr(), dX.data_ptr(), dy.data_ptr(), stream)
     return y_host
+
+
+_solvers: dict = {}
+
+
+def bicgstab_solver(n: int, device: torch.device) -> "L.BiCGSTAB":
+    """Cached solver for n x n systems on `device` with its zero-filled workspace."""
+    key = (int(n), device.index)
+    with _cache_lock:
+        ent = _solvers.get(key)
+        if ent is not None:
+            return ent[0]
+    S = L.BiCGSTAB(n)
+    ws = torch.zeros(S.workspace_bytes, dtype=torch.uint8, device=device)
+    S.set_workspace(ws.data_ptr(), S.workspace_bytes)
+    with _cache_lock:
+        _solvers.setdefault(key, (S, ws))
+        return _solvers[key][0]
+
+
+def bicgstab(A: torch.Tensor, b: torch.Tensor, *, tol: float = 1e-6, max_iters: int = 1000,
+             check_every: int = 8, out=None):
+    """Solve A x = b (A [n, n] float32 CUDA, nonsymmetric) with BiCGSTAB on the adaptive MV
+    (the paper's Sec. 5.2.2 case study).  Returns (x, iterations, relative residual)."""
+    if A.dim() != 2 or A.shape[0] != A.shape[1] or b.shape != (A.shape[0],):
+        raise ValueError(f"bicgstab: A must be [n, n] and b [n], got {tuple(A.shape)}, {tuple(b.shape)}")
+    dev = _check_dev(A, b)
+    if A.dtype != torch.float32:
+        raise TypeError("bicgstab takes float32")
+    x = torch.empty_like(b) if out is None else out
+    S = bicgstab_solver(A.shape[0], dev)
+    stream = torch.cuda.current_stream(dev).cuda_stream
+    it, rel = S.solve(A.data_ptr(), b.data_ptr(), x.data_ptr(), max_iters, tol, check_every, stream)
+    return x, it, rel

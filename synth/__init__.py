@@ -27,6 +27,8 @@ value distribution):
     perm      : 1 if c == R-1-r else 0      (matrices only; the reversal permutation)
     diag      : uniform(i) if r == c else 0 (matrices only)
     rowscale  : uniform(i) * 2^((r mod 41) - 20)       (fp32 matrices only)
+    diagdom   : uniform(i) if r != c else C            (matrices only; strictly diagonally
+                dominant since |uniform| < 1: the BiCGSTAB systems)
 * seeds: seed(config, role) = 20120611 + 1000*config + {A: 0, x: 1, b: 2}.
 """
 from __future__ import annotations
@@ -40,7 +42,7 @@ _M2 = 0x94D049BB133111EB
 _MASK64 = (1 << 64) - 1
 
 KINDS = ("uniform", "positive", "ones", "smallint", "smallint4",
-         "identity", "perm", "diag", "rowscale")
+         "identity", "perm", "diag", "rowscale", "diagdom")
 VECTOR_KINDS = ("uniform", "positive", "ones", "smallint", "smallint4")
 KIND_CODE = {k: i for i, k in enumerate(KINDS)}
 
@@ -75,7 +77,7 @@ def hash64(s: int, idx: np.ndarray) -> np.ndarray:
 
 def _from_hash(h: np.ndarray, dtype, kind: str) -> np.ndarray:
     dtype = np.dtype(dtype)
-    if kind in ("uniform", "diag", "rowscale"):
+    if kind in ("uniform", "diag", "rowscale", "diagdom"):
         if dtype == np.float32:
             v = ((h >> np.uint64(40)) & np.uint64(0xFFFFFF)).astype(np.int64) - (1 << 23)
             return (v.astype(np.float32) * np.float32(2.0 ** -23)).astype(np.float32)
@@ -134,6 +136,8 @@ def matrix(R: int, C: int, layout: str, dtype, kind: str, s: int,
             blk = _from_hash(hash64(s, idx), dtype, kind)
             if kind == "diag":
                 blk = np.where(r == c, blk, dtype.type(0)).astype(dtype)
+            elif kind == "diagdom":
+                blk = np.where(r == c, dtype.type(C), blk).astype(dtype)
             elif kind == "rowscale":
                 if dtype != np.float32:
                     raise ValueError("rowscale is fp32 only")

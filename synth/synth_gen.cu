@@ -7,7 +7,7 @@
 //
 //   h = splitmix64(seed ^ (i * 0x9E3779B97F4A7C15)),  i = r*C + c (logical index)
 //   kinds: 0 uniform, 1 positive, 2 ones, 3 smallint, 4 smallint4, 5 identity,
-//          6 perm, 7 diag, 8 rowscale   (see synth/__init__.py for the formulas)
+//          6 perm, 7 diag, 8 rowscale, 9 diagdom   (see synth/__init__.py for the formulas)
 #include <cstdint>
 #include <type_traits>
 #include <cuda_runtime.h>
@@ -49,6 +49,7 @@ template <> __device__ __forceinline__ float elem<float>(uint64_t seed, int kind
     float v = f32_of(splitmix64(seed ^ (i * 0x9E3779B97F4A7C15ull)), kind);
     if (kind == 7) return r == c ? v : 0.f;
     if (kind == 8) return v * ldexpf(1.f, int(r % 41) - 20);
+    if (kind == 9) return r == c ? float(C) : v;
     return v;
 }
 template <> __device__ __forceinline__ int32_t elem<int32_t>(uint64_t seed, int kind, int64_t R, int64_t C, int64_t r, int64_t c) {
@@ -58,6 +59,7 @@ template <> __device__ __forceinline__ int32_t elem<int32_t>(uint64_t seed, int 
     const uint64_t i = uint64_t(r) * uint64_t(C) + uint64_t(c);
     int32_t v = i32_of(splitmix64(seed ^ (i * 0x9E3779B97F4A7C15ull)), kind);
     if (kind == 7) return r == c ? v : 0;
+    if (kind == 9) return r == c ? int32_t(C) : v;
     return v;
 }
 

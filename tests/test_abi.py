@@ -27,7 +27,7 @@ def test_library_exports_every_declared_symbol():
     for name in declared:
         assert hasattr(lib, name), name
     assert sorted(L.SYMBOLS) == declared
-    assert L.lib().adaptic_abi_version() == 3
+    assert L.lib().adaptic_abi_version() == 4
 
 
 def test_enums_match_header():
