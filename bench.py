@@ -50,9 +50,9 @@ def parse():
     ap.add_argument("--impl", choices=["adaptic", "reference"], default="adaptic")
     ap.add_argument("--workload", choices=["sweep", "rowshard", "splitk", "dot", "blas1", "config0", "multi", "bicgstab"], default="sweep")
     ap.add_argument("--variant", default="AUTO", help="force one variant (fixed-variant sweeps)")
-    ap.add_argument("--streams", type=int, default=1,
-                    help="issue the step's independent problems round-robin on this many CUDA streams "
-                         "(joined by events at the end of every step)")
+    ap.add_argument("--streams", type=int, default=2,
+                    help="the step's independent problems go through adaptic_run_batch on this many "
+                         "concurrent streams (1 = one after another on one stream)")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -254,37 +254,22 @@ def run_adaptic(args):
     n = len(probs)
     step_bytes = sum(p.bytes for p in probs)
 
-    # optional multi-stream issue: problem i on stream i % streams; each side stream's
-    # problems get their own plan (and so their own workspace)
+    # the step: every problem through the C ABI's batched entry (adaptic_run_batch), which
+    # issues them round-robin on `--streams` concurrent streams forked from / joined to the
+    # current stream; per-launch events (--kernel-events-in-timed) need one stream
+    from paper_conf_pldi_samadihmlm12_b200 import _lib as L
     main = torch.cuda.current_stream()
-    side = [torch.cuda.Stream() for _ in range(max(1, args.streams) - 1)]
-    if side:
-        import paper_conf_pldi_samadihmlm12_b200 as adaptic
-        from paper_conf_pldi_samadihmlm12_b200 import _lib as L
-        for i, p in enumerate(probs):
-            k = i % (len(side) + 1)
-            if k:
-                p.stream = side[k - 1].cuda_stream
-                p.plan = adaptic.get_plan(L.OPS[p.op], p.R, p.C, L.F32, torch.device("cuda", torch.cuda.current_device()),
-                                          args.variant, None, p.stream)
-    fork = torch.cuda.Event()
-    joins = [torch.cuda.Event() for _ in side]
+    nstreams = max(1, args.streams) if not args.kernel_events_in_timed else 1
+    batch = L.Batch([(p.plan, *p.ptrs) for p in probs])
 
     def one_step(evs=None):
-        if side and evs is None:
-            fork.record(main)
-            for st in side:
-                st.wait_event(fork)
-        for i, p in enumerate(probs):
-            if evs is not None:
+        if evs is None:
+            batch.run(nstreams, main.cuda_stream)
+        else:
+            for i, p in enumerate(probs):
                 evs[i].record()
-            p.launch()
-        if evs is not None:
+                p.launch()
             evs[n].record()
-        if side and evs is None:
-            for st, ev in zip(side, joins):
-                ev.record(st)
-                main.wait_event(ev)
         if splitk:
             dist.all_reduce(probs[0].y, op=dist.ReduceOp.SUM)
 
@@ -388,7 +373,8 @@ def run_adaptic(args):
                 "kernel_timing": ("per-launch CUDA events inside the timed region" if inner else
                                   f"per-kernel CUDA events after the timed region: each kernel 5x back to back, "
                                   f"{kev_steps} samples (the timed region itself has events only at its ends)"),
-                "kernel_sum_ms": kernel_sum_ms, "latency_us": latency, "streams": max(1, args.streams),
+                "kernel_sum_ms": kernel_sum_ms, "latency_us": latency, "streams": nstreams,
+                "issue": f"adaptic_run_batch over {nstreams} stream(s) per step",
                 "gpu_launches": n * args.steps, "clocks": clk,
                 "selected": {q["op"] + f" {q['R']}x{q['C']}": [q["variant"], round(q["frac"], 3)] for q in per}}
         print(json.dumps(line), flush=True)

@@ -31,7 +31,7 @@ P_LANES, P_SPLITS, P_CTAS_PER_SM, P_UNROLL, P_XSMEM, P_BLOCK, P_ROWS, P_ORDER, P
 
 # every symbol the header declares (tests check they are all exported)
 SYMBOLS = ("adaptic_plan", "adaptic_plan_forced", "adaptic_plan_multi", "adaptic_plan_variant", "adaptic_plan_describe",
-           "adaptic_plan_workspace_bytes", "adaptic_plan_set_workspace", "adaptic_run",
+           "adaptic_plan_workspace_bytes", "adaptic_plan_set_workspace", "adaptic_run", "adaptic_run_batch",
            "adaptic_run_host", "adaptic_plan_destroy", "adaptic_status_string",
            "adaptic_variant_name", "adaptic_last_cuda_error", "adaptic_abi_version",
            "adaptic_bicgstab_create", "adaptic_bicgstab_workspace_bytes", "adaptic_bicgstab_set_workspace",
@@ -83,6 +83,9 @@ def lib():
         L.adaptic_plan_set_workspace.restype = i32
         L.adaptic_run.argtypes = [vp, vp, vp, vp, vp]
         L.adaptic_run.restype = i32
+        L.adaptic_run_batch.argtypes = [ctypes.c_int32, ctypes.POINTER(vp), ctypes.POINTER(vp), ctypes.POINTER(vp),
+                                        ctypes.POINTER(vp), ctypes.c_int32, vp]
+        L.adaptic_run_batch.restype = i32
         L.adaptic_run_host.argtypes = [vp, vp, vp, vp, vp, vp, vp, vp]
         L.adaptic_run_host.restype = i32
         L.adaptic_plan_destroy.argtypes = [vp]
@@ -119,6 +122,24 @@ def lib():
 def _check(status: int, where: str):
     if status != OK:
         raise AdapticError(status, where)
+
+
+class Batch:
+    """Marshalled arguments of adaptic_run_batch for a fixed list of (plan, A, x, y)."""
+
+    def __init__(self, items):
+        n = len(items)
+        self.n = n
+        self._plans = [it[0] for it in items]                 # keep the plans alive
+        arr = lambda vals: (ctypes.c_void_p * max(1, n))(*[ctypes.c_void_p(v or None) for v in vals])  # noqa: E731
+        self.plans = (ctypes.c_void_p * max(1, n))(*[p.handle for p in self._plans])
+        self.A = arr([it[1] for it in items])
+        self.x = arr([it[2] for it in items])
+        self.y = arr([it[3] for it in items])
+
+    def run(self, streams: int, stream: int = 0):
+        _check(lib().adaptic_run_batch(self.n, self.plans, self.A, self.x, self.y, int(streams),
+                                       ctypes.c_void_p(stream or None)), "adaptic_run_batch")
 
 
 class Plan:

@@ -553,11 +553,15 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
             if (!p->path_ok[(p->vec_shape || mis) ? 1 : 0]) return ADAPTIC_ERR_UNSUPPORTED;
             return ADAPTIC_OK;
         }
-        // ---- MV_TPR proper (vector path only; scalar path = the group fallback above)
+        // ---- MV_TPR proper: index 1 = the TMA-staged kernel (128-bit shared reads, or 32-bit
+        // ones for C % 4 != 0 -- then p->mis marks it); index 0 = the group fallback above
+        // (pointers the bulk copies cannot use)
         const int64_t fb_grid = p->grid[0];
         const int64_t fb_chain = p->chain[0], fb_depth = p->depth[0];
         const bool fb_ok = p->path_ok[0];
-        if (!p->vec_shape || C > 256) return ADAPTIC_ERR_UNSUPPORTED;
+        if (C > 256) return ADAPTIC_ERR_UNSUPPORTED;
+        const bool scal = !p->vec_shape;
+        p->mis = scal;
         int NT = par(ADAPTIC_P_LANES);
         if (NT <= 0) NT = (C <= 32) ? 256 : 128;
         if (NT != 128 && NT != 256) return ADAPTIC_ERR_INVALID_ARG;
@@ -574,11 +578,11 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
         p->stages = stages;
         p->block = NT;
         p->smem = xbytes + size_t(stages) * stage_bytes;
-        const int occ = occupancy(tpr_fn(dt, NT, px), NT, p->smem, dev.present, cps_t);
+        const int occ = occupancy(tpr_fn(dt, NT, px, scal), NT, p->smem, dev.present, cps_t);
         p->ctas_per_sm = std::min(cps_t, occ);
         p->grid[1] = std::max<int64_t>(1, std::min<int64_t>(ceil_div(R, NT), int64_t(dev.sms) * p->ctas_per_sm));
-        p->chain[1] = ceil_div(C / 4, 2);
-        p->depth[1] = 3;
+        p->chain[1] = scal ? ceil_div(C, 2) : ceil_div(C / 4, 2);
+        p->depth[1] = scal ? 2 : 3;
         p->path_ok[1] = (dt == DT_I32) || bound_ok(p->chain[1] + p->depth[1]);
         p->grid[0] = fb_grid; p->chain[0] = fb_chain; p->depth[0] = fb_depth; p->path_ok[0] = fb_ok;
         if (!p->path_ok[1]) return ADAPTIC_ERR_UNSUPPORTED;
@@ -886,8 +890,8 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
         }
     } else switch (p->variant) {
         case ADAPTIC_V_MV_TPR:
-            if (vec) {
-                fn = tpr_fn(dt, p->lanes, px);
+            if (vec || mis) {
+                fn = tpr_fn(dt, p->lanes, px, mis);
                 smem = p->smem;
                 cudaError_t e = ensure_smem_attr(fn, smem);
                 if (e != cudaSuccess) return cuda_fail(e);
@@ -1048,11 +1052,82 @@ adaptic_status adaptic_run(adaptic_plan_t p, const void* A, const void* x, void*
         else vec = aligned(A, 16) && aligned(x, 16);
     }
     // misaligned-row kernels: any 4-byte aligned A; DOT's b must share A's address modulo 16
-    const bool mis = !vec && p->mis &&
-                     (p->op != ADAPTIC_OP_DOT ||   // TMV / MV: any 4-byte alignment
-                      ((reinterpret_cast<uintptr_t>(A) - reinterpret_cast<uintptr_t>(x)) & 15u) == 0);
+    bool mis = !vec && p->mis &&
+               (p->op != ADAPTIC_OP_DOT ||   // TMV / MV: any 4-byte alignment
+                ((reinterpret_cast<uintptr_t>(A) - reinterpret_cast<uintptr_t>(x)) & 15u) == 0);
+    if (mis && p->variant == ADAPTIC_V_MV_TPR)   // bulk copies of row tiles: 16-byte aligned bases
+        mis = aligned(A, 16) && (p->op != ADAPTIC_OP_DOT || aligned(x, 16));
     if (!p->path_ok[(vec || mis) ? 1 : 0]) return ADAPTIC_ERR_MISALIGNED;   // scalar path would break the error bound
     return launch(p, A, x, y, stream, vec, mis);
+}
+
+// ---- batched issue over concurrent streams (per host thread, per device)
+namespace {
+constexpr int kMaxBatchStreams = 8;
+struct StreamPool {
+    int dev = -1;
+    cudaStream_t side[kMaxBatchStreams - 1] = {};
+    cudaEvent_t fork = nullptr, join[kMaxBatchStreams - 1] = {};
+};
+thread_local StreamPool g_pools[8];
+
+cudaError_t pool_for_current_device(StreamPool** out) {
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    if (dev < 0 || dev >= 8) return cudaErrorInvalidDevice;
+    StreamPool& P = g_pools[dev];
+    if (P.dev != dev) {
+        for (int i = 0; i < kMaxBatchStreams - 1; ++i) {
+            if ((e = cudaStreamCreateWithFlags(&P.side[i], cudaStreamNonBlocking)) != cudaSuccess) return e;
+            if ((e = cudaEventCreateWithFlags(&P.join[i], cudaEventDisableTiming)) != cudaSuccess) return e;
+        }
+        if ((e = cudaEventCreateWithFlags(&P.fork, cudaEventDisableTiming)) != cudaSuccess) return e;
+        P.dev = dev;
+    }
+    *out = &P;
+    return cudaSuccess;
+}
+}  // namespace
+
+adaptic_status adaptic_run_batch(int32_t n, const adaptic_plan_t* plans, const void* const* A,
+                                 const void* const* x, void* const* y, int32_t streams, void* stream_) {
+    if (n < 0 || streams < 1 || streams > kMaxBatchStreams) return ADAPTIC_ERR_INVALID_ARG;
+    if (n == 0) return ADAPTIC_OK;
+    if (!plans || !A || !x || !y) return ADAPTIC_ERR_INVALID_ARG;
+    for (int32_t i = 0; i < n; ++i) {                   // all-or-nothing: validate before issuing
+        if (!plans[i]) return ADAPTIC_ERR_INVALID_ARG;
+        const adaptic_status st = check_run(plans[i], A[i], x[i], y[i]);
+        if (st != ADAPTIC_OK) return st;
+    }
+    cudaStream_t stream = static_cast<cudaStream_t>(stream_);
+    const int k = std::min<int>(streams, n);
+    if (k == 1) {
+        for (int32_t i = 0; i < n; ++i) {
+            const adaptic_status st = adaptic_run(plans[i], A[i], x[i], y[i], stream_);
+            if (st != ADAPTIC_OK) return st;
+        }
+        return ADAPTIC_OK;
+    }
+    StreamPool* P = nullptr;
+    cudaError_t e = pool_for_current_device(&P);
+    if (e != cudaSuccess) return cuda_fail(e);
+    if ((e = cudaEventRecord(P->fork, stream)) != cudaSuccess) return cuda_fail(e);
+    for (int j = 0; j < k - 1; ++j)
+        if ((e = cudaStreamWaitEvent(P->side[j], P->fork, 0)) != cudaSuccess) return cuda_fail(e);
+    adaptic_status st = ADAPTIC_OK;
+    for (int32_t i = 0; i < n && st == ADAPTIC_OK; ++i) {
+        int lane = i % k;
+        for (int32_t q = 0; q < i; ++q)                   // a plan's workspace serialises its runs:
+            if (plans[q] == plans[i] && plans[i]->ws_bytes > 0) { lane = q % k; break; }   // same stream
+        cudaStream_t s = lane == 0 ? stream : P->side[lane - 1];
+        st = adaptic_run(plans[i], A[i], x[i], y[i], s);
+    }
+    for (int j = 0; j < k - 1; ++j) {                    // join (also after a failure)
+        if ((e = cudaEventRecord(P->join[j], P->side[j])) != cudaSuccess) return cuda_fail(e);
+        if ((e = cudaStreamWaitEvent(stream, P->join[j], 0)) != cudaSuccess) return cuda_fail(e);
+    }
+    return st;
 }
 
 adaptic_status adaptic_run_host(adaptic_plan_t p, const void* A_host, const void* x_host, void* y_host,

@@ -49,19 +49,20 @@ void* cta_fn(int dtype, int NT, int RB, int U, bool vec, int xm, bool pipe) {
     return dtype == DT_F32 ? cta_fn_t<float>(NT, RB, U, vec, xm, pipe) : cta_fn_t<uint32_t>(NT, RB, U, vec, xm, pipe);
 }
 
-template <class T>
-static void* tpr_fn_t(int NT, bool px) {
+template <class T, bool SC>
+static void* tpr_fn_s(int NT, bool px) {
     switch (NT) {
-        case 128: return px ? reinterpret_cast<void*>(&mv_tpr_kernel<T, 128, true>)
-                            : reinterpret_cast<void*>(&mv_tpr_kernel<T, 128, false>);
-        case 256: return px ? reinterpret_cast<void*>(&mv_tpr_kernel<T, 256, true>)
-                            : reinterpret_cast<void*>(&mv_tpr_kernel<T, 256, false>);
+        case 128: return px ? reinterpret_cast<void*>(&mv_tpr_kernel<T, 128, true, SC>)
+                            : reinterpret_cast<void*>(&mv_tpr_kernel<T, 128, false, SC>);
+        case 256: return px ? reinterpret_cast<void*>(&mv_tpr_kernel<T, 256, true, SC>)
+                            : reinterpret_cast<void*>(&mv_tpr_kernel<T, 256, false, SC>);
         default: return nullptr;
     }
 }
 
-void* tpr_fn(int dtype, int NT, bool px) {
-    return dtype == DT_F32 ? tpr_fn_t<float>(NT, px) : tpr_fn_t<uint32_t>(NT, px);
+void* tpr_fn(int dtype, int NT, bool px, bool scal) {
+    if (dtype == DT_F32) return scal ? tpr_fn_s<float, true>(NT, px) : tpr_fn_s<float, false>(NT, px);
+    return scal ? tpr_fn_s<uint32_t, true>(NT, px) : tpr_fn_s<uint32_t, false>(NT, px);
 }
 
 }  // namespace adaptic

@@ -33,7 +33,7 @@ void* group_fn_i32(int G, int U, bool vec, int xmode);
 void* tmv_fn_f32(int LR, int U, bool vec, int NT);
 void* tmv_fn_i32(int LR, int U, bool vec, int NT);
 void* cta_fn(int dtype, int NT, int RB, int U, bool vec, int xmode, bool pipe);
-void* tpr_fn(int dtype, int NT, bool perrowx);
+void* tpr_fn(int dtype, int NT, bool perrowx, bool scal = false);   // scal: C % 4 != 0 rows
 
 // Misaligned-row MV/DOT (mv_mis_kernels.cuh; C % 4 != 0, 128-bit body + scalar head/tail):
 //   group: (const T* A, const T* X, T* y, int64_t R, int64_t C), RB = max(1, 4/U)

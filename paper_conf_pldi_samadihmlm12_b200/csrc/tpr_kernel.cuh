@@ -11,6 +11,12 @@
 // STAGES-deep ring guarded by mbarriers, and each thread then reduces its own
 // row out of shared memory.  The rotation k' = (k + t) mod (C/4) makes the
 // 128-bit shared loads of 8 consecutive threads hit distinct banks.
+// SCAL (C % 4 != 0): a tile is still a contiguous NT*C*4-byte block whose size is a
+// multiple of 16 (NT*4 = 512 or 1024), so the bulk copies stay 16-byte granular;
+// only the last, partial tile copies its < 16-byte remainder with plain loads, and
+// x (C*4 bytes) is staged by the threads.  Rows are read as 32-bit words; thread t
+// starts at word t*C + rot*t with rot = (C odd ? 0 : 1), so the C+rot words between
+// neighbouring threads are odd and the 32 lanes hit 32 distinct banks.
 #pragma once
 
 #include "common.cuh"
@@ -20,7 +26,7 @@ namespace adaptic {
 constexpr int TPR_MAX_STAGES = 8;
 
 // Dynamic smem layout: [x: C elems][stage 0: NT*C (+ NT*C for DOT's b)] ... ; 16B aligned.
-template <class T, int NT, bool PERROWX>
+template <class T, int NT, bool PERROWX, bool SCAL = false>
 __global__ void __launch_bounds__(NT)
 mv_tpr_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restrict__ y,
               int64_t R, int64_t C, int stages)
@@ -53,29 +59,69 @@ mv_tpr_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restrict__ 
         const int64_t tile = blockIdx.x + i * gridDim.x;
         const int64_t r0 = tile * NT;
         const int64_t nrows = min(int64_t(NT), R - r0);
-        const uint32_t bytes = uint32_t(nrows * C * sizeof(T));
+        const uint32_t bytes = uint32_t(nrows * C * sizeof(T)) & (SCAL ? ~15u : ~0u);
         T* dst = ring + size_t(i % stages) * stage_elems;
         uint64_t* bar = &full[i % stages];
         mbar_arrive_expect_tx(bar, PERROWX ? 2 * bytes : bytes);
-        bulk_g2s(dst, A + r0 * C, bytes, bar);
-        if (PERROWX) bulk_g2s(dst + tile_elems, X + r0 * C, bytes, bar);
+        if (bytes) {
+            bulk_g2s(dst, A + r0 * C, bytes, bar);
+            if (PERROWX) bulk_g2s(dst + tile_elems, X + r0 * C, bytes, bar);
+        }
     };
 
     if (tid == 0) {
-        if (!PERROWX) {
+        if (!PERROWX && !SCAL) {
             mbar_arrive_expect_tx(&xbar, uint32_t(C * sizeof(T)));
             bulk_g2s_keep(xs, X, uint32_t(C * sizeof(T)), &xbar);
         }
         const int64_t pre = min(int64_t(stages), my_tiles);
         for (int64_t i = 0; i < pre; ++i) issue(i);
     }
-    if (!PERROWX) mbar_wait(&xbar, 0);
+    if (!PERROWX && !SCAL) mbar_wait(&xbar, 0);
+    if (!PERROWX && SCAL) {
+        for (int64_t c = tid; c < C; c += NT) xs[c] = ld_x(X + c);
+        __syncthreads();
+    }
 
     const V* xv = reinterpret_cast<const V*>(xs);
     for (int64_t i = 0; i < my_tiles; ++i) {
         const int st = int(i % stages);
         mbar_wait(&full[st], uint32_t((i / stages) & 1));
         const int64_t r0 = (blockIdx.x + i * gridDim.x) * int64_t(NT);
+        if constexpr (SCAL) {
+            T* stg = ring + size_t(st) * stage_elems;
+            const int64_t nel = min(int64_t(NT), R - r0) * C;
+            const int64_t bulk = int64_t((uint64_t(nel) * sizeof(T)) & ~uint64_t(15)) / int64_t(sizeof(T));
+            if (bulk < nel) {                 // last partial tile: < 16-byte remainder
+                for (int64_t e = bulk + tid; e < nel; e += NT) {
+                    stg[e] = A[r0 * C + e];
+                    if (PERROWX) stg[tile_elems + e] = X[r0 * C + e];
+                }
+                __syncthreads();
+            }
+            const T* ar = stg + size_t(tid) * C;
+            const T* br = PERROWX ? stg + tile_elems + size_t(tid) * C : xs;
+            if (r0 + tid < R) {
+                const int Ci = int(C);
+                T acc0 = T(0), acc1 = T(0);
+                int k = (Ci & 1) ? 0 : tid % Ci;
+                int n = 0;
+                for (; n + 1 < Ci; n += 2) {
+                    const int k1 = (k + 1 == Ci) ? 0 : k + 1;
+                    acc0 = mac(ar[k], br[k], acc0);
+                    acc1 = mac(ar[k1], br[k1], acc1);
+                    k = (k1 + 1 == Ci) ? 0 : k1 + 1;
+                }
+                if (n < Ci) acc0 = mac(ar[k], br[k], acc0);
+                y[r0 + tid] = acc0 + acc1;
+            }
+            __syncthreads();
+            if (tid == 0 && i + stages < my_tiles) {
+                fence_proxy_async();
+                issue(i + stages);
+            }
+            continue;
+        }
         const V* av = reinterpret_cast<const V*>(ring + size_t(st) * stage_elems) + size_t(tid) * c4;
         const V* bv = PERROWX ? reinterpret_cast<const V*>(ring + size_t(st) * stage_elems + tile_elems) + size_t(tid) * c4
                               : xv;

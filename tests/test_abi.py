@@ -27,7 +27,7 @@ def test_library_exports_every_declared_symbol():
     for name in declared:
         assert hasattr(lib, name), name
     assert sorted(L.SYMBOLS) == declared
-    assert L.lib().adaptic_abi_version() == 4
+    assert L.lib().adaptic_abi_version() == 5
 
 
 def test_enums_match_header():
@@ -165,3 +165,19 @@ def test_plan_is_o1_host_only():
         adaptic.plan("tmv", 8192, 8192)
     dt = (time.perf_counter() - t) / 2000
     assert dt < 2e-3, dt
+
+
+def test_run_batch_host_checks():
+    lib = L.lib()
+    VP = ctypes.c_void_p
+    one = (VP * 1)(VP(None))
+    assert lib.adaptic_run_batch(0, None, None, None, None, 1, None) == L.OK
+    assert lib.adaptic_run_batch(-1, one, one, one, one, 1, None) == L.ERR_INVALID_ARG
+    assert lib.adaptic_run_batch(1, one, one, one, one, 0, None) == L.ERR_INVALID_ARG
+    assert lib.adaptic_run_batch(1, one, one, one, one, 9, None) == L.ERR_INVALID_ARG
+    assert lib.adaptic_run_batch(1, one, one, one, one, 2, None) == L.ERR_INVALID_ARG   # NULL plan
+    p = adaptic.plan("mv", 16, 16)
+    b = L.Batch([(p, 0x10000000, 0x20000000, 0x10000040)])                          # y inside A
+    with pytest.raises(adaptic.AdapticError) as e:
+        b.run(2)
+    assert e.value.status == L.ERR_ALIAS

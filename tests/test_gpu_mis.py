@@ -163,3 +163,26 @@ def test_tmv_misaligned_base_and_output():
                     assert e.status == L.ERR_UNSUPPORTED
                     continue
                 check(yb[off:off + R].cpu().numpy(), oracle.tmv(B, x), "f32", f"tmv off {off} {R}x{C} {v}")
+
+
+@pytest.mark.parametrize("dt", ["f32", "i32"])
+def test_tpr_rows_off_the_16_byte_grid(dt):
+    """MV_TPR with C % 4 != 0: tiles are still 16-byte-granular bulk copies (the last,
+    partial tile's remainder by plain loads), rows read as 32-bit words."""
+    npdt = np.float32 if dt == "f32" else np.int32
+    for R, C in [(1, 5), (3, 17), (255, 9), (256, 13), (1000, 65), (4097, 33), (100003, 7), (777, 2)]:
+        for op in ("mv", "dot"):
+            A = synth.matrix(R, C, "mv", npdt, "uniform", 31 + R + C)
+            X = (synth.matrix(R, C, "mv", npdt, "uniform", 32 + R) if op == "dot"
+                 else synth.vector(C, npdt, "uniform", 33 + C))
+            for p in (None, [128, 0, 0, 2], [256, 0, 0, 4]):
+                try:
+                    plan = adaptic.plan(op, R, C, dt, variant="MV_TPR", params=p)
+                except adaptic.AdapticError as e:
+                    assert e.status == L.ERR_UNSUPPORTED
+                    continue
+                assert plan.describe()["mis"]
+                fn = adaptic.mv if op == "mv" else adaptic.dot
+                y = fn(torch.from_numpy(A).to(DEV), torch.from_numpy(X).to(DEV), variant="MV_TPR", params=p)
+                ref = oracle.mv(A, X) if op == "mv" else oracle.dot(A, X)
+                check(y.cpu().numpy(), ref, dt, f"tpr {op} {dt} {R}x{C} {p}")

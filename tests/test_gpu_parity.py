@@ -341,7 +341,7 @@ def test_workspace_stays_zero_and_reruns_are_identical():
     for y in ys[1:]:
         assert np.array_equal(y, ys[0])
     check(ys[0], oracle.mv(A, x), "f32")
-    ws = adaptic.ops._cache[(L.OP_MV, R, C, L.F32, "MV_SPLIT", None, 0, stream)][1]
+    ws = adaptic.ops._cache[(L.OP_MV, R, C, L.F32, "MV_SPLIT", None, 0, stream, 1)][1]
     cnt_off = plan.describe()["workspace_bytes"] - R * 4
     assert int(ws[cnt_off:].sum().item()) == 0                  # tickets re-armed
 
@@ -463,3 +463,38 @@ def test_config4_tmv_1024x16M_sampled():
     idx = _sample_rows(R, 12)
     sub = M.view(C, R)[:, torch.from_numpy(idx).to(DEV)].t().contiguous().cpu().numpy()
     check(y[torch.from_numpy(idx).to(DEV)].cpu().numpy(), oracle.mv(sub, x.cpu().numpy()), "f32", "config4")
+
+
+def test_run_batch_equals_single_runs():
+    """adaptic_run_batch: independent problems on 1..4 concurrent streams give exactly the
+    single-call results (same plans, same kernels); a plan with a workspace repeated in a
+    batch stays on one stream; validation is all-or-nothing."""
+    dev = torch.device(DEV)
+    stream = torch.cuda.current_stream().cuda_stream
+    shapes = [("mv", 8, 1 << 20), ("tmv", 1 << 16, 64), ("mv", 4096, 1001), ("tmv", 9, 100000), ("dot", 3, 1 << 18)]
+    items, refs = [], []
+    for op, R, C in shapes:
+        M, X = make_inputs(op, R, C, "f32")
+        Md, Xd = torch.from_numpy(M).to(dev), torch.from_numpy(X).to(dev)
+        plan = adaptic.get_plan({"mv": L.OP_MV, "tmv": L.OP_TMV, "dot": L.OP_DOT}[op], R, C, L.F32, dev, "AUTO", None, stream)
+        y = torch.full((R,), float("nan"), device=dev)
+        items.append((plan, Md.data_ptr(), Xd.data_ptr(), y.data_ptr(), Md, Xd, y))
+        refs.append(run_gpu(op, M, X))
+    # the same split plan twice (workspace): second copy with its own output
+    p0 = items[0]
+    y2 = torch.full_like(p0[6], float("nan"))
+    items.append((p0[0], p0[1], p0[2], y2.data_ptr(), p0[4], p0[5], y2))
+    refs.append(refs[0])
+    for k in (1, 2, 3, 4):
+        for it in items:
+            it[6].fill_(float("nan"))
+        L.Batch([it[:4] for it in items]).run(k, stream)
+        for it, ref in zip(items, refs):
+            assert np.array_equal(it[6].cpu().numpy(), ref), k
+    bad = list(items[:2]) + [(items[2][0], items[2][1], items[2][2], items[2][1])]     # y aliases A
+    items[0][6].fill_(7.0)
+    with pytest.raises(adaptic.AdapticError) as e:
+        L.Batch([it[:4] for it in bad]).run(2, stream)
+    assert e.value.status == L.ERR_ALIAS
+    torch.cuda.synchronize()
+    assert (items[0][6] == 7.0).all()                    # nothing was issued

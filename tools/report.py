@@ -19,17 +19,25 @@ def main():
     ap.add_argument("--peak", type=float, default=None, help="HBM GB/s (default MEASURED_PEAKS.json)")
     ap.add_argument("--md", default=None)
     ap.add_argument("--min-bytes", type=float, default=256 * 2 ** 20, help="gate applies at >= this many bytes")
+    ap.add_argument("--best-from", nargs="*", default=[],
+                    help="sweeps whose fixed-variant runs give 'best fixed' (AUTO is taken from the inputs)")
     a = ap.parse_args()
     peak = a.peak
     if peak is None:
         p = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "MEASURED_PEAKS.json")
         peak = json.load(open(p))["hbm_gbs"] if os.path.exists(p) else 6650.0
-    rows = []
-    for path in a.inputs:
-        import gzip
-        op = gzip.open if path.endswith(".gz") else open
-        with op(path, "rt") as f:
-            rows += [json.loads(l) for l in f if l.strip()]
+    import gzip
+
+    def load(paths):
+        out = []
+        for path in paths:
+            op = gzip.open if path.endswith(".gz") else open
+            with op(path, "rt") as f:
+                out += [json.loads(l) for l in f if l.strip()]
+        return out
+    rows = load(a.inputs)
+    if a.best_from:
+        rows = [r for r in rows if r["req"] == "AUTO"] + [r for r in load(a.best_from) if r["req"] != "AUTO"]
     by = collections.defaultdict(list)
     for r in rows:
         by[(r["op"], r["dtype"], r["R"], r["C"])].append(r)

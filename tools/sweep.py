@@ -75,7 +75,8 @@ def grids(op, R, C):
         if C <= 256:
             for nt in (128, 256):
                 for st in (2, 4, 8):
-                    out.append(("MV_TPR", [nt, 0, 0, st]))
+                    for cps in (0, 1):
+                        out.append(("MV_TPR", [nt, 0, cps, st]))
     else:
         rv = R // 4 if R % 4 == 0 else R
         for u in (2, 4, 8):
