@@ -44,6 +44,7 @@ struct adaptic_plan_s {
     size_t smem;           // dynamic shared memory bytes (TPR ring, or staged x)
     int block;
     bool vec_shape;        // C % 4 == 0 (MV/DOT) or R % 4 == 0 (TMV)
+    bool flat;             // TMV_REGTILE with R <= 64, R % 4 != 0: the flat-stream kernel
     bool mis;              // MV/DOT with C % 4 != 0: index 1 describes the misaligned-row
                            // kernels (128-bit body + scalar head/tail, mv_mis_kernels.cuh)
     int64_t grid[2];       // [scalar, vector] instance
@@ -212,6 +213,7 @@ int heuristic_variant(int op, int64_t R, int64_t C, int sms) {
         return ADAPTIC_V_MV_SPLIT;
     }
     if (op == ADAPTIC_OP_TMV) {
+        if (R % 4 != 0 && R <= TMV_FLAT_MAX_R) return ADAPTIC_V_TMV_REGTILE;     // flat stream
         const int64_t rv = (R % 4 == 0) ? R / 4 : R;
         if (rv >= int64_t(sms) * 512 && C <= 4096) return ADAPTIC_V_TMV_COL;
         if (rv <= 256) return ADAPTIC_V_TMV_REGTILE;
@@ -312,11 +314,18 @@ adaptic_status derive_multi(adaptic_plan_s* p, const int32_t* params, const DevI
     }
     if (op == ADAPTIC_OP_MV && (v == ADAPTIC_V_MV_CPR || v == ADAPTIC_V_MV_SPLIT)) {
         const int NT = 256, RB = 8 / K;
+        const int64_t nvr = p->vec_shape ? C / 4 : C;
         int U = par(ADAPTIC_P_UNROLL);
-        if (U <= 0) U = 2;
+        if (U <= 0) U = nvr >= 2 * NT ? 2 : 1;             // short rows: do not idle half the CTA
         if (U != 1 && U != 2) return ADAPTIC_ERR_INVALID_ARG;
+        // x of all K vectors in shared memory when small (param XSMEM: 1 off, 2 on)
+        const int xreq = par(ADAPTIC_P_XSMEM);
+        const bool xs = xreq == 2 ? (K * C * 4 <= kXsMaxBytes) : (xreq != 1 && K * C * 4 <= kXsAutoBytes * 2);
+        if (xreq == 2 && !xs) return ADAPTIC_ERR_UNSUPPORTED;
+        p->xmode = xs ? 1 : 0;
+        p->smem = xs ? size_t(K) * size_t(C) * 4 : 0;
         int cps = par(ADAPTIC_P_CTAS_PER_SM);
-        if (cps <= 0) cps = occupancy(mmv_cta_fn(K, U, p->vec_shape), NT, 0, dev.present, 2048 / NT);
+        if (cps <= 0) cps = occupancy(mmv_cta_fn(K, U, p->vec_shape, xs), NT, p->smem, dev.present, 2048 / NT);
         p->lanes = NT; p->unroll = U; p->block = NT; p->rb = RB; p->ctas_per_sm = cps;
         const int64_t slots = int64_t(dev.sms) * cps;
         const int64_t groups = ceil_div(R, RB);
@@ -659,6 +668,31 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
     // R % 4 != 0: the misaligned-row kernel (two aligned loads + funnel shift) keeps the
     // stream 128-bit over ceil(R/4) output vectors; it handles any B / y alignment, so no
     // scalar path is planned for these shapes
+    p->flat = false;
+    if (!p->vec_shape && v == ADAPTIC_V_TMV_REGTILE && R <= TMV_FLAT_MAX_R) {
+        // few outputs off the 16-byte grid: stream B as one flat array (tmv_flat_kernel.cuh)
+        int U = par(ADAPTIC_P_UNROLL);
+        if (U <= 0) U = 4;
+        if (U != 2 && U != 4 && U != 8) return ADAPTIC_ERR_INVALID_ARG;
+        const int NTa = (TMV_FLAT_NT / int(R)) * int(R);
+        int cps = par(ADAPTIC_P_CTAS_PER_SM);
+        if (cps <= 0) cps = occupancy(tmv_flat_fn(dt, U), TMV_FLAT_NT, 0, dev.present, 4);
+        const int64_t slots = int64_t(dev.sms) * cps;
+        const int64_t nvec = ceil_div(R * C, 4) + 1;
+        const int64_t G = std::max<int64_t>(1, std::min<int64_t>(slots, ceil_div(nvec, int64_t(NTa) * U)));
+        const int64_t iters = ceil_div(nvec, G * NTa);
+        p->flat = true; p->mis = true;
+        p->lanes = NTa; p->unroll = U; p->block = TMV_FLAT_NT; p->ctas_per_sm = cps; p->splits = 1;
+        p->grid[1] = G;
+        p->chain[1] = fold_chain(iters);
+        p->depth[1] = 2 + NTa / R + ceil_div(G, NTa / R) + NTa / R + 1;
+        p->path_ok[1] = (dt == DT_I32) || bound_ok(p->chain[1] + p->depth[1]);
+        if (!p->path_ok[1]) return ADAPTIC_ERR_UNSUPPORTED;
+        const size_t part = ((size_t(G) * size_t(R) * 4 + 255) / 256) * 256;
+        p->cnt_off = part;
+        p->ws_bytes = part + 256;
+        return ADAPTIC_OK;
+    }
     const bool tmis = !p->vec_shape && R >= 8;
     p->mis = tmis;
     const int64_t rv1 = p->vec_shape ? R / 4 : tmis ? ceil_div(R, 4) : R;
@@ -868,7 +902,7 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
         const int K = p->nvec;
         if (p->op == ADAPTIC_OP_TMV) fn = tmmv_fn(K, p->lanes, p->unroll, vec);
         else if (p->variant == ADAPTIC_V_MV_SUBWARP || p->variant == ADAPTIC_V_MV_WPR) fn = mmv_group_fn(K, p->lanes, p->unroll, vec);
-        else fn = mmv_cta_fn(K, p->unroll, vec);
+        else { fn = mmv_cta_fn(K, p->unroll, vec, p->xmode == 1); smem = p->smem; }
         if (p->op == ADAPTIC_OP_MV && (p->variant == ADAPTIC_V_MV_SUBWARP || p->variant == ADAPTIC_V_MV_WPR)) {
             args6[0] = &A; args6[1] = &X; args6[2] = &y; args6[3] = &R; args6[4] = &C;
             args = args6;
@@ -921,6 +955,13 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
             args = args9;
             break;
         default:
+            if (p->flat && mis) {
+                fn = tmv_flat_fn(dt, p->unroll);
+                args7[0] = &A; args7[1] = &X; args7[2] = &y; args7[3] = &R; args7[4] = &C;
+                args7[5] = &part; args7[6] = &cnt;
+                args = args7;
+                break;
+            }
             fn = mis ? tmv_mis_fn(dt, p->lanes, p->unroll) : tmv_fn(dt, p->lanes, p->unroll, vec, p->block);
             args8[0] = &A; args8[1] = &X; args8[2] = &y; args8[3] = &R; args8[4] = &C;
             args8[5] = &S; args8[6] = &part; args8[7] = &cnt;

@@ -1,6 +1,6 @@
 // Instances of the multi-vector kernels (mmv_kernels.cuh), fp32, K in {2, 4, 8}:
 //   group: G in {1,2,4,8,16,32} x U in {1,2,4} (K*U <= 16) x VEC, RB = 2
-//   cta  : NT = 256, U in {1, 2} x VEC
+//   cta  : NT = 256, U in {1, 2} x VEC x x-in-shared-memory
 //   tmmv : LR in {1,...,256} x VEC x U in {2, 4} (4 only for K <= 4), NT = 256
 #include "mmv_kernels.cuh"
 
@@ -31,10 +31,12 @@ static void* mg_g(int G, int U) {
 }
 
 template <int K, bool VEC>
-static void* mc_u(int U) {
-    switch (U) {
-        case 1: return reinterpret_cast<void*>(&mmv_cta_kernel<K, 256, 1, VEC>);
-        case 2: return reinterpret_cast<void*>(&mmv_cta_kernel<K, 256, 2, VEC>);
+static void* mc_u(int U, bool xs) {
+    switch (U * 2 + (xs ? 1 : 0)) {
+        case 2: return reinterpret_cast<void*>(&mmv_cta_kernel<K, 256, 1, VEC, false>);
+        case 3: return reinterpret_cast<void*>(&mmv_cta_kernel<K, 256, 1, VEC, true>);
+        case 4: return reinterpret_cast<void*>(&mmv_cta_kernel<K, 256, 2, VEC, false>);
+        case 5: return reinterpret_cast<void*>(&mmv_cta_kernel<K, 256, 2, VEC, true>);
         default: return nullptr;
     }
 }
@@ -71,7 +73,7 @@ static void* mt_l(int LR, int U) {
     }
 
 void* mmv_group_fn(int K, int G, int U, bool vec) { ADAPTIC_K(mg_g, G, U) }
-void* mmv_cta_fn(int K, int U, bool vec) { ADAPTIC_K(mc_u, U) }
+void* mmv_cta_fn(int K, int U, bool vec, bool xs) { ADAPTIC_K(mc_u, U, xs) }
 void* tmmv_fn(int K, int LR, int U, bool vec) { ADAPTIC_K(mt_l, LR, U) }
 #undef ADAPTIC_K
 

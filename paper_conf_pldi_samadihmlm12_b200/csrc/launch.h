@@ -46,6 +46,11 @@ void* mis_cta_fn_i32(int NT, int U, int xmode);
 //   (const T* B, const T* X, T* y, int64_t R, int64_t C, int S, T* part, unsigned* cnt)
 void* tmv_mis_fn_f32(int LR, int U);
 void* tmv_mis_fn_i32(int LR, int U);
+// Flat-stream TMV for few outputs (tmv_flat_kernel.cuh; R <= 64, R % 4 != 0), NT = 256:
+//   (const T* B, const T* X, T* y, int64_t R, int64_t C, T* part, unsigned* cnt)
+constexpr int TMV_FLAT_NT = 256;
+constexpr int TMV_FLAT_MAX_R = 64;
+void* tmv_flat_fn(int dtype, int U);
 
 // Multi-vector MV / TMV (mmv_kernels.cuh), fp32, K in {2, 4, 8}; X is K x C, Y is K x R:
 //   group: (const float* A, const float* X, float* Y, int64_t R, int64_t C), rows of <= G*U vectors
@@ -53,7 +58,7 @@ void* tmv_mis_fn_i32(int LR, int U);
 //   tmmv : (B, X, Y, R, C, int S, float* part, unsigned* cnt), NT = 256, U in {2, 4}
 constexpr int MMV_GROUP_RB = 2;
 void* mmv_group_fn(int K, int G, int U, bool vec);
-void* mmv_cta_fn(int K, int U, bool vec);
+void* mmv_cta_fn(int K, int U, bool vec, bool xs);   // xs: K*C*4 bytes of x staged in smem
 void* tmmv_fn(int K, int LR, int U, bool vec);
 
 // BLAS-1 reductions (blas1_kernels.cuh), fp32 input, one translation unit per operator:

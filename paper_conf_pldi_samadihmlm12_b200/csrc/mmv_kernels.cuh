@@ -86,12 +86,25 @@ mmv_group_kernel(const float* __restrict__ A, const float* __restrict__ X, float
 // ------------------------------------------------------------------ MV, CTA per RB rows (+ splits)
 // RB = 8 / K rows per CTA step share every x load (x traffic K/RB times the matrix
 // bytes instead of K); S CTAs per row group interleave in steps of NT*U vectors.
-template <int K, int NT, int U, bool VEC>
+// XS: the K x-vectors (K*C*4 bytes, small) are staged once per CTA in shared memory
+// (TMA bulk copy on the 128-bit path), so x reads leave L1/L2 alone.
+template <int K, int NT, int U, bool VEC, bool XS = false>
 __global__ void __launch_bounds__(NT)
 mmv_cta_kernel(const float* __restrict__ A, const float* __restrict__ X, float* __restrict__ Y,
                int64_t R, int64_t C, int S, float* __restrict__ ws_part, unsigned int* __restrict__ ws_cnt)
 {
     pdl_prologue();
+    if constexpr (XS) {
+        extern __shared__ __align__(128) unsigned char dyn_smem[];
+        __shared__ __align__(8) uint64_t xbar;
+        float* xs = reinterpret_cast<float*>(dyn_smem);
+        if (VEC) stage_to_smem(xs, X, uint32_t(K * C * 4), &xbar);
+        else {
+            for (int64_t i = threadIdx.x; i < K * C; i += NT) xs[i] = X[i];
+            __syncthreads();
+        }
+        X = xs;
+    }
     using E = typename ElemOf<float, VEC>::type;
     constexpr int W = VEC ? 4 : 1;
     constexpr int RB = (8 / K) > 0 ? 8 / K : 1;
@@ -132,7 +145,7 @@ mmv_cta_kernel(const float* __restrict__ A, const float* __restrict__ X, float* 
             for (int u = 0; u < U; ++u)
 #pragma unroll
                 for (int j = 0; j < K; ++j) {
-                    const E xv = ld_x(Xv + j * nv + b + tid + int64_t(NT) * u);
+                    const E xv = XS ? Xv[j * nv + b + tid + int64_t(NT) * u] : ld_x(Xv + j * nv + b + tid + int64_t(NT) * u);
 #pragma unroll
                     for (int i = 0; i < RB; ++i) emac(acc[i][j], a[i][u], xv);
                 }
@@ -151,7 +164,7 @@ mmv_cta_kernel(const float* __restrict__ A, const float* __restrict__ X, float* 
             for (int i = 0; i < RB; ++i) a[i] = ld_stream(Av + off[i] + v);
 #pragma unroll
             for (int j = 0; j < K; ++j) {
-                const E xv = ld_x(Xv + j * nv + v);
+                const E xv = XS ? Xv[j * nv + v] : ld_x(Xv + j * nv + v);
 #pragma unroll
                 for (int i = 0; i < RB; ++i) emac(acc[i][j], a[i], xv);
             }

@@ -131,7 +131,8 @@ TMV_FORCED = [("AUTO", None), ("TMV_COL", [0, 0, 0, 4]), ("TMV_COL", [0, 0, 0, 8
 def test_tmv_misaligned_rows_every_variant(dt):
     """R % 4 != 0: B's rows start at every alignment; two aligned loads + funnel shift."""
     npdt = np.float32 if dt == "f32" else np.int32
-    shapes = [(9, 33), (13, 1000), (63, 257), (129, 4099), (1023, 65), (5, 100003), (1001, 1001), (30, 7)]
+    shapes = [(9, 33), (13, 1000), (63, 257), (129, 4099), (1023, 65), (5, 100003), (1001, 1001), (30, 7),
+              (1, 1000), (2, 77), (3, 100000), (1, 1), (7, 3), (62, 1 << 16)]
 
     def case(R, C, v, p):
         B = synth.matrix(R, C, "tmv", npdt, "uniform", synth.seed(12, "A") + R + C)
