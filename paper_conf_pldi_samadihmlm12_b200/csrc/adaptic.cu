@@ -1057,13 +1057,13 @@ int adaptic_plan_describe(adaptic_plan_t p, char* buf, size_t cap) {
         tmp, sizeof(tmp),
         "{\"op\":\"%s\",\"dtype\":\"%s\",\"rows\":%lld,\"cols\":%lld,\"variant\":\"%s\",\"source\":\"%s\","
         "\"nvec\":%d,\"sms\":%d,\"lanes\":%d,\"unroll\":%d,\"rows_per_group\":%d,\"splits\":%d,\"block\":%d,"
-        "\"ctas_per_sm\":%d,\"stages\":%d,\"xmode\":%d,\"ilv\":%d,\"pipe\":%d,\"smem\":%zu,\"vec_shape\":%s,\"mis\":%s,"
+        "\"ctas_per_sm\":%d,\"stages\":%d,\"xmode\":%d,\"ilv\":%d,\"pipe\":%d,\"smem\":%zu,\"vec_shape\":%s,\"mis\":%s,\"flat\":%s,"
         "\"grid\":[%lld,%lld],\"chain\":[%lld,%lld],\"depth\":[%lld,%lld],\"path_ok\":[%s,%s],"
         "\"fallback_lanes\":%d,\"fallback_unroll\":%d,\"workspace_bytes\":%zu}",
         ops[p->op], p->dtype == ADAPTIC_F32 ? "f32" : "i32", (long long)p->R, (long long)p->C,
         kVariantNames[p->variant], src[p->source], p->nvec, p->sms, p->lanes, p->unroll, p->rb, p->splits, p->block,
         p->ctas_per_sm, p->stages, p->xmode, p->ilv, p->pipe, p->smem, p->vec_shape ? "true" : "false",
-        p->mis ? "true" : "false",
+        p->mis ? "true" : "false", p->flat ? "true" : "false",
         (long long)p->grid[0], (long long)p->grid[1], (long long)p->chain[0], (long long)p->chain[1],
         (long long)p->depth[0], (long long)p->depth[1], p->path_ok[0] ? "true" : "false",
         p->path_ok[1] ? "true" : "false", p->fb_lanes, p->fb_unroll, p->ws_bytes);
