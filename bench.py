@@ -50,6 +50,8 @@ def parse():
     ap.add_argument("--impl", choices=["adaptic", "reference"], default="adaptic")
     ap.add_argument("--workload", choices=["sweep", "rowshard", "splitk", "dot", "blas1", "config0", "multi", "bicgstab"], default="sweep")
     ap.add_argument("--variant", default="AUTO", help="force one variant (fixed-variant sweeps)")
+    ap.add_argument("--dtype", choices=["f32", "i32"], default="f32",
+                    help="element type of the MV/TMV/DOT workloads (i32: arithmetic modulo 2^32)")
     ap.add_argument("--streams", type=int, default=2,
                     help="the step's independent problems go through adaptic_run_batch on this many "
                          "concurrent streams (1 = one after another on one stream)")
@@ -173,7 +175,7 @@ def algo_bytes(op, R, C, nvec=1):
 class Problem:
     """One (op, R, C) instance, resident in HBM, with its selected plan."""
 
-    def __init__(self, op, R, C, cfg, variant="AUTO", shard=None, full=None, nvec=1):
+    def __init__(self, op, R, C, cfg, variant="AUTO", shard=None, full=None, nvec=1, dtype="f32"):
         import torch
         import synth
         import paper_conf_pldi_samadihmlm12_b200 as adaptic
@@ -182,22 +184,24 @@ class Problem:
         dev = torch.device("cuda", torch.cuda.current_device())
         Rf, Cf = full if full else (R, C)           # logical full problem (shards are slices)
         rows, cols = shard if shard else ((0, R), (0, C))
-        self.M = torch.empty(R * C, dtype=torch.float32, device=dev)
+        tdt = torch.int32 if dtype == "i32" else torch.float32
+        self.dtype = dtype
+        self.M = torch.empty(R * C, dtype=tdt, device=dev)
         layout = "tmv" if op == "tmv" else "mv"
         synth.device_matrix(self.M, Rf, Cf, layout, "uniform", synth.seed(cfg, "A"), rows=rows, cols=cols)
         if op in B1_OPS:
             self.X = torch.empty(0, dtype=torch.float32, device=dev)      # unused
         elif op == "dot":
-            self.X = torch.empty(R * C, dtype=torch.float32, device=dev)
+            self.X = torch.empty(R * C, dtype=tdt, device=dev)
             synth.device_matrix(self.X, Rf, Cf, "mv", "uniform", synth.seed(cfg, "b"), rows=rows, cols=cols)
         else:
-            self.X = torch.empty(C * nvec, dtype=torch.float32, device=dev)
+            self.X = torch.empty(C * nvec, dtype=tdt, device=dev)
             synth.device_vector(self.X, "uniform", synth.seed(cfg, "x"), start=cols[0])
         self.y = torch.empty(R * (4 if op == "b1all" else nvec),
-                             dtype=torch.int32 if op in ("iamax", "iamin") else torch.float32, device=dev)
+                             dtype=torch.int32 if op in ("iamax", "iamin") else tdt, device=dev)
         opc = L.OPS[op]
         self.stream = torch.cuda.current_stream().cuda_stream
-        self.plan = adaptic.get_plan(opc, R, C, L.F32, dev, variant, None, self.stream, nvec)
+        self.plan = adaptic.get_plan(opc, R, C, L.I32 if dtype == "i32" else L.F32, dev, variant, None, self.stream, nvec)
         self.desc = self.plan.describe()
         self.bytes = algo_bytes(op, R, C, nvec)
         self.ptrs = (self.M.data_ptr(), self.X.data_ptr(), self.y.data_ptr())
@@ -211,7 +215,7 @@ class Problem:
 
 def build_problems(args, world, rank):
     if args.workload == "sweep":
-        return [Problem(op, 1 << k, 1 << (26 - k), 1, args.variant)
+        return [Problem(op, 1 << k, 1 << (26 - k), 1, args.variant, dtype=args.dtype)
                 for k in range(3, 24) for op in ("mv", "tmv")], \
             {"workload": "configs[1]: TMV/MV fp32 shape sweep at 256 MiB, 8Mx8 .. 8192x8192 .. 8x8M, "
                          "both layouts, variant selector", "shapes": 42, "per_gpu": "full sweep (weak)"}
@@ -229,8 +233,8 @@ def build_problems(args, world, rank):
                          "(B1ALL, horizontal actor integration) fp32 at 256 MiB, N x L = 1x2^26 .. 2^22x16",
              "shapes": len(B1_SHAPES) * len(B1_OPS)}
     if args.workload == "dot":
-        return [Problem("dot", 1, 1 << k, 2, args.variant) for k in range(10, 31)], \
-            {"workload": "configs[2]: scalar product fp32 N=1, L=2^10..2^30", "shapes": 21}
+        return [Problem("dot", 1, 1 << k, 2, args.variant, dtype=args.dtype) for k in range(10, 31)], \
+            {"workload": f"configs[2]: scalar product {args.dtype} N=1, L=2^10..2^30", "shapes": 21}
     from paper_conf_pldi_samadihmlm12_b200.dist import shard_range
     if args.workload == "rowshard":
         R, C = 131072, 32768
@@ -361,7 +365,8 @@ def run_adaptic(args):
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": elapsed_ms / args.steps, "higher_is_better": True,
                 "scaling": "weak" if args.workload in ("sweep", "dot") else "strong",
-                "vs_baseline": None, "dtype": "f32", "data": "synthetic (seeded splitmix64, U[-1,1))",
+                "vs_baseline": None, "dtype": args.dtype,
+                "data": "synthetic (seeded splitmix64; fp32 U[-1,1), int32 U{-128..127})",
                 "config": dict(config, bytes_per_step_per_gpu=step_bytes, variant=args.variant,
                                l2=("every input >= 256 MiB > 126 MB L2 and problems alternate; no flush needed"
                                    if args.workload in ("sweep", "blas1") else
@@ -429,8 +434,8 @@ def measure_e2e(args, probs, world):
         sel = probs[:: max(1, len(probs) // k)]
     hosts = []
     for p in sel:
-        Mh = torch.empty(p.M.numel(), dtype=torch.float32, pin_memory=True)
-        Xh = torch.empty(p.X.numel(), dtype=torch.float32, pin_memory=True)
+        Mh = torch.empty(p.M.numel(), dtype=p.M.dtype, pin_memory=True)
+        Xh = torch.empty(p.X.numel(), dtype=p.X.dtype, pin_memory=True)
         Mh.copy_(p.M)
         Xh.copy_(p.X)
         yh = torch.empty(p.y.numel(), dtype=p.y.dtype, pin_memory=True)

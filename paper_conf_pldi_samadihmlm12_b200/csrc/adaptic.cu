@@ -671,18 +671,19 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
     p->flat = false;
     if (!p->vec_shape && v == ADAPTIC_V_TMV_REGTILE && R <= TMV_FLAT_MAX_R) {
         // few outputs off the 16-byte grid: stream B as one flat array (tmv_flat_kernel.cuh)
+        const int FNT = R <= TMV_FLAT_NT_SMALL_R ? 256 : 1024;
         int U = par(ADAPTIC_P_UNROLL);
         if (U <= 0) U = 4;
-        if (U != 2 && U != 4 && U != 8) return ADAPTIC_ERR_INVALID_ARG;
-        const int NTa = (TMV_FLAT_NT / int(R)) * int(R);
+        if (U != 2 && U != 4 && !(U == 8 && FNT == 256)) return ADAPTIC_ERR_INVALID_ARG;
+        const int NTa = (FNT / int(R)) * int(R);
         int cps = par(ADAPTIC_P_CTAS_PER_SM);
-        if (cps <= 0) cps = occupancy(tmv_flat_fn(dt, U), TMV_FLAT_NT, 0, dev.present, 4);
+        if (cps <= 0) cps = occupancy(tmv_flat_fn(dt, U, FNT), FNT, 0, dev.present, 2048 / FNT);
         const int64_t slots = int64_t(dev.sms) * cps;
         const int64_t nvec = ceil_div(R * C, 4) + 1;
         const int64_t G = std::max<int64_t>(1, std::min<int64_t>(slots, ceil_div(nvec, int64_t(NTa) * U)));
         const int64_t iters = ceil_div(nvec, G * NTa);
         p->flat = true; p->mis = true;
-        p->lanes = NTa; p->unroll = U; p->block = TMV_FLAT_NT; p->ctas_per_sm = cps; p->splits = 1;
+        p->lanes = NTa; p->unroll = U; p->block = FNT; p->ctas_per_sm = cps; p->splits = 1;
         p->grid[1] = G;
         p->chain[1] = fold_chain(iters);
         p->depth[1] = 2 + NTa / R + ceil_div(G, NTa / R) + NTa / R + 1;
@@ -956,7 +957,7 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
             break;
         default:
             if (p->flat && mis) {
-                fn = tmv_flat_fn(dt, p->unroll);
+                fn = tmv_flat_fn(dt, p->unroll, p->block);
                 args7[0] = &A; args7[1] = &X; args7[2] = &y; args7[3] = &R; args7[4] = &C;
                 args7[5] = &part; args7[6] = &cnt;
                 args = args7;

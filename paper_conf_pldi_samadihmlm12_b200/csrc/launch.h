@@ -46,11 +46,12 @@ void* mis_cta_fn_i32(int NT, int U, int xmode);
 //   (const T* B, const T* X, T* y, int64_t R, int64_t C, int S, T* part, unsigned* cnt)
 void* tmv_mis_fn_f32(int LR, int U);
 void* tmv_mis_fn_i32(int LR, int U);
-// Flat-stream TMV for few outputs (tmv_flat_kernel.cuh; R <= 64, R % 4 != 0), NT = 256:
+// Flat-stream TMV for few outputs (tmv_flat_kernel.cuh; R <= 256, R % 4 != 0), NT = 256
+// (R <= 64) or 1024 (R > 64):
 //   (const T* B, const T* X, T* y, int64_t R, int64_t C, T* part, unsigned* cnt)
-constexpr int TMV_FLAT_NT = 256;
-constexpr int TMV_FLAT_MAX_R = 64;
-void* tmv_flat_fn(int dtype, int U);
+constexpr int TMV_FLAT_MAX_R = 256;
+constexpr int TMV_FLAT_NT_SMALL_R = 64;     // R above this: 1024-thread CTAs
+void* tmv_flat_fn(int dtype, int U, int NT);
 
 // Multi-vector MV / TMV (mmv_kernels.cuh), fp32, K in {2, 4, 8}; X is K x C, Y is K x R:
 //   group: (const float* A, const float* X, float* Y, int64_t R, int64_t C), rows of <= G*U vectors
