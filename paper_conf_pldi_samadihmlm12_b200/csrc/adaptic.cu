@@ -213,7 +213,6 @@ int heuristic_variant(int op, int64_t R, int64_t C, int sms) {
         return ADAPTIC_V_MV_SPLIT;
     }
     if (op == ADAPTIC_OP_TMV) {
-        if (R % 4 != 0 && R <= TMV_FLAT_MAX_R) return ADAPTIC_V_TMV_REGTILE;     // flat stream
         const int64_t rv = (R % 4 == 0) ? R / 4 : R;
         if (rv >= int64_t(sms) * 512 && C <= 4096) return ADAPTIC_V_TMV_COL;
         if (rv <= 256) return ADAPTIC_V_TMV_REGTILE;
