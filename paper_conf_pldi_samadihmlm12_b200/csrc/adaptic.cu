@@ -285,6 +285,22 @@ adaptic_status derive_multi(adaptic_plan_s* p, const int32_t* params, const DevI
         const int64_t f = FOLD / U;
         return int64_t(U) * std::min<int64_t>(iters, f) + iters / f;
     };
+    if (op == ADAPTIC_OP_MV && v == ADAPTIC_V_MV_WPR && p->vec_shape && int64_t(K) * C * 4 <= MMV_WARP_SMEM &&
+        C / 4 > int64_t(32) * (K == 8 ? 2 : 4)) {
+        // medium rows: warp per row, all K x-vectors staged in shared memory (mmv_warp_kernel)
+        const int NT = 256, RB = 1, U = 2;
+        p->smem = size_t(K) * size_t(C) * 4;
+        p->xmode = 3;
+        int cps = par(ADAPTIC_P_CTAS_PER_SM);
+        if (cps <= 0) cps = occupancy(mmv_warp_fn(K), NT, p->smem, dev.present, 4);
+        p->lanes = 32; p->unroll = U; p->block = NT; p->rb = RB; p->ctas_per_sm = cps;
+        const int64_t iters = ceil_div(C / 4, int64_t(32) * U);
+        p->grid[1] = std::max<int64_t>(1, std::min<int64_t>(ceil_div(R, int64_t(RB) * (NT / 32)), int64_t(dev.sms) * cps));
+        p->chain[1] = chain_of(iters, U);
+        p->depth[1] = 2 + 5 + 1;
+        p->path_ok[1] = bound_ok(p->chain[1] + p->depth[1]);
+        return p->path_ok[1] ? ADAPTIC_OK : ADAPTIC_ERR_UNSUPPORTED;
+    }
     if (op == ADAPTIC_OP_MV && (v == ADAPTIC_V_MV_SUBWARP || v == ADAPTIC_V_MV_WPR)) {
         // short rows, x in registers: each lane covers <= U vectors of a row.  Only the
         // plan's own load path is planned (G and U depend on the row length in loads),
@@ -797,6 +813,8 @@ adaptic_status make_plan(int op, int64_t rows, int64_t cols, int dtype, int vari
         const int64_t nv = (cols % 4 == 0) ? cols / 4 : cols;
         if (op == ADAPTIC_OP_TMV) p->variant = heuristic_variant(op, rows, cols, dev.sms);
         else if (nv <= 32 * (nvec == 8 ? 2 : 4)) p->variant = ADAPTIC_V_MV_SUBWARP;
+        else if (cols % 4 == 0 && int64_t(nvec) * cols * 4 <= MMV_WARP_SMEM)
+            p->variant = ADAPTIC_V_MV_WPR;                                 // warp per row, x in smem
         else if (rows >= 4 * int64_t(dev.sms)) p->variant = ADAPTIC_V_MV_CPR;
         else p->variant = ADAPTIC_V_MV_SPLIT;
         p->source = 2;
@@ -901,11 +919,12 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
     if (p->nvec > 1) {
         const int K = p->nvec;
         if (p->op == ADAPTIC_OP_TMV) fn = tmmv_fn(K, p->lanes, p->unroll, vec);
+        else if (p->xmode == 3) { fn = mmv_warp_fn(K); smem = p->smem; }
         else if (p->variant == ADAPTIC_V_MV_SUBWARP || p->variant == ADAPTIC_V_MV_WPR) fn = mmv_group_fn(K, p->lanes, p->unroll, vec);
         else { fn = mmv_cta_fn(K, p->unroll, vec, p->xmode == 1); smem = p->smem; }
         if (p->op == ADAPTIC_OP_MV && (p->variant == ADAPTIC_V_MV_SUBWARP || p->variant == ADAPTIC_V_MV_WPR)) {
             args6[0] = &A; args6[1] = &X; args6[2] = &y; args6[3] = &R; args6[4] = &C;
-            args = args6;
+            args = args6;                        // register-x group kernel or the warp kernel (xmode 3)
         } else {
             args8[0] = &A; args8[1] = &X; args8[2] = &y; args8[3] = &R; args8[4] = &C;
             args8[5] = &S; args8[6] = &part; args8[7] = &cnt;

@@ -64,6 +64,16 @@ static void* mt_l(int LR, int U) {
     return nullptr;
 }
 
+// warp-per-row kernel with x in shared memory: RB = 1, U = 2, NT = 256
+void* mmv_warp_fn(int K) {
+    switch (K) {
+        case 2: return reinterpret_cast<void*>(&mmv_warp_kernel<2, 1, 2, 256>);
+        case 4: return reinterpret_cast<void*>(&mmv_warp_kernel<4, 1, 2, 256>);
+        case 8: return reinterpret_cast<void*>(&mmv_warp_kernel<8, 1, 2, 256>);
+        default: return nullptr;
+    }
+}
+
 #define ADAPTIC_K(FN, ...)                                                       \
     switch (K) {                                                                 \
         case 2: return vec ? FN<2, true>(__VA_ARGS__) : FN<2, false>(__VA_ARGS__); \

@@ -61,6 +61,9 @@ constexpr int MMV_GROUP_RB = 2;
 void* mmv_group_fn(int K, int G, int U, bool vec);
 void* mmv_cta_fn(int K, int U, bool vec, bool xs);   // xs: K*C*4 bytes of x staged in smem
 void* tmmv_fn(int K, int LR, int U, bool vec);
+//   warp : (A, X, Y, R, C), warp per row, all K x-vectors in smem (K * C * 4 <= MMV_WARP_SMEM)
+void* mmv_warp_fn(int K);
+constexpr int MMV_WARP_SMEM = 40 * 1024;
 
 // BLAS-1 reductions (blas1_kernels.cuh), fp32 input, one translation unit per operator:
 //   b1 group: (const float* A, void* y, int64_t R, int64_t C); rbu 0 = (RB 4, U 2), 1 = (RB 1, U 8)

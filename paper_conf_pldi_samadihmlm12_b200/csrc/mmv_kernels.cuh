@@ -199,6 +199,82 @@ mmv_cta_kernel(const float* __restrict__ A, const float* __restrict__ X, float* 
     }
 }
 
+// ------------------------------------------------------------------ MV, medium rows: warp per row, x in smem
+// All K x-vectors (K*C*4 bytes <= 48 KB) are staged once per CTA by TMA; each warp then
+// streams whole rows (RB per step, U loads per row in flight) and reduces with shuffles:
+// no CTA-wide barrier per row (the CTA-per-row kernel's per-row reduction and the
+// measured alternative that staged x in column chunks with a per-block ticket dominated rows of a few KB).
+template <int K, int RB, int U, int NT>
+__global__ void __launch_bounds__(NT, 4)
+mmv_warp_kernel(const float* __restrict__ A, const float* __restrict__ X, float* __restrict__ Y,
+                int64_t R, int64_t C)
+{
+    pdl_prologue();
+    extern __shared__ __align__(128) unsigned char dyn_smem[];
+    __shared__ __align__(8) uint64_t xbar;
+    float4* xs = reinterpret_cast<float4*>(dyn_smem);   // [K][nv]
+    const int64_t nv = C / 4;
+    stage_to_smem(xs, X, uint32_t(K * C * 4), &xbar);
+    const float4* __restrict__ Av = reinterpret_cast<const float4*>(A);
+    const int lane = threadIdx.x & 31;
+    const int64_t warp = (int64_t(blockIdx.x) * NT + threadIdx.x) >> 5;
+    const int64_t nwarps = (int64_t(gridDim.x) * NT) >> 5;
+    for (int64_t base = warp * RB; base < R; base += nwarps * RB) {
+        int64_t off[RB];
+#pragma unroll
+        for (int i = 0; i < RB; ++i) off[i] = (base + i < R ? base + i : 0) * nv;
+        float4 acc[RB][K];
+#pragma unroll
+        for (int i = 0; i < RB; ++i)
+#pragma unroll
+            for (int j = 0; j < K; ++j) acc[i][j] = make_float4(0.f, 0.f, 0.f, 0.f);
+        float outer[RB][K];
+#pragma unroll
+        for (int i = 0; i < RB; ++i)
+#pragma unroll
+            for (int j = 0; j < K; ++j) outer[i][j] = 0.f;
+        int it = 0;
+        int64_t v = lane;
+        for (; v + 32 * (U - 1) < nv; v += 32 * U) {
+            float4 a[RB][U];
+#pragma unroll
+            for (int u = 0; u < U; ++u)
+#pragma unroll
+                for (int i = 0; i < RB; ++i) a[i][u] = ld_stream(Av + off[i] + v + 32 * u);
+#pragma unroll
+            for (int u = 0; u < U; ++u)
+#pragma unroll
+                for (int j = 0; j < K; ++j) {
+                    const float4 xv = xs[j * nv + v + 32 * u];
+#pragma unroll
+                    for (int i = 0; i < RB; ++i) vmac(acc[i][j], a[i][u], xv);
+                }
+            if (++it == FOLD / U) {
+                it = 0;
+#pragma unroll
+                for (int i = 0; i < RB; ++i)
+#pragma unroll
+                    for (int j = 0; j < K; ++j) { outer[i][j] += vsum(acc[i][j]); acc[i][j] = make_float4(0.f, 0.f, 0.f, 0.f); }
+            }
+        }
+        for (; v < nv; v += 32) {
+#pragma unroll
+            for (int i = 0; i < RB; ++i) {
+                const float4 a = ld_stream(Av + off[i] + v);
+#pragma unroll
+                for (int j = 0; j < K; ++j) vmac(acc[i][j], a, xs[j * nv + v]);
+            }
+        }
+#pragma unroll
+        for (int i = 0; i < RB; ++i)
+#pragma unroll
+            for (int j = 0; j < K; ++j) {
+                const float t = group_sum<32>(outer[i][j] + vsum(acc[i][j]));
+                if (lane == 0 && base + i < R) Y[j * R + base + i] = t;
+            }
+    }
+}
+
 // ------------------------------------------------------------------ TMV tiles
 // As tmv_kernel: CTA tile of LR output vectors x LC = NT/LR c-lanes, S c-ranges,
 // with K accumulators per thread (one per vector) and the lc-combine per vector.
