@@ -213,3 +213,21 @@ def iamin(a: np.ndarray) -> np.ndarray:
     y = np.empty(a.shape[0], np.int64)
     assert _blas1_lib().oracle_iamaxmin(_ptr(a), a.shape[0], a.shape[1], -1, _ptr(y)) == 0
     return y
+
+
+def stencil5(u: np.ndarray, c: float, n: float):
+    """Five-point stencil of an H x W fp32 grid (oracle.c oracle_stencil5_f64): returns
+    (v, S) in float64, v = c u + n (T + B + L + R) inside, v = u on the edge."""
+    u = _c(u, np.float32)
+    H, W = u.shape
+    v = np.empty((H, W), np.float64)
+    S = np.empty((H, W), np.float64)
+    lib = _load()
+    if not getattr(lib, "_st5_ready", False):
+        P = ctypes.c_void_p
+        I = ctypes.c_int64
+        lib.oracle_stencil5_f64.argtypes = [P, I, I, ctypes.c_double, ctypes.c_double, P, P]
+        lib.oracle_stencil5_f64.restype = ctypes.c_int
+        lib._st5_ready = True
+    assert lib.oracle_stencil5_f64(_ptr(u), H, W, float(c), float(n), _ptr(v), _ptr(S)) == 0
+    return v, S

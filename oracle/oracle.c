@@ -236,3 +236,31 @@ int oracle_iamaxmin(const float* a, int64_t N, int64_t L, int which, int64_t* id
     }
     return 0;
 }
+
+/* ---- five-point stencil (second item) -----------------------
+ * The paper's neighbouring-access actor (Sec. 4.1.2, Fig. 4a): every
+ * point reads its top, bottom, left and right neighbours and itself and pushes
+ * func(Top, Bottom, Right, Left, Center); points on the edge are skipped ("if (not on
+ * edge)").  func is not printed; reading R19: the weighted Jacobi form
+ *   v[i][j] = c * u[i][j] + n * (u[i-1][j] + u[i+1][j] + u[i][j-1] + u[i][j+1])
+ * for 1 <= i < H-1, 1 <= j < W-1, and v = u on the edge.  u, v are H x W row-major
+ * fp32; the oracle evaluates in double (products of fp32 values are exact) and
+ * returns S = |c u| + |n| (|T| + |B| + |L| + |R|) per point for the tolerance. */
+int oracle_stencil5_f64(const float* u, int64_t H, int64_t W, double c, double n, double* v, double* S)
+{
+    if (H < 0 || W < 0) return 1;
+    for (int64_t i = 0; i < H; ++i) {
+        for (int64_t j = 0; j < W; ++j) {
+            const int64_t k = i * W + j;
+            if (i == 0 || j == 0 || i == H - 1 || j == W - 1) {
+                v[k] = (double)u[k];
+                if (S) S[k] = fabs((double)u[k]);
+                continue;
+            }
+            const double t = u[k - W], b = u[k + W], l = u[k - 1], r = u[k + 1], ce = u[k];
+            v[k] = c * ce + n * (t + b + l + r);
+            if (S) S[k] = fabs(c * ce) + fabs(n) * (fabs(t) + fabs(b) + fabs(l) + fabs(r));
+        }
+    }
+    return 0;
+}
