@@ -122,7 +122,7 @@
 extern "C" {
 #endif
 
-#define ADAPTIC_ABI_VERSION 5
+#define ADAPTIC_ABI_VERSION 6
 
 typedef enum {
     ADAPTIC_OK = 0,
@@ -144,9 +144,13 @@ typedef enum {
     ADAPTIC_OP_NRM2 = 4,  /* float y[N] = sqrt(sum_e a_n[e]^2)                      */
     ADAPTIC_OP_IAMAX = 5, /* int32 y[N] = smallest 1-based e maximising |a_n[e]|    */
     ADAPTIC_OP_IAMIN = 6, /* int32 y[N] = smallest 1-based e minimising |a_n[e]|    */
-    ADAPTIC_OP_B1ALL = 7  /* all four in ONE pass over a (horizontal actor integration,
+    ADAPTIC_OP_B1ALL = 7, /* all four in ONE pass over a (horizontal actor integration,
                            * P:600): y = [asum N floats | nrm2 N floats | iamax N int32 |
                            * iamin N int32], 16*N bytes                               */
+    /* Five-point stencil (the paper's neighbouring-access actor, Sec. 4.1.2, Fig. 4a):
+     * A = u (rows = H, cols = W, fp32 row-major), x = {c, n} (2 device floats),
+     * y = v (H x W): v = c u + n (T + B + L + R) inside, v = u on the edge.        */
+    ADAPTIC_OP_STENCIL5 = 8
 } adaptic_op;
 
 typedef enum {
@@ -164,7 +168,9 @@ typedef enum {
     ADAPTIC_V_TMV_COL = 6,
     ADAPTIC_V_TMV_SPLITK = 7,
     ADAPTIC_V_TMV_REGTILE = 8,
-    ADAPTIC_V_COUNT = 9
+    ADAPTIC_V_ST_DIRECT = 9,   /* stencil: no shared memory, neighbours from L1/L2          */
+    ADAPTIC_V_ST_TILE = 10,    /* stencil: TMA-staged super tiles, double-buffered */
+    ADAPTIC_V_COUNT = 11
 } adaptic_variant;
 
 /* Optional parameters for adaptic_plan_forced: an array of ADAPTIC_NPARAMS
@@ -188,7 +194,10 @@ typedef enum {
  *                      the row, 2 = the splits interleave in steps of
  *                      threads*unroll vectors (default when splits > 1).
  *   [ADAPTIC_P_PIPE]   MV_CPR / MV_SPLIT with 256 threads: 1 = single-buffered
- *                      loads (default), 2 = register double-buffered main loop. */
+ *                      loads (default), 2 = register double-buffered main loop.
+ *   ST_TILE: [ADAPTIC_P_ROWS] super-tile height TH in {4, 8, 16, 32}, [ADAPTIC_P_LANES]
+ *                      width TW in {128, 256, 512} (default: the paper's reuse metric
+ *                      sum(accesses)/halo, among tilings with enough blocks). */
 #define ADAPTIC_P_LANES 0
 #define ADAPTIC_P_SPLITS 1
 #define ADAPTIC_P_CTAS_PER_SM 2

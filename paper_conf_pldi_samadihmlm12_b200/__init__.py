@@ -13,7 +13,7 @@ There is no CPU fallback: without ``libadaptic.so`` every call raises.
 """
 from ._lib import BiCGSTAB, VARIANTS, MV_VARIANTS, TMV_VARIANTS, AdapticError, Plan, lib  # noqa: F401
 from .ops import (asum, b1all, bicgstab, bicgstab_solver, clear_cache, dot, get_plan, iamax, iamin, mv, mv_multi, nrm2, plan,  # noqa: F401
-                  run_host, tmv, tmv_multi)
+                  run_host, stencil5, tmv, tmv_multi)
 
-__all__ = ["mv", "tmv", "dot", "asum", "nrm2", "iamax", "iamin", "b1all", "mv_multi", "tmv_multi", "bicgstab", "bicgstab_solver", "plan", "run_host", "Plan", "AdapticError", "lib",
+__all__ = ["mv", "tmv", "dot", "asum", "nrm2", "iamax", "iamin", "b1all", "mv_multi", "tmv_multi", "bicgstab", "bicgstab_solver", "stencil5", "plan", "run_host", "Plan", "AdapticError", "lib",
            "VARIANTS", "MV_VARIANTS", "TMV_VARIANTS", "get_plan", "clear_cache"]

@@ -17,13 +17,14 @@ LIB_PATH = os.environ.get("ADAPTIC_LIB", os.path.join(HERE, "libadaptic.so"))
 # enums (mirror include/adaptic.h)
 OK, ERR_INVALID_ARG, ERR_UNSUPPORTED, ERR_MISALIGNED, ERR_ALIAS, ERR_NO_WORKSPACE, ERR_CUDA = range(7)
 OP_MV, OP_TMV, OP_DOT = 0, 1, 2
-OP_ASUM, OP_NRM2, OP_IAMAX, OP_IAMIN, OP_B1ALL = 3, 4, 5, 6, 7
+OP_ASUM, OP_NRM2, OP_IAMAX, OP_IAMIN, OP_B1ALL, OP_STENCIL5 = 3, 4, 5, 6, 7, 8
 OPS = {"mv": OP_MV, "tmv": OP_TMV, "dot": OP_DOT, "asum": OP_ASUM, "nrm2": OP_NRM2,
-       "iamax": OP_IAMAX, "iamin": OP_IAMIN, "b1all": OP_B1ALL}
+       "iamax": OP_IAMAX, "iamin": OP_IAMIN, "b1all": OP_B1ALL, "stencil5": OP_STENCIL5}
 B1_VARIANTS = ("MV_SUBWARP", "MV_WPR", "MV_CPR", "MV_SPLIT")
 F32, I32 = 0, 1
 VARIANTS = ("AUTO", "MV_TPR", "MV_SUBWARP", "MV_WPR", "MV_CPR", "MV_SPLIT",
-            "TMV_COL", "TMV_SPLITK", "TMV_REGTILE")
+            "TMV_COL", "TMV_SPLITK", "TMV_REGTILE", "ST_DIRECT", "ST_TILE")
+ST_VARIANTS = ("ST_DIRECT", "ST_TILE")
 V = {name: i for i, name in enumerate(VARIANTS)}
 MV_VARIANTS = ("MV_TPR", "MV_SUBWARP", "MV_WPR", "MV_CPR", "MV_SPLIT")
 TMV_VARIANTS = ("TMV_COL", "TMV_SPLITK", "TMV_REGTILE")

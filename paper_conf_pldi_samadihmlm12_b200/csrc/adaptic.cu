@@ -74,7 +74,7 @@ const int kTableN = int(sizeof(kTable) / sizeof(kTable[0])) - 1;
 
 const char* const kVariantNames[ADAPTIC_V_COUNT] = {
     "AUTO", "MV_TPR", "MV_SUBWARP", "MV_WPR", "MV_CPR", "MV_SPLIT",
-    "TMV_COL", "TMV_SPLITK", "TMV_REGTILE"};
+    "TMV_COL", "TMV_SPLITK", "TMV_REGTILE", "ST_DIRECT", "ST_TILE"};
 
 constexpr double kUnitRoundoff = 5.9604644775390625e-08;  // 2^-24
 constexpr double kTol = 1e-4;                              // north_star tolerance
@@ -106,6 +106,8 @@ bool is_b1_op(int op) { return op >= ADAPTIC_OP_ASUM && op <= ADAPTIC_OP_B1ALL; 
 size_t y_bytes_per_row(int op) { return op == ADAPTIC_OP_B1ALL ? 16 : 4; }
 bool is_b1_variant(int v) { return v >= ADAPTIC_V_MV_SUBWARP && v <= ADAPTIC_V_MV_SPLIT; }
 bool op_has_variant(int op, int v) {
+    if (op == ADAPTIC_OP_STENCIL5) return v == ADAPTIC_V_ST_DIRECT || v == ADAPTIC_V_ST_TILE;
+    if (v == ADAPTIC_V_ST_DIRECT || v == ADAPTIC_V_ST_TILE) return false;
     if (op == ADAPTIC_OP_TMV) return is_tmv_family(v);
     if (is_b1_op(op)) return is_b1_variant(v);
     return is_mv_family(v);
@@ -201,6 +203,7 @@ int64_t pick_splits(int64_t units, int64_t slots, int64_t smax, int64_t smin) {
 
 // ---------------------------------------------------------------- heuristic (no table cell)
 int heuristic_variant(int op, int64_t R, int64_t C, int sms) {
+    if (op == ADAPTIC_OP_STENCIL5) return (C % 4 == 0) ? ADAPTIC_V_ST_TILE : ADAPTIC_V_ST_DIRECT;
     if (is_b1_op(op)) {
         // the paper's regimes (Fig. 1) for a unary reduction: lane groups
         // for many short rows, a CTA per row once rows are long and numerous
@@ -268,6 +271,70 @@ const TableEntry* table_lookup(int op, int dtype, int64_t R, int64_t C, bool* pr
     // int32 moves the same bytes as fp32: use the fp32 cells when int32 was not swept
     if (dtype != ADAPTIC_F32) return table_lookup(op, ADAPTIC_F32, R, C, projected);
     return nullptr;
+}
+
+// Five-point stencil: ST_DIRECT (no shared memory) or ST_TILE (TMA-staged super tiles,
+// the paper's neighbouring-access optimization).  The super tile follows the
+// input: the largest reuse metric sum(element accesses) / halo among tilings that
+// still give every SM two CTAs' worth of tiles ("for small input sizes ... smaller super
+// tiles in order to have more blocks").  Index 0 = the scalar direct kernel (fallback for
+// misaligned pointers), index 1 = the planned kernel on the 128-bit path.
+adaptic_status derive_stencil(adaptic_plan_s* p, const int32_t* params, const DevInfo& dev) {
+    const int v = p->variant;
+    const int64_t H = p->R, W = p->C;
+    auto par = [&](int i) -> int { return params ? params[i] : 0; };
+    p->vec_shape = (W % 4 == 0);
+    p->mis = false; p->flat = false; p->splits = 1; p->smem = 0; p->stages = 0; p->xmode = 0; p->ilv = 0;
+    p->pipe = 0; p->rb = 1; p->fb_lanes = 0; p->fb_unroll = 0; p->ws_bytes = 0; p->cnt_off = 0; p->unroll = 1;
+    p->block = 256;
+    const int cps_d = occupancy(st_direct_fn(false), 256, 0, dev.present, 8);
+    p->grid[0] = std::max<int64_t>(1, std::min<int64_t>(ceil_div(H * W, 256), int64_t(dev.sms) * cps_d));
+    p->chain[0] = p->chain[1] = 0;                    // no reduction: 3 roundings per point
+    p->depth[0] = p->depth[1] = 3;
+    p->path_ok[0] = true;
+    p->grid[1] = 0; p->path_ok[1] = false;
+    if (v == ADAPTIC_V_ST_DIRECT) {
+        p->lanes = 4; p->ctas_per_sm = cps_d;
+        if (p->vec_shape) {
+            const int cps = occupancy(st_direct_fn(true), 256, 0, dev.present, 8);
+            p->grid[1] = std::max<int64_t>(1, std::min<int64_t>(ceil_div(H * (W / 4), 256), int64_t(dev.sms) * cps));
+            p->path_ok[1] = true;
+        }
+        return ADAPTIC_OK;
+    }
+    if (!p->vec_shape) return ADAPTIC_ERR_UNSUPPORTED;   // TMA rows need C % 4 == 0
+    static const int kTH[] = {4, 8, 16, 32}, kTW[] = {128, 256, 512};
+    int TH = par(ADAPTIC_P_ROWS), TW = par(ADAPTIC_P_LANES);
+    if (TH > 0 || TW > 0) {
+        if (TH <= 0) TH = 8;
+        if (TW <= 0) TW = 256;
+        if (!st_tile_fn(TH, TW)) return ADAPTIC_ERR_INVALID_ARG;
+    } else {
+        double best = -1.0, best_tiles = -1.0;
+        int bth = 4, btw = 128;
+        const double want = 2.0 * dev.sms;
+        for (int th : kTH)
+            for (int tw : kTW) {
+                if (tw > std::max<int64_t>(128, pow2_ceil(W))) continue;
+                const double tiles = double(ceil_div(H, th)) * double(ceil_div(W, tw));
+                const double reuse = 5.0 * th * tw / double((th + 2) * (tw + 8) - th * tw);
+                const bool enough = tiles >= want;
+                // prefer tilings with enough blocks, then the reuse metric; if none has
+                // enough blocks, the one with the most tiles
+                const double key = enough ? 1e9 + reuse : tiles;
+                if (key > best || (key == best && tiles > best_tiles)) { best = key; best_tiles = tiles; bth = th; btw = tw; }
+            }
+        TH = bth; TW = btw;
+    }
+    p->rb = TH; p->lanes = TW;
+    p->smem = size_t(2) * size_t(TH + 2) * size_t(TW + 8) * 4;
+    int cps = par(ADAPTIC_P_CTAS_PER_SM);
+    if (cps <= 0) cps = occupancy(st_tile_fn(TH, TW), 256, p->smem, dev.present, 2);
+    p->ctas_per_sm = std::max(1, cps);
+    const int64_t tiles = ceil_div(H, TH) * ceil_div(W, TW);
+    p->grid[1] = std::max<int64_t>(1, std::min<int64_t>(tiles, int64_t(dev.sms) * p->ctas_per_sm));
+    p->path_ok[1] = true;
+    return ADAPTIC_OK;
 }
 
 // Multi-vector MV / TMV (adaptic_plan_multi): K = nvec vectors share one pass over the
@@ -517,6 +584,7 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
     const int v = p->variant;
     if (!op_has_variant(op, v)) return ADAPTIC_ERR_UNSUPPORTED;
     if (p->nvec > 1) return derive_multi(p, params, dev);
+    if (op == ADAPTIC_OP_STENCIL5) return derive_stencil(p, params, dev);
     if (is_b1_op(op)) return derive_b1(p, params, dev);
 
     p->vec_shape = (op == ADAPTIC_OP_TMV) ? (R % 4 == 0) : (C % 4 == 0);
@@ -768,7 +836,8 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
 }
 
 adaptic_status validate_shape(int op, int64_t rows, int64_t cols, int dtype) {
-    if (op < ADAPTIC_OP_MV || op > ADAPTIC_OP_B1ALL) return ADAPTIC_ERR_INVALID_ARG;
+    if (op < ADAPTIC_OP_MV || op > ADAPTIC_OP_STENCIL5) return ADAPTIC_ERR_INVALID_ARG;
+    if (op == ADAPTIC_OP_STENCIL5 && dtype != ADAPTIC_F32) return ADAPTIC_ERR_UNSUPPORTED;
     if (dtype != ADAPTIC_F32 && dtype != ADAPTIC_I32) return ADAPTIC_ERR_INVALID_ARG;
     if (rows < 0 || cols < 0) return ADAPTIC_ERR_INVALID_ARG;
     if (is_b1_op(op) && dtype != ADAPTIC_F32) return ADAPTIC_ERR_UNSUPPORTED;
@@ -916,7 +985,16 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
     int stages = p->stages;
 
     void* args7[7];
-    if (p->nvec > 1) {
+    if (p->op == ADAPTIC_OP_STENCIL5) {
+        if (p->variant == ADAPTIC_V_ST_TILE && vec) {
+            fn = st_tile_fn(p->rb, p->lanes);
+            smem = p->smem;
+        } else {
+            fn = st_direct_fn(vec);
+        }
+        args6[0] = &A; args6[1] = &X; args6[2] = &y; args6[3] = &R; args6[4] = &C;
+        args = args6;
+    } else if (p->nvec > 1) {
         const int K = p->nvec;
         if (p->op == ADAPTIC_OP_TMV) fn = tmmv_fn(K, p->lanes, p->unroll, vec);
         else if (p->xmode == 3) { fn = mmv_warp_fn(K); smem = p->smem; }
@@ -1019,9 +1097,10 @@ adaptic_status check_run(const adaptic_plan_s* p, const void* A, const void* x, 
     const bool b1 = is_b1_op(p->op);          // BLAS-1: x is unused (may be NULL)
     if (!A || (!x && !b1)) return ADAPTIC_ERR_INVALID_ARG;
     if (!aligned(A, 4) || (!b1 && !aligned(x, 4))) return ADAPTIC_ERR_MISALIGNED;
-    const size_t ybytes = size_t(p->R) * y_bytes_per_row(p->op) * size_t(p->nvec);
+    const bool st = p->op == ADAPTIC_OP_STENCIL5;
     const size_t abytes = size_t(p->R) * size_t(p->C) * 4;
-    const size_t xbytes = b1 ? 0 : (p->op == ADAPTIC_OP_DOT ? abytes : size_t(p->C) * 4 * size_t(p->nvec));
+    const size_t ybytes = st ? abytes : size_t(p->R) * y_bytes_per_row(p->op) * size_t(p->nvec);
+    const size_t xbytes = b1 ? 0 : st ? 8 : (p->op == ADAPTIC_OP_DOT ? abytes : size_t(p->C) * 4 * size_t(p->nvec));
     if (overlap(y, ybytes, A, abytes) || (!b1 && overlap(y, ybytes, x, xbytes))) return ADAPTIC_ERR_ALIAS;
     if (p->ws_bytes > 0 && (p->ws == nullptr || p->ws_cap < p->ws_bytes)) return ADAPTIC_ERR_NO_WORKSPACE;
     return ADAPTIC_OK;
@@ -1069,7 +1148,7 @@ adaptic_status adaptic_plan_set_workspace(adaptic_plan_t plan, void* dev_ptr, si
 
 int adaptic_plan_describe(adaptic_plan_t p, char* buf, size_t cap) {
     if (!p) return -1;
-    static const char* ops[] = {"MV", "TMV", "DOT", "ASUM", "NRM2", "IAMAX", "IAMIN", "B1ALL"};
+    static const char* ops[] = {"MV", "TMV", "DOT", "ASUM", "NRM2", "IAMAX", "IAMIN", "B1ALL", "STENCIL5"};
     static const char* src[] = {"forced", "table", "heuristic"};
     char tmp[1024];
     const int n = std::snprintf(
@@ -1100,11 +1179,14 @@ adaptic_status adaptic_run(adaptic_plan_t p, const void* A, const void* x, void*
     adaptic_status st = check_run(p, A, x, y);
     if (st != ADAPTIC_OK || p->R == 0) return st;
     if (p->C == 0) {
+        if (p->op == ADAPTIC_OP_STENCIL5) return ADAPTIC_OK;          // H x 0 grid: nothing to write
         cudaError_t e = cudaMemsetAsync(y, 0, size_t(p->R) * y_bytes_per_row(p->op) * size_t(p->nvec), stream);
         return e == cudaSuccess ? ADAPTIC_OK : cuda_fail(e);
     }
     bool vec = p->vec_shape;
-    if (vec && p->nvec > 1) {
+    if (vec && p->op == ADAPTIC_OP_STENCIL5) {
+        vec = aligned(A, 16) && aligned(y, 16);
+    } else if (vec && p->nvec > 1) {
         vec = aligned(A, 16) && aligned(x, 16) && aligned(y, 16);
     } else if (vec) {
         if (p->op == ADAPTIC_OP_TMV) vec = aligned(A, 16) && aligned(y, 16);
@@ -1199,8 +1281,10 @@ adaptic_status adaptic_run_host(adaptic_plan_t p, const void* A_host, const void
     if (!y_host || (p->C > 0 && (!A_host || (!x_host && !b1)))) return ADAPTIC_ERR_INVALID_ARG;
     adaptic_status st = check_run(p, dA, dx, dy);
     if (st != ADAPTIC_OK) return st;
+    const bool sten = p->op == ADAPTIC_OP_STENCIL5;
     const size_t abytes = size_t(p->R) * size_t(p->C) * 4;
-    const size_t xbytes = (p->op == ADAPTIC_OP_DOT ? abytes : size_t(p->C) * 4 * size_t(p->nvec));
+    const size_t xbytes = sten ? 8 : (p->op == ADAPTIC_OP_DOT ? abytes : size_t(p->C) * 4 * size_t(p->nvec));
+    const size_t ybytes = sten ? abytes : size_t(p->R) * y_bytes_per_row(p->op) * size_t(p->nvec);
     cudaError_t e;
     if (p->C > 0) {
         if (!b1 && (e = cudaMemcpyAsync(dx, x_host, xbytes, cudaMemcpyHostToDevice, stream)) != cudaSuccess)
@@ -1209,10 +1293,7 @@ adaptic_status adaptic_run_host(adaptic_plan_t p, const void* A_host, const void
     }
     st = adaptic_run(p, dA, dx, dy, stream_);
     if (st != ADAPTIC_OK) return st;
-    if ((e = cudaMemcpyAsync(y_host, dy, size_t(p->R) * y_bytes_per_row(p->op) * size_t(p->nvec), cudaMemcpyDeviceToHost,
-                             stream)) !=
-        cudaSuccess)
-        return cuda_fail(e);
+    if ((e = cudaMemcpyAsync(y_host, dy, ybytes, cudaMemcpyDeviceToHost, stream)) != cudaSuccess) return cuda_fail(e);
     return ADAPTIC_OK;
 }
 

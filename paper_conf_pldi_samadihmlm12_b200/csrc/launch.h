@@ -63,6 +63,12 @@ void* mmv_cta_fn(int K, int U, bool vec, bool xs);   // xs: K*C*4 bytes of x sta
 void* tmmv_fn(int K, int LR, int U, bool vec);
 //   warp : (A, X, Y, R, C), warp per row, all K x-vectors in smem (K * C * 4 <= MMV_WARP_SMEM)
 void* mmv_warp_fn(int K);
+
+// Five-point stencil (stencil_kernels.cu), 256 threads:
+//   direct: (const float* u, const float* coef, float* v, int64_t H, int64_t W)
+//   tile  : same arguments, dynamic smem 2 * (TH + 2) * (TW + 8) * 4 bytes
+void* st_direct_fn(bool vec);
+void* st_tile_fn(int TH, int TW);
 constexpr int MMV_WARP_SMEM = 40 * 1024;
 
 // BLAS-1 reductions (blas1_kernels.cuh), fp32 input, one translation unit per operator:

@@ -1,0 +1,163 @@
+// stencil_kernels.cu -- five-point stencil with input-adaptive super tiles (SURVEY 8(f)
+// rank 4, second item), sm_100a.
+//
+// The paper's neighbouring-access optimization (Sec. 4.1.2): a point and
+// its four neighbours are read for every output, so reading them straight from
+// global memory touches the input five times; instead each block brings a tile plus
+// its halo into shared memory, and to shrink the halo overhead several tiles are
+// merged into a SUPER TILE whose size and shape follow the input: "for small input
+// sizes it is beneficial to use smaller super tiles in order to have more blocks.
+// Large super tiles are advantageous for large input sizes", chosen by the reuse
+// metric sum(element accesses) / halo size.  v = c u + n (T + B + L + R)
+// inside, v = u on the edge (reading R19); x holds {c, n} on the device.
+//
+//   st_direct_kernel  no shared memory: 4 outputs per thread, neighbours from L1/L2
+//                     (a grid-stride sweep keeps the rows above and below L2-resident)
+//   st_tile_kernel    super tiles of TH x TW outputs; the (TH+2) x (TW+8) input block
+//                     (16-byte-aligned halo of 4 columns; 1 used) arrives by TMA bulk
+//                     copies, one per row, double-buffered: the next super tile of the
+//                     CTA streams in while the current one is computed.
+#include "common.cuh"
+#include "launch.h"
+
+namespace adaptic {
+
+__device__ __forceinline__ float st_point(float c, float n, float ce, float t, float b, float l, float r) {
+    return fmaf(c, ce, n * ((t + b) + (l + r)));
+}
+
+// --------------------------------------------------------------------------- direct
+template <bool VEC, int NT>
+__global__ void __launch_bounds__(NT)
+st_direct_kernel(const float* __restrict__ u, const float* __restrict__ coef, float* __restrict__ v,
+                 int64_t H, int64_t W)
+{
+    pdl_prologue();
+    const float c = __ldg(coef), n = __ldg(coef + 1);
+    const int64_t nvr = VEC ? W / 4 : W;              // vectors per row
+    const int64_t total = H * nvr;
+    for (int64_t q = int64_t(blockIdx.x) * NT + threadIdx.x; q < total; q += int64_t(gridDim.x) * NT) {
+        const int64_t i = q / nvr, k = q - i * nvr;
+        const int64_t at = i * W + (VEC ? 4 * k : k);
+        if constexpr (VEC) {
+            const float4 ce = *reinterpret_cast<const float4*>(u + at);
+            float4 o = ce;
+            if (i > 0 && i < H - 1) {
+                const float4 t = __ldg(reinterpret_cast<const float4*>(u + at - W));
+                const float4 b = __ldg(reinterpret_cast<const float4*>(u + at + W));
+                const float l = k > 0 ? __ldg(u + at - 1) : 0.f;
+                const float r = k < nvr - 1 ? __ldg(u + at + 4) : 0.f;
+                if (k > 0) o.x = st_point(c, n, ce.x, t.x, b.x, l, ce.y);
+                o.y = st_point(c, n, ce.y, t.y, b.y, ce.x, ce.z);
+                o.z = st_point(c, n, ce.z, t.z, b.z, ce.y, ce.w);
+                if (k < nvr - 1) o.w = st_point(c, n, ce.w, t.w, b.w, ce.z, r);
+            }
+            *reinterpret_cast<float4*>(v + at) = o;
+        } else {
+            const float ce = u[at];
+            float o = ce;
+            if (i > 0 && i < H - 1 && k > 0 && k < W - 1)
+                o = st_point(c, n, ce, __ldg(u + at - W), __ldg(u + at + W), __ldg(u + at - 1), __ldg(u + at + 1));
+            v[at] = o;
+        }
+    }
+}
+
+// --------------------------------------------------------------------------- super tiles
+// Shared buffer b holds input rows row0-1 .. row0+TH (clamped to the grid) and columns
+// col0-4 .. col0+TW+3 (clamped), at smem column (global column - col0 + 4).
+template <int TH, int TW, int NT>
+__global__ void __launch_bounds__(NT)
+st_tile_kernel(const float* __restrict__ u, const float* __restrict__ coef, float* __restrict__ v,
+               int64_t H, int64_t W)
+{
+    pdl_prologue();
+    constexpr int SW = TW + 8;                        // smem row pitch (floats), 16-byte multiple
+    constexpr int SH = TH + 2;
+    extern __shared__ __align__(128) unsigned char dyn_smem[];
+    float* buf = reinterpret_cast<float*>(dyn_smem);  // [2][SH][SW]
+    __shared__ __align__(8) uint64_t bar[2];
+    const float c = __ldg(coef), n = __ldg(coef + 1);
+    const int64_t tiles_c = (W + TW - 1) / TW, tiles_r = (H + TH - 1) / TH;
+    const int64_t ntiles = tiles_r * tiles_c;
+    const int tid = threadIdx.x;
+    const int64_t my = blockIdx.x < ntiles ? (ntiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+
+    auto issue = [&](int64_t li) {                    // thread 0: local tile li -> buffer li & 1
+        const int64_t tile = blockIdx.x + li * gridDim.x;
+        const int64_t tr = tile / tiles_c, tc = tile - tr * tiles_c;
+        const int64_t row0 = tr * TH, col0 = tc * TW;
+        const int64_t r_lo = max(row0 - 1, int64_t(0)), r_hi = min(row0 + TH + 1, H);
+        const int64_t c_lo = max(col0 - 4, int64_t(0)), c_hi = min(col0 + TW + 4, W);
+        const uint32_t bytes = uint32_t(c_hi - c_lo) * 4u;
+        float* dst = buf + (li & 1) * (SH * SW);
+        mbar_arrive_expect_tx(&bar[li & 1], bytes * uint32_t(r_hi - r_lo));
+        for (int64_t r = r_lo; r < r_hi; ++r)
+            bulk_g2s(dst + (r - row0 + 1) * SW + (c_lo - col0 + 4), u + r * W + c_lo, bytes, &bar[li & 1]);
+    };
+    if (tid == 0) {
+        mbar_init(&bar[0], 1); mbar_init(&bar[1], 1);
+        fence_mbar_init();
+        if (my > 0) issue(0);
+        if (my > 1) issue(1);
+    }
+    __syncthreads();
+    constexpr int TWV = TW / 4;
+    for (int64_t li = 0; li < my; ++li) {
+        const int64_t tile = blockIdx.x + li * gridDim.x;
+        const int64_t tr = tile / tiles_c, tc = tile - tr * tiles_c;
+        const int64_t row0 = tr * TH, col0 = tc * TW;
+        mbar_wait(&bar[li & 1], uint32_t((li >> 1) & 1));
+        const float* s = buf + (li & 1) * (SH * SW);
+        for (int e = tid; e < TH * TWV; e += NT) {
+            const int rr = e / TWV, kv = e - rr * TWV;
+            const int64_t i = row0 + rr, j = col0 + 4 * kv;
+            if (i >= H || j >= W) continue;
+            const float* sc = s + (rr + 1) * SW + 4 + 4 * kv;
+            const float4 ce = *reinterpret_cast<const float4*>(sc);
+            float4 o = ce;
+            if (i > 0 && i < H - 1) {
+                const float4 t = *reinterpret_cast<const float4*>(sc - SW);
+                const float4 b = *reinterpret_cast<const float4*>(sc + SW);
+                if (j > 0) o.x = st_point(c, n, ce.x, t.x, b.x, sc[-1], ce.y);
+                o.y = st_point(c, n, ce.y, t.y, b.y, ce.x, ce.z);
+                o.z = st_point(c, n, ce.z, t.z, b.z, ce.y, ce.w);
+                if (j + 4 < W) o.w = st_point(c, n, ce.w, t.w, b.w, ce.z, sc[4]);
+            }
+            *reinterpret_cast<float4*>(v + i * W + j) = o;
+        }
+        __syncthreads();                              // buffer li & 1 is free again
+        if (tid == 0 && li + 2 < my) {
+            fence_proxy_async();
+            issue(li + 2);
+        }
+    }
+}
+
+// --------------------------------------------------------------------------- instances
+void* st_direct_fn(bool vec) {
+    return vec ? reinterpret_cast<void*>(&st_direct_kernel<true, 256>)
+               : reinterpret_cast<void*>(&st_direct_kernel<false, 256>);
+}
+
+template <int TH>
+static void* st_tile_w(int TW) {
+    switch (TW) {
+        case 128: return reinterpret_cast<void*>(&st_tile_kernel<TH, 128, 256>);
+        case 256: return reinterpret_cast<void*>(&st_tile_kernel<TH, 256, 256>);
+        case 512: return reinterpret_cast<void*>(&st_tile_kernel<TH, 512, 256>);
+        default: return nullptr;
+    }
+}
+
+void* st_tile_fn(int TH, int TW) {
+    switch (TH) {
+        case 4: return st_tile_w<4>(TW);
+        case 8: return st_tile_w<8>(TW);
+        case 16: return st_tile_w<16>(TW);
+        case 32: return st_tile_w<32>(TW);
+        default: return nullptr;
+    }
+}
+
+}  // namespace adaptic

@@ -267,3 +267,30 @@ def bicgstab(A: torch.Tensor, b: torch.Tensor, *, tol: float = 1e-6, max_iters: 
     stream = torch.cuda.current_stream(dev).cuda_stream
     it, rel = S.solve(A.data_ptr(), b.data_ptr(), x.data_ptr(), max_iters, tol, check_every, stream)
     return x, it, rel
+
+
+_coefs: dict = {}
+
+
+def stencil5(u: torch.Tensor, c: float, n: float, *, variant="AUTO", params=None, out=None) -> torch.Tensor:
+    """Five-point stencil of an H x W float32 grid (the paper's neighbouring-access
+    actor, Sec. 4.1.2): v = c u + n (T + B + L + R) inside, v = u on the edge."""
+    if u.dim() != 2:
+        raise ValueError(f"stencil5: u must be [H, W], got {tuple(u.shape)}")
+    dev = _check_dev(u)
+    if u.dtype != torch.float32:
+        raise TypeError("stencil5 takes float32")
+    H, W = u.shape
+    key = (float(c), float(n), dev.index)
+    coef = _coefs.get(key)
+    if coef is None:
+        coef = torch.tensor([c, n], dtype=torch.float32, device=dev)
+        _coefs[key] = coef
+    if out is None:
+        out = torch.empty_like(u)
+    elif out.shape != u.shape or out.dtype != u.dtype or not out.is_contiguous():
+        raise ValueError("out must be a contiguous float32 tensor shaped like u")
+    stream = torch.cuda.current_stream(dev).cuda_stream
+    plan = get_plan(L.OP_STENCIL5, H, W, L.F32, dev, variant, params, stream)
+    plan.run(u.data_ptr(), coef.data_ptr(), out.data_ptr(), stream)
+    return out

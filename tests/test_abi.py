@@ -27,7 +27,7 @@ def test_library_exports_every_declared_symbol():
     for name in declared:
         assert hasattr(lib, name), name
     assert sorted(L.SYMBOLS) == declared
-    assert L.lib().adaptic_abi_version() == 5
+    assert L.lib().adaptic_abi_version() == 6
 
 
 def test_enums_match_header():
@@ -106,7 +106,7 @@ def test_invalid_args():
     h = ctypes.c_void_p()
     assert lib.adaptic_plan(0, -1, 5, 0, ctypes.byref(h)) == L.ERR_INVALID_ARG
     assert lib.adaptic_plan(0, 5, -1, 0, ctypes.byref(h)) == L.ERR_INVALID_ARG
-    assert lib.adaptic_plan(8, 5, 5, 0, ctypes.byref(h)) == L.ERR_INVALID_ARG
+    assert lib.adaptic_plan(9, 5, 5, 0, ctypes.byref(h)) == L.ERR_INVALID_ARG
     assert lib.adaptic_plan(0, 5, 5, 9, ctypes.byref(h)) == L.ERR_INVALID_ARG
     assert lib.adaptic_plan(0, 1 << 40, 1 << 40, 0, ctypes.byref(h)) == L.ERR_INVALID_ARG  # byte overflow
     assert lib.adaptic_plan(0, 5, 5, 0, None) == L.ERR_INVALID_ARG
