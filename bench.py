@@ -48,7 +48,7 @@ def parse():
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", choices=["adaptic", "reference"], default="adaptic")
-    ap.add_argument("--workload", choices=["sweep", "rowshard", "splitk", "dot", "blas1", "config0", "multi", "bicgstab"], default="sweep")
+    ap.add_argument("--workload", choices=["sweep", "rowshard", "splitk", "dot", "blas1", "config0", "multi", "bicgstab", "stencil"], default="sweep")
     ap.add_argument("--variant", default="AUTO", help="force one variant (fixed-variant sweeps)")
     ap.add_argument("--dtype", choices=["f32", "i32"], default="f32",
                     help="element type of the MV/TMV/DOT workloads (i32: arithmetic modulo 2^32)")
@@ -159,6 +159,7 @@ def max_over_ranks(v: float, world: int) -> float:
 
 # ------------------------------------------------------------------------------ problems
 B1_OPS = ("asum", "nrm2", "iamax", "iamin", "b1all")
+ST_SHAPES = [(1 << k, 1 << (26 - k)) for k in range(8, 19)]
 B1_SHAPES = [(1, 1 << 26), (64, 1 << 20), (4096, 1 << 14), (1 << 16, 1024), (1 << 20, 64), (1 << 22, 16)]
 
 
@@ -169,6 +170,8 @@ def algo_bytes(op, R, C, nvec=1):
         return 4 * (2 * R * C + R)
     if op in B1_OPS:
         return 4 * (R * C + (4 if op == "b1all" else 1) * R)
+    if op == "stencil5":
+        return 4 * (2 * R * C + 2)                 # u read once, v written once, {c, n}
     return 4 * (R * C + nvec * (C + R))
 
 
@@ -191,13 +194,15 @@ class Problem:
         synth.device_matrix(self.M, Rf, Cf, layout, "uniform", synth.seed(cfg, "A"), rows=rows, cols=cols)
         if op in B1_OPS:
             self.X = torch.empty(0, dtype=torch.float32, device=dev)      # unused
+        elif op == "stencil5":
+            self.X = torch.tensor([0.6, 0.1], dtype=torch.float32, device=dev)   # {c, n}
         elif op == "dot":
             self.X = torch.empty(R * C, dtype=tdt, device=dev)
             synth.device_matrix(self.X, Rf, Cf, "mv", "uniform", synth.seed(cfg, "b"), rows=rows, cols=cols)
         else:
             self.X = torch.empty(C * nvec, dtype=tdt, device=dev)
             synth.device_vector(self.X, "uniform", synth.seed(cfg, "x"), start=cols[0])
-        self.y = torch.empty(R * (4 if op == "b1all" else nvec),
+        self.y = torch.empty(R * C if op == "stencil5" else R * (4 if op == "b1all" else nvec),
                              dtype=torch.int32 if op in ("iamax", "iamin") else tdt, device=dev)
         opc = L.OPS[op]
         self.stream = torch.cuda.current_stream().cuda_stream
@@ -232,6 +237,11 @@ def build_problems(args, world, rank):
             {"workload": "SURVEY 8(f)#1-2: BLAS-1 Sasum/Snrm2/Isamax/Isamin + the four fused in one pass "
                          "(B1ALL, horizontal actor integration) fp32 at 256 MiB, N x L = 1x2^26 .. 2^22x16",
              "shapes": len(B1_SHAPES) * len(B1_OPS)}
+    if args.workload == "stencil":
+        return [Problem("stencil5", H, W, 9, args.variant) for H, W in ST_SHAPES], \
+            {"workload": "SURVEY 8(f)#4: five-point stencil fp32 with input-adaptive super tiles, 256 MiB grids "
+                         "H x W = 256x256K .. 8192^2 .. 256Kx256 (the paper's Convolution Separable aspect "
+                         "ratios, P:796-874, scaled to B200)", "shapes": len(ST_SHAPES)}
     if args.workload == "dot":
         return [Problem("dot", 1, 1 << k, 2, args.variant, dtype=args.dtype) for k in range(10, 31)], \
             {"workload": f"configs[2]: scalar product {args.dtype} N=1, L=2^10..2^30", "shapes": 21}
@@ -364,12 +374,12 @@ def run_adaptic(args):
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": elapsed_ms / args.steps, "higher_is_better": True,
-                "scaling": "weak" if args.workload in ("sweep", "dot") else "strong",
+                "scaling": "strong" if args.workload in ("rowshard", "splitk") else "weak",
                 "vs_baseline": None, "dtype": args.dtype,
                 "data": "synthetic (seeded splitmix64; fp32 U[-1,1), int32 U{-128..127})",
                 "config": dict(config, bytes_per_step_per_gpu=step_bytes, variant=args.variant,
                                l2=("every input >= 256 MiB > 126 MB L2 and problems alternate; no flush needed"
-                                   if args.workload in ("sweep", "blas1") else
+                                   if args.workload in ("sweep", "blas1", "stencil") else
                                    "L2-resident by design (256 KiB): latency-bound, see latency_us"
                                    if args.workload == "config0" else
                                    "dot: lengths 2^10..2^30 back to back; the >= 2^25 ones exceed L2"
@@ -484,6 +494,8 @@ def cpu_baseline(probs, args, budget_s: float = 20.0):
         elif p.op == "tmv":
             for j in range(p.nvec):
                 oracle.tmv(M.reshape(p.C, p.R), X[j * p.C:(j + 1) * p.C])
+        elif p.op == "stencil5":
+            oracle.stencil5(M.reshape(p.R, p.C), float(X[0]), float(X[1]))
         elif p.op in B1_OPS:
             for f in (("asum", "nrm2", "iamax", "iamin") if p.op == "b1all" else (p.op,)):
                 getattr(oracle, f)(M.reshape(p.R, p.C))
@@ -522,6 +534,9 @@ def run_reference(args):
     elif args.workload == "blas1":
         pool = [(op, 1, 1 << 24) for op in B1_OPS[:4]] + [(op, 1 << 16, 256) for op in B1_OPS[:4]]
         cfg = 7
+    elif args.workload == "stencil":
+        pool = [("stencil5", 1024, 1 << 14), ("stencil5", 1 << 14, 1024)]
+        cfg = 9
     else:
         pool = [("tmv", 1024, 1 << 16)]
         cfg = 4
@@ -531,7 +546,7 @@ def run_reference(args):
             a = synth.matrix(R, C, "mv", np.float32, "uniform", synth.seed(cfg, "A"))
             b = synth.matrix(R, C, "mv", np.float32, "uniform", synth.seed(cfg, "b"))
             data.append((op, R, C, a, b, 4 * (2 * R * C + R)))
-        elif op in B1_OPS:
+        elif op in B1_OPS or op == "stencil5":
             a = synth.matrix(R, C, "mv", np.float32, "uniform", synth.seed(cfg, "A"))
             data.append((op, R, C, a, None, algo_bytes(op, R, C)))
         else:
@@ -540,6 +555,7 @@ def run_reference(args):
             data.append((op, R, C, M, x, 4 * (R * C + R + C)))
     fns = {"mv": oracle.mv, "tmv": oracle.tmv, "dot": oracle.dot}
     fns.update({op: (lambda M, X, f=getattr(oracle, op): f(M)) for op in B1_OPS if op != "b1all"})
+    fns["stencil5"] = lambda M, X: oracle.stencil5(M, 0.6, 0.1)
     for s in range(args.warmup):
         op, R, C, M, X, _ = data[s % len(data)]
         fns[op](M, X)

@@ -95,9 +95,10 @@ def test_large_grid_device_generated():
     o = out.cpu().numpy()
     ref, S = oracle.stencil5(u[:64], C0, N0)
     err = np.abs(o[:64].astype(np.float64) - ref)
-    assert (err <= 1e-6 * S).all()
+    assert (err[:-1] <= 1e-6 * S[:-1]).all()              # row 63 is an edge only in the slice
     ref, S = oracle.stencil5(u[-64:], C0, N0)
     err = np.abs(o[-64:].astype(np.float64) - ref)
     assert (err[1:] <= 1e-6 * S[1:]).all()                # row 0 of the slice is an edge only in the slice
-    mid, _ = oracle.stencil5(u[2000:2100], C0, N0)           # a band in the middle (interior rows 1..98)
-    assert np.allclose(o[2001:2099], mid[1:-1], rtol=0, atol=1e-6 * np.abs(mid).max())
+    mid, S = oracle.stencil5(u[2000:2100], C0, N0)           # a band in the middle (interior rows 1..98)
+    err = np.abs(o[2001:2099].astype(np.float64) - mid[1:-1])
+    assert (err <= 1e-6 * S[1:-1]).all()
