@@ -82,6 +82,7 @@ constexpr double kTol = 1e-4;                              // north_star toleran
 int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
 int ilog2_floor(int64_t v) { int k = -1; while (v > 0) { v >>= 1; ++k; } return k; }
 int64_t pow2_ceil(int64_t v) { int64_t p = 1; while (p < v) p <<= 1; return p; }
+int64_t pow2_floor(int64_t v) { int64_t p = 1; while (p * 2 <= v) p <<= 1; return p; }
 int clampi(int64_t v, int lo, int hi) { return int(std::max<int64_t>(lo, std::min<int64_t>(hi, v))); }
 
 struct DevInfo { int dev; int sms; bool present; };
@@ -203,7 +204,9 @@ int64_t pick_splits(int64_t units, int64_t slots, int64_t smax, int64_t smin) {
 
 // ---------------------------------------------------------------- heuristic (no table cell)
 int heuristic_variant(int op, int64_t R, int64_t C, int sms) {
-    if (op == ADAPTIC_OP_STENCIL5) return (C % 4 == 0) ? ADAPTIC_V_ST_TILE : ADAPTIC_V_ST_DIRECT;
+    // measured on B200 (profiles/r1_stencil_sweep.md): the L2-strip direct kernel beats
+    // the shared-memory super tiles on every shape >= 64 MiB and on the L2-resident ones
+    if (op == ADAPTIC_OP_STENCIL5) return ADAPTIC_V_ST_DIRECT;
     if (is_b1_op(op)) {
         // the paper's regimes (Fig. 1) for a unary reduction: lane groups
         // for many short rows, a CTA per row once rows are long and numerous
@@ -296,8 +299,20 @@ adaptic_status derive_stencil(adaptic_plan_s* p, const int32_t* params, const De
     if (v == ADAPTIC_V_ST_DIRECT) {
         p->lanes = 4; p->ctas_per_sm = cps_d;
         if (p->vec_shape) {
-            const int cps = occupancy(st_direct_fn(true), 256, 0, dev.present, 8);
-            p->grid[1] = std::max<int64_t>(1, std::min<int64_t>(ceil_div(H * (W / 4), 256), int64_t(dev.sms) * cps));
+            // rows of >= 2 MB: (strip, row) items strip-major (param ORDER 1 = the plain
+            // row-major grid-stride sweep, 2 = strips).  Measured (profiles/r1_stencil_sweep.md):
+            // equal up to 1-2 MB rows, strips +3..60 % beyond (8 x 8M: 3.9 -> 6.2 TB/s)
+            const int ord = par(ADAPTIC_P_ORDER);
+            p->xmode = (ord == 2 || (ord <= 0 && W / 4 >= ST_STRIP_MIN_ROW)) ? 1 : 0;
+            if (p->xmode == 1) {
+                const int cps = occupancy(st_strip_fn(), 256, 0, dev.present, 8);
+                const int64_t items = ceil_div(W / 4, int64_t(ST_STRIP_SV)) * H;
+                p->grid[1] = std::max<int64_t>(1, std::min<int64_t>(items, int64_t(dev.sms) * cps));
+                p->ctas_per_sm = cps;
+            } else {
+                const int cps = occupancy(st_direct_fn(true), 256, 0, dev.present, 8);
+                p->grid[1] = std::max<int64_t>(1, std::min<int64_t>(ceil_div(H * (W / 4), 256), int64_t(dev.sms) * cps));
+            }
             p->path_ok[1] = true;
         }
         return ADAPTIC_OK;
@@ -393,6 +408,50 @@ adaptic_status derive_multi(adaptic_plan_s* p, const int32_t* params, const DevI
             p->path_ok[w] = bound_ok(p->chain[w] + p->depth[w]);
         }
         return p->path_ok[p->vec_shape ? 1 : 0] ? ADAPTIC_OK : ADAPTIC_ERR_UNSUPPORTED;
+    }
+    if (op == ADAPTIC_OP_MV && (v == ADAPTIC_V_MV_CPR || v == ADAPTIC_V_MV_SPLIT) && p->vec_shape &&
+        (par(ADAPTIC_P_XSMEM) == 3 ||
+         (par(ADAPTIC_P_XSMEM) <= 0 && v == ADAPTIC_V_MV_SPLIT && par(ADAPTIC_P_SPLITS) <= 0))) {
+        // x tiles in shared memory, stream-K ranges of (chunk, row) units (mmv_tile_kernel):
+        // params LANES = chunk width CW (values), ROWS = rows per merge ticket MB
+        const int NT = 256, U = 2;                   // RB = 4 rows per warp step (2 at K = 8)
+        int64_t CW = par(ADAPTIC_P_LANES);
+        if (CW <= 0) CW = (int64_t(K) * C * 4 <= MMV_TILE_ONE_CHUNK) ? C : MMV_TILE_XBYTES / (4 * K);
+        if (CW <= 0 || CW % 4 != 0 || 2 * int64_t(K) * CW * 4 > kXsMaxBytes) return ADAPTIC_ERR_INVALID_ARG;
+        CW = std::min<int64_t>(CW, C);
+        const int64_t nch = ceil_div(C, CW);
+        int MB = par(ADAPTIC_P_ROWS);
+        if (MB <= 0) {
+            // merge work per block: K MB outputs x nch chunks over NT threads, <= ~16 chunks each
+            const int64_t emax = std::max<int64_t>(1, std::min<int64_t>(NT, int64_t(NT) * 16 / nch));
+            MB = clampi(int(pow2_floor(std::max<int64_t>(1, emax / K))), 1, 64);
+        }
+        if (nch * R > (int64_t(1) << 62) / 256) return ADAPTIC_ERR_UNSUPPORTED;
+        if (nch > 1 && int64_t(std::min<int64_t>(MB, R)) * nch > int64_t(UINT_MAX)) return ADAPTIC_ERR_UNSUPPORTED;
+        p->smem = (nch > 1 ? 2 : 1) * size_t(K) * size_t(CW) * 4;   // x chunks, double-buffered
+        p->xmode = 4;
+        int cps = par(ADAPTIC_P_CTAS_PER_SM);
+        if (cps <= 0) cps = occupancy(mmv_tile_fn(K), NT, p->smem, dev.present, 2);
+        p->lanes = int(CW); p->unroll = U; p->block = NT; p->rb = MB; p->ctas_per_sm = cps;
+        p->splits = int(std::min<int64_t>(nch, INT_MAX));
+        p->grid[1] = std::max<int64_t>(1, std::min<int64_t>(nch * R, int64_t(dev.sms) * cps));
+        const int64_t per_lane = ceil_div(CW / 4, int64_t(32));
+        int64_t merge = 0;
+        if (nch > 1) {
+            const int64_t E = int64_t(K) * MB;
+            const int64_t G = E <= NT ? NT / E : 1;
+            const int64_t per = ceil_div(nch, G);
+            merge = std::min<int64_t>(per, 32) + per / 32 + G;
+        }
+        p->chain[1] = 4 * per_lane;
+        p->depth[1] = 5 + merge + 1;
+        p->path_ok[1] = bound_ok(p->chain[1] + p->depth[1]);
+        if (nch > 1) {
+            const size_t part = ((size_t(nch) * size_t(K) * size_t(R) * 4 + 255) / 256) * 256;
+            p->cnt_off = part;
+            p->ws_bytes = part + size_t(ceil_div(R, int64_t(MB))) * 4;
+        }
+        return p->path_ok[1] ? ADAPTIC_OK : ADAPTIC_ERR_UNSUPPORTED;
     }
     if (op == ADAPTIC_OP_MV && (v == ADAPTIC_V_MV_CPR || v == ADAPTIC_V_MV_SPLIT)) {
         const int NT = 256, RB = 8 / K;
@@ -520,11 +579,13 @@ adaptic_status derive_b1(adaptic_plan_s* p, const int32_t* params, const DevInfo
         int rb = par(ADAPTIC_P_ROWS);
         if (rb <= 0) rb = (v == ADAPTIC_V_MV_WPR && nv1 >= 512) ? 1 : 4;
         if (rb != 1 && rb != 4) return ADAPTIC_ERR_INVALID_ARG;
-        const int U = rb == 1 ? 8 : 2;
+        const int rbu = rb == 1 ? 1 : 0;
+        if (op == ADAPTIC_OP_B1ALL && rb == 4) rb = 2;      // the fused op's multi-row instance: 2 rows x 4 loads
+        const int U = rb == 1 ? 8 : (rb == 2 ? 4 : 2);
         p->lanes = G; p->unroll = U; p->rb = rb; p->block = GROUP_NT;
         const int rows_per_cta = rb * (32 / G) * (GROUP_NT / 32);
         int cps = par(ADAPTIC_P_CTAS_PER_SM);
-        if (cps <= 0) cps = occupancy(b1_group_fn(op, G, rb == 1 ? 1 : 0, p->vec_shape), GROUP_NT, 0, dev.present, 4);
+        if (cps <= 0) cps = occupancy(b1_group_fn(op, G, rbu, p->vec_shape), GROUP_NT, 0, dev.present, 4);
         p->ctas_per_sm = cps;
         for (int w = 0; w < 2; ++w) {
             if (w == 1 && !p->vec_shape) continue;
@@ -882,8 +943,7 @@ adaptic_status make_plan(int op, int64_t rows, int64_t cols, int dtype, int vari
         const int64_t nv = (cols % 4 == 0) ? cols / 4 : cols;
         if (op == ADAPTIC_OP_TMV) p->variant = heuristic_variant(op, rows, cols, dev.sms);
         else if (nv <= 32 * (nvec == 8 ? 2 : 4)) p->variant = ADAPTIC_V_MV_SUBWARP;
-        else if (cols % 4 == 0 && int64_t(nvec) * cols * 4 <= MMV_WARP_SMEM)
-            p->variant = ADAPTIC_V_MV_WPR;                                 // warp per row, x in smem
+        else if (cols % 4 == 0) p->variant = ADAPTIC_V_MV_SPLIT;         // x tiles in smem, stream-K
         else if (rows >= 4 * int64_t(dev.sms)) p->variant = ADAPTIC_V_MV_CPR;
         else p->variant = ADAPTIC_V_MV_SPLIT;
         p->source = 2;
@@ -980,6 +1040,7 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
     void* args8[8];
     void* args9[9];
     int ilv = p->ilv;
+    int tile_cw = p->lanes, tile_mb = p->rb;        // mmv_tile_kernel chunk width / ticket rows
     void* args6[6];
     void** args = nullptr;
     int stages = p->stages;
@@ -989,6 +1050,8 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
         if (p->variant == ADAPTIC_V_ST_TILE && vec) {
             fn = st_tile_fn(p->rb, p->lanes);
             smem = p->smem;
+        } else if (vec && p->xmode == 1) {
+            fn = st_strip_fn();
         } else {
             fn = st_direct_fn(vec);
         }
@@ -997,10 +1060,15 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
     } else if (p->nvec > 1) {
         const int K = p->nvec;
         if (p->op == ADAPTIC_OP_TMV) fn = tmmv_fn(K, p->lanes, p->unroll, vec);
+        else if (p->xmode == 4) { fn = vec ? mmv_tile_fn(K) : nullptr; smem = p->smem; }
         else if (p->xmode == 3) { fn = mmv_warp_fn(K); smem = p->smem; }
         else if (p->variant == ADAPTIC_V_MV_SUBWARP || p->variant == ADAPTIC_V_MV_WPR) fn = mmv_group_fn(K, p->lanes, p->unroll, vec);
         else { fn = mmv_cta_fn(K, p->unroll, vec, p->xmode == 1); smem = p->smem; }
-        if (p->op == ADAPTIC_OP_MV && (p->variant == ADAPTIC_V_MV_SUBWARP || p->variant == ADAPTIC_V_MV_WPR)) {
+        if (p->op == ADAPTIC_OP_MV && p->xmode == 4) {
+            args9[0] = &A; args9[1] = &X; args9[2] = &y; args9[3] = &R; args9[4] = &C;
+            args9[5] = &tile_cw; args9[6] = &tile_mb; args9[7] = &part; args9[8] = &cnt;
+            args = args9;
+        } else if (p->op == ADAPTIC_OP_MV && (p->variant == ADAPTIC_V_MV_SUBWARP || p->variant == ADAPTIC_V_MV_WPR)) {
             args6[0] = &A; args6[1] = &X; args6[2] = &y; args6[3] = &R; args6[4] = &C;
             args = args6;                        // register-x group kernel or the warp kernel (xmode 3)
         } else {

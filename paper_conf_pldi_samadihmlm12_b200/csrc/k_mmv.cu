@@ -74,6 +74,16 @@ void* mmv_warp_fn(int K) {
     }
 }
 
+// x-tiled stream-K kernel: RB = 4 rows per warp step, U = 2, NT = 256
+void* mmv_tile_fn(int K) {
+    switch (K) {
+        case 2: return reinterpret_cast<void*>(&mmv_tile_kernel<2, 4, 2, 256>);
+        case 4: return reinterpret_cast<void*>(&mmv_tile_kernel<4, 4, 2, 256>);
+        case 8: return reinterpret_cast<void*>(&mmv_tile_kernel<8, 2, 2, 256>);
+        default: return nullptr;
+    }
+}
+
 #define ADAPTIC_K(FN, ...)                                                       \
     switch (K) {                                                                 \
         case 2: return vec ? FN<2, true>(__VA_ARGS__) : FN<2, false>(__VA_ARGS__); \

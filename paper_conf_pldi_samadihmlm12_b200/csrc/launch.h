@@ -63,11 +63,20 @@ void* mmv_cta_fn(int K, int U, bool vec, bool xs);   // xs: K*C*4 bytes of x sta
 void* tmmv_fn(int K, int LR, int U, bool vec);
 //   warp : (A, X, Y, R, C), warp per row, all K x-vectors in smem (K * C * 4 <= MMV_WARP_SMEM)
 void* mmv_warp_fn(int K);
+//   tile : (A, X, Y, R, C, int CW, int MB, float* part, unsigned* cnt), x chunks of CW values
+//          staged in smem per piece of a stream-K range of (chunk, row) units, NT = 256
+void* mmv_tile_fn(int K);
+constexpr int64_t MMV_TILE_XBYTES = 32 * 1024;       // x bytes per piece (all K vectors)
+constexpr int64_t MMV_TILE_ONE_CHUNK = 48 * 1024;    // up to this K C 4: one chunk, no merge
 
 // Five-point stencil (stencil_kernels.cu), 256 threads:
 //   direct: (const float* u, const float* coef, float* v, int64_t H, int64_t W)
 //   tile  : same arguments, dynamic smem 2 * (TH + 2) * (TW + 8) * 4 bytes
 void* st_direct_fn(bool vec);
+//   strip : same arguments; (strip of ST_STRIP_SV float4 columns, row) items, strip-major
+void* st_strip_fn();
+constexpr int ST_STRIP_SV = 256 * 4;
+constexpr int64_t ST_STRIP_MIN_ROW = 131072;       // float4 per row from which strips are used
 void* st_tile_fn(int TH, int TW);
 constexpr int MMV_WARP_SMEM = 40 * 1024;
 

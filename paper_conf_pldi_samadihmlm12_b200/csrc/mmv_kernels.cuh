@@ -275,6 +275,254 @@ mmv_warp_kernel(const float* __restrict__ A, const float* __restrict__ X, float*
     }
 }
 
+// ------------------------------------------------------------------ MV, x tiles in smem (any row length)
+// Reduce N = 2^n values across a warp at once (a reduce-scatter butterfly): N - 1 + (5 - n)
+// shuffles instead of 5 N.  On return every lane holds the warp total of v[lane >> (5 - n)];
+// the addition tree is fixed, so the result is deterministic.
+template <int N> __device__ __forceinline__ float warp_multi_sum(float (&v)[N]) {
+    static_assert(N >= 1 && N <= 32 && (N & (N - 1)) == 0, "N: power of two <= 32");
+    const int lane = threadIdx.x & 31;
+    int o = 16;
+#pragma unroll
+    for (int h = N / 2; h >= 1; h >>= 1, o >>= 1) {
+        const bool up = (lane & o) != 0;
+#pragma unroll
+        for (int i = 0; i < h; ++i) {
+            const float send = up ? v[i] : v[i + h];
+            const float keep = up ? v[i + h] : v[i];
+            v[i] = keep + __shfl_xor_sync(0xffffffffu, send, o);
+        }
+    }
+    float r = v[0];
+#pragma unroll
+    for (; o >= 1; o >>= 1) r += __shfl_xor_sync(0xffffffffu, r, o);
+    return r;
+}
+
+// The matrix is cut into column chunks of CW values; the work units are (chunk, row)
+// pairs in chunk-major order and CTA b of G owns units [b T / G, (b+1) T / G) (T = nch R),
+// so every CTA streams the same number of row segments (no wave tail) and its range is
+// a few PIECES (chunk, contiguous rows).  Per piece the K x-chunks (K CW 4 bytes) are
+// staged in shared memory by TMA, double-buffered (the next piece's x streams in while
+// this one computes); each warp streams RB rows at a time, U 128-bit loads per row in
+// flight, every x float4 read from smem feeding RB rows, and reduces the RB K dot
+// products with one reduce-scatter butterfly.  A piece with fewer than NW RB rows (few
+// long rows) also splits its columns over the idle warps; their sums are combined in
+// warp order through shared memory.  One chunk: y is written directly; otherwise
+// per-(chunk, row) partials go to the workspace and the CTA that completes a block of MB
+// rows (ticket = rows x chunks delivered) sums the chunks in chunk order (G thread groups
+// over chunk ranges, second-level accumulator every 32 chunks, groups combined in
+// order) -- deterministic, same launch.  x traffic per piece: K CW 4 bytes.
+template <int K, int RB, int U, int NT>
+__global__ void __launch_bounds__(NT, 2)
+mmv_tile_kernel(const float* __restrict__ A, const float* __restrict__ X, float* __restrict__ Y,
+                int64_t R, int64_t C, int CW, int MB, float* __restrict__ part, unsigned int* __restrict__ cnt)
+{
+    constexpr int N = RB * K;
+    constexpr int NW = NT / 32;
+    constexpr int LOGN = (N >= 32) ? 5 : (N >= 16) ? 4 : (N >= 8) ? 3 : (N >= 4) ? 2 : (N >= 2) ? 1 : 0;
+    static_assert((1 << LOGN) == N, "RB * K must be a power of two");
+    pdl_prologue();
+    extern __shared__ __align__(128) unsigned char dyn_smem[];
+    __shared__ __align__(8) uint64_t xbar[2];
+    __shared__ unsigned int s_last[NT];
+    __shared__ float s_red[NT];
+    __shared__ float s_part[NW][N];
+    float4* xs0 = reinterpret_cast<float4*>(dyn_smem);         // [2][K][CW / 4]
+    const int CWV = CW / 4;
+    const int64_t nch = (C + CW - 1) / CW;
+    const int64_t T = nch * R;
+    const int64_t u_beg = T * int64_t(blockIdx.x) / gridDim.x;
+    const int64_t u_end = T * (int64_t(blockIdx.x) + 1) / gridDim.x;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const int64_t nvr = C / 4;                                  // float4 per matrix row
+    const float4* __restrict__ Av = reinterpret_cast<const float4*>(A);
+    auto next_u = [&](int64_t u) {                              // first unit of the following piece
+        const int64_t ra = u % R;
+        return u + (min(R, ra + (u_end - u)) - ra);
+    };
+    auto issue = [&](int64_t u, int buf) {                      // thread 0: x chunk of piece u -> buf
+        const int64_t c0 = (u / R) * CW;
+        const int cw = int(min(int64_t(CW), C - c0));
+        mbar_arrive_expect_tx(&xbar[buf], uint32_t(K) * uint32_t(cw) * 4u);
+#pragma unroll
+        for (int j = 0; j < K; ++j)
+            bulk_g2s_keep(xs0 + (buf * K + j) * CWV, X + int64_t(j) * C + c0, uint32_t(cw) * 4u, &xbar[buf]);
+    };
+    if (threadIdx.x == 0) {
+        mbar_init(&xbar[0], 1); mbar_init(&xbar[1], 1);
+        fence_mbar_init();
+        if (u_beg < u_end) issue(u_beg, 0);
+        const int64_t u1 = u_beg < u_end ? next_u(u_beg) : u_end;
+        if (u1 < u_end) issue(u1, 1);
+    }
+    __syncthreads();
+    int k = 0;
+    for (int64_t u = u_beg; u < u_end; ++k) {
+        const int64_t ch = u / R;
+        const int64_t ra = u - ch * R;
+        const int64_t rb = min(R, ra + (u_end - u));
+        const int64_t c0 = ch * CW;
+        const int nvv = int(min(int64_t(CW), C - c0)) / 4;
+        const int buf = k & 1;
+        const float4* xs = xs0 + buf * K * CWV;
+        mbar_wait(&xbar[buf], uint32_t((k >> 1) & 1));
+        const int nrg = int((rb - ra + RB - 1) / RB);           // row groups of this piece
+        const int cs = nrg >= NW ? 1 : NW / nrg;                // warps per row group
+        const int rg_first = cs == 1 ? warp : warp % nrg;
+        const int sub = cs == 1 ? 0 : warp / nrg;
+        const int v_lo = int(int64_t(nvv) * sub / cs), v_hi = int(int64_t(nvv) * (sub + 1) / cs);
+        for (int rg = rg_first; rg < nrg && sub < cs; rg += (cs == 1 ? NW : nrg)) {
+            const int64_t r0 = ra + int64_t(rg) * RB;
+            const float4* rowp[RB];
+#pragma unroll
+            for (int i = 0; i < RB; ++i) rowp[i] = Av + (r0 + i < rb ? r0 + i : r0) * nvr + c0 / 4;
+            float acc[RB][K];
+#pragma unroll
+            for (int i = 0; i < RB; ++i)
+#pragma unroll
+                for (int j = 0; j < K; ++j) acc[i][j] = 0.f;
+            int v = v_lo + lane;
+            for (; v + 32 * (U - 1) < v_hi; v += 32 * U) {
+                float4 a[RB][U];
+#pragma unroll
+                for (int uu = 0; uu < U; ++uu)
+#pragma unroll
+                    for (int i = 0; i < RB; ++i) a[i][uu] = ld_stream(rowp[i] + v + 32 * uu);
+#pragma unroll
+                for (int uu = 0; uu < U; ++uu)
+#pragma unroll
+                    for (int j = 0; j < K; ++j) {
+                        const float4 xv = xs[j * CWV + v + 32 * uu];
+#pragma unroll
+                        for (int i = 0; i < RB; ++i) {
+                            float t = acc[i][j];
+                            t = fmaf(a[i][uu].x, xv.x, t);
+                            t = fmaf(a[i][uu].y, xv.y, t);
+                            t = fmaf(a[i][uu].z, xv.z, t);
+                            acc[i][j] = fmaf(a[i][uu].w, xv.w, t);
+                        }
+                    }
+            }
+            for (; v < v_hi; v += 32) {
+                float4 a[RB];
+#pragma unroll
+                for (int i = 0; i < RB; ++i) a[i] = ld_stream(rowp[i] + v);
+#pragma unroll
+                for (int j = 0; j < K; ++j) {
+                    const float4 xv = xs[j * CWV + v];
+#pragma unroll
+                    for (int i = 0; i < RB; ++i) {
+                        float t = acc[i][j];
+                        t = fmaf(a[i].x, xv.x, t);
+                        t = fmaf(a[i].y, xv.y, t);
+                        t = fmaf(a[i].z, xv.z, t);
+                        acc[i][j] = fmaf(a[i].w, xv.w, t);
+                    }
+                }
+            }
+            float flat[N];
+#pragma unroll
+            for (int i = 0; i < RB; ++i)
+#pragma unroll
+                for (int j = 0; j < K; ++j) flat[i * K + j] = acc[i][j];
+            const float tot = warp_multi_sum<N>(flat);
+            const int idx = lane >> (5 - LOGN);
+            if ((lane & ((1 << (5 - LOGN)) - 1)) == 0) {
+                if (cs > 1) {
+                    s_part[warp][idx] = tot;
+                } else {
+                    const int i = idx / K, j = idx - (idx / K) * K;
+                    const int64_t row = r0 + i;
+                    if (row < rb) {
+                        if (nch == 1) Y[int64_t(j) * R + row] = tot;
+                        else part[(ch * K + j) * R + row] = tot;
+                    }
+                }
+            }
+        }
+        if (cs > 1) {                                           // combine the column splits in warp order
+            __syncthreads();
+            for (int t = threadIdx.x; t < nrg * N; t += NT) {
+                const int rg = t / N, idx = t - rg * N;
+                float s = 0.f;
+                for (int q = 0; q < cs; ++q) s += s_part[q * nrg + rg][idx];
+                const int i = idx / K, j = idx - (idx / K) * K;
+                const int64_t row = ra + int64_t(rg) * RB + i;
+                if (row < rb) {
+                    if (nch == 1) Y[int64_t(j) * R + row] = s;
+                    else part[(ch * K + j) * R + row] = s;
+                }
+            }
+        }
+        if (nch > 1) {
+            // tickets: rows x chunks delivered per block of MB rows
+            __threadfence();
+            __syncthreads();
+            const int64_t b0 = ra / MB, b1 = (rb - 1) / MB;
+            for (int64_t bb = b0; bb <= b1; bb += NT) {
+                const int64_t blk = bb + threadIdx.x;
+                unsigned int last = 0u;
+                if (blk <= b1) {
+                    const int64_t lo = blk * MB, hi = min(R, lo + MB);
+                    const unsigned int mine = unsigned(min(hi, rb) - max(lo, ra));
+                    const unsigned int need = unsigned(hi - lo) * unsigned(nch);
+                    const unsigned int old = atomicAdd(cnt + blk, mine);
+                    if (old + mine == need) { cnt[blk] = 0u; last = 1u; }
+                }
+                s_last[threadIdx.x] = last;
+                __syncthreads();
+                __threadfence();
+                const int nb = int(min(int64_t(NT), b1 - bb + 1));
+                for (int q = 0; q < nb; ++q) {
+                    if (!s_last[q]) continue;
+                    const int64_t lo = (bb + q) * MB, hi = min(R, lo + MB);
+                    const int rows = int(hi - lo);
+                    const int E = K * rows;                     // outputs of the block
+                    const int G = E <= NT ? NT / E : 1;         // thread groups over chunk ranges
+                    for (int e0 = 0; e0 < E; e0 += NT) {
+                        const int e = G > 1 ? int(threadIdx.x) % E : e0 + int(threadIdx.x);
+                        const int g = G > 1 ? int(threadIdx.x) / E : 0;
+                        float val = 0.f;
+                        if (g < G && e < E) {
+                            const int j = e / rows;
+                            const int64_t r = lo + (e - j * rows);
+                            const int64_t c_lo = nch * g / G, c_hi = nch * (g + 1) / G;
+                            float outer = 0.f, inner = 0.f;
+                            int n32 = 0;
+#pragma unroll 8
+                            for (int64_t c = c_lo; c < c_hi; ++c) {
+                                inner += ld_partial(part + (c * K + j) * R + r);
+                                if (++n32 == 32) { outer += inner; inner = 0.f; n32 = 0; }
+                            }
+                            val = outer + inner;
+                        }
+                        s_red[threadIdx.x] = val;
+                        __syncthreads();
+                        const int ne = G > 1 ? E : min(E - e0, NT);
+                        if (int(threadIdx.x) < ne) {
+                            float t = 0.f;
+                            for (int gg = 0; gg < G; ++gg) t += s_red[gg * E + int(threadIdx.x)];
+                            const int ee = e0 + int(threadIdx.x);
+                            const int j = ee / rows;
+                            Y[int64_t(j) * R + lo + (ee - j * rows)] = t;
+                        }
+                        __syncthreads();
+                    }
+                }
+                __syncthreads();
+            }
+        }
+        __syncthreads();                                        // every warp is done with xs[buf]
+        const int64_t un = u + (rb - ra);
+        if (threadIdx.x == 0 && un < u_end) {
+            const int64_t u2 = next_u(un);
+            if (u2 < u_end) { fence_proxy_async(); issue(u2, buf); }
+        }
+        u = un;
+    }
+}
+
 // ------------------------------------------------------------------ TMV tiles
 // As tmv_kernel: CTA tile of LR output vectors x LC = NT/LR c-lanes, S c-ranges,
 // with K accumulators per thread (one per vector) and the lc-combine per vector.

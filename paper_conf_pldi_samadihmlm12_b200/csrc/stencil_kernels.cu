@@ -63,6 +63,62 @@ st_direct_kernel(const float* __restrict__ u, const float* __restrict__ coef, fl
     }
 }
 
+// --------------------------------------------------------------------------- L2 strips
+// The B200 form of the paper's super tile: the grid is cut into vertical strips of SV
+// = NT V float4 columns and the work items (strip, row) are taken strip-major, so the
+// CTAs in flight at any time cover a band of consecutive rows of ONE strip and a row's
+// top and bottom neighbours are read by concurrently running CTAs -- the reuse is
+// captured by L2 (126 MB) instead of a shared-memory halo.  Without strips a long row
+// (8 x 8M: 32 MB per row) is evicted before the next row needs it (measured 3.9 TB/s
+// row-major vs 6.2 with strips; equal for rows up to ~2 MB).  Each thread issues its V centre/top/bottom float4 loads and its
+// 2 V edge scalars before the first FMA; v is stored evict-first.
+template <int NT, int V>
+__global__ void __launch_bounds__(NT)
+st_strip_kernel(const float* __restrict__ u, const float* __restrict__ coef, float* __restrict__ v,
+                int64_t H, int64_t W)
+{
+    pdl_prologue();
+    constexpr int SV = NT * V;
+    const float c = __ldg(coef), n = __ldg(coef + 1);
+    const int64_t nvr = W / 4;
+    const int64_t nstrips = (nvr + SV - 1) / SV;
+    const int64_t items = nstrips * H;
+    const float4* __restrict__ u4 = reinterpret_cast<const float4*>(u);
+    float4* __restrict__ v4 = reinterpret_cast<float4*>(v);
+    for (int64_t it = blockIdx.x; it < items; it += gridDim.x) {
+        const int64_t s = it / H, i = it - s * H;
+        const bool inner = i > 0 && i < H - 1;
+        const int64_t row = i * nvr;
+        float4 ce[V], t[V], b[V];
+        float l[V], r[V];
+#pragma unroll
+        for (int q = 0; q < V; ++q) {
+            const int64_t k = s * SV + q * NT + threadIdx.x;
+            const int64_t kk = k < nvr ? k : nvr - 1;             // stay in bounds; result discarded
+            ce[q] = __ldg(u4 + row + kk);
+            if (inner) {
+                t[q] = __ldg(u4 + row - nvr + kk);
+                b[q] = __ldg(u4 + row + nvr + kk);
+                l[q] = kk > 0 ? __ldg(u + 4 * (row + kk) - 1) : 0.f;
+                r[q] = kk < nvr - 1 ? __ldg(u + 4 * (row + kk) + 4) : 0.f;
+            }
+        }
+#pragma unroll
+        for (int q = 0; q < V; ++q) {
+            const int64_t k = s * SV + q * NT + threadIdx.x;
+            if (k >= nvr) continue;
+            float4 o = ce[q];
+            if (inner) {
+                if (k > 0) o.x = st_point(c, n, ce[q].x, t[q].x, b[q].x, l[q], ce[q].y);
+                o.y = st_point(c, n, ce[q].y, t[q].y, b[q].y, ce[q].x, ce[q].z);
+                o.z = st_point(c, n, ce[q].z, t[q].z, b[q].z, ce[q].y, ce[q].w);
+                if (k < nvr - 1) o.w = st_point(c, n, ce[q].w, t[q].w, b[q].w, ce[q].z, r[q]);
+            }
+            __stcs(v4 + row + k, o);
+        }
+    }
+}
+
 // --------------------------------------------------------------------------- super tiles
 // Shared buffer b holds input rows row0-1 .. row0+TH (clamped to the grid) and columns
 // col0-4 .. col0+TW+3 (clamped), at smem column (global column - col0 + 4).
@@ -139,6 +195,8 @@ void* st_direct_fn(bool vec) {
     return vec ? reinterpret_cast<void*>(&st_direct_kernel<true, 256>)
                : reinterpret_cast<void*>(&st_direct_kernel<false, 256>);
 }
+
+void* st_strip_fn() { return reinterpret_cast<void*>(&st_strip_kernel<256, 4>); }
 
 template <int TH>
 static void* st_tile_w(int TW) {

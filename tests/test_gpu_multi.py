@@ -19,7 +19,9 @@ DEV = "cuda:0"
 TOL = 1e-4
 MV_FORCED = [("AUTO", None)] + [("MV_SUBWARP", [g, 0, 0, u]) for g in (1, 4, 16) for u in (1, 2, 4)] + \
             [("MV_WPR", [0, 0, 0, u]) for u in (1, 2)] + [("MV_CPR", [0, 0, 0, u]) for u in (1, 2)] + \
-            [("MV_SPLIT", [0, s, 0, 2]) for s in (2, 7)]
+            [("MV_SPLIT", [0, s, 0, 2]) for s in (2, 7)] + \
+            [("MV_SPLIT", [0, 0, 0, 0, 3]), ("MV_SPLIT", [128, 0, 0, 0, 3, 0, 1]), ("MV_SPLIT", [256, 0, 1, 0, 3, 0, 3]),
+             ("MV_CPR", [1024, 0, 0, 0, 3, 0, 64])]   # x-tile stream-K kernel: default, many chunks, odd MB
 TMV_FORCED = [("AUTO", None), ("TMV_COL", None)] + [("TMV_SPLITK", [lr, s]) for lr in (1, 8, 64) for s in (0, 3)] + \
              [("TMV_REGTILE", None)]
 
@@ -89,11 +91,12 @@ def test_exact_on_integer_data_and_equal_to_single_calls():
 
 
 def test_device_generated_256MiB():
-    for op, (R, C) in (("mv", (4096, 16384)), ("tmv", (16384, 4096))):
+    for op, (R, C), K in (("mv", (4096, 16384), 4), ("tmv", (16384, 4096), 4), ("mv", (64, 1 << 20), 4),
+                          ("mv", (64, 1 << 20), 8), ("mv", (8192, 8192), 2), ("mv", (65536, 1024), 8)):
         t = torch.empty(R * C, dtype=torch.float32, device=DEV)
         synth.device_matrix(t, R, C, op, "uniform", synth.seed(14, "A"))
         M = t.cpu().numpy().reshape((R, C) if op == "mv" else (C, R))
-        X = synth.matrix(4, C, "mv", np.float32, "uniform", 15)
+        X = synth.matrix(K, C, "mv", np.float32, "uniform", 15)
         fn = adaptic.mv_multi if op == "mv" else adaptic.tmv_multi
         Y = fn(t.view(M.shape), torch.from_numpy(X).to(DEV)).cpu().numpy()
-        check(Y, M, X, op, f"{op} 256MiB")
+        check(Y, M, X, op, f"{op} {R}x{C} K={K} 256MiB")

@@ -44,8 +44,9 @@ def _collect(cases):
 
 
 SHAPES = [(1, 4), (2, 8), (3, 3), (5, 12), (33, 100), (64, 256), (65, 260), (129, 1000), (300, 516), (1000, 64),
-          (7, 4096), (2049, 132)]
-FORCED = [("AUTO", None), ("ST_DIRECT", None)] + \
+          (7, 4096), (2049, 132), (5, 8200), (9, 16384), (1, 8192)]
+FORCED = [("AUTO", None), ("ST_DIRECT", None), ("ST_DIRECT", [0, 0, 0, 0, 0, 0, 0, 1]),
+          ("ST_DIRECT", [0, 0, 0, 0, 0, 0, 0, 2])] + \
          [("ST_TILE", [tw, 0, 0, 0, 0, 0, th]) for th in (4, 8, 16, 32) for tw in (128, 256, 512)]
 
 
