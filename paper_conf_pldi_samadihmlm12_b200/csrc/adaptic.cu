@@ -202,6 +202,23 @@ int64_t pick_splits(int64_t units, int64_t slots, int64_t smax, int64_t smin) {
     return best;
 }
 
+// Split count for persistent grid-stride kernels whose blocks are long: the smallest S
+// whose blocks fill the last wave to >= 90 % (one partly idle wave of long blocks costs
+// less than a second wave plus twice the partials to merge).
+int64_t pick_splits_wave(int64_t units, int64_t slots, int64_t smax) {
+    units = std::max<int64_t>(1, units);
+    int64_t best = 1;
+    double best_eff = -1.0;
+    for (int64_t S = 1; S <= std::max<int64_t>(1, smax); ++S) {
+        const int64_t nblk = units * S;
+        const double eff = double(nblk) / double(ceil_div(nblk, slots) * slots);
+        if (eff >= 0.9) return S;
+        if (eff > best_eff + 1e-9) { best_eff = eff; best = S; }
+        if (nblk > 4 * slots) break;
+    }
+    return best;
+}
+
 // ---------------------------------------------------------------- heuristic (no table cell)
 int heuristic_variant(int op, int64_t R, int64_t C, int sms) {
     // measured on B200 (profiles/r1_stencil_sweep.md): the L2-strip direct kernel beats
@@ -303,8 +320,15 @@ adaptic_status derive_stencil(adaptic_plan_s* p, const int32_t* params, const De
             // row-major grid-stride sweep, 2 = strips).  Measured (profiles/r1_stencil_sweep.md):
             // equal up to 1-2 MB rows, strips +3..60 % beyond (8 x 8M: 3.9 -> 6.2 TB/s)
             const int ord = par(ADAPTIC_P_ORDER);
-            p->xmode = (ord == 2 || (ord <= 0 && W / 4 >= ST_STRIP_MIN_ROW)) ? 1 : 0;
-            if (p->xmode == 1) {
+            p->xmode = (ord == 2 || (ord <= 0 && W / 4 >= ST_STRIP_MIN_ROW)) ? 1 : (ord == 3 ? 2 : 0);
+            if (p->xmode == 2) {                             // column sweep, register sliding window
+                const int th = par(ADAPTIC_P_ROWS) > 0 ? par(ADAPTIC_P_ROWS) : 64;
+                p->rb = th;
+                const int cps = occupancy(st_column_fn(), 256, 0, dev.present, 8);
+                const int64_t tiles = ceil_div(W / 4, int64_t(256)) * ceil_div(H, int64_t(th));
+                p->grid[1] = std::max<int64_t>(1, std::min<int64_t>(tiles, int64_t(dev.sms) * cps));
+                p->ctas_per_sm = cps;
+            } else if (p->xmode == 1) {
                 const int cps = occupancy(st_strip_fn(), 256, 0, dev.present, 8);
                 const int64_t items = ceil_div(W / 4, int64_t(ST_STRIP_SV)) * H;
                 p->grid[1] = std::max<int64_t>(1, std::min<int64_t>(items, int64_t(dev.sms) * cps));
@@ -411,7 +435,8 @@ adaptic_status derive_multi(adaptic_plan_s* p, const int32_t* params, const DevI
     }
     if (op == ADAPTIC_OP_MV && (v == ADAPTIC_V_MV_CPR || v == ADAPTIC_V_MV_SPLIT) && p->vec_shape &&
         (par(ADAPTIC_P_XSMEM) == 3 ||
-         (par(ADAPTIC_P_XSMEM) <= 0 && v == ADAPTIC_V_MV_SPLIT && par(ADAPTIC_P_SPLITS) <= 0))) {
+         (par(ADAPTIC_P_XSMEM) <= 0 && v == ADAPTIC_V_MV_SPLIT && par(ADAPTIC_P_SPLITS) <= 0 && R > 16))) {
+        // (R <= 16: the interleaved-split kernel with x through L1 measured 1.3x faster at 8 rows)
         // x tiles in shared memory, stream-K ranges of (chunk, row) units (mmv_tile_kernel):
         // params LANES = chunk width CW (values), ROWS = rows per merge ticket MB
         const int NT = 256, U = 2;                   // RB = 4 rows per warp step (2 at K = 8)
@@ -422,8 +447,9 @@ adaptic_status derive_multi(adaptic_plan_s* p, const int32_t* params, const DevI
         const int64_t nch = ceil_div(C, CW);
         int MB = par(ADAPTIC_P_ROWS);
         if (MB <= 0) {
-            // merge work per block: K MB outputs x nch chunks over NT threads, <= ~16 chunks each
-            const int64_t emax = std::max<int64_t>(1, std::min<int64_t>(NT, int64_t(NT) * 16 / nch));
+            // merge work per block: K MB outputs x nch chunks over NT threads, <= ~64 chunks each
+            // (measured, 64 x 1M K = 4: MB 8 -> 4.25 TB/s, MB 2 -> 3.45, MB 64 -> 3.45)
+            const int64_t emax = std::max<int64_t>(1, std::min<int64_t>(NT, int64_t(NT) * 64 / nch));
             MB = clampi(int(pow2_floor(std::max<int64_t>(1, emax / K))), 1, 64);
         }
         if (nch * R > (int64_t(1) << 62) / 256) return ADAPTIC_ERR_UNSUPPORTED;
@@ -510,9 +536,73 @@ adaptic_status derive_multi(adaptic_plan_s* p, const int32_t* params, const DevI
     const int64_t rv1 = p->vec_shape ? R / 4 : R;
     int LR = par(ADAPTIC_P_LANES);
     if (LR <= 0) LR = (v == ADAPTIC_V_TMV_COL) ? 256 : (v == ADAPTIC_V_TMV_REGTILE) ? clampi(pow2_ceil(rv1), 1, 256)
-                                                                                  : clampi(pow2_ceil(rv1), 1, 64);
+                                                                                  : clampi(pow2_ceil(rv1), 1, rv1 <= 256 ? 32 : 64);
     if (LR < 1 || LR > 256 || (LR & (LR - 1))) return ADAPTIC_ERR_INVALID_ARG;
     if (v == ADAPTIC_V_TMV_REGTILE && rv1 > LR) return ADAPTIC_ERR_UNSUPPORTED;
+    // B rows staged by TMA (tmmv_tma_kernel; param XSMEM 1 = the register-fed kernel)
+    // measured (profiles/r1c_multi_tmv.md): TMA staging wins for few outputs (R <= 256: one
+    // contiguous bulk copy per stage, +23-34 % at K = 4) and for R >= 256K with C >= 128 (+14-25 %);
+    // elsewhere both are within a few % and the register-fed kernel is kept.
+    // param XSMEM: 3 = TMA-staged, 1 = register-fed, 0 = this rule
+    const int xreq = par(ADAPTIC_P_XSMEM);
+    const bool tma_rule = rv1 <= 64 || (rv1 >= 65536 && C >= 128);
+    if (p->vec_shape && rv1 >= 16 && v != ADAPTIC_V_TMV_COL && (xreq == 3 || (xreq <= 0 && tma_rule)) &&
+        (par(ADAPTIC_P_LANES) <= 0 || par(ADAPTIC_P_LANES) >= 16)) {
+        // LR: the widest tile (longest bulk copies) whose split count still fills the GPU with
+        // at most 16 LC partials to merge per thread (the merging CTA reads S / LC per thread)
+        p->smem = size_t(TMMV_TMA_STAGES) * TMMV_TMA_STAGE_V4 * 16;
+        int cps = par(ADAPTIC_P_CTAS_PER_SM);
+        if (cps <= 0) cps = occupancy(tmmv_tma_fn(K, 64), NT, p->smem, dev.present, 2);
+        const int64_t slots = int64_t(dev.sms) * cps;
+        auto splits_for = [&](int lr) -> int64_t {
+            const int64_t tiles = ceil_div(rv1, int64_t(lr));
+            const int64_t cr = TMMV_TMA_STAGE_V4 / lr;
+            const int64_t O = int64_t(K) * std::min<int64_t>(lr, rv1);            // float4 outputs per tile
+            const int64_t cap = std::max<int64_t>(1, std::min<int64_t>(tiles == 1 ? 1024 : 64 * std::max<int64_t>(1, NT / O),
+                                                                     ceil_div(C, cr)));
+            return pick_splits(tiles, slots, cap, 1);
+        };
+        bool one_split = false;
+        if (par(ADAPTIC_P_LANES) <= 0 && rv1 <= 256) {
+            LR = int(std::max<int64_t>(16, pow2_ceil(rv1)));      // one tile: contiguous stages
+        } else if (par(ADAPTIC_P_LANES) <= 0 && xreq <= 0) {
+            LR = 256;                                              // huge R: 4 KB row copies, no split
+            one_split = true;
+        } else if (par(ADAPTIC_P_LANES) <= 0) {
+            // wave efficiency of each tile width; the widest within 5 % of the best (longer copies)
+            double eff[5] = {0, 0, 0, 0, 0}, best_eff = 0.0;
+            for (int i = 0, lr = 256; lr >= 16; lr >>= 1, ++i) {
+                if (lr > std::max<int64_t>(16, pow2_ceil(rv1))) continue;
+                const int64_t blocks = ceil_div(rv1, int64_t(lr)) * splits_for(lr);
+                eff[i] = double(blocks) / double(ceil_div(blocks, slots) * slots);
+                best_eff = std::max(best_eff, eff[i]);
+            }
+            LR = 16;
+            for (int i = 0, lr = 256; lr >= 16; lr >>= 1, ++i)
+                if (eff[i] > 0.0 && eff[i] >= best_eff - 0.05) { LR = lr; break; }
+        }
+        if (!tmmv_tma_fn(K, LR)) return ADAPTIC_ERR_INVALID_ARG;
+        const int LC = NT / LR;
+        p->xmode = 5;
+        p->lanes = LR; p->unroll = 1; p->block = NT; p->ctas_per_sm = cps;
+        const int64_t tiles = ceil_div(rv1, int64_t(LR));
+        const int64_t cr = TMMV_TMA_STAGE_V4 / LR;
+        int64_t S = par(ADAPTIC_P_SPLITS) > 0 ? par(ADAPTIC_P_SPLITS) : one_split ? 1 : splits_for(LR);
+        const int64_t rows = ceil_div(ceil_div(C, S), int64_t(LC));
+        p->chain[1] = std::min<int64_t>(rows, FOLD + cr / LC) + rows / FOLD;
+        const int64_t Gm = std::max<int64_t>(1, NT / (int64_t(K) * std::min<int64_t>(LR, rv1)));
+        p->depth[1] = ilog2c(LC) + (S > 1 ? ceil_div(S, Gm) + Gm : 0) + 1;
+        p->path_ok[1] = bound_ok(p->chain[1] + p->depth[1]);
+        p->grid[1] = std::max<int64_t>(1, std::min<int64_t>(tiles * S, slots));
+        if (S > INT_MAX || !p->path_ok[1]) return ADAPTIC_ERR_UNSUPPORTED;
+        p->splits = int(S);
+        if (S > 1) {
+            const size_t part = ((size_t(R) * size_t(K) * size_t(S) * 4 + 255) / 256) * 256;
+            p->cnt_off = part;
+            p->ws_bytes = part + size_t(tiles) * 4;
+        }
+        return ADAPTIC_OK;
+    }
     int cps = par(ADAPTIC_P_CTAS_PER_SM);
     if (cps <= 0) cps = occupancy(tmmv_fn(K, LR, U, p->vec_shape), NT, 0, dev.present, 2048 / NT);
     p->lanes = LR; p->unroll = U; p->block = NT; p->ctas_per_sm = cps;
@@ -520,7 +610,7 @@ adaptic_status derive_multi(adaptic_plan_s* p, const int32_t* params, const DevI
     const int64_t slots = int64_t(dev.sms) * cps;
     int64_t S = 1;
     if (par(ADAPTIC_P_SPLITS) > 0) S = par(ADAPTIC_P_SPLITS);
-    else if (v != ADAPTIC_V_TMV_COL) S = pick_splits(ceil_div(rv1, LR), slots, std::max<int64_t>(1, ceil_div(C, int64_t(LC) * U)), 1);
+    else if (v != ADAPTIC_V_TMV_COL) S = pick_splits_wave(ceil_div(rv1, LR), slots, std::max<int64_t>(1, ceil_div(C, int64_t(LC) * U)));
     for (;;) {
         bool ok_all = true;
         for (int w = 0; w < 2; ++w) {
@@ -570,11 +660,6 @@ adaptic_status derive_b1(adaptic_plan_s* p, const int32_t* params, const DevInfo
     const int64_t nv1 = p->vec_shape ? C / 4 : C;
 
     if (v == ADAPTIC_V_MV_SUBWARP || v == ADAPTIC_V_MV_WPR) {
-        int G;
-        if (v == ADAPTIC_V_MV_WPR) G = 32;
-        else if (par(ADAPTIC_P_LANES) > 0) G = par(ADAPTIC_P_LANES);
-        else G = clampi(pow2_ceil(ceil_div(std::max<int64_t>(1, nv1), 2)), 1, 16);
-        if (G < 1 || G > 32 || (G & (G - 1)) || (v == ADAPTIC_V_MV_SUBWARP && G > 16)) return ADAPTIC_ERR_INVALID_ARG;
         // (RB, U): 4 rows x 2 loads (short rows) or 1 row x 8 loads (long rows)
         int rb = par(ADAPTIC_P_ROWS);
         if (rb <= 0) rb = (v == ADAPTIC_V_MV_WPR && nv1 >= 512) ? 1 : 4;
@@ -582,6 +667,12 @@ adaptic_status derive_b1(adaptic_plan_s* p, const int32_t* params, const DevInfo
         const int rbu = rb == 1 ? 1 : 0;
         if (op == ADAPTIC_OP_B1ALL && rb == 4) rb = 2;      // the fused op's multi-row instance: 2 rows x 4 loads
         const int U = rb == 1 ? 8 : (rb == 2 ? 4 : 2);
+        // lanes per row: a row is one step of G x U loads (so the unrolled main loop runs)
+        int G;
+        if (v == ADAPTIC_V_MV_WPR) G = 32;
+        else if (par(ADAPTIC_P_LANES) > 0) G = par(ADAPTIC_P_LANES);
+        else G = clampi(pow2_ceil(ceil_div(std::max<int64_t>(1, nv1), U)), 1, 16);
+        if (G < 1 || G > 32 || (G & (G - 1)) || (v == ADAPTIC_V_MV_SUBWARP && G > 16)) return ADAPTIC_ERR_INVALID_ARG;
         p->lanes = G; p->unroll = U; p->rb = rb; p->block = GROUP_NT;
         const int rows_per_cta = rb * (32 / G) * (GROUP_NT / 32);
         int cps = par(ADAPTIC_P_CTAS_PER_SM);
@@ -941,7 +1032,15 @@ adaptic_status make_plan(int op, int64_t rows, int64_t cols, int dtype, int vari
     }
     if (nvec > 1) {                    // multi-vector: the regime rules of the paper (Fig. 1)
         const int64_t nv = (cols % 4 == 0) ? cols / 4 : cols;
-        if (op == ADAPTIC_OP_TMV) p->variant = heuristic_variant(op, rows, cols, dev.sms);
+        if (op == ADAPTIC_OP_TMV) {
+            // measured (profiles/r1c_multi_tmv.md): TMA-staged tiles for R <= 256 and for R >= 256K
+            // with C >= 128 (derive_multi's rule); register-fed SPLITK tiles with one wave of
+            // splits elsewhere; TMV_COL for huge R with few rows of B
+            const int64_t rv = rows / 4;
+            if (rows % 4 == 0 && rv >= 65536 && cols < 128) p->variant = ADAPTIC_V_TMV_COL;
+            else if (rows % 4 == 0 && rv >= 16) p->variant = ADAPTIC_V_TMV_SPLITK;
+            else p->variant = heuristic_variant(op, rows, cols, dev.sms);
+        }
         else if (nv <= 32 * (nvec == 8 ? 2 : 4)) p->variant = ADAPTIC_V_MV_SUBWARP;
         else if (cols % 4 == 0) p->variant = ADAPTIC_V_MV_SPLIT;         // x tiles in smem, stream-K
         else if (rows >= 4 * int64_t(dev.sms)) p->variant = ADAPTIC_V_MV_CPR;
@@ -1052,14 +1151,21 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
             smem = p->smem;
         } else if (vec && p->xmode == 1) {
             fn = st_strip_fn();
+        } else if (vec && p->xmode == 2) {
+            fn = st_column_fn();
+            args7[0] = &A; args7[1] = &X; args7[2] = &y; args7[3] = &R; args7[4] = &C; args7[5] = &tile_mb;
+            args = args7;
         } else {
             fn = st_direct_fn(vec);
         }
-        args6[0] = &A; args6[1] = &X; args6[2] = &y; args6[3] = &R; args6[4] = &C;
-        args = args6;
+        if (!args) {
+            args6[0] = &A; args6[1] = &X; args6[2] = &y; args6[3] = &R; args6[4] = &C;
+            args = args6;
+        }
     } else if (p->nvec > 1) {
         const int K = p->nvec;
-        if (p->op == ADAPTIC_OP_TMV) fn = tmmv_fn(K, p->lanes, p->unroll, vec);
+        if (p->op == ADAPTIC_OP_TMV && p->xmode == 5) { fn = vec ? tmmv_tma_fn(K, p->lanes) : nullptr; smem = p->smem; }
+        else if (p->op == ADAPTIC_OP_TMV) fn = tmmv_fn(K, p->lanes, p->unroll, vec);
         else if (p->xmode == 4) { fn = vec ? mmv_tile_fn(K) : nullptr; smem = p->smem; }
         else if (p->xmode == 3) { fn = mmv_warp_fn(K); smem = p->smem; }
         else if (p->variant == ADAPTIC_V_MV_SUBWARP || p->variant == ADAPTIC_V_MV_WPR) fn = mmv_group_fn(K, p->lanes, p->unroll, vec);

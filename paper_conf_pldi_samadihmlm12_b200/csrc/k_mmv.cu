@@ -84,6 +84,27 @@ void* mmv_tile_fn(int K) {
     }
 }
 
+template <int K>
+static void* tt_l(int LR) {
+    switch (LR) {
+        case 16: return reinterpret_cast<void*>(&tmmv_tma_kernel<K, 16, 256>);
+        case 32: return reinterpret_cast<void*>(&tmmv_tma_kernel<K, 32, 256>);
+        case 64: return reinterpret_cast<void*>(&tmmv_tma_kernel<K, 64, 256>);
+        case 128: return reinterpret_cast<void*>(&tmmv_tma_kernel<K, 128, 256>);
+        case 256: return reinterpret_cast<void*>(&tmmv_tma_kernel<K, 256, 256>);
+        default: return nullptr;
+    }
+}
+
+void* tmmv_tma_fn(int K, int LR) {
+    switch (K) {
+        case 2: return tt_l<2>(LR);
+        case 4: return tt_l<4>(LR);
+        case 8: return tt_l<8>(LR);
+        default: return nullptr;
+    }
+}
+
 #define ADAPTIC_K(FN, ...)                                                       \
     switch (K) {                                                                 \
         case 2: return vec ? FN<2, true>(__VA_ARGS__) : FN<2, false>(__VA_ARGS__); \

@@ -66,6 +66,11 @@ void* mmv_warp_fn(int K);
 //   tile : (A, X, Y, R, C, int CW, int MB, float* part, unsigned* cnt), x chunks of CW values
 //          staged in smem per piece of a stream-K range of (chunk, row) units, NT = 256
 void* mmv_tile_fn(int K);
+//   tmma : tmmv arguments; B rows staged by TMA in TMMV_TMA_STAGES stages of
+//          TMMV_TMA_STAGE_V4 float4 (CR = STAGE_V4 / LR rows of LR float4), NT = 256, LR in {16..256}
+void* tmmv_tma_fn(int K, int LR);
+constexpr int TMMV_TMA_STAGE_V4 = 2048;              // 32 KB per stage
+constexpr int TMMV_TMA_STAGES = 3;
 constexpr int64_t MMV_TILE_XBYTES = 32 * 1024;       // x bytes per piece (all K vectors)
 constexpr int64_t MMV_TILE_ONE_CHUNK = 48 * 1024;    // up to this K C 4: one chunk, no merge
 
@@ -75,6 +80,9 @@ constexpr int64_t MMV_TILE_ONE_CHUNK = 48 * 1024;    // up to this K C 4: one ch
 void* st_direct_fn(bool vec);
 //   strip : same arguments; (strip of ST_STRIP_SV float4 columns, row) items, strip-major
 void* st_strip_fn();
+//   column: (u, coef, v, H, W, int TH): NT = 256 float4 columns x TH rows per tile, register
+//           sliding window down each column (D = 4 rows loaded ahead)
+void* st_column_fn();
 constexpr int ST_STRIP_SV = 256 * 4;
 constexpr int64_t ST_STRIP_MIN_ROW = 131072;       // float4 per row from which strips are used
 void* st_tile_fn(int TH, int TW);

@@ -603,4 +603,177 @@ tmmv_kernel(const float* __restrict__ B, const float* __restrict__ X, float* __r
     }
 }
 
+// ------------------------------------------------------------------ TMV tiles, TMA-staged
+// Same tiling and split/merge as tmmv_kernel, but the B rows of a (tile, split) block
+// arrive in shared memory by TMA bulk copies (one per B row segment of 16 LR bytes,
+// issued by the lanes of warp 0) into an ST-deep ring of CR-row stages, so the bytes in
+// flight (ST CR LR 16 per CTA) no longer cost registers: with K accumulators per
+// thread the register-fed kernel kept only U = 4 float4 in flight per thread and was
+// latency-bound (ncu: long-scoreboard stalls, 16 warps/SM, ~4.3 TB/s).  The ring runs
+// across the CTA's blocks (stage i + ST is issued as soon as stage i is consumed).
+// Threads read b = stage[row][lr] (a warp reads 32 consecutive float4, conflict-free)
+// and x_j[c] through L1 (one broadcast per warp when LR >= 32).  When one tile covers
+// all outputs (R <= 4 LR) consecutive B rows are contiguous and a stage is ONE bulk copy
+// (row pitch R/4 in shared memory): per-row copies of a few hundred bytes ran at 1.9 TB/s.
+template <int K, int LR, int NT>
+__global__ void __launch_bounds__(NT, 2)
+tmmv_tma_kernel(const float* __restrict__ B, const float* __restrict__ X, float* __restrict__ Y,
+                int64_t R, int64_t C, int S, float* __restrict__ ws_part, unsigned int* __restrict__ ws_cnt)
+{
+    pdl_prologue();
+    constexpr int LC = NT / LR;
+    constexpr int CR = TMMV_TMA_STAGE_V4 / LR;           // B rows per stage
+    constexpr int ST = TMMV_TMA_STAGES;
+    static_assert(CR % LC == 0 && CR >= LC, "stage rows: a multiple of the c-lanes");
+    extern __shared__ __align__(128) unsigned char dyn_smem[];
+    float4* ring = reinterpret_cast<float4*>(dyn_smem);  // [ST][CR][LR]
+    __shared__ __align__(8) uint64_t full[ST];
+    __shared__ float4 red[LC > 1 ? NT : 1];
+    __shared__ float4 s_merge[NT];
+    __shared__ unsigned int flag;
+    const int64_t rv = R / 4;
+    const int64_t ntiles = (rv + LR - 1) / LR;
+    const int64_t chunk = (C + S - 1) / S;
+    const float4* __restrict__ Bv = reinterpret_cast<const float4*>(B);
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int lr = tid % LR, lc = tid / LR;
+    const int64_t nblk = ntiles * S;
+    const int64_t my_blks = blockIdx.x < nblk ? (nblk - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+    auto geom = [&](int64_t m, int64_t& tile, int& s, int64_t& c0, int64_t& c1, int& w) {
+        const int64_t blk = blockIdx.x + m * gridDim.x;
+        tile = blk % ntiles;
+        s = int(blk / ntiles);
+        c0 = min(C, int64_t(s) * chunk);
+        c1 = min(C, c0 + chunk);
+        w = int(min(int64_t(LR), rv - tile * LR));
+    };
+    // producer (warp 0, uniform state): next (block, stage) to issue
+    int64_t pm = 0, pst = 0, issued = 0;
+    auto produce = [&]() {
+        int64_t tile, c0, c1, nst = 0; int s, w;
+        for (; pm < my_blks; ++pm) {                      // skip empty splits
+            geom(pm, tile, s, c0, c1, w);
+            nst = (c1 - c0 + CR - 1) / CR;
+            if (nst > 0) break;
+        }
+        if (pm >= my_blks) return;
+        const int64_t r_lo = c0 + pst * CR;
+        const int nr = int(min(int64_t(CR), c1 - r_lo));
+        const int slot = int(issued % ST);
+        if (lane == 0) mbar_arrive_expect_tx(&full[slot], uint32_t(nr) * uint32_t(w) * 16u);
+        __syncwarp();
+        fence_proxy_async();
+        if (ntiles == 1) {                                // whole rows: the stage is one contiguous block
+            if (lane == 0)
+                bulk_g2s(ring + size_t(slot) * CR * LR, Bv + r_lo * rv, uint32_t(nr) * uint32_t(w) * 16u, &full[slot]);
+        } else {
+            for (int q = lane; q < nr; q += 32)
+                bulk_g2s(ring + (size_t(slot) * CR + q) * LR, Bv + (r_lo + q) * rv + tile * LR, uint32_t(w) * 16u, &full[slot]);
+        }
+        ++issued;
+        if (++pst == nst) { pst = 0; ++pm; }
+    };
+    if (tid == 0) {
+        for (int i = 0; i < ST; ++i) mbar_init(&full[i], 1);
+        fence_mbar_init();
+    }
+    __syncthreads();
+    if (warp == 0)
+        while (issued < ST && pm < my_blks) produce();
+    int64_t consumed = 0;
+    float4* yv = reinterpret_cast<float4*>(Y);
+    float4* pv = reinterpret_cast<float4*>(ws_part);
+    for (int64_t m = 0; m < my_blks; ++m) {
+        int64_t tile, c0, c1; int s, w;
+        geom(m, tile, s, c0, c1, w);
+        const int64_t nst = (c1 - c0 + CR - 1) / CR;
+        const int64_t r4 = tile * LR + lr;
+        const bool rok = lr < w;
+        float4 acc[K], outer[K];
+#pragma unroll
+        for (int j = 0; j < K; ++j) { acc[j] = make_float4(0.f, 0.f, 0.f, 0.f); outer[j] = acc[j]; }
+        int rows_acc = 0;
+        for (int64_t st = 0; st < nst; ++st, ++consumed) {
+            const int slot = int(consumed % ST);
+            const int64_t r_lo = c0 + st * CR;
+            const int nr = int(min(int64_t(CR), c1 - r_lo));
+            mbar_wait(&full[slot], uint32_t((consumed / ST) & 1));
+            const float4* sb = ring + size_t(slot) * CR * LR;
+            const int P = ntiles == 1 ? w : LR;           // smem row pitch (float4)
+            if (rok) {
+                if (nr == CR) {
+#pragma unroll (K <= 4 ? 4 : 2)
+                    for (int q = lc; q < CR; q += LC) {
+                        const float4 b = sb[q * P + lr];
+#pragma unroll
+                        for (int j = 0; j < K; ++j) esmac(acc[j], b, ld_x(X + j * C + r_lo + q));
+                    }
+                } else {
+                    for (int q = lc; q < nr; q += LC) {
+                        const float4 b = sb[q * P + lr];
+#pragma unroll
+                        for (int j = 0; j < K; ++j) esmac(acc[j], b, ld_x(X + j * C + r_lo + q));
+                    }
+                }
+            }
+            rows_acc += CR / LC;
+            if (rows_acc >= FOLD) {                       // bounded fp32 chains (planner: chain_of)
+                rows_acc = 0;
+#pragma unroll
+                for (int j = 0; j < K; ++j) { outer[j] = eadd(outer[j], acc[j]); acc[j] = make_float4(0.f, 0.f, 0.f, 0.f); }
+            }
+            __syncthreads();                              // every thread is done with the slot
+            if (warp == 0 && pm < my_blks) produce();
+        }
+#pragma unroll
+        for (int j = 0; j < K; ++j) {
+            const float4 tot = lc_combine<NT, LR>(eadd(outer[j], acc[j]), red);
+            if (S == 1) {
+                if (tid < LR && rok) yv[j * rv + r4] = tot;
+            } else if (tid < LR && rok) {
+                pv[(int64_t(s) * K + j) * rv + r4] = tot;
+            }
+            __syncthreads();                              // red[] reuse by the next vector
+        }
+        if (S > 1 && ticket_is_last(ws_cnt + tile, unsigned(S), &flag)) {
+            // O = K w float4 outputs x S partials: G = NT / O thread groups each sum a contiguous
+            // slot range with 4 independent accumulators, then the groups combine in order
+            const int O = K * w;
+            const int G = O <= NT ? NT / O : 1;
+            for (int o0 = 0; o0 < O; o0 += NT) {
+                const int o = G > 1 ? tid % O : o0 + tid;
+                const int g = G > 1 ? tid / O : 0;
+                float4 mm = make_float4(0.f, 0.f, 0.f, 0.f);
+                if (g < G && o < O) {
+                    const int j = o / w, q = o - (o / w) * w;
+                    const float4* base = pv + int64_t(j) * rv + tile * LR + q;
+                    const int64_t stride = int64_t(K) * rv;
+                    const int64_t s_lo = int64_t(S) * g / G, s_hi = int64_t(S) * (g + 1) / G;
+                    float4 m1 = mm, m2 = mm, m3 = mm;
+                    int64_t sl = s_lo;
+                    for (; sl + 3 < s_hi; sl += 4) {
+                        const float4 t0 = ld_partial(base + sl * stride), t1 = ld_partial(base + (sl + 1) * stride);
+                        const float4 t2 = ld_partial(base + (sl + 2) * stride), t3 = ld_partial(base + (sl + 3) * stride);
+                        mm = eadd(mm, t0); m1 = eadd(m1, t1); m2 = eadd(m2, t2); m3 = eadd(m3, t3);
+                    }
+                    for (; sl < s_hi; ++sl) mm = eadd(mm, ld_partial(base + sl * stride));
+                    mm = eadd(eadd(mm, m1), eadd(m2, m3));
+                }
+                s_merge[tid] = mm;
+                __syncthreads();
+                const int no = G > 1 ? O : min(O - o0, NT);
+                if (tid < no) {
+                    float4 t = make_float4(0.f, 0.f, 0.f, 0.f);
+                    for (int gg = 0; gg < G; ++gg) t = eadd(t, s_merge[gg * (G > 1 ? O : 0) + tid]);
+                    const int oo = o0 + tid;
+                    const int j = oo / w, q = oo - (oo / w) * w;
+                    yv[int64_t(j) * rv + tile * LR + q] = t;
+                }
+                __syncthreads();
+            }
+        }
+        __syncthreads();
+    }
+}
+
 }  // namespace adaptic

@@ -119,6 +119,70 @@ st_strip_kernel(const float* __restrict__ u, const float* __restrict__ coef, flo
     }
 }
 
+// --------------------------------------------------------------------------- column sweep
+// Register sliding window: a CTA owns NT float4 columns x TH rows and each thread walks
+// down its column keeping rows i-1, i, i+1 in registers, so every input float4 is loaded
+// ONCE (plus 2 halo rows per tile) instead of three times through L1/L2; the left/right
+// neighbours come from the adjacent lanes by shuffles (scalar loads only at the warp
+// edges).  The next D rows are loaded together (D float4 in flight per thread).  Tiles
+// are taken column-strip-major so vertically adjacent tiles -- which share halo rows --
+// run at the same time.
+template <int NT, int D>
+__global__ void __launch_bounds__(NT)
+st_column_kernel(const float* __restrict__ u, const float* __restrict__ coef, float* __restrict__ v,
+                 int64_t H, int64_t W, int TH)
+{
+    pdl_prologue();
+    const float c = __ldg(coef), n = __ldg(coef + 1);
+    const int64_t nvr = W / 4;
+    const int64_t tiles_c = (nvr + NT - 1) / NT, tiles_r = (H + TH - 1) / TH;
+    const int64_t ntiles = tiles_c * tiles_r;
+    const float4* __restrict__ u4 = reinterpret_cast<const float4*>(u);
+    float4* __restrict__ v4 = reinterpret_cast<float4*>(v);
+    const int lane = threadIdx.x & 31;
+    const float4 z = make_float4(0.f, 0.f, 0.f, 0.f);
+    for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+        const int64_t tc = t / tiles_r, tr = t - tc * tiles_r;
+        const int64_t k = tc * NT + threadIdx.x;
+        const bool ok = k < nvr;
+        const int64_t kk = ok ? k : nvr - 1;                    // in bounds; results discarded
+        const int64_t r0 = tr * TH, r1 = min(H, r0 + TH);
+        const bool lo_edge = (k == 0), hi_edge = (k == nvr - 1);
+        // lane 0 / lane 31 (and the last column) take their outer neighbour from memory
+        const bool need_l = (lane == 0) && k > 0;
+        const bool need_r = (lane == 31 || k == nvr - 1 || threadIdx.x == NT - 1) && k < nvr - 1;
+        float4 up = r0 > 0 ? __ldg(u4 + (r0 - 1) * nvr + kk) : z;
+        float4 q[D + 1];
+#pragma unroll
+        for (int d = 0; d <= D; ++d) q[d] = (r0 + d < H) ? __ldg(u4 + (r0 + d) * nvr + kk) : z;
+        for (int64_t i = r0; i < r1; i += D) {
+#pragma unroll
+            for (int d = 0; d < D; ++d) {
+                const int64_t row = i + d;
+                if (row >= r1) break;
+                const float4 ce = q[d], dn = q[d + 1];
+                float l = __shfl_up_sync(0xffffffffu, ce.w, 1);
+                float r = __shfl_down_sync(0xffffffffu, ce.x, 1);
+                if (need_l) l = __ldg(u + 4 * (row * nvr + kk) - 1);
+                if (need_r) r = __ldg(u + 4 * (row * nvr + kk) + 4);
+                float4 o = ce;
+                if (row > 0 && row < H - 1) {
+                    if (!lo_edge) o.x = st_point(c, n, ce.x, up.x, dn.x, l, ce.y);
+                    o.y = st_point(c, n, ce.y, up.y, dn.y, ce.x, ce.z);
+                    o.z = st_point(c, n, ce.z, up.z, dn.z, ce.y, ce.w);
+                    if (!hi_edge) o.w = st_point(c, n, ce.w, up.w, dn.w, ce.z, r);
+                }
+                if (ok) __stcs(v4 + row * nvr + k, o);
+                up = ce;
+            }
+            q[0] = q[D];
+#pragma unroll
+            for (int d = 1; d <= D; ++d)                        // rows up to r1 (the last row's dn)
+                q[d] = (i + D + d < H && i + D + d <= r1) ? __ldg(u4 + (i + D + d) * nvr + kk) : z;
+        }
+    }
+}
+
 // --------------------------------------------------------------------------- super tiles
 // Shared buffer b holds input rows row0-1 .. row0+TH (clamped to the grid) and columns
 // col0-4 .. col0+TW+3 (clamped), at smem column (global column - col0 + 4).
@@ -197,6 +261,7 @@ void* st_direct_fn(bool vec) {
 }
 
 void* st_strip_fn() { return reinterpret_cast<void*>(&st_strip_kernel<256, 4>); }
+void* st_column_fn() { return reinterpret_cast<void*>(&st_column_kernel<256, 4>); }
 
 template <int TH>
 static void* st_tile_w(int TW) {

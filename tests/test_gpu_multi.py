@@ -23,7 +23,9 @@ MV_FORCED = [("AUTO", None)] + [("MV_SUBWARP", [g, 0, 0, u]) for g in (1, 4, 16)
             [("MV_SPLIT", [0, 0, 0, 0, 3]), ("MV_SPLIT", [128, 0, 0, 0, 3, 0, 1]), ("MV_SPLIT", [256, 0, 1, 0, 3, 0, 3]),
              ("MV_CPR", [1024, 0, 0, 0, 3, 0, 64])]   # x-tile stream-K kernel: default, many chunks, odd MB
 TMV_FORCED = [("AUTO", None), ("TMV_COL", None)] + [("TMV_SPLITK", [lr, s]) for lr in (1, 8, 64) for s in (0, 3)] + \
-             [("TMV_REGTILE", None)]
+             [("TMV_REGTILE", None), ("TMV_SPLITK", [64, 0, 0, 0, 1]), ("TMV_SPLITK", [16, 5, 0, 0, 3]),
+              ("TMV_SPLITK", [256, 3, 1, 0, 3]), ("TMV_SPLITK", [0, 0, 0, 0, 3]),
+              ("TMV_REGTILE", [0, 0, 0, 0, 3])]    # register-fed kernel; TMA-staged (XSMEM 3)
 
 
 def check(Y, M, X, op, what):
@@ -47,7 +49,8 @@ def _collect(cases):
 @pytest.mark.parametrize("op", ["mv", "tmv"])
 @pytest.mark.parametrize("K", [2, 4, 8])
 def test_every_variant(op, K):
-    shapes = [(1, 1), (3, 5), (33, 64), (100, 257), (517, 1024), (7, 40000), (1000, 12), (64, 100), (5000, 8)]
+    shapes = [(1, 1), (3, 5), (33, 64), (100, 257), (517, 1024), (7, 40000), (1000, 12), (64, 100), (5000, 8),
+              (256, 40000), (1024, 3001), (2048, 17)]
     forced = MV_FORCED if op == "mv" else TMV_FORCED
 
     def case(R, C, v, p):
@@ -92,7 +95,8 @@ def test_exact_on_integer_data_and_equal_to_single_calls():
 
 def test_device_generated_256MiB():
     for op, (R, C), K in (("mv", (4096, 16384), 4), ("tmv", (16384, 4096), 4), ("mv", (64, 1 << 20), 4),
-                          ("mv", (64, 1 << 20), 8), ("mv", (8192, 8192), 2), ("mv", (65536, 1024), 8)):
+                          ("mv", (64, 1 << 20), 8), ("mv", (8192, 8192), 2), ("mv", (65536, 1024), 8),
+                          ("tmv", (64, 1 << 20), 4), ("tmv", (8192, 8192), 8), ("tmv", (1 << 20, 64), 2)):
         t = torch.empty(R * C, dtype=torch.float32, device=DEV)
         synth.device_matrix(t, R, C, op, "uniform", synth.seed(14, "A"))
         M = t.cpu().numpy().reshape((R, C) if op == "mv" else (C, R))

@@ -46,7 +46,8 @@ def _collect(cases):
 SHAPES = [(1, 4), (2, 8), (3, 3), (5, 12), (33, 100), (64, 256), (65, 260), (129, 1000), (300, 516), (1000, 64),
           (7, 4096), (2049, 132), (5, 8200), (9, 16384), (1, 8192)]
 FORCED = [("AUTO", None), ("ST_DIRECT", None), ("ST_DIRECT", [0, 0, 0, 0, 0, 0, 0, 1]),
-          ("ST_DIRECT", [0, 0, 0, 0, 0, 0, 0, 2])] + \
+          ("ST_DIRECT", [0, 0, 0, 0, 0, 0, 0, 2]), ("ST_DIRECT", [0, 0, 0, 0, 0, 0, 0, 3]),
+          ("ST_DIRECT", [0, 0, 0, 0, 0, 0, 3, 3]), ("ST_DIRECT", [0, 0, 0, 0, 0, 0, 9, 3])] + \
          [("ST_TILE", [tw, 0, 0, 0, 0, 0, th]) for th in (4, 8, 16, 32) for tw in (128, 256, 512)]
 
 
@@ -82,9 +83,10 @@ def test_harmonic_field_is_reproduced():
     H, W = 200, 640
     i, j = np.meshgrid(np.arange(H), np.arange(W), indexing="ij")
     u = (i + 2 * j).astype(np.float32)
-    for v in ("ST_DIRECT", "ST_TILE"):
-        out = adaptic.stencil5(torch.from_numpy(u).to(DEV), 0.5, 0.125, variant=v).cpu().numpy()
-        assert np.array_equal(out, u), v
+    for v, p in (("ST_DIRECT", None), ("ST_TILE", None), ("ST_DIRECT", [0, 0, 0, 0, 0, 0, 0, 2]),
+                 ("ST_DIRECT", [0, 0, 0, 0, 0, 0, 0, 3])):
+        out = adaptic.stencil5(torch.from_numpy(u).to(DEV), 0.5, 0.125, variant=v, params=p).cpu().numpy()
+        assert np.array_equal(out, u), (v, p)
 
 
 def test_large_grid_device_generated():

@@ -30,7 +30,11 @@ TW = (128, 256, 512)
 
 
 def grid(W):
-    out = [("AUTO", None), ("ST_DIRECT", None)]
+    out = [("AUTO", None), ("ST_DIRECT", [0, 0, 0, 0, 0, 0, 0, 1])]
+    if W >= 4096:
+        out.append(("ST_DIRECT", [0, 0, 0, 0, 0, 0, 0, 2]))
+    for th in (16, 32, 64, 128):
+        out.append(("ST_DIRECT", [0, 0, 0, 0, 0, 0, th, 3]))
     for th in TH:
         for tw in TW:
             if tw > max(128, W):
