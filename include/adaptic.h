@@ -187,6 +187,13 @@ typedef enum {
  *   [ADAPTIC_P_XSMEM]  MV_SUBWARP / MV_WPR / MV_CPR: 1 = read x through the
  *                      read-only cache path, 2 = stage x in shared memory once per
  *                      CTA with a TMA bulk copy (needs cols*4 <= 200 KB).
+ *                      MV_CPR / MV_SPLIT, fp32, cols % 4 == 0: 3 = the x-tile
+ *                      stream-K kernel (column chunks of [ADAPTIC_P_LANES] values,
+ *                      x chunks TMA-staged and double-buffered, (chunk, row) units
+ *                      split evenly over the CTAs, chunk partials merged in order
+ *                      per block of [ADAPTIC_P_ROWS] rows); 4-byte-aligned pointers
+ *                      then run the CTA-per-row kernel.  Multi-vector TMV: 3 = B
+ *                      rows staged by TMA, 1 = register-fed tiles.
  *   [ADAPTIC_P_BLOCK]  TMV_*: threads per CTA, 256 or 1024 (unroll <= 4 at 1024).
  *   [ADAPTIC_P_ROWS]   MV_CPR / MV_SPLIT: rows per CTA step sharing each x load,
  *                      (rows, unroll) in {(1,2),(1,4),(1,8),(2,2),(2,4),(4,2)}.
@@ -195,6 +202,9 @@ typedef enum {
  *                      threads*unroll vectors (default when splits > 1).
  *   [ADAPTIC_P_PIPE]   MV_CPR / MV_SPLIT with 256 threads: 1 = single-buffered
  *                      loads (default), 2 = register double-buffered main loop.
+ *   ST_DIRECT: [ADAPTIC_P_ORDER] 1 = row-major grid-stride sweep, 2 = L2 strips
+ *                      (default for rows >= 2 MB), 3 = register sliding window down
+ *                      float4 columns, [ADAPTIC_P_ROWS] rows per tile (default 64).
  *   ST_TILE: [ADAPTIC_P_ROWS] super-tile height TH in {4, 8, 16, 32}, [ADAPTIC_P_LANES]
  *                      width TW in {128, 256, 512} (default: the paper's reuse metric
  *                      sum(accesses)/halo, among tilings with enough blocks). */

@@ -457,7 +457,7 @@ adaptic_status derive_multi(adaptic_plan_s* p, const int32_t* params, const DevI
         p->smem = (nch > 1 ? 2 : 1) * size_t(K) * size_t(CW) * 4;   // x chunks, double-buffered
         p->xmode = 4;
         int cps = par(ADAPTIC_P_CTAS_PER_SM);
-        if (cps <= 0) cps = occupancy(mmv_tile_fn(K), NT, p->smem, dev.present, 2);
+        if (cps <= 0) cps = occupancy(mmv_tile_fn(p->dtype, K), NT, p->smem, dev.present, 2);
         p->lanes = int(CW); p->unroll = U; p->block = NT; p->rb = MB; p->ctas_per_sm = cps;
         p->splits = int(std::min<int64_t>(nch, INT_MAX));
         p->grid[1] = std::max<int64_t>(1, std::min<int64_t>(nch * R, int64_t(dev.sms) * cps));
@@ -736,6 +736,10 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
     const int v = p->variant;
     if (!op_has_variant(op, v)) return ADAPTIC_ERR_UNSUPPORTED;
     if (p->nvec > 1) return derive_multi(p, params, dev);
+    // single-vector MV (fp32 or int32) on the x-tile stream-K kernel (param XSMEM 3)
+    if (op == ADAPTIC_OP_MV && (v == ADAPTIC_V_MV_CPR || v == ADAPTIC_V_MV_SPLIT) &&
+        par(ADAPTIC_P_XSMEM) == 3 && C % 4 == 0)
+        return derive_multi(p, params, dev);
     if (op == ADAPTIC_OP_STENCIL5) return derive_stencil(p, params, dev);
     if (is_b1_op(op)) return derive_b1(p, params, dev);
 
@@ -1166,7 +1170,7 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
         const int K = p->nvec;
         if (p->op == ADAPTIC_OP_TMV && p->xmode == 5) { fn = vec ? tmmv_tma_fn(K, p->lanes) : nullptr; smem = p->smem; }
         else if (p->op == ADAPTIC_OP_TMV) fn = tmmv_fn(K, p->lanes, p->unroll, vec);
-        else if (p->xmode == 4) { fn = vec ? mmv_tile_fn(K) : nullptr; smem = p->smem; }
+        else if (p->xmode == 4) { fn = vec ? mmv_tile_fn(ADAPTIC_F32, K) : nullptr; smem = p->smem; }
         else if (p->xmode == 3) { fn = mmv_warp_fn(K); smem = p->smem; }
         else if (p->variant == ADAPTIC_V_MV_SUBWARP || p->variant == ADAPTIC_V_MV_WPR) fn = mmv_group_fn(K, p->lanes, p->unroll, vec);
         else { fn = mmv_cta_fn(K, p->unroll, vec, p->xmode == 1); smem = p->smem; }
@@ -1218,6 +1222,14 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
             break;
         case ADAPTIC_V_MV_CPR:
         case ADAPTIC_V_MV_SPLIT:
+            if (p->xmode == 4) {                          // x-tile stream-K kernel, K = 1
+                fn = vec ? mmv_tile_fn(dt, 1) : nullptr;
+                smem = p->smem;
+                args9[0] = &A; args9[1] = &X; args9[2] = &y; args9[3] = &R; args9[4] = &C;
+                args9[5] = &tile_cw; args9[6] = &tile_mb; args9[7] = &part; args9[8] = &cnt;
+                args = args9;
+                break;
+            }
             fn = mis ? mis_cta_fn(dt, p->lanes, p->unroll, p->xmode)
                      : cta_fn(dt, p->lanes, p->rb, p->unroll, vec, p->xmode, p->pipe != 0);
             smem = p->smem;
@@ -1373,6 +1385,17 @@ adaptic_status adaptic_run(adaptic_plan_t p, const void* A, const void* x, void*
                 ((reinterpret_cast<uintptr_t>(A) - reinterpret_cast<uintptr_t>(x)) & 15u) == 0);
     if (mis && p->variant == ADAPTIC_V_MV_TPR)   // bulk copies of row tiles: 16-byte aligned bases
         mis = aligned(A, 16) && (p->op != ADAPTIC_OP_DOT || aligned(x, 16));
+    if (!vec && p->nvec == 1 && p->xmode == 4) {
+        // the x-tile kernel needs 16-byte rows and bases (TMA): a single-vector plan run on
+        // 4-byte-aligned pointers takes the CTA-per-row kernel of the same shape instead
+        adaptic_plan_s fb = *p;
+        fb.variant = ADAPTIC_V_MV_CPR;
+        fb.ws = nullptr;
+        if (derive(&fb, nullptr, device_info()) != ADAPTIC_OK || fb.ws_bytes != 0) return ADAPTIC_ERR_UNSUPPORTED;
+        const bool fmis = fb.mis;
+        if (!fb.path_ok[fmis ? 1 : 0]) return ADAPTIC_ERR_MISALIGNED;
+        return launch(&fb, A, x, y, stream, false, fmis);
+    }
     if (!p->path_ok[(vec || mis) ? 1 : 0]) return ADAPTIC_ERR_MISALIGNED;   // scalar path would break the error bound
     return launch(p, A, x, y, stream, vec, mis);
 }

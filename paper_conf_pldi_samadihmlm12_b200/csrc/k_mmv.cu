@@ -3,6 +3,7 @@
 //   cta  : NT = 256, U in {1, 2} x VEC x x-in-shared-memory
 //   tmmv : LR in {1,...,256} x VEC x U in {2, 4} (4 only for K <= 4), NT = 256
 #include "mmv_kernels.cuh"
+#include "adaptic.h"
 
 namespace adaptic {
 
@@ -74,12 +75,15 @@ void* mmv_warp_fn(int K) {
     }
 }
 
-// x-tiled stream-K kernel: RB = 4 rows per warp step, U = 2, NT = 256
-void* mmv_tile_fn(int K) {
+// x-tiled stream-K kernel: RB = 4 rows per warp step (2 at K = 8), U = 2 (4 at K = 1), NT = 256;
+// K = 1 also for int32 (dt = ADAPTIC_I32)
+void* mmv_tile_fn(int dt, int K) {
+    if (dt == ADAPTIC_I32) return K == 1 ? reinterpret_cast<void*>(&mmv_tile_kernel<uint32_t, 1, 4, 4, 256>) : nullptr;
     switch (K) {
-        case 2: return reinterpret_cast<void*>(&mmv_tile_kernel<2, 4, 2, 256>);
-        case 4: return reinterpret_cast<void*>(&mmv_tile_kernel<4, 4, 2, 256>);
-        case 8: return reinterpret_cast<void*>(&mmv_tile_kernel<8, 2, 2, 256>);
+        case 1: return reinterpret_cast<void*>(&mmv_tile_kernel<float, 1, 4, 4, 256>);
+        case 2: return reinterpret_cast<void*>(&mmv_tile_kernel<float, 2, 4, 2, 256>);
+        case 4: return reinterpret_cast<void*>(&mmv_tile_kernel<float, 4, 4, 2, 256>);
+        case 8: return reinterpret_cast<void*>(&mmv_tile_kernel<float, 8, 2, 2, 256>);
         default: return nullptr;
     }
 }

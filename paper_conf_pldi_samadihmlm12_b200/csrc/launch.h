@@ -65,7 +65,7 @@ void* tmmv_fn(int K, int LR, int U, bool vec);
 void* mmv_warp_fn(int K);
 //   tile : (A, X, Y, R, C, int CW, int MB, float* part, unsigned* cnt), x chunks of CW values
 //          staged in smem per piece of a stream-K range of (chunk, row) units, NT = 256
-void* mmv_tile_fn(int K);
+void* mmv_tile_fn(int dt, int K);
 //   tmma : tmmv arguments; B rows staged by TMA in TMMV_TMA_STAGES stages of
 //          TMMV_TMA_STAGE_V4 float4 (CR = STAGE_V4 / LR rows of LR float4), NT = 256, LR in {16..256}
 void* tmmv_tma_fn(int K, int LR);

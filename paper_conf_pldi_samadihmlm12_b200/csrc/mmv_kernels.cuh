@@ -279,7 +279,7 @@ mmv_warp_kernel(const float* __restrict__ A, const float* __restrict__ X, float*
 // Reduce N = 2^n values across a warp at once (a reduce-scatter butterfly): N - 1 + (5 - n)
 // shuffles instead of 5 N.  On return every lane holds the warp total of v[lane >> (5 - n)];
 // the addition tree is fixed, so the result is deterministic.
-template <int N> __device__ __forceinline__ float warp_multi_sum(float (&v)[N]) {
+template <int N, class T> __device__ __forceinline__ T warp_multi_sum(T (&v)[N]) {
     static_assert(N >= 1 && N <= 32 && (N & (N - 1)) == 0, "N: power of two <= 32");
     const int lane = threadIdx.x & 31;
     int o = 16;
@@ -288,12 +288,12 @@ template <int N> __device__ __forceinline__ float warp_multi_sum(float (&v)[N]) 
         const bool up = (lane & o) != 0;
 #pragma unroll
         for (int i = 0; i < h; ++i) {
-            const float send = up ? v[i] : v[i + h];
-            const float keep = up ? v[i + h] : v[i];
+            const T send = up ? v[i] : v[i + h];
+            const T keep = up ? v[i + h] : v[i];
             v[i] = keep + __shfl_xor_sync(0xffffffffu, send, o);
         }
     }
-    float r = v[0];
+    T r = v[0];
 #pragma unroll
     for (; o >= 1; o >>= 1) r += __shfl_xor_sync(0xffffffffu, r, o);
     return r;
@@ -313,11 +313,13 @@ template <int N> __device__ __forceinline__ float warp_multi_sum(float (&v)[N]) 
 // rows (ticket = rows x chunks delivered) sums the chunks in chunk order (G thread groups
 // over chunk ranges, second-level accumulator every 32 chunks, groups combined in
 // order) -- deterministic, same launch.  x traffic per piece: K CW 4 bytes.
-template <int K, int RB, int U, int NT>
+// T = float or uint32_t (int32 modulo 2^32: any order is exact); K > 1 is fp32 only.
+template <class T, int K, int RB, int U, int NT>
 __global__ void __launch_bounds__(NT, 2)
-mmv_tile_kernel(const float* __restrict__ A, const float* __restrict__ X, float* __restrict__ Y,
-                int64_t R, int64_t C, int CW, int MB, float* __restrict__ part, unsigned int* __restrict__ cnt)
+mmv_tile_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restrict__ Y,
+                int64_t R, int64_t C, int CW, int MB, T* __restrict__ part, unsigned int* __restrict__ cnt)
 {
+    using V = vec4_t<T>;
     constexpr int N = RB * K;
     constexpr int NW = NT / 32;
     constexpr int LOGN = (N >= 32) ? 5 : (N >= 16) ? 4 : (N >= 8) ? 3 : (N >= 4) ? 2 : (N >= 2) ? 1 : 0;
@@ -326,17 +328,17 @@ mmv_tile_kernel(const float* __restrict__ A, const float* __restrict__ X, float*
     extern __shared__ __align__(128) unsigned char dyn_smem[];
     __shared__ __align__(8) uint64_t xbar[2];
     __shared__ unsigned int s_last[NT];
-    __shared__ float s_red[NT];
-    __shared__ float s_part[NW][N];
-    float4* xs0 = reinterpret_cast<float4*>(dyn_smem);         // [2][K][CW / 4]
+    __shared__ T s_red[NT];
+    __shared__ T s_part[NW][N];
+    V* xs0 = reinterpret_cast<V*>(dyn_smem);                   // [2][K][CW / 4]
     const int CWV = CW / 4;
     const int64_t nch = (C + CW - 1) / CW;
-    const int64_t T = nch * R;
-    const int64_t u_beg = T * int64_t(blockIdx.x) / gridDim.x;
-    const int64_t u_end = T * (int64_t(blockIdx.x) + 1) / gridDim.x;
+    const int64_t TU = nch * R;                                // (chunk, row) units
+    const int64_t u_beg = TU * int64_t(blockIdx.x) / gridDim.x;
+    const int64_t u_end = TU * (int64_t(blockIdx.x) + 1) / gridDim.x;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int64_t nvr = C / 4;                                  // float4 per matrix row
-    const float4* __restrict__ Av = reinterpret_cast<const float4*>(A);
+    const V* __restrict__ Av = reinterpret_cast<const V*>(A);
     auto next_u = [&](int64_t u) {                              // first unit of the following piece
         const int64_t ra = u % R;
         return u + (min(R, ra + (u_end - u)) - ra);
@@ -365,7 +367,7 @@ mmv_tile_kernel(const float* __restrict__ A, const float* __restrict__ X, float*
         const int64_t c0 = ch * CW;
         const int nvv = int(min(int64_t(CW), C - c0)) / 4;
         const int buf = k & 1;
-        const float4* xs = xs0 + buf * K * CWV;
+        const V* xs = xs0 + buf * K * CWV;
         mbar_wait(&xbar[buf], uint32_t((k >> 1) & 1));
         const int nrg = int((rb - ra + RB - 1) / RB);           // row groups of this piece
         const int cs = nrg >= NW ? 1 : NW / nrg;                // warps per row group
@@ -374,17 +376,17 @@ mmv_tile_kernel(const float* __restrict__ A, const float* __restrict__ X, float*
         const int v_lo = int(int64_t(nvv) * sub / cs), v_hi = int(int64_t(nvv) * (sub + 1) / cs);
         for (int rg = rg_first; rg < nrg && sub < cs; rg += (cs == 1 ? NW : nrg)) {
             const int64_t r0 = ra + int64_t(rg) * RB;
-            const float4* rowp[RB];
+            const V* rowp[RB];
 #pragma unroll
             for (int i = 0; i < RB; ++i) rowp[i] = Av + (r0 + i < rb ? r0 + i : r0) * nvr + c0 / 4;
-            float acc[RB][K];
+            T acc[RB][K];
 #pragma unroll
             for (int i = 0; i < RB; ++i)
 #pragma unroll
-                for (int j = 0; j < K; ++j) acc[i][j] = 0.f;
+                for (int j = 0; j < K; ++j) acc[i][j] = T(0);
             int v = v_lo + lane;
             for (; v + 32 * (U - 1) < v_hi; v += 32 * U) {
-                float4 a[RB][U];
+                V a[RB][U];
 #pragma unroll
                 for (int uu = 0; uu < U; ++uu)
 #pragma unroll
@@ -393,40 +395,40 @@ mmv_tile_kernel(const float* __restrict__ A, const float* __restrict__ X, float*
                 for (int uu = 0; uu < U; ++uu)
 #pragma unroll
                     for (int j = 0; j < K; ++j) {
-                        const float4 xv = xs[j * CWV + v + 32 * uu];
+                        const V xv = xs[j * CWV + v + 32 * uu];
 #pragma unroll
                         for (int i = 0; i < RB; ++i) {
-                            float t = acc[i][j];
-                            t = fmaf(a[i][uu].x, xv.x, t);
-                            t = fmaf(a[i][uu].y, xv.y, t);
-                            t = fmaf(a[i][uu].z, xv.z, t);
-                            acc[i][j] = fmaf(a[i][uu].w, xv.w, t);
+                            T t = acc[i][j];
+                            t = mac(a[i][uu].x, xv.x, t);
+                            t = mac(a[i][uu].y, xv.y, t);
+                            t = mac(a[i][uu].z, xv.z, t);
+                            acc[i][j] = mac(a[i][uu].w, xv.w, t);
                         }
                     }
             }
             for (; v < v_hi; v += 32) {
-                float4 a[RB];
+                V a[RB];
 #pragma unroll
                 for (int i = 0; i < RB; ++i) a[i] = ld_stream(rowp[i] + v);
 #pragma unroll
                 for (int j = 0; j < K; ++j) {
-                    const float4 xv = xs[j * CWV + v];
+                    const V xv = xs[j * CWV + v];
 #pragma unroll
                     for (int i = 0; i < RB; ++i) {
-                        float t = acc[i][j];
-                        t = fmaf(a[i].x, xv.x, t);
-                        t = fmaf(a[i].y, xv.y, t);
-                        t = fmaf(a[i].z, xv.z, t);
-                        acc[i][j] = fmaf(a[i].w, xv.w, t);
+                        T t = acc[i][j];
+                        t = mac(a[i].x, xv.x, t);
+                        t = mac(a[i].y, xv.y, t);
+                        t = mac(a[i].z, xv.z, t);
+                        acc[i][j] = mac(a[i].w, xv.w, t);
                     }
                 }
             }
-            float flat[N];
+            T flat[N];
 #pragma unroll
             for (int i = 0; i < RB; ++i)
 #pragma unroll
                 for (int j = 0; j < K; ++j) flat[i * K + j] = acc[i][j];
-            const float tot = warp_multi_sum<N>(flat);
+            const T tot = warp_multi_sum<N>(flat);
             const int idx = lane >> (5 - LOGN);
             if ((lane & ((1 << (5 - LOGN)) - 1)) == 0) {
                 if (cs > 1) {
@@ -445,7 +447,7 @@ mmv_tile_kernel(const float* __restrict__ A, const float* __restrict__ X, float*
             __syncthreads();
             for (int t = threadIdx.x; t < nrg * N; t += NT) {
                 const int rg = t / N, idx = t - rg * N;
-                float s = 0.f;
+                T s = T(0);
                 for (int q = 0; q < cs; ++q) s += s_part[q * nrg + rg][idx];
                 const int i = idx / K, j = idx - (idx / K) * K;
                 const int64_t row = ra + int64_t(rg) * RB + i;
@@ -483,17 +485,17 @@ mmv_tile_kernel(const float* __restrict__ A, const float* __restrict__ X, float*
                     for (int e0 = 0; e0 < E; e0 += NT) {
                         const int e = G > 1 ? int(threadIdx.x) % E : e0 + int(threadIdx.x);
                         const int g = G > 1 ? int(threadIdx.x) / E : 0;
-                        float val = 0.f;
+                        T val = T(0);
                         if (g < G && e < E) {
                             const int j = e / rows;
                             const int64_t r = lo + (e - j * rows);
                             const int64_t c_lo = nch * g / G, c_hi = nch * (g + 1) / G;
-                            float outer = 0.f, inner = 0.f;
+                            T outer = T(0), inner = T(0);
                             int n32 = 0;
 #pragma unroll 8
                             for (int64_t c = c_lo; c < c_hi; ++c) {
                                 inner += ld_partial(part + (c * K + j) * R + r);
-                                if (++n32 == 32) { outer += inner; inner = 0.f; n32 = 0; }
+                                if (++n32 == 32) { outer += inner; inner = T(0); n32 = 0; }
                             }
                             val = outer + inner;
                         }
@@ -501,7 +503,7 @@ mmv_tile_kernel(const float* __restrict__ A, const float* __restrict__ X, float*
                         __syncthreads();
                         const int ne = G > 1 ? E : min(E - e0, NT);
                         if (int(threadIdx.x) < ne) {
-                            float t = 0.f;
+                            T t = T(0);
                             for (int gg = 0; gg < G; ++gg) t += s_red[gg * E + int(threadIdx.x)];
                             const int ee = e0 + int(threadIdx.x);
                             const int j = ee / rows;

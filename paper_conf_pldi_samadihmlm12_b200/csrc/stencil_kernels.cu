@@ -27,6 +27,20 @@ __device__ __forceinline__ float st_point(float c, float n, float ce, float t, f
 }
 
 // --------------------------------------------------------------------------- direct
+// q / nvr by multiply-high (Granlund-Montgomery, 33-bit magic 2^32 + m): exact for every
+// 32-bit q; a 64-bit division per element cost ~60 integer instructions (half the issue
+// slots of the kernel, SASS count) -- grids below 2^32 vectors take this path.
+struct FastDiv32 {
+    uint32_t d, m, l;
+    __device__ explicit FastDiv32(uint32_t dd) : d(dd) {
+        l = dd > 1 ? 32u - uint32_t(__clz(dd - 1u)) : 0u;
+        m = uint32_t((((uint64_t(1) << l) - dd) << 32) / dd + 1u);
+    }
+    __device__ __forceinline__ uint32_t div(uint32_t q) const {
+        return uint32_t((uint64_t(__umulhi(q, m)) + q) >> l);
+    }
+};
+
 template <bool VEC, int NT>
 __global__ void __launch_bounds__(NT)
 st_direct_kernel(const float* __restrict__ u, const float* __restrict__ coef, float* __restrict__ v,
@@ -36,8 +50,12 @@ st_direct_kernel(const float* __restrict__ u, const float* __restrict__ coef, fl
     const float c = __ldg(coef), n = __ldg(coef + 1);
     const int64_t nvr = VEC ? W / 4 : W;              // vectors per row
     const int64_t total = H * nvr;
+    const bool small = total <= int64_t(0xffffffffu) - int64_t(gridDim.x) * NT;
+    const FastDiv32 fd(uint32_t(small ? nvr : 1));
     for (int64_t q = int64_t(blockIdx.x) * NT + threadIdx.x; q < total; q += int64_t(gridDim.x) * NT) {
-        const int64_t i = q / nvr, k = q - i * nvr;
+        int64_t i, k;
+        if (small) { i = fd.div(uint32_t(q)); k = q - i * nvr; }
+        else { i = q / nvr; k = q - i * nvr; }
         const int64_t at = i * W + (VEC ? 4 * k : k);
         if constexpr (VEC) {
             const float4 ce = *reinterpret_cast<const float4*>(u + at);
@@ -149,8 +167,8 @@ st_column_kernel(const float* __restrict__ u, const float* __restrict__ coef, fl
         const int64_t r0 = tr * TH, r1 = min(H, r0 + TH);
         const bool lo_edge = (k == 0), hi_edge = (k == nvr - 1);
         // lane 0 / lane 31 (and the last column) take their outer neighbour from memory
-        const bool need_l = (lane == 0) && k > 0;
-        const bool need_r = (lane == 31 || k == nvr - 1 || threadIdx.x == NT - 1) && k < nvr - 1;
+        const bool need_l = (lane == 0) && k > 0 && ok;          // (idle lanes read nothing: kk is clamped)
+        const bool need_r = (lane == 31 || threadIdx.x == NT - 1) && k < nvr - 1;
         float4 up = r0 > 0 ? __ldg(u4 + (r0 - 1) * nvr + kk) : z;
         float4 q[D + 1];
 #pragma unroll

@@ -25,16 +25,23 @@ import paper_conf_pldi_samadihmlm12_b200 as adaptic  # noqa: E402
 from paper_conf_pldi_samadihmlm12_b200 import _lib as L  # noqa: E402
 
 OPC = L.OPS
-B1 = ("asum", "nrm2", "iamax", "iamin")
+B1 = ("asum", "nrm2", "iamax", "iamin", "b1all")
 
 
 CTA_GRID = [(256, rb, u, pp) for rb, u in ((1, 2), (1, 4), (1, 8), (2, 2), (2, 4), (4, 2)) for pp in (1, 2)] + \
            [(1024, 1, 2, 1), (1024, 1, 4, 1), (1024, 2, 2, 1)]
 
 
-def grids(op, R, C):
+def tile_grid(op, R, C, dtype):
+    """The x-tile stream-K kernel (XSMEM 3; fp32 MV on the 128-bit path): chunk widths."""
+    if op != "mv" or dtype != "f32" or C % 4 != 0 or C < 512:
+        return []
+    return [("MV_SPLIT", [cw, 0, 0, 0, 3, 0, 0]) for cw in (0, 8192, 16384) if cw <= C]
+
+
+def grids(op, R, C, dtype="f32"):
     """(variant, params) candidates; params = [lanes, splits, ctas_per_sm, unroll, xsmem, block, rows], 0 = auto."""
-    out = [("AUTO", None)]
+    out = [("AUTO", None)] + tile_grid(op, R, C, dtype)
     if op in B1:
         nv = C // 4 if C % 4 == 0 else C
         if nv <= 64:
@@ -128,6 +135,7 @@ def main():
                          "output count (TMV: R+1) off the 128-bit path, for the scalar-shape table cells")
     ap.add_argument("--perturb-only", action="store_true", help="only the perturbed (off-128-bit-path) shapes")
     ap.add_argument("--auto-only", action="store_true", help="time only the selector's pick (validation runs)")
+    ap.add_argument("--tile-only", action="store_true", help="time only the x-tile stream-K candidates (+ AUTO)")
     a = ap.parse_args()
     dev = torch.device("cuda:0")
     tdt = torch.float32 if a.dtype == "f32" else torch.int32
@@ -149,7 +157,7 @@ def main():
     maxel = max(R * C for R, C, _ in shapes) + max(R + C for R, C, _ in shapes)
     M = torch.empty(maxel * (2 if "dot" in a.ops else 1), dtype=tdt, device=dev)
     X = torch.empty(max(C for _, C, _ in shapes) + 1, dtype=tdt, device=dev)
-    Y = torch.empty(max(R for R, _, _ in shapes) + 1, dtype=tdt, device=dev)   # 4-byte y (int32 for IAMAX/IAMIN)
+    Y = torch.empty(4 * (max(R for R, _, _ in shapes) + 1), dtype=tdt, device=dev)   # 4-byte y; B1ALL: 4 per row
     synth.device_matrix(M, 1, M.numel(), "mv", "uniform", 11)
     synth.device_vector(X, "uniform", 12)
     t0 = time.time()
@@ -159,14 +167,17 @@ def main():
                 R, C = (R0 + pert, C0) if op == "tmv" else (R0, C0 + pert)
                 Xp = M.data_ptr() + R * C * 4 if op == "dot" else X.data_ptr()
                 ptrs = (M.data_ptr(), Xp, Y.data_ptr())
-                for variant, params in (grids(op, R, C) if not a.auto_only else [("AUTO", None)]):
+                cands = ([("AUTO", None)] if a.auto_only else
+                         [("AUTO", None)] + tile_grid(op, R, C, a.dtype) if a.tile_only else grids(op, R, C, a.dtype))
+                for variant, params in cands:
                     try:
                         plan = adaptic.get_plan(OPC[op], R, C, dtc, dev, variant, params, stream)
                     except adaptic.AdapticError:
                         continue
                     ts = time_plan(plan, ptrs, stream, a.reps)
                     med = statistics.median(ts)
-                    nbytes = 4 * (R * C * (2 if op == "dot" else 1) + R + (0 if op in ("dot",) + B1 else C))
+                    nbytes = 4 * (R * C * (2 if op == "dot" else 1) + (4 if op == "b1all" else 1) * R
+                                  + (0 if op in ("dot",) + B1 else C))
                     d = plan.describe()
                     f.write(json.dumps({"op": op, "dtype": a.dtype, "R": R, "C": C, "variant": d["variant"],
                                         "req": variant, "params": params, "us": med, "us_min": min(ts),
