@@ -428,8 +428,21 @@ def measure_latency(p, reps=200):
         evs[1].record(stream)
         torch.cuda.synchronize()
         amort = evs[0].elapsed_time(evs[1]) * 1e3 / (5 * reps)
+        # L2-cold: a write of 2x the L2 size between launches evicts B and x
+        l2 = torch.cuda.get_device_properties(torch.cuda.current_device()).L2_cache_size
+        scratch = torch.empty(2 * l2 // 4 + 1024, dtype=torch.float32, device=torch.cuda.current_device())
+        cold = []
+        for _ in range(30):
+            scratch.fill_(1.0)
+            evs[0].record(stream)
+            p.plan.run(*p.ptrs, s)
+            evs[1].record(stream)
+            evs[1].synchronize()
+            cold.append(evs[0].elapsed_time(evs[1]) * 1e3)
     return {"single_launch_median": statistics.median(single), "single_launch_min": min(single),
-            "graph_amortized": amort, "graph_launches": reps, "variant": p.desc["variant"]}
+            "graph_amortized": amort, "graph_launches": reps,
+            "l2_cold_median": statistics.median(cold), "l2_cold_note": "2x L2 scratch write before each launch",
+            "variant": p.desc["variant"]}
 
 
 def measure_e2e(args, probs, world):

@@ -1106,11 +1106,16 @@ bool pdl_enabled() {
 std::mutex g_attr_mu;
 // (device, kernel) pairs that already have their dynamic-smem limit raised
 struct AttrKey { int dev; void* fn; size_t smem; };
-AttrKey g_attr_done[64];
+constexpr int kAttrCache = 256;
+AttrKey g_attr_done[kAttrCache];
 int g_attr_n = 0;
 
 cudaError_t ensure_smem_attr(void* fn, size_t smem) {
-    if (smem <= 48 * 1024) return cudaSuccess;
+    // the 48 KB default covers static + dynamic shared memory; kernels here declare up to
+    // ~8 KB statically, so every dynamic size above 32 KB raises the limit explicitly
+    // (found by a run with the caching allocator off: a 48 KB TPR ring + 72 B of
+    // mbarriers failed to launch)
+    if (smem <= 32 * 1024) return cudaSuccess;
     int dev = 0;
     cudaError_t e = cudaGetDevice(&dev);
     if (e != cudaSuccess) return e;
@@ -1123,7 +1128,7 @@ cudaError_t ensure_smem_attr(void* fn, size_t smem) {
     if (e != cudaSuccess) return e;
     for (int i = 0; i < g_attr_n; ++i)
         if (g_attr_done[i].dev == dev && g_attr_done[i].fn == fn) { g_attr_done[i].smem = smem; return cudaSuccess; }
-    if (g_attr_n < 64) g_attr_done[g_attr_n++] = AttrKey{dev, fn, smem};
+    if (g_attr_n < kAttrCache) g_attr_done[g_attr_n++] = AttrKey{dev, fn, smem};
     return cudaSuccess;
 }
 
@@ -1252,7 +1257,7 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
             break;
     }
     if (!fn) return ADAPTIC_ERR_UNSUPPORTED;
-    if (smem > 48 * 1024) {
+    if (smem > 32 * 1024) {
         cudaError_t ea = ensure_smem_attr(fn, smem);
         if (ea != cudaSuccess) return cuda_fail(ea);
     }

@@ -77,12 +77,18 @@ tmv_flat_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restrict_
         }
         // the rest, one vector at a time, words outside B masked
         for (; q < qend; q += T_) {
-            const E a = ld_stream(Ba + q);
-            const T av[4] = {a.x, a.y, a.z, a.w};
+            const int64_t f0 = 4 * q - b0;
+            if (f0 >= 0 && f0 + 3 < total) {
+                const E a = ld_stream(Ba + q);
+                const T av[4] = {a.x, a.y, a.z, a.w};
 #pragma unroll
-            for (int j = 0; j < 4; ++j) {
-                const int64_t f = 4 * q + j - b0;
-                if (f >= 0 && f < total) acc[j] = mac(av[j], ld_x(X + f / R), acc[j]);
+                for (int j = 0; j < 4; ++j) acc[j] = mac(av[j], ld_x(X + (f0 + j) / R), acc[j]);
+            } else {                                    // B's first / last vector: only its own words
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    const int64_t f = f0 + j;
+                    if (f >= 0 && f < total) acc[j] = mac(ld_stream(B + f), ld_x(X + f / R), acc[j]);
+                }
             }
         }
 #pragma unroll

@@ -29,6 +29,21 @@ template <class V> __device__ __forceinline__ V funnel4(const V& lo, const V& hi
     return r;
 }
 
+// Aligned vector q of the aligned view (element e of B is element b0 + e of the view):
+// one 128-bit load when all four words lie inside B, else the words inside B one by one
+// (zeros elsewhere) -- the first vector of B starts b0 words early and the last may end
+// up to 3 words late; those words are never selected, and are not read either.
+template <class E, class T> __device__ __forceinline__ E ld_inside(const E* Ba, const T* B, int64_t q, int b0, int64_t total) {
+    const int64_t f0 = 4 * q - b0;                    // element of B at lane 0
+    if (f0 >= 0 && f0 + 3 < total) return ld_stream(Ba + q);
+    E v = zero_of<E>();
+    if (f0 >= 0 && f0 < total) v.x = ld_stream(B + f0);
+    if (f0 + 1 >= 0 && f0 + 1 < total) v.y = ld_stream(B + f0 + 1);
+    if (f0 + 2 >= 0 && f0 + 2 < total) v.z = ld_stream(B + f0 + 2);
+    if (f0 + 3 >= 0 && f0 + 3 < total) v.w = ld_stream(B + f0 + 3);
+    return v;
+}
+
 template <class T, int LR, int U, int NT>
 __global__ void __launch_bounds__(NT, U <= 2 ? 4 : U <= 4 ? 3 : 2)
 tmv_mis_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restrict__ y,
@@ -76,8 +91,8 @@ tmv_mis_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restrict__
                 const int64_t f = b0 + cc * R + col;             // aligned-view element index
                 const int64_t q = f >> 2;
                 sh[u] = int(f & 3);
-                lo[u] = ld_stream(Ba + q);
-                hi[u] = ld_stream(Ba + min(q + 1, qmax));
+                lo[u] = ld_inside(Ba, B, q, b0, R * C);
+                hi[u] = ld_inside(Ba, B, min(q + 1, qmax), b0, R * C);
                 xs[u] = ld_x(X + cc);
             }
 #pragma unroll
@@ -92,7 +107,8 @@ tmv_mis_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restrict__
         for (; c < c1; c += LC) {
             const int64_t f = b0 + c * R + col;
             const int64_t q = f >> 2;
-            esmac(acc[0], funnel4(ld_stream(Ba + q), ld_stream(Ba + min(q + 1, qmax)), int(f & 3)), ld_x(X + c));
+            esmac(acc[0], funnel4(ld_inside(Ba, B, q, b0, R * C), ld_inside(Ba, B, min(q + 1, qmax), b0, R * C),
+                                  int(f & 3)), ld_x(X + c));
         }
         E tot = eadd(outer, tree_sum<U>(acc));
         tot = lc_combine<NT, LR>(tot, red);

@@ -105,3 +105,16 @@ def test_large_grid_device_generated():
     mid, S = oracle.stencil5(u[2000:2100], C0, N0)           # a band in the middle (interior rows 1..98)
     err = np.abs(o[2001:2099].astype(np.float64) - mid[1:-1])
     assert (err <= 1e-6 * S[1:-1]).all()
+
+
+def test_run_host_end_to_end():
+    """Host buffers through the C ABI (adaptic_run_host: H2D of u and {c, n}, kernel, D2H of v)."""
+    H, W = 300, 1028
+    u = synth.matrix(H, W, "mv", np.float32, "uniform", 77)
+    uh = torch.from_numpy(u).pin_memory()
+    ch = torch.tensor([C0, N0], dtype=torch.float32).pin_memory()
+    vh = torch.empty(H, W, dtype=torch.float32).pin_memory()
+    du, dc, dv = torch.empty(H, W, device=DEV), torch.empty(2, device=DEV), torch.empty(H, W, device=DEV)
+    adaptic.run_host("stencil5", uh, ch, vh, du, dc, dv)
+    torch.cuda.synchronize()
+    check(vh.numpy(), u, C0, N0, "run_host")
