@@ -1,0 +1,62 @@
+"""Host-side planner rules added for the stencil, the x-tile stream-K MV kernel and the
+multi-vector TMA/TMV choices.  No GPU needed: plans are built and
+described, nothing is launched (no device: occupancy takes its documented fallback)."""
+import pytest
+
+import paper_conf_pldi_samadihmlm12_b200 as adaptic
+
+
+def d(op, R, C, dtype="f32", variant="AUTO", params=None, nvec=1):
+    return adaptic.plan(op, R, C, dtype, variant=variant, params=params, nvec=nvec).describe()
+
+
+def test_stencil_selector_and_orders():
+    assert d("stencil5", 8192, 8192)["variant"] == "ST_DIRECT"
+    assert d("stencil5", 8192, 8192)["xmode"] == 0                 # rows < 2 MB: row-major sweep
+    assert d("stencil5", 8, 1 << 23)["xmode"] == 1                 # 32 MB rows: L2 strips
+    assert d("stencil5", 64, 4096, variant="ST_DIRECT", params=[0, 0, 0, 0, 0, 0, 0, 2])["xmode"] == 1
+    col = d("stencil5", 64, 4096, variant="ST_DIRECT", params=[0, 0, 0, 0, 0, 0, 16, 3])
+    assert col["xmode"] == 2 and col["rows_per_group"] == 16
+    assert d("stencil5", 100, 101)["vec_shape"] is False           # odd width: scalar direct kernel
+    t = d("stencil5", 4096, 16384, variant="ST_TILE")               # the paper's reuse-metric super tile
+    assert t["variant"] == "ST_TILE" and t["smem"] > 0
+    with pytest.raises(adaptic.AdapticError):
+        d("stencil5", 64, 64, "i32")
+
+
+def test_tile_kernel_cells_fp32_and_int32():
+    for dt in ("f32", "i32"):
+        p = d("mv", 4096, 16384, dt)
+        assert p["variant"] == "MV_SPLIT" and p["xmode"] == 4, p
+        assert p["lanes"] == 16384 and p["path_ok"][1]
+    p = d("mv", 300, 50000, variant="MV_SPLIT", params=[1024, 0, 0, 0, 3, 0, 2])
+    assert p["xmode"] == 4 and p["lanes"] == 1024 and p["rows_per_group"] == 2
+    assert p["splits"] == -(-50000 // 1024) and p["workspace_bytes"] > 0
+    # one chunk: no merge, no workspace
+    assert d("mv", 300, 1024, variant="MV_SPLIT", params=[0, 0, 0, 0, 3])["workspace_bytes"] == 0
+    # rows off the 16-byte grid never take the tile kernel
+    assert d("mv", 300, 1027, variant="MV_SPLIT", params=[0, 0, 0, 0, 3])["xmode"] != 4
+
+
+def test_multi_vector_rules():
+    assert d("mv", 8192, 8192, nvec=4)["xmode"] == 4               # x-tile stream-K
+    assert d("mv", 8, 1 << 23, nvec=4)["xmode"] != 4               # R <= 16: interleaved splits
+    assert d("mv", 1 << 20, 64, nvec=4)["variant"] == "MV_SUBWARP"  # short rows: x in registers
+    few = d("tmv", 64, 1 << 20, nvec=4)
+    assert few["xmode"] == 5 and few["lanes"] == 16                 # one contiguous TMA tile
+    huge = d("tmv", 262144, 256, nvec=4)
+    assert huge["xmode"] == 5 and huge["lanes"] == 256 and huge["splits"] == 1
+    mid = d("tmv", 8192, 8192, nvec=4)
+    assert mid["xmode"] == 0 and mid["variant"] == "TMV_SPLITK"     # register-fed tiles
+    assert d("tmv", 1 << 20, 64, nvec=4)["variant"] == "TMV_COL"
+    forced = d("tmv", 8192, 8192, variant="TMV_SPLITK", params=[128, 9, 0, 0, 3], nvec=8)
+    assert forced["xmode"] == 5 and forced["splits"] == 9
+
+
+@pytest.mark.parametrize("K", [2, 4, 8])
+def test_multi_plans_respect_the_error_bound(K):
+    for op in ("mv", "tmv"):
+        for k in range(3, 24, 2):
+            p = d(op, 1 << k, 1 << (26 - k), nvec=K)
+            w = 1 if p["vec_shape"] else 0
+            assert p["path_ok"][w], (op, k, p)
