@@ -320,8 +320,12 @@ adaptic_status derive_stencil(adaptic_plan_s* p, const int32_t* params, const De
             // row-major grid-stride sweep, 2 = strips).  Measured (profiles/r1_stencil_sweep.md):
             // equal up to 1-2 MB rows, strips +3..60 % beyond (8 x 8M: 3.9 -> 6.2 TB/s)
             const int ord = par(ADAPTIC_P_ORDER);
-            p->xmode = (ord == 2 || (ord <= 0 && W / 4 >= ST_STRIP_MIN_ROW)) ? 1 : (ord == 3 ? 2 : 0);
-            if (p->xmode == 2) {                             // column sweep, register sliding window
+            p->xmode = (ord == 2 || (ord <= 0 && W / 4 >= ST_STRIP_MIN_ROW)) ? 1 : (ord == 3 ? 2 : ord == 4 ? 3 : 0);
+            if (p->xmode == 3) {                             // row-major, 2 float4 per thread per step
+                const int cps = occupancy(st_direct2_fn(), 256, 0, dev.present, 8);
+                p->grid[1] = std::max<int64_t>(1, std::min<int64_t>(ceil_div(H * (W / 4), 512), int64_t(dev.sms) * cps));
+                p->ctas_per_sm = cps;
+            } else if (p->xmode == 2) {                             // column sweep, register sliding window
                 const int th = par(ADAPTIC_P_ROWS) > 0 ? par(ADAPTIC_P_ROWS) : 64;
                 p->rb = th;
                 const int cps = occupancy(st_column_fn(), 256, 0, dev.present, 8);
@@ -1160,6 +1164,8 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
             smem = p->smem;
         } else if (vec && p->xmode == 1) {
             fn = st_strip_fn();
+        } else if (vec && p->xmode == 3) {
+            fn = st_direct2_fn();
         } else if (vec && p->xmode == 2) {
             fn = st_column_fn();
             args7[0] = &A; args7[1] = &X; args7[2] = &y; args7[3] = &R; args7[4] = &C; args7[5] = &tile_mb;

@@ -83,6 +83,8 @@ void* st_strip_fn();
 //   column: (u, coef, v, H, W, int TH): NT = 256 float4 columns x TH rows per tile, register
 //           sliding window down each column (D = 4 rows loaded ahead)
 void* st_column_fn();
+//   direct2: direct arguments; row-major, two float4 outputs per thread per step (ORDER 4)
+void* st_direct2_fn();
 constexpr int ST_STRIP_SV = 256 * 4;
 constexpr int64_t ST_STRIP_MIN_ROW = 131072;       // float4 per row from which strips are used
 void* st_tile_fn(int TH, int TW);

@@ -81,6 +81,57 @@ st_direct_kernel(const float* __restrict__ u, const float* __restrict__ coef, fl
     }
 }
 
+// Row-major sweep, two float4 outputs per thread per step (q and q + stride): all six
+// float4 and four scalar loads are issued before the first FMA, v is stored evict-first
+// (keeps u's neighbour rows in L2 longer).  Planner ORDER 4.
+template <int NT>
+__global__ void __launch_bounds__(NT)
+st_direct2_kernel(const float* __restrict__ u, const float* __restrict__ coef, float* __restrict__ v,
+                  int64_t H, int64_t W)
+{
+    pdl_prologue();
+    const float c = __ldg(coef), n = __ldg(coef + 1);
+    const int64_t nvr = W / 4;
+    const int64_t total = H * nvr;
+    const int64_t stride = int64_t(gridDim.x) * NT;
+    const bool small = total + stride <= int64_t(0xffffffffu);
+    const FastDiv32 fd(uint32_t(small ? nvr : 1));
+    const float4* __restrict__ u4 = reinterpret_cast<const float4*>(u);
+    float4* __restrict__ v4 = reinterpret_cast<float4*>(v);
+    for (int64_t q0 = int64_t(blockIdx.x) * NT + threadIdx.x; q0 < total; q0 += 2 * stride) {
+        int64_t qq[2], i[2], k[2];
+        bool ok[2], in[2];
+        float4 ce[2], t[2], b[2];
+        float l[2], r[2];
+#pragma unroll
+        for (int e = 0; e < 2; ++e) {
+            qq[e] = q0 + e * stride;
+            ok[e] = qq[e] < total;
+            const int64_t q = ok[e] ? qq[e] : q0;
+            i[e] = small ? int64_t(fd.div(uint32_t(q))) : q / nvr;
+            k[e] = q - i[e] * nvr;
+            in[e] = i[e] > 0 && i[e] < H - 1;
+            ce[e] = __ldg(u4 + q);
+            t[e] = in[e] ? __ldg(u4 + q - nvr) : ce[e];
+            b[e] = in[e] ? __ldg(u4 + q + nvr) : ce[e];
+            l[e] = (in[e] && k[e] > 0) ? __ldg(u + 4 * q - 1) : 0.f;
+            r[e] = (in[e] && k[e] < nvr - 1) ? __ldg(u + 4 * q + 4) : 0.f;
+        }
+#pragma unroll
+        for (int e = 0; e < 2; ++e) {
+            if (!ok[e]) continue;
+            float4 o = ce[e];
+            if (in[e]) {
+                if (k[e] > 0) o.x = st_point(c, n, ce[e].x, t[e].x, b[e].x, l[e], ce[e].y);
+                o.y = st_point(c, n, ce[e].y, t[e].y, b[e].y, ce[e].x, ce[e].z);
+                o.z = st_point(c, n, ce[e].z, t[e].z, b[e].z, ce[e].y, ce[e].w);
+                if (k[e] < nvr - 1) o.w = st_point(c, n, ce[e].w, t[e].w, b[e].w, ce[e].z, r[e]);
+            }
+            __stcs(v4 + qq[e], o);
+        }
+    }
+}
+
 // --------------------------------------------------------------------------- L2 strips
 // The B200 form of the paper's super tile: the grid is cut into vertical strips of SV
 // = NT V float4 columns and the work items (strip, row) are taken strip-major, so the
@@ -279,6 +330,7 @@ void* st_direct_fn(bool vec) {
 }
 
 void* st_strip_fn() { return reinterpret_cast<void*>(&st_strip_kernel<256, 4>); }
+void* st_direct2_fn() { return reinterpret_cast<void*>(&st_direct2_kernel<256>); }
 void* st_column_fn() { return reinterpret_cast<void*>(&st_column_kernel<256, 4>); }
 
 template <int TH>

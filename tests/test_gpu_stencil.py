@@ -47,7 +47,8 @@ SHAPES = [(1, 4), (2, 8), (3, 3), (5, 12), (33, 100), (64, 256), (65, 260), (129
           (7, 4096), (2049, 132), (5, 8200), (9, 16384), (1, 8192)]
 FORCED = [("AUTO", None), ("ST_DIRECT", None), ("ST_DIRECT", [0, 0, 0, 0, 0, 0, 0, 1]),
           ("ST_DIRECT", [0, 0, 0, 0, 0, 0, 0, 2]), ("ST_DIRECT", [0, 0, 0, 0, 0, 0, 0, 3]),
-          ("ST_DIRECT", [0, 0, 0, 0, 0, 0, 3, 3]), ("ST_DIRECT", [0, 0, 0, 0, 0, 0, 9, 3])] + \
+          ("ST_DIRECT", [0, 0, 0, 0, 0, 0, 3, 3]), ("ST_DIRECT", [0, 0, 0, 0, 0, 0, 9, 3]),
+          ("ST_DIRECT", [0, 0, 0, 0, 0, 0, 0, 4])] + \
          [("ST_TILE", [tw, 0, 0, 0, 0, 0, th]) for th in (4, 8, 16, 32) for tw in (128, 256, 512)]
 
 

@@ -30,7 +30,7 @@ TW = (128, 256, 512)
 
 
 def grid(W):
-    out = [("AUTO", None), ("ST_DIRECT", [0, 0, 0, 0, 0, 0, 0, 1])]
+    out = [("AUTO", None), ("ST_DIRECT", [0, 0, 0, 0, 0, 0, 0, 1]), ("ST_DIRECT", [0, 0, 0, 0, 0, 0, 0, 4])]
     if W >= 4096:
         out.append(("ST_DIRECT", [0, 0, 0, 0, 0, 0, 0, 2]))
     for th in (16, 32, 64, 128):
