@@ -194,6 +194,20 @@ typedef enum {
  *                      per block of [ADAPTIC_P_ROWS] rows); 4-byte-aligned pointers
  *                      then run the CTA-per-row kernel.  Multi-vector TMV: 3 = B
  *                      rows staged by TMA, 1 = register-fed tiles.
+ *                      MV_SUBWARP / MV_WPR (MV and DOT, fp32 / int32, cols <= 32 *
+ *                      lanes): 4 = row tiles -- [ADAPTIC_P_ROWS] consecutive rows
+ *                      (0: ~24 KB; -n: ~n KB) bulk-copied (TMA) as one 16-byte-
+ *                      aligned block into a ring of [ADAPTIC_P_UNROLL] stages, each
+ *                      row reduced by [ADAPTIC_P_LANES] lanes with x held in
+ *                      registers ([ADAPTIC_P_BLOCK] 256 or 512 threads).  A, and
+ *                      DOT's b, must be 16-byte aligned for it; other pointers run
+ *                      the variant's direct kernel.  TMV_REGTILE (rows <= 1024):
+ *                      4 = tiles of [ADAPTIC_P_ROWS] rows of B (a multiple of 4;
+ *                      0 / -n as above) and their x values staged by TMA, thread
+ *                      (r, slice) accumulating output r over its rows of every
+ *                      tile, [ADAPTIC_P_BLOCK] 256 / 512 / 1024 >= rows threads;
+ *                      16-byte-aligned B and x, else the direct kernel.  A tile
+ *                      height is capped so that two ring stages fit.
  *   [ADAPTIC_P_BLOCK]  TMV_*: threads per CTA, 256 or 1024 (unroll <= 4 at 1024).
  *   [ADAPTIC_P_ROWS]   MV_CPR / MV_SPLIT: rows per CTA step sharing each x load,
  *                      (rows, unroll) in {(1,2),(1,4),(1,8),(2,2),(2,4),(4,2)}.

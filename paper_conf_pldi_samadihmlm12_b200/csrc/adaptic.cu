@@ -55,6 +55,7 @@ struct adaptic_plan_s {
     int fb_lanes, fb_unroll;
     // workspace
     size_t ws_bytes, cnt_off;
+    size_t fb_ws_off;      // staged-tile plans: the direct-kernel fallback's workspace starts here
     void* ws;
     size_t ws_cap;
 };
@@ -731,6 +732,124 @@ adaptic_status derive_b1(adaptic_plan_s* p, const int32_t* params, const DevInfo
     return ADAPTIC_OK;
 }
 
+adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& dev);
+
+// MV / DOT lane groups on TMA-staged row tiles (rowtile_kernel.cuh): MV_SUBWARP / MV_WPR
+// with [ADAPTIC_P_XSMEM] = 4.  [LANES] G (WPR: 32), [BLOCK] threads 256 | 512, [ROWS]
+// rows per tile k, [UNROLL] ring stages, [CTAS_PER_SM] resident CTAs the ring is sized
+// for.  Needs C <= 32*G (x slice in registers); 16-byte-aligned A (and b) at run time,
+// else adaptic_run takes the same variant's direct kernel.
+adaptic_status derive_rowtile(adaptic_plan_s* p, const int32_t* params, const DevInfo& dev) {
+    auto par = [&](int i) -> int { return params ? params[i] : 0; };
+    const bool px = (p->op == ADAPTIC_OP_DOT);
+    const int64_t R = p->R, C = p->C;
+    int G = p->variant == ADAPTIC_V_MV_WPR ? 32 : par(ADAPTIC_P_LANES);
+    if (G <= 0) G = clampi(pow2_ceil(ceil_div(C, 8)), 1, 16);
+    if (G < 1 || G > 32 || (G & (G - 1)) || (p->variant == ADAPTIC_V_MV_SUBWARP && G > 16))
+        return ADAPTIC_ERR_INVALID_ARG;
+    if (C > int64_t(RT_MAX_C_PER_LANE) * G) return ADAPTIC_ERR_UNSUPPORTED;
+    int NT = par(ADAPTIC_P_BLOCK);
+    if (NT <= 0) NT = 256;
+    if (NT != 256 && NT != 512) return ADAPTIC_ERR_INVALID_ARG;
+    const int ngr = NT / G;
+    const int64_t opb = int64_t(px ? 2 : 1) * 4;             // staged bytes per element
+    int64_t k = par(ADAPTIC_P_ROWS);
+    if (k <= 0) {          // 0: ~24 KB of matrix per tile; -n: ~n KB (fitted tables); whole warps of rows
+        const int64_t kb = k < 0 ? -k : 24;
+        k = std::max<int64_t>(1, (kb * 1024) / (C * opb));
+        if (k >= ngr) k = k / ngr * ngr;
+    }
+    k = std::min<int64_t>(k, std::max<int64_t>(1, R));
+    int cps = par(ADAPTIC_P_CTAS_PER_SM);
+    if (cps <= 0) cps = 2;
+    // a tile height fitted on a shorter row (table cells span a factor of 2 in C) is
+    // capped so that two stages still fit the ring budget
+    const int64_t kmax2 = ((int64_t(220) * 1024 / cps / 2) / (4 * (px ? 2 : 1)) - 9) / C;
+    if (kmax2 < 1) return ADAPTIC_ERR_UNSUPPORTED;
+    k = std::min(k, kmax2);
+    const size_t stage_bytes = rowtile_tile_words(k, C) * 4 * (px ? 2 : 1);
+    if (stage_bytes > 200 * 1024) return ADAPTIC_ERR_UNSUPPORTED;
+    int stages = int(std::min<size_t>(RT_MAX_STAGES_H, (size_t(220) * 1024 / size_t(cps)) / stage_bytes));
+    if (par(ADAPTIC_P_UNROLL) > 0) stages = std::min(stages, par(ADAPTIC_P_UNROLL));
+    if (stages < 2) return ADAPTIC_ERR_UNSUPPORTED;
+    p->smem = size_t(stages) * stage_bytes;
+    void* fn = rowtile_fn(p->dtype, NT, G, px);
+    if (!fn) return ADAPTIC_ERR_UNSUPPORTED;
+    const int occ = occupancy(fn, NT, p->smem, dev.present, cps);
+    if (occ < 1) return ADAPTIC_ERR_UNSUPPORTED;
+    p->ctas_per_sm = std::min(cps, occ);
+    p->lanes = G; p->block = NT; p->rb = int(k); p->stages = stages; p->unroll = stages;
+    p->xmode = 4;
+    p->mis = !p->vec_shape;
+    const int64_t ntiles = ceil_div(R, k);
+    p->grid[1] = std::max<int64_t>(1, std::min<int64_t>(ntiles, int64_t(dev.sms) * p->ctas_per_sm));
+    p->chain[1] = ceil_div(ceil_div(C, G), 2);
+    p->depth[1] = ilog2c(G) + 1;
+    p->path_ok[1] = (p->dtype == DT_I32) || bound_ok(p->chain[1] + p->depth[1]);
+    if (!p->path_ok[1]) return ADAPTIC_ERR_UNSUPPORTED;
+    return ADAPTIC_OK;
+}
+
+// TMV with few outputs on TMA-staged tiles of B (tmv_rowtile_kernel.cuh): TMV_REGTILE with
+// [ADAPTIC_P_XSMEM] = 4.  [BLOCK] threads 256 | 512 | 1024 (>= R), [ROWS] rows of B per
+// tile k (a multiple of 4), [UNROLL] ring stages, [CTAS_PER_SM].  16-byte-aligned B and x
+// at run time, else adaptic_run takes the variant's direct kernel.
+adaptic_status derive_tmv_rowtile(adaptic_plan_s* p, const int32_t* params, const DevInfo& dev) {
+    auto par = [&](int i) -> int { return params ? params[i] : 0; };
+    const int64_t R = p->R, C = p->C;
+    if (R > 1024) return ADAPTIC_ERR_UNSUPPORTED;
+    int NT = par(ADAPTIC_P_BLOCK);
+    if (NT <= 0) NT = R <= 64 ? 256 : 1024;
+    if ((NT != 256 && NT != 512 && NT != 1024) || R > NT) return ADAPTIC_ERR_INVALID_ARG;
+    int cps = par(ADAPTIC_P_CTAS_PER_SM);
+    if (cps <= 0) cps = 1024 / NT;
+    int64_t k = par(ADAPTIC_P_ROWS);
+    if (k < 0) {                        // -n: ~n KB of B and x per tile (fitted tables)
+        k = std::max<int64_t>(4, (int64_t(-k) * 1024 / 4) / (R + 1) / 4 * 4);
+    } else if (k == 0) {                // ~24 KB of B per tile, and at least 3 stages in the budget
+        const int64_t words = std::min<int64_t>(24 * 1024, (int64_t(220) * 1024 / cps) / 3) / 4 - 9;
+        k = std::max<int64_t>(4, words / (R + 1) / 4 * 4);
+    }
+    if (k % 4 != 0) return ADAPTIC_ERR_INVALID_ARG;
+    k = std::min<int64_t>(k, ceil_div(C, 4) * 4);
+    // cap a tile height fitted on fewer outputs so that two stages fit the ring budget
+    const int64_t kmax2 = (((int64_t(220) * 1024 / cps / 2) / 4 - 9) / (R + 1)) / 4 * 4;
+    if (kmax2 < 4) return ADAPTIC_ERR_UNSUPPORTED;
+    k = std::min(k, kmax2);
+    const size_t stage_bytes = (rowtile_tile_words(k, R) + size_t(k)) * 4;
+    if (stage_bytes > 200 * 1024) return ADAPTIC_ERR_UNSUPPORTED;
+    int stages = int(std::min<size_t>(8, (size_t(220) * 1024 / size_t(cps)) / stage_bytes));
+    if (par(ADAPTIC_P_UNROLL) > 0) stages = std::min(stages, par(ADAPTIC_P_UNROLL));
+    if (stages < 2) return ADAPTIC_ERR_UNSUPPORTED;
+    p->smem = size_t(stages) * stage_bytes;
+    void* fn = tmv_rowtile_fn(p->dtype, NT);
+    const int occ = occupancy(fn, NT, p->smem, dev.present, cps);
+    if (occ < 1) return ADAPTIC_ERR_UNSUPPORTED;
+    p->ctas_per_sm = std::min(cps, occ);
+    const int64_t ntiles = ceil_div(C, k);
+    const int64_t G = std::max<int64_t>(1, std::min<int64_t>(ntiles, int64_t(dev.sms) * p->ctas_per_sm));
+    const int64_t nsl = NT / R;
+    p->lanes = int(R); p->block = NT; p->rb = int(k); p->stages = stages; p->unroll = stages;
+    p->xmode = 4; p->splits = 1; p->mis = !p->vec_shape;
+    p->grid[1] = G;
+    const int64_t rows_per_thread = ceil_div(ceil_div(ntiles, G) * k, nsl);
+    p->chain[1] = fold_chain(ceil_div(rows_per_thread, 4)) + 1;
+    const int64_t ngroups = ceil_div(G, 16);                  // TRT_GROUP CTAs per merge group
+    p->depth[1] = 3 + 2 * nsl + ceil_div(16, nsl) + ceil_div(ngroups, nsl);
+    p->path_ok[1] = (p->dtype == DT_I32) || bound_ok(p->chain[1] + p->depth[1]);
+    if (!p->path_ok[1]) return ADAPTIC_ERR_UNSUPPORTED;
+    // CTA partials (G x R), group partials (ngroups x R), then 1 + ngroups counters
+    const size_t part = ((size_t(G + ngroups) * size_t(R) * 4 + 255) / 256) * 256;
+    p->cnt_off = part;
+    p->ws_bytes = part + ((size_t(1 + ngroups) * 4 + 255) / 256) * 256;
+    // pointers the bulk copies cannot use run the variant's direct kernel on its own
+    // (disjoint, hence still zeroed) part of this workspace
+    adaptic_plan_s fb = *p;
+    p->fb_ws_off = p->ws_bytes;
+    if (derive(&fb, nullptr, dev) == ADAPTIC_OK) p->ws_bytes += fb.ws_bytes;
+    return ADAPTIC_OK;
+}
+
 // Fill the kernel parameters of `p` for p->variant.  params: user overrides or nullptr.
 adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& dev) {
     const int op = p->op, dt = p->dtype;
@@ -762,6 +881,8 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
     p->cnt_off = 0;
 
     for (int w = 0; w < 2; ++w) { p->grid[w] = 0; p->chain[w] = 0; p->depth[w] = 0; p->path_ok[w] = false; }
+    if ((v == ADAPTIC_V_MV_SUBWARP || v == ADAPTIC_V_MV_WPR) && par(ADAPTIC_P_XSMEM) == 4)
+        return derive_rowtile(p, params, dev);
 
     // rows not 16-byte aligned (C % 4 != 0): the misaligned-row kernels keep the matrix
     // stream 128-bit; the plain scalar kernels (index 0) remain for DOT operands whose
@@ -912,6 +1033,7 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
     // stream 128-bit over ceil(R/4) output vectors; it handles any B / y alignment, so no
     // scalar path is planned for these shapes
     p->flat = false;
+    if (v == ADAPTIC_V_TMV_REGTILE && par(ADAPTIC_P_XSMEM) == 4) return derive_tmv_rowtile(p, params, dev);
     if (!p->vec_shape && v == ADAPTIC_V_TMV_REGTILE && R <= TMV_FLAT_MAX_R) {
         // few outputs off the 16-byte grid: stream B as one flat array (tmv_flat_kernel.cuh)
         const int FNT = R <= TMV_FLAT_NT_SMALL_R ? 256 : 1024;
@@ -1022,7 +1144,7 @@ adaptic_status make_plan(int op, int64_t rows, int64_t cols, int dtype, int vari
     adaptic_plan_s* p = new (std::nothrow) adaptic_plan_s();
     if (!p) return ADAPTIC_ERR_INVALID_ARG;
     p->op = op; p->dtype = dtype; p->R = rows; p->C = cols; p->sms = dev.sms; p->nvec = nvec;
-    p->ws = nullptr; p->ws_cap = 0;
+    p->ws = nullptr; p->ws_cap = 0; p->fb_ws_off = 0;
 
     if (variant != ADAPTIC_V_AUTO) {
         p->variant = variant; p->source = 0;
@@ -1226,6 +1348,14 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
             break;
         case ADAPTIC_V_MV_SUBWARP:
         case ADAPTIC_V_MV_WPR:
+            if (p->xmode == 4) {                          // TMA-staged row tiles
+                fn = rowtile_fn(dt, p->block, p->lanes, px);
+                smem = p->smem;
+                args7[0] = &A; args7[1] = &X; args7[2] = &y; args7[3] = &R; args7[4] = &C;
+                args7[5] = &tile_mb; args7[6] = &stages;
+                args = args7;
+                break;
+            }
             fn = mis ? mis_group_fn(dt, p->lanes, p->unroll, p->xmode) : group_fn(dt, p->lanes, p->unroll, vec, p->xmode);
             smem = p->smem;
             args6[0] = &A; args6[1] = &X; args6[2] = &y; args6[3] = &R; args6[4] = &C;
@@ -1249,6 +1379,14 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
             args = args9;
             break;
         default:
+            if (p->xmode == 4) {                          // TMV on staged tiles of B
+                fn = tmv_rowtile_fn(dt, p->block);
+                smem = p->smem;
+                args9[0] = &A; args9[1] = &X; args9[2] = &y; args9[3] = &R; args9[4] = &C;
+                args9[5] = &tile_mb; args9[6] = &stages; args9[7] = &part; args9[8] = &cnt;
+                args = args9;
+                break;
+            }
             if (p->flat && mis) {
                 fn = tmv_flat_fn(dt, p->unroll, p->block);
                 args7[0] = &A; args7[1] = &X; args7[2] = &y; args7[3] = &R; args7[4] = &C;
@@ -1396,6 +1534,23 @@ adaptic_status adaptic_run(adaptic_plan_t p, const void* A, const void* x, void*
                 ((reinterpret_cast<uintptr_t>(A) - reinterpret_cast<uintptr_t>(x)) & 15u) == 0);
     if (mis && p->variant == ADAPTIC_V_MV_TPR)   // bulk copies of row tiles: 16-byte aligned bases
         mis = aligned(A, 16) && (p->op != ADAPTIC_OP_DOT || aligned(x, 16));
+    if (p->nvec == 1 && p->xmode == 4 && (p->variant == ADAPTIC_V_MV_SUBWARP || p->variant == ADAPTIC_V_MV_WPR ||
+                                           p->variant == ADAPTIC_V_TMV_REGTILE)) {
+        // row tiles are bulk-copied from 16-byte-aligned bases; other pointers take the
+        // direct kernel of the same variant and shape
+        if (aligned(A, 16) && (p->op == ADAPTIC_OP_MV || aligned(x, 16)))
+            return launch(p, A, x, y, stream, p->vec_shape, p->mis);
+        adaptic_plan_s fb = *p;
+        if (derive(&fb, nullptr, device_info()) != ADAPTIC_OK) return ADAPTIC_ERR_UNSUPPORTED;
+        if (fb.ws_bytes > 0) {                    // its own zeroed slice of p's workspace
+            if (!p->ws || p->fb_ws_off + fb.ws_bytes > p->ws_cap) return ADAPTIC_ERR_NO_WORKSPACE;
+            fb.ws = static_cast<char*>(p->ws) + p->fb_ws_off;
+            fb.ws_cap = p->ws_cap - p->fb_ws_off;
+        } else {
+            fb.ws = nullptr; fb.ws_cap = 0;
+        }
+        return adaptic_run(&fb, A, x, y, stream_);
+    }
     if (!vec && p->nvec == 1 && p->xmode == 4) {
         // the x-tile kernel needs 16-byte rows and bases (TMA): a single-vector plan run on
         // 4-byte-aligned pointers takes the CTA-per-row kernel of the same shape instead

@@ -1,0 +1,54 @@
+// Instances of mv_rowtile_kernel (MV_SUBWARP / MV_WPR with [ADAPTIC_P_XSMEM] = 4):
+// G in {1, 2, 4, 8, 16, 32} lanes per row, 256 or 512 threads, fp32 / int32, MV / DOT.
+#include "launch.h"
+#include "rowtile_kernel.cuh"
+#include "tmv_rowtile_kernel.cuh"
+
+namespace adaptic {
+
+template <class T, int NT, bool PX>
+static void* rt_g(int G) {
+    switch (G) {
+        case 1: return reinterpret_cast<void*>(&mv_rowtile_kernel<T, NT, 1, PX>);
+        case 2: return reinterpret_cast<void*>(&mv_rowtile_kernel<T, NT, 2, PX>);
+        case 4: return reinterpret_cast<void*>(&mv_rowtile_kernel<T, NT, 4, PX>);
+        case 8: return reinterpret_cast<void*>(&mv_rowtile_kernel<T, NT, 8, PX>);
+        case 16: return reinterpret_cast<void*>(&mv_rowtile_kernel<T, NT, 16, PX>);
+        case 32: return reinterpret_cast<void*>(&mv_rowtile_kernel<T, NT, 32, PX>);
+        default: return nullptr;
+    }
+}
+
+template <class T>
+static void* rt_t(int NT, int G, bool px) {
+    if (NT == 256) return px ? rt_g<T, 256, true>(G) : rt_g<T, 256, false>(G);
+    if (NT == 512) return px ? rt_g<T, 512, true>(G) : rt_g<T, 512, false>(G);
+    return nullptr;
+}
+
+void* rowtile_fn(int dtype, int NT, int G, bool px) {
+    return dtype == DT_F32 ? rt_t<float>(NT, G, px) : rt_t<uint32_t>(NT, G, px);
+}
+
+}  // namespace adaptic
+
+namespace adaptic {
+// words per operand tile (the kernel's tile_w): k*C plus up to 3 head and 3 tail words,
+// rounded up to 16 bytes
+size_t rowtile_tile_words(int64_t k, int64_t C) { return size_t((k * C + 6 + 3) / 4) * 4; }
+}  // namespace adaptic
+
+namespace adaptic {
+// TMV on staged tiles of B (tmv_rowtile_kernel.cuh): 256, 512 or 1024 threads
+void* tmv_rowtile_fn(int dtype, int NT) {
+    switch (NT) {
+        case 256: return dtype == DT_F32 ? reinterpret_cast<void*>(&tmv_rowtile_kernel<float, 256>)
+                                         : reinterpret_cast<void*>(&tmv_rowtile_kernel<uint32_t, 256>);
+        case 512: return dtype == DT_F32 ? reinterpret_cast<void*>(&tmv_rowtile_kernel<float, 512>)
+                                         : reinterpret_cast<void*>(&tmv_rowtile_kernel<uint32_t, 512>);
+        case 1024: return dtype == DT_F32 ? reinterpret_cast<void*>(&tmv_rowtile_kernel<float, 1024>)
+                                          : reinterpret_cast<void*>(&tmv_rowtile_kernel<uint32_t, 1024>);
+        default: return nullptr;
+    }
+}
+}  // namespace adaptic

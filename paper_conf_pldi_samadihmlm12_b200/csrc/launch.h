@@ -53,6 +53,18 @@ constexpr int TMV_FLAT_MAX_R = 256;
 constexpr int TMV_FLAT_NT_SMALL_R = 64;     // R above this: 1024-thread CTAs
 void* tmv_flat_fn(int dtype, int U, int NT);
 
+// Lane groups on TMA-staged row tiles (rowtile_kernel.cuh; MV_SUBWARP / MV_WPR with
+// [ADAPTIC_P_XSMEM] = 4), C <= 32*G, 16-byte-aligned A (and DOT's b), NT in {256, 512}:
+//   (const T* A, const T* X, T* y, int64_t R, int64_t C, int k, int stages)   [dynamic smem]
+constexpr int RT_MAX_C_PER_LANE = 32;
+constexpr int RT_MAX_STAGES_H = 8;          // == RT_MAX_STAGES (mbarriers per CTA)
+void* rowtile_fn(int dtype, int NT, int G, bool px);
+size_t rowtile_tile_words(int64_t k, int64_t C);
+// TMV with R <= NT outputs on staged tiles of B (tmv_rowtile_kernel.cuh; TMV_REGTILE with
+// [ADAPTIC_P_XSMEM] = 4), 16-byte-aligned B and x, k % 4 == 0, NT in {256, 512, 1024}:
+//   (const T* B, const T* X, T* y, int64_t R, int64_t C, int k, int stages, T* part, unsigned* cnt)
+void* tmv_rowtile_fn(int dtype, int NT);
+
 // Multi-vector MV / TMV (mmv_kernels.cuh), fp32, K in {2, 4, 8}; X is K x C, Y is K x R:
 //   group: (const float* A, const float* X, float* Y, int64_t R, int64_t C), rows of <= G*U vectors
 //   cta  : (A, X, Y, R, C, int S, float* part, unsigned* cnt), RB = 8/K rows per CTA, NT = 256

@@ -1,0 +1,136 @@
+// rowtile_kernel.cuh -- MV / DOT lane groups on TMA-staged row tiles (sm_100a).
+//
+// The paper's K4/K3 thread shapes ("several threads ... the dot product of
+// one row", rows merged adaptively into one block) for rows of C <= 32*G elements
+// whose start is NOT 16-byte aligned (C % 4 != 0) -- the held-out 3*2^k shapes where
+// the direct kernels (mv_mis_kernels.cuh: 128-bit body + scalar head/tail) run at
+// 0.4-0.7 of the copy peak because a short row leaves each lane one or two loads in
+// flight.  Here the load side and the reduction side are decoupled:
+//
+//  * k consecutive rows are one contiguous run of k*C words.  Thread 0 copies the
+//    16-byte-aligned cover of that run ([floor4(r0*C), ceil4((r0+k)*C)) words) with
+//    one cp.async.bulk into a STAGES-deep ring guarded by mbarriers, so every SM
+//    keeps STAGES-1 whole tiles (tens of KB) in flight no matter how short the rows.
+//    Only the last tile of the matrix may end inside a 16-byte word group; its < 4
+//    remaining words are copied by the threads (no read past the matrix).
+//  * G lanes reduce one row out of shared memory: lane li reads words li + G*m
+//    (consecutive lanes, consecutive banks), x[li + G*m] lives in registers for the
+//    whole kernel (it is the same for every row), and the G partials are combined
+//    with a log2(G)-step butterfly (group_sum).  DOT (PERROWX) stages its second
+//    operand tile beside the first; both bases are 16-byte aligned, so the two tiles
+//    share the head offset.
+//
+// Accumulation order per row is fixed (lane partials over m in two interleaved
+// chains, then the butterfly), so a plan is deterministic (P7 invariants).
+#pragma once
+
+#include "common.cuh"
+
+namespace adaptic {
+
+constexpr int RT_MAX_STAGES = 8;
+constexpr int RT_MAXM = 32;          // x values per lane: C <= 32*G
+
+template <class T, int NT, int G, bool PERROWX>
+__global__ void __launch_bounds__(NT)
+mv_rowtile_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restrict__ y,
+                  int64_t R, int64_t C, int k, int stages)
+{
+    pdl_prologue();
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    __shared__ __align__(8) uint64_t full[RT_MAX_STAGES];
+
+    const int tid = threadIdx.x;
+    const int li = tid % G;
+    constexpr int NGR = NT / G;
+    const int Ci = int(C);
+    const int64_t total = R * C;
+    const int64_t ntiles = (R + k - 1) / k;
+    // words per operand tile: k*C plus up to 3 head and 3 tail words, rounded to 16 bytes
+    const int64_t tile_w = ((int64_t(k) * C + 6 + 3) / 4) * 4;
+    T* ring = reinterpret_cast<T*>(smem_raw);
+    const int64_t stage_w = tile_w * (PERROWX ? 2 : 1);
+    const int64_t my_tiles = blockIdx.x < ntiles ? (ntiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+
+    if (tid == 0) {
+        for (int s = 0; s < stages; ++s) mbar_init(&full[s], 1);
+        fence_mbar_init();
+    }
+    __syncthreads();
+
+    // local tile i -> stage i % stages (thread 0 only)
+    auto issue = [&](int64_t i) {
+        const int64_t r0 = (blockIdx.x + i * gridDim.x) * int64_t(k);
+        const int64_t w0 = r0 * C, w1 = min(R, r0 + k) * C;
+        const int64_t a0 = w0 & ~int64_t(3);
+        int64_t a1 = (w1 + 3) & ~int64_t(3);
+        if (a1 > total) a1 = w1 & ~int64_t(3);          // last tile: never read past the matrix
+        const uint32_t bytes = uint32_t((a1 - a0) * int64_t(sizeof(T)));
+        T* dst = ring + (i % stages) * stage_w;
+        uint64_t* bar = &full[i % stages];
+        mbar_arrive_expect_tx(bar, PERROWX ? 2 * bytes : bytes);
+        if (bytes) {
+            bulk_g2s(dst, A + a0, bytes, bar);
+            if (PERROWX) bulk_g2s(dst + tile_w, X + a0, bytes, bar);
+        }
+    };
+
+    if (tid == 0) {
+        const int64_t pre = min(int64_t(stages), my_tiles);
+        for (int64_t i = 0; i < pre; ++i) issue(i);
+    }
+
+    // x slice of this lane, kept in registers across all rows (MV only)
+    T xr[RT_MAXM];
+    if constexpr (!PERROWX) {
+#pragma unroll
+        for (int m = 0; m < RT_MAXM; ++m) {
+            const int c = li + G * m;
+            xr[m] = c < Ci ? ld_x(X + c) : T(0);
+        }
+    }
+
+    for (int64_t i = 0; i < my_tiles; ++i) {
+        const int st = int(i % stages);
+        const int64_t r0 = (blockIdx.x + i * gridDim.x) * int64_t(k);
+        const int nrows = int(min(int64_t(k), R - r0));
+        const int64_t w0 = r0 * C;
+        const int head = int(w0 & 3);
+        T* stg = ring + st * stage_w;
+        mbar_wait(&full[st], uint32_t((i / stages) & 1));
+        const int64_t w1 = w0 + int64_t(nrows) * C;
+        if (((w1 + 3) & ~int64_t(3)) > total && (w1 & 3)) {  // the matrix's last < 4 words
+            const int64_t a0 = w0 & ~int64_t(3);
+            for (int64_t e = (w1 & ~int64_t(3)) + tid; e < w1; e += NT) {
+                stg[e - a0] = A[e];
+                if (PERROWX) stg[tile_w + e - a0] = X[e];
+            }
+            __syncthreads();
+        }
+        const T* base = stg + head;
+        // whole warps step together (the butterfly needs all 32 lanes): groups whose
+        // row is past the tile contribute nothing and write nothing
+        for (int rb = (tid >> 5) * (32 / G); rb < nrows; rb += NGR) {
+            const int row = rb + (tid & 31) / G;
+            const bool live = row < nrows;
+            const T* ar = base + int64_t(live ? row : 0) * Ci;
+            T acc0 = T(0), acc1 = T(0);
+#pragma unroll
+            for (int m = 0; m < RT_MAXM; m += 2) {
+                if (G * m >= Ci) break;                 // uniform: C is the same for every lane
+                const int c0 = li + G * m, c1 = c0 + G;
+                if (live && c0 < Ci) acc0 = mac(ar[c0], PERROWX ? ar[tile_w + c0] : xr[m], acc0);
+                if (live && c1 < Ci) acc1 = mac(ar[c1], PERROWX ? ar[tile_w + c1] : xr[m + 1], acc1);
+            }
+            const T s = group_sum<G>(acc0 + acc1);
+            if (live && li == 0) y[r0 + row] = s;
+        }
+        __syncthreads();                                // every thread is done with stage st
+        if (tid == 0 && i + stages < my_tiles) {
+            fence_proxy_async();                        // generic-proxy reads before the async refill
+            issue(i + stages);
+        }
+    }
+}
+
+}  // namespace adaptic

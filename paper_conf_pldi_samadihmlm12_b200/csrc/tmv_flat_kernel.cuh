@@ -43,17 +43,33 @@ tmv_flat_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restrict_
     T acc[4] = {T(0), T(0), T(0), T(0)}, outer[4] = {T(0), T(0), T(0), T(0)};
     if (tid < NTa) {
         const int64_t t = int64_t(blockIdx.x) * NTa + tid;
+        // one vector whose words may lie outside B (the first and the last): masked, with
+        // the x index by division
+        auto edge_vec = [&](int64_t q) {
+            const int64_t f0 = 4 * q - b0;
+            if (f0 >= 0 && f0 + 3 < total) {
+                const E a = ld_stream(Ba + q);
+                const T av[4] = {a.x, a.y, a.z, a.w};
+#pragma unroll
+                for (int j = 0; j < 4; ++j) acc[j] = mac(av[j], ld_x(X + (f0 + j) / R), acc[j]);
+            } else {
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    const int64_t f = f0 + j;
+                    if (f >= 0 && f < total) acc[j] = mac(ld_stream(B + f), ld_x(X + f / R), acc[j]);
+                }
+            }
+        };
+        int64_t q = t;
+        // vector 0 may start before B (b0 > 0): peel it, so that the unrolled loop below
+        // runs for every thread (thread 0 included) with nonnegative word indices
+        if (q == 0) { if (qend > 0) edge_vec(0); q = T_; }
         int64_t c[4];
 #pragma unroll
-        for (int j = 0; j < 4; ++j) {                   // word f = 4t + j - b0 (may be < 0 for t = 0)
-            const int64_t f = 4 * t + j - b0;
-            c[j] = f >= 0 ? f / R : -1;
-        }
+        for (int j = 0; j < 4; ++j) c[j] = (4 * q + j - b0) / R;     // word 4q + j - b0 >= 1
         int it = 0;
-        int64_t q = t;
         // interior vectors (every word inside B): q in [1, qend - 1)
         for (; q + T_ * (U - 1) < qend - 1; q += T_ * U) {
-            if (q == 0) break;                          // the first vector may start before B
             E a[U];
             T xv[U][4];
 #pragma unroll
@@ -76,21 +92,7 @@ tmv_flat_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restrict_
             }
         }
         // the rest, one vector at a time, words outside B masked
-        for (; q < qend; q += T_) {
-            const int64_t f0 = 4 * q - b0;
-            if (f0 >= 0 && f0 + 3 < total) {
-                const E a = ld_stream(Ba + q);
-                const T av[4] = {a.x, a.y, a.z, a.w};
-#pragma unroll
-                for (int j = 0; j < 4; ++j) acc[j] = mac(av[j], ld_x(X + (f0 + j) / R), acc[j]);
-            } else {                                    // B's first / last vector: only its own words
-#pragma unroll
-                for (int j = 0; j < 4; ++j) {
-                    const int64_t f = f0 + j;
-                    if (f >= 0 && f < total) acc[j] = mac(ld_stream(B + f), ld_x(X + f / R), acc[j]);
-                }
-            }
-        }
+        for (; q < qend; q += T_) edge_vec(q);
 #pragma unroll
         for (int j = 0; j < 4; ++j) P[4 * tid + j] = outer[j] + acc[j];
     }

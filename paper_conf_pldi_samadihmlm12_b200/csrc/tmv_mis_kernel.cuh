@@ -85,15 +85,34 @@ tmv_mis_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restrict__
             E lo[U], hi[U];
             T xs[U];
             int sh[U];
+            // aligned vectors grow with c: when the first load's low vector starts inside B
+            // and the last load's high vector ends inside it, every word of every load is
+            // inside B and no per-word masking is needed (only the very first / last 16
+            // bytes of B take the masked path)
+            const int64_t qf = (b0 + c * R + col) >> 2;
+            const int64_t ql = (b0 + (c + int64_t(LC) * (U - 1)) * R + col) >> 2;
+            if (4 * qf - b0 >= 0 && 4 * (ql + 1) - b0 + 3 < R * C) {
 #pragma unroll
-            for (int u = 0; u < U; ++u) {
-                const int64_t cc = c + int64_t(LC) * u;
-                const int64_t f = b0 + cc * R + col;             // aligned-view element index
-                const int64_t q = f >> 2;
-                sh[u] = int(f & 3);
-                lo[u] = ld_inside(Ba, B, q, b0, R * C);
-                hi[u] = ld_inside(Ba, B, min(q + 1, qmax), b0, R * C);
-                xs[u] = ld_x(X + cc);
+                for (int u = 0; u < U; ++u) {
+                    const int64_t cc = c + int64_t(LC) * u;
+                    const int64_t f = b0 + cc * R + col;
+                    const int64_t q = f >> 2;
+                    sh[u] = int(f & 3);
+                    lo[u] = ld_stream(Ba + q);
+                    hi[u] = ld_stream(Ba + q + 1);
+                    xs[u] = ld_x(X + cc);
+                }
+            } else {
+#pragma unroll
+                for (int u = 0; u < U; ++u) {
+                    const int64_t cc = c + int64_t(LC) * u;
+                    const int64_t f = b0 + cc * R + col;         // aligned-view element index
+                    const int64_t q = f >> 2;
+                    sh[u] = int(f & 3);
+                    lo[u] = ld_inside(Ba, B, q, b0, R * C);
+                    hi[u] = ld_inside(Ba, B, min(q + 1, qmax), b0, R * C);
+                    xs[u] = ld_x(X + cc);
+                }
             }
 #pragma unroll
             for (int u = 0; u < U; ++u) esmac(acc[u], funnel4(lo[u], hi[u], sh[u]), xs[u]);

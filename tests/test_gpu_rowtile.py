@@ -1,0 +1,216 @@
+"""Lane groups on TMA-staged row tiles (csrc/rowtile_kernel.cuh; MV_SUBWARP / MV_WPR
+with [ADAPTIC_P_XSMEM] = 4) against the oracle -- needs a GPU.
+
+fp32 within 1e-4 * S_r (north_star), int32 bit-exact, P5 (integer-valued fp32) exact.
+Covers every lane-group width, tiles of 1 .. many rows, ragged last tiles, a matrix
+whose word count is not a multiple of 4 (the last tile's remainder copied by the
+threads), rows at every 16-byte phase (C % 4 = 1, 2, 3 and 0), 256/512-thread CTAs,
+2..8 ring stages, DOT, and base pointers that are not 16-byte aligned (those run the
+variant's direct kernel)."""
+import itertools
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import synth
+
+pytestmark = pytest.mark.gpu
+
+if torch.cuda.is_available():
+    import paper_conf_pldi_samadihmlm12_b200 as adaptic
+    from paper_conf_pldi_samadihmlm12_b200 import _lib as L
+
+DEV = "cuda:0"
+TOL = 1e-4
+
+
+def check(y, ref, dt, what):
+    if dt == "i32":
+        assert np.array_equal(y, ref), f"{what}: int32 mismatch at {np.nonzero(y != ref)[0][:8]}"
+    else:
+        yr, S = ref
+        err = np.abs(y.astype(np.float64) - yr)
+        bad = ~(err <= TOL * S)
+        assert not bad.any(), f"{what}: {bad.sum()} out of tolerance, worst {np.max(err - TOL * S)}"
+
+
+def _collect(cases):
+    fails = []
+    for what, fn in cases:
+        try:
+            fn()
+        except Exception as e:  # noqa: BLE001 -- report every failing case at once
+            fails.append(f"{what}: {type(e).__name__}: {str(e)[:200]}")
+    assert not fails, f"{len(fails)} failures:\n" + "\n".join(fails[:40])
+
+
+def rt_params(g, nt=0, k=0, stages=0, cps=0):
+    """[lanes, splits, ctas_per_sm, unroll(stages), xsmem=4, block, rows]"""
+    return [g, 0, cps, stages, 4, nt, k]
+
+
+SHAPES = [(1, 5), (3, 17), (7, 9), (33, 19), (64, 31), (65, 127), (130, 257), (257, 66), (1000, 21),
+          (999, 513), (4097, 33), (12345, 9), (100003, 7), (5, 1024), (300, 100), (2, 1), (17, 2), (31, 3)]
+PLANS = [("MV_SUBWARP", rt_params(g, nt, k, st)) for g in (1, 2, 4, 8, 16) for nt, k, st in
+         ((0, 0, 0), (512, 0, 2), (256, 1, 4), (256, 37, 8))] + \
+        [("MV_WPR", rt_params(32, nt, k, st)) for nt, k, st in ((0, 0, 0), (512, 3, 3), (256, 64, 2))]
+
+
+@pytest.mark.parametrize("op", ["mv", "dot"])
+@pytest.mark.parametrize("dt", ["f32", "i32"])
+def test_rowtile_every_width_and_tile(op, dt):
+    npdt = np.float32 if dt == "f32" else np.int32
+
+    def case(R, C, v, p):
+        A = synth.matrix(R, C, "mv", npdt, "uniform", synth.seed(21, "A") + R + C)
+        X = (synth.matrix(R, C, "mv", npdt, "uniform", synth.seed(21, "b") + R) if op == "dot"
+             else synth.vector(C, npdt, "uniform", synth.seed(21, "x") + C))
+        try:
+            plan = adaptic.plan(op, R, C, dt, variant=v, params=p)
+        except adaptic.AdapticError as e:
+            assert e.status == L.ERR_UNSUPPORTED, str(e)
+            # auto tile height always fits; a forced one may leave < 2 stages of ring
+            assert C > 32 * p[0] or p[6] > 0, f"unexpected UNSUPPORTED {R}x{C} {p}"
+            return
+        d = plan.describe()
+        assert d["xmode"] == 4 and d["stages"] >= 2, d
+        fn = adaptic.mv if op == "mv" else adaptic.dot
+        y = fn(torch.from_numpy(A).to(DEV), torch.from_numpy(X).to(DEV), variant=v, params=p).cpu().numpy()
+        ref = oracle.mv(A, X) if op == "mv" else oracle.dot(A, X)
+        check(y, ref, dt, f"{op} {dt} {R}x{C} {v} {p}")
+    _collect([(f"{R}x{C} {v} {p}", lambda R=R, C=C, v=v, p=p: case(R, C, v, p))
+              for (R, C), (v, p) in itertools.product(SHAPES, PLANS)])
+
+
+def test_rowtile_exact_on_integer_valued_fp32():
+    """P5: every partial sum exact, so the staged kernel equals the oracle bit for bit."""
+    for R, C, g in [(4099, 257, 16), (100003, 9, 1), (2049, 1023, 32), (777, 130, 8)]:
+        A = synth.matrix(R, C, "mv", np.float32, "smallint", 41 + C)
+        x = synth.vector(C, np.float32, "smallint", 42 + C)
+        v = "MV_WPR" if g == 32 else "MV_SUBWARP"
+        y = adaptic.mv(torch.from_numpy(A).to(DEV), torch.from_numpy(x).to(DEV), variant=v,
+                       params=rt_params(g)).cpu().numpy()
+        assert np.array_equal(y.astype(np.float64), oracle.mv(A, x)[0]), f"P5 {R}x{C} g{g}"
+
+
+def test_rowtile_deterministic_scaling_and_negation():
+    """P7: the same plan on 2^k x and -x gives exactly 2^k y and -y (fixed order)."""
+    R, C = 5000, 171
+    A = torch.from_numpy(synth.matrix(R, C, "mv", np.float32, "uniform", 51)).to(DEV)
+    x = torch.from_numpy(synth.vector(C, np.float32, "uniform", 52)).to(DEV)
+    p = rt_params(8)
+    y = adaptic.mv(A, x, variant="MV_SUBWARP", params=p)
+    assert torch.equal(adaptic.mv(A, x * 8, variant="MV_SUBWARP", params=p), y * 8)
+    assert torch.equal(adaptic.mv(A, -x, variant="MV_SUBWARP", params=p), -y)
+    assert torch.equal(adaptic.mv(A, x, variant="MV_SUBWARP", params=p), y)
+
+
+def test_rowtile_unaligned_bases_fall_back():
+    """A (or DOT's b) not 16-byte aligned: the variant's direct kernel, same results."""
+    for R, C, off in [(31, 37, 1), (640, 101, 2), (9, 500, 3), (1000, 16, 1)]:
+        A = synth.matrix(R, C, "mv", np.float32, "uniform", 5 + C)
+        x = synth.vector(C, np.float32, "uniform", 6 + C)
+        big = torch.zeros(R * C + 8, dtype=torch.float32, device=DEV)
+        big[off:off + R * C] = torch.from_numpy(A.reshape(-1)).to(DEV)
+        Ad = big[off:off + R * C].view(R, C)
+        for v, g in (("MV_SUBWARP", 4), ("MV_WPR", 32)):
+            p = rt_params(g)
+            try:
+                adaptic.plan("mv", R, C, "f32", variant=v, params=p)
+            except adaptic.AdapticError:
+                continue
+            y = adaptic.mv(Ad, torch.from_numpy(x).to(DEV), variant=v, params=p).cpu().numpy()
+            check(y, oracle.mv(A, x), "f32", f"off {off} {R}x{C} {v}")
+    R, C = 333, 129
+    a = synth.matrix(R, C, "mv", np.int32, "uniform", 71)
+    b = synth.matrix(R, C, "mv", np.int32, "uniform", 72)
+    bb = torch.zeros(R * C + 4, dtype=torch.int32, device=DEV)
+    bb[1:1 + R * C] = torch.from_numpy(b.reshape(-1)).to(DEV)
+    y = adaptic.dot(torch.from_numpy(a).to(DEV), bb[1:1 + R * C].view(R, C), variant="MV_SUBWARP",
+                    params=rt_params(8)).cpu().numpy()
+    check(y, oracle.dot(a, b), "i32", "dot b off by 4 bytes")
+
+
+def test_rowtile_large_held_out_shape_sampled():
+    """A 256 MiB held-out shape at full size in the bench's configuration (AUTO and the
+    forced staged plan): sampled rows against the oracle row by row."""
+    R, C = 262144, 257
+    A = torch.empty(R * C, dtype=torch.float32, device=DEV)
+    synth.device_matrix(A, R, C, "mv", "uniform", 61)
+    x = torch.empty(C, dtype=torch.float32, device=DEV)
+    synth.device_vector(x, "uniform", 62)
+    xs = x.cpu().numpy()
+    rows = np.unique(np.concatenate([np.arange(0, 64), np.arange(R - 64, R),
+                                     np.random.default_rng(3).integers(0, R, 256)]))
+    for v, p in (("AUTO", None), ("MV_WPR", rt_params(32)), ("MV_SUBWARP", rt_params(16, 512))):
+        y = adaptic.mv(A.view(R, C), x, variant=v, params=p).cpu().numpy()
+        Arows = A.view(R, C)[torch.from_numpy(rows).to(DEV)].cpu().numpy()
+        yr, S = oracle.mv(Arows, xs)
+        err = np.abs(y[rows].astype(np.float64) - yr)
+        assert np.all(err <= TOL * S), f"{v} {p}"
+
+
+# ---------------------------------------------------------------- TMV on staged tiles of B
+def trt_params(nt=0, k=0, stages=0, cps=0):
+    """TMV_REGTILE [lanes, splits, ctas_per_sm, unroll(stages), xsmem=4, block, rows]"""
+    return [0, 0, cps, stages, 4, nt, k]
+
+
+TMV_SHAPES = [(1, 1), (1, 1000), (2, 77), (3, 100003), (5, 7), (9, 4099), (13, 1000), (63, 257), (64, 333),
+              (129, 4099), (255, 100), (256, 17), (257, 999), (513, 1001), (1023, 65), (1024, 9), (4, 3), (30, 7)]
+TMV_PLANS = [trt_params()] + [trt_params(nt, k, st) for nt, k, st in
+                              ((256, 4, 0), (512, 8, 2), (1024, 0, 3), (1024, 4, 8), (256, 64, 2))]
+
+
+@pytest.mark.parametrize("dt", ["f32", "i32"])
+def test_tmv_rowtile_shapes_and_tiles(dt):
+    npdt = np.float32 if dt == "f32" else np.int32
+
+    def case(R, C, p):
+        B = synth.matrix(R, C, "tmv", npdt, "uniform", synth.seed(22, "A") + R + C)
+        x = synth.vector(C, npdt, "uniform", synth.seed(22, "x") + C)
+        try:
+            plan = adaptic.plan("tmv", R, C, dt, variant="TMV_REGTILE", params=p)
+        except adaptic.AdapticError as e:
+            assert e.status in (L.ERR_UNSUPPORTED, L.ERR_INVALID_ARG), str(e)
+            # forced shapes may exceed the CTA (R > threads), the ring budget (< 2 stages) or
+            # the error bound (slice sums of 1024 threads for R = 1); the default plan may not
+            assert p != trt_params() or R > 1024, f"unexpected {e} for {R}x{C} {p}"
+            return
+        assert plan.describe()["xmode"] == 4
+        y = adaptic.tmv(torch.from_numpy(B).to(DEV), torch.from_numpy(x).to(DEV), variant="TMV_REGTILE", params=p)
+        check(y.cpu().numpy(), oracle.tmv(B, x), dt, f"tmv {dt} {R}x{C} {p}")
+    _collect([(f"{R}x{C} {p}", lambda R=R, C=C, p=p: case(R, C, p))
+              for (R, C), p in itertools.product(TMV_SHAPES, TMV_PLANS)])
+
+
+def test_tmv_rowtile_exact_and_deterministic():
+    """P5 exact at 2^22 elements with R off the 16-byte grid; P7 scaling/negation."""
+    for R in (9, 129, 513):
+        C = (1 << 22) // R
+        B = synth.matrix(R, C, "tmv", np.float32, "smallint", 81 + R)
+        x = synth.vector(C, np.float32, "smallint", 82 + R)
+        Bd, xd = torch.from_numpy(B).to(DEV), torch.from_numpy(x).to(DEV)
+        y = adaptic.tmv(Bd, xd, variant="TMV_REGTILE", params=trt_params())
+        assert np.array_equal(y.cpu().numpy().astype(np.float64), oracle.tmv(B, x)[0]), f"P5 {R}x{C}"
+        Bu = torch.from_numpy(synth.matrix(R, C, "tmv", np.float32, "uniform", 83 + R)).to(DEV)
+        yu = adaptic.tmv(Bu, xd, variant="TMV_REGTILE", params=trt_params())
+        assert torch.equal(adaptic.tmv(Bu, xd * 4, variant="TMV_REGTILE", params=trt_params()), yu * 4)
+        assert torch.equal(adaptic.tmv(Bu, -xd, variant="TMV_REGTILE", params=trt_params()), -yu)
+
+
+def test_tmv_rowtile_unaligned_bases_fall_back():
+    for R, C in [(9, 1000), (61, 333), (517, 64)]:
+        B = synth.matrix(R, C, "tmv", np.float32, "uniform", 91 + R)
+        x = synth.vector(C, np.float32, "uniform", 92 + C)
+        for off in (1, 2, 3):
+            big = torch.zeros(R * C + 8, dtype=torch.float32, device=DEV)
+            big[off:off + R * C] = torch.from_numpy(B.reshape(-1)).to(DEV)
+            xb = torch.zeros(C + 8, dtype=torch.float32, device=DEV)
+            xb[off:off + C] = torch.from_numpy(x).to(DEV)
+            for Bv, xv in ((big[off:off + R * C].view(C, R), torch.from_numpy(x).to(DEV)),
+                           (torch.from_numpy(B).to(DEV), xb[off:off + C])):
+                y = adaptic.tmv(Bv, xv, variant="TMV_REGTILE", params=trt_params())
+                check(y.cpu().numpy(), oracle.tmv(B, x), "f32", f"tmv off {off} {R}x{C}")

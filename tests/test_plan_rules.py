@@ -60,3 +60,39 @@ def test_multi_plans_respect_the_error_bound(K):
             p = d(op, 1 << k, 1 << (26 - k), nvec=K)
             w = 1 if p["vec_shape"] else 0
             assert p["path_ok"][w], (op, k, p)
+
+
+def test_staged_row_tiles_mv_dot():
+    """XSMEM 4 on MV_SUBWARP / MV_WPR: the staged row-tile kernel (rowtile_kernel.cuh)."""
+    p = d("mv", 262144, 257, variant="MV_WPR", params=[0, 0, 0, 0, 4])
+    assert p["xmode"] == 4 and p["lanes"] == 32 and p["stages"] >= 2 and p["mis"]
+    assert p["rows_per_group"] % 8 == 0                               # whole warps of rows (256/32 groups)
+    assert p["chain"][1] == 5 and p["path_ok"][1]                      # ceil(ceil(257/32)/2)
+    # ROWS = -n: an ~n KB tile (the fitted tables' portable form); DOT stages b too
+    assert d("mv", 100000, 100, variant="MV_SUBWARP", params=[4, 0, 0, 0, 4, 256, -12])["rows_per_group"] == 30
+    assert d("dot", 100000, 100, variant="MV_SUBWARP", params=[4, 0, 0, 0, 4, 256, -12])["rows_per_group"] == 15
+    # an explicit height too tall for two stages is capped, not refused
+    capped = d("mv", 3145728, 22, variant="MV_SUBWARP", params=[1, 0, 0, 0, 4, 256, 722])
+    assert capped["rows_per_group"] < 722 and capped["stages"] == 2
+    # x must fit the registers: C <= 32 * G
+    with pytest.raises(adaptic.AdapticError):
+        d("mv", 1000, 300, variant="MV_SUBWARP", params=[8, 0, 0, 0, 4])
+    # the fitted table takes the staged kernel on the off-grid short-row shapes
+    for op, R, C in (("mv", 262144, 257), ("mv", 8388608, 9), ("dot", 524288, 129)):
+        assert d(op, R, C)["xmode"] == 4, (op, R, C)
+
+
+def test_staged_tmv_tiles():
+    """XSMEM 4 on TMV_REGTILE: tiles of B + x chunks (tmv_rowtile_kernel.cuh), R <= 1024."""
+    p = d("tmv", 9, 8388608, variant="TMV_REGTILE", params=[0, 0, 0, 0, 4])
+    assert p["xmode"] == 4 and p["block"] == 256 and p["rows_per_group"] % 4 == 0 and p["stages"] >= 3
+    assert p["workspace_bytes"] > 0 and p["path_ok"][1]
+    assert d("tmv", 513, 131072, variant="TMV_REGTILE", params=[0, 0, 0, 0, 4])["block"] == 1024
+    with pytest.raises(adaptic.AdapticError):                          # more outputs than threads
+        d("tmv", 300, 1000, variant="TMV_REGTILE", params=[0, 0, 0, 0, 4, 256])
+    with pytest.raises(adaptic.AdapticError):                          # R > 1024
+        d("tmv", 1025, 1000, variant="TMV_REGTILE", params=[0, 0, 0, 0, 4])
+    with pytest.raises(adaptic.AdapticError):                          # tile height not a multiple of 4
+        d("tmv", 9, 1000, variant="TMV_REGTILE", params=[0, 0, 0, 0, 4, 256, 6])
+    for R, C in ((9, 8388608), (129, 524288), (14, 5162220)):
+        assert d("tmv", R, C)["xmode"] == 4, (R, C)

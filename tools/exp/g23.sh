@@ -1,0 +1,17 @@
+#!/bin/bash
+# parity of the staged MV/DOT/TMV kernels, then the full candidate grid on the off-grid
+# shapes they serve (fresh data for every candidate, same box) for the table refit
+set -u
+mkdir -p gpurun_out
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/g23_build.log 2>&1 || { echo build-failed; tail -30 gpurun_out/g23_build.log; exit 1; }
+timeout 900 python -m pytest tests/test_gpu_rowtile.py tests/test_gpu_mis.py -x -q > gpurun_out/g23_pytest.log 2>&1
+echo "pytest rc=$?"; tail -5 gpurun_out/g23_pytest.log
+out=gpurun_out/sweep_r1f_offgrid.jsonl
+rm -f $out
+for e in 20 21 22 23 24 25 26; do
+  timeout 900 python tools/sweep.py --out $out --elems $e --perturb-only --ops mv,dot --kmin $((e-9)) --reps 7 >> gpurun_out/g23_sweep.log 2>&1
+  timeout 900 python tools/sweep.py --out $out --elems $e --perturb-only --ops tmv --kmin 3 --kmax 9 --reps 7 >> gpurun_out/g23_sweep.log 2>&1
+done
+timeout 900 python tools/sweep.py --out $out --elems 26 --kmin 30 --ops mv,dot --extra 393216x171,3145728x22 --reps 7 >> gpurun_out/g23_sweep.log 2>&1
+timeout 900 python tools/sweep.py --out $out --elems 26 --kmin 30 --ops tmv --extra 14x5162220,98x691870 --reps 7 >> gpurun_out/g23_sweep.log 2>&1
+wc -l $out

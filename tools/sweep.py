@@ -39,9 +39,32 @@ def tile_grid(op, R, C, dtype):
     return [("MV_SPLIT", [cw, 0, 0, 0, 3, 0, 0]) for cw in (0, 8192, 16384) if cw <= C]
 
 
+def rowtile_grid(op, R, C):
+    """Lane groups on TMA-staged row tiles (XSMEM 4; MV/DOT, C <= 32*G): lanes per row G,
+    threads per CTA and tile height (rows per ~12 / 24 (auto) / 48 KB of staged data)."""
+    if op == "tmv":
+        if R > 1024:
+            return []
+        return [("TMV_REGTILE", [0, 0, 0, 0, 4, nt, k]) for nt in (256, 512, 1024) if nt >= R
+                for k in sorted({0, max(4, 12 * 1024 // (4 * R) // 4 * 4), max(4, 48 * 1024 // (4 * R) // 4 * 4)})]
+    if op not in ("mv", "dot") or C > 1024:
+        return []
+    out = []
+    opb = 8 if op == "dot" else 4
+    for g in (1, 2, 4, 8, 16, 32):
+        if C > 32 * g or (g > 1 and C < 2 * g):
+            continue
+        v = "MV_WPR" if g == 32 else "MV_SUBWARP"
+        for nt in (256, 512):
+            for kb in (0, 12, 48):
+                k = 0 if kb == 0 else max(1, kb * 1024 // (C * opb))
+                out.append((v, [g, 0, 0, 0, 4, nt, k]))
+    return out
+
+
 def grids(op, R, C, dtype="f32"):
     """(variant, params) candidates; params = [lanes, splits, ctas_per_sm, unroll, xsmem, block, rows], 0 = auto."""
-    out = [("AUTO", None)] + tile_grid(op, R, C, dtype)
+    out = [("AUTO", None)] + tile_grid(op, R, C, dtype) + rowtile_grid(op, R, C)
     if op in B1:
         nv = C // 4 if C % 4 == 0 else C
         if nv <= 64:
@@ -136,6 +159,8 @@ def main():
     ap.add_argument("--perturb-only", action="store_true", help="only the perturbed (off-128-bit-path) shapes")
     ap.add_argument("--auto-only", action="store_true", help="time only the selector's pick (validation runs)")
     ap.add_argument("--tile-only", action="store_true", help="time only the x-tile stream-K candidates (+ AUTO)")
+    ap.add_argument("--rowtile-only", action="store_true", help="time only the staged row-tile candidates (+ AUTO)")
+    ap.add_argument("--flat-only", action="store_true", help="time only the flat-stream TMV candidates (+ AUTO)")
     a = ap.parse_args()
     dev = torch.device("cuda:0")
     tdt = torch.float32 if a.dtype == "f32" else torch.int32
@@ -167,8 +192,17 @@ def main():
                 R, C = (R0 + pert, C0) if op == "tmv" else (R0, C0 + pert)
                 Xp = M.data_ptr() + R * C * 4 if op == "dot" else X.data_ptr()
                 ptrs = (M.data_ptr(), Xp, Y.data_ptr())
-                cands = ([("AUTO", None)] if a.auto_only else
-                         [("AUTO", None)] + tile_grid(op, R, C, a.dtype) if a.tile_only else grids(op, R, C, a.dtype))
+                if a.auto_only:
+                    cands = [("AUTO", None)]
+                elif a.tile_only:
+                    cands = [("AUTO", None)] + tile_grid(op, R, C, a.dtype)
+                elif a.rowtile_only:
+                    cands = [("AUTO", None)] + rowtile_grid(op, R, C)
+                elif a.flat_only:
+                    cands = [("AUTO", None)] + [("TMV_REGTILE", [0, 0, 0, u]) for u in (2, 4, 8)] + \
+                        rowtile_grid(op, R, C)
+                else:
+                    cands = grids(op, R, C, a.dtype)
                 for variant, params in cands:
                     try:
                         plan = adaptic.get_plan(OPC[op], R, C, dtc, dev, variant, params, stream)
