@@ -6,6 +6,8 @@ Workloads (``--workload``):
   sweep    (default, BJ:configs[1]) one step = the selector-chosen kernel on all 42
            problems of the fixed-256-MiB shape sweep: R x C = 2^k x 2^(26-k),
            k = 3..23, in both layouts (MV: A row-major R x C; TMV: B = A^T).
+  offgrid  the same 42 problems with C+1 (MV) / R+1 (TMV): rows off the 16-byte grid
+           (misaligned 128-bit body kernels, staged row tiles).
   rowshard (BJ:configs[3]) MV 131072 x 32768 fp32, rows sharded over ranks.
   splitk   (BJ:configs[4]) TMV 1024 x 16M fp32, C split over ranks + NCCL all-reduce.
   dot      (BJ:configs[2]) scalar product N = 1, L = 2^10..2^30 (fp32).
@@ -48,7 +50,7 @@ def parse():
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", choices=["adaptic", "reference"], default="adaptic")
-    ap.add_argument("--workload", choices=["sweep", "rowshard", "splitk", "dot", "blas1", "config0", "multi", "bicgstab", "stencil"], default="sweep")
+    ap.add_argument("--workload", choices=["sweep", "offgrid", "rowshard", "splitk", "dot", "blas1", "config0", "multi", "bicgstab", "stencil"], default="sweep")
     ap.add_argument("--variant", default="AUTO", help="force one variant (fixed-variant sweeps)")
     ap.add_argument("--dtype", choices=["f32", "i32"], default="f32",
                     help="element type of the MV/TMV/DOT workloads (i32: arithmetic modulo 2^32)")
@@ -224,6 +226,12 @@ def build_problems(args, world, rank):
                 for k in range(3, 24) for op in ("mv", "tmv")], \
             {"workload": "configs[1]: TMV/MV fp32 shape sweep at 256 MiB, 8Mx8 .. 8192x8192 .. 8x8M, "
                          "both layouts, variant selector", "shapes": 42, "per_gpu": "full sweep (weak)"}
+    if args.workload == "offgrid":
+        return [Problem(op, (1 << k) + (op == "tmv"), (1 << (26 - k)) + (op == "mv"), 1, args.variant,
+                        dtype=args.dtype) for k in range(3, 24) for op in ("mv", "tmv")], \
+            {"workload": "configs[1] off the 16-byte grid: the sweep's 21 shapes with C+1 (MV) / R+1 (TMV), "
+                         "256 MiB each, rows not 16-byte aligned, variant selector", "shapes": 42,
+             "per_gpu": "full sweep (weak)"}
     if args.workload == "multi":
         shapes = [(8192, 8192), (65536, 1024), (1 << 20, 64), (64, 1 << 20)]
         return [Problem(op, R, C, 8, args.variant, nvec=4) for R, C in shapes for op in ("mv", "tmv")], \
@@ -379,7 +387,7 @@ def run_adaptic(args):
                 "data": "synthetic (seeded splitmix64; fp32 U[-1,1), int32 U{-128..127})",
                 "config": dict(config, bytes_per_step_per_gpu=step_bytes, variant=args.variant,
                                l2=("every input >= 256 MiB > 126 MB L2 and problems alternate; no flush needed"
-                                   if args.workload in ("sweep", "blas1", "stencil") else
+                                   if args.workload in ("sweep", "offgrid", "blas1", "stencil") else
                                    "L2-resident by design (256 KiB): latency-bound, see latency_us"
                                    if args.workload == "config0" else
                                    "dot: lengths 2^10..2^30 back to back; the >= 2^25 ones exceed L2"
@@ -548,6 +556,10 @@ def run_reference(args):
     import synth
     if args.workload == "sweep":
         pool = [("mv", 1 << 13, 1 << 13), ("tmv", 1 << 13, 1 << 13), ("mv", 1 << 20, 64), ("tmv", 64, 1 << 20)]
+        cfg = 1
+    elif args.workload == "offgrid":
+        pool = [("mv", 1 << 13, (1 << 13) + 1), ("tmv", (1 << 13) + 1, 1 << 13), ("mv", 1 << 20, 65),
+                ("tmv", 65, 1 << 20)]
         cfg = 1
     elif args.workload == "dot":
         pool = [("dot", 1, 1 << 26)]

@@ -1569,10 +1569,12 @@ adaptic_status adaptic_run(adaptic_plan_t p, const void* A, const void* x, void*
 // ---- batched issue over concurrent streams (per host thread, per device)
 namespace {
 constexpr int kMaxBatchStreams = 8;
+constexpr size_t kExclusiveSmem = 64 * 1024;     // dynamic smem per CTA of a staged-tile plan
 struct StreamPool {
     int dev = -1;
     cudaStream_t side[kMaxBatchStreams - 1] = {};
     cudaEvent_t fork = nullptr, join[kMaxBatchStreams - 1] = {};
+    cudaEvent_t mainev = nullptr;          // the caller's stream, for exclusive plans
 };
 thread_local StreamPool g_pools[8];
 
@@ -1588,6 +1590,7 @@ cudaError_t pool_for_current_device(StreamPool** out) {
             if ((e = cudaEventCreateWithFlags(&P.join[i], cudaEventDisableTiming)) != cudaSuccess) return e;
         }
         if ((e = cudaEventCreateWithFlags(&P.fork, cudaEventDisableTiming)) != cudaSuccess) return e;
+        if ((e = cudaEventCreateWithFlags(&P.mainev, cudaEventDisableTiming)) != cudaSuccess) return e;
         P.dev = dev;
     }
     *out = &P;
@@ -1621,12 +1624,33 @@ adaptic_status adaptic_run_batch(int32_t n, const adaptic_plan_t* plans, const v
     for (int j = 0; j < k - 1; ++j)
         if ((e = cudaStreamWaitEvent(P->side[j], P->fork, 0)) != cudaSuccess) return cuda_fail(e);
     adaptic_status st = ADAPTIC_OK;
+    auto lane_stream = [&](int l) { return l == 0 ? stream : P->side[l - 1]; };
+    auto lane_event = [&](int l) { return l == 0 ? P->mainev : P->join[l - 1]; };
     for (int32_t i = 0; i < n && st == ADAPTIC_OK; ++i) {
         int lane = i % k;
         for (int32_t q = 0; q < i; ++q)                   // a plan's workspace serialises its runs:
             if (plans[q] == plans[i] && plans[i]->ws_bytes > 0) { lane = q % k; break; }   // same stream
-        cudaStream_t s = lane == 0 ? stream : P->side[lane - 1];
+        cudaStream_t s = lane_stream(lane);
+        // Staged-tile kernels size a persistent grid for the whole GPU and hold most of an
+        // SM's shared memory: next to another stream's kernel their late CTAs stretch the
+        // launch (offgrid step 2.29 -> 2.81 ms measured), so they run alone -- after every
+        // lane's earlier work, and before any lane's later work.
+        const bool excl = plans[i]->smem >= kExclusiveSmem;
+        if (excl)
+            for (int l = 0; l < k; ++l) {
+                if (l == lane) continue;
+                if ((e = cudaEventRecord(lane_event(l), lane_stream(l))) != cudaSuccess ||
+                    (e = cudaStreamWaitEvent(s, lane_event(l), 0)) != cudaSuccess) { st = cuda_fail(e); break; }
+            }
+        if (st != ADAPTIC_OK) break;
         st = adaptic_run(plans[i], A[i], x[i], y[i], s);
+        if (excl && st == ADAPTIC_OK) {
+            if ((e = cudaEventRecord(lane_event(lane), s)) != cudaSuccess) { st = cuda_fail(e); break; }
+            for (int l = 0; l < k; ++l)
+                if (l != lane && (e = cudaStreamWaitEvent(lane_stream(l), lane_event(lane), 0)) != cudaSuccess) {
+                    st = cuda_fail(e); break;
+                }
+        }
     }
     for (int j = 0; j < k - 1; ++j) {                    // join (also after a failure)
         if ((e = cudaEventRecord(P->join[j], P->side[j])) != cudaSuccess) return cuda_fail(e);

@@ -104,9 +104,14 @@ template <class T> __device__ __forceinline__ T ld_partial_any(const T* p) { ret
 // therefore wait for that grid (and its memory) before touching inputs, and it
 // immediately allows the NEXT kernel to be scheduled into SMs its own CTAs free.
 // Without PDL both instructions are no-ops.
+#ifndef ADAPTIC_PDL_EARLY_TRIGGER
+#define ADAPTIC_PDL_EARLY_TRIGGER 0
+#endif
 __device__ __forceinline__ void pdl_prologue() {
     asm volatile("griddepcontrol.wait;" ::: "memory");
+#if ADAPTIC_PDL_EARLY_TRIGGER
     asm volatile("griddepcontrol.launch_dependents;" :::);
+#endif
 }
 
 // ---------------------------------------------------------------- TMA bulk copy + mbarrier

@@ -99,23 +99,26 @@ tmv_rowtile_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restri
             __syncthreads();
         }
         if (active) {
-            const T* bt = stg + (w0 & 3) + r;
-            const T* xt = stg + tile_w;
+            // running 32-bit smem offsets (a stage is < 256 KB): one add per row, no multiplies
+            const T* pb = stg + (w0 & 3) + r + s * R;
+            const T* px = stg + tile_w + s;
+            const int sb = nsl * R;                     // words between a thread's rows
             int c = s;
             for (; c + 3 * nsl < nc; c += 4 * nsl) {
-                acc[0] = mac(bt[int64_t(c) * R], xt[c], acc[0]);
-                acc[1] = mac(bt[int64_t(c + nsl) * R], xt[c + nsl], acc[1]);
-                acc[2] = mac(bt[int64_t(c + 2 * nsl) * R], xt[c + 2 * nsl], acc[2]);
-                acc[3] = mac(bt[int64_t(c + 3 * nsl) * R], xt[c + 3 * nsl], acc[3]);
+                acc[0] = mac(pb[0], px[0], acc[0]);
+                acc[1] = mac(pb[sb], px[nsl], acc[1]);
+                acc[2] = mac(pb[2 * sb], px[2 * nsl], acc[2]);
+                acc[3] = mac(pb[3 * sb], px[3 * nsl], acc[3]);
+                pb += 4 * sb; px += 4 * nsl;
                 if (++steps == FOLD) {
                     steps = 0;
                     outer += (acc[0] + acc[1]) + (acc[2] + acc[3]);
                     acc[0] = acc[1] = acc[2] = acc[3] = T(0);
                 }
             }
-            if (c < nc) acc[0] = mac(bt[int64_t(c) * R], xt[c], acc[0]);             // < 4 rows left
-            if (c + nsl < nc) acc[1] = mac(bt[int64_t(c + nsl) * R], xt[c + nsl], acc[1]);
-            if (c + 2 * nsl < nc) acc[2] = mac(bt[int64_t(c + 2 * nsl) * R], xt[c + 2 * nsl], acc[2]);
+            if (c < nc) acc[0] = mac(pb[0], px[0], acc[0]);                            // < 4 rows left
+            if (c + nsl < nc) acc[1] = mac(pb[sb], px[nsl], acc[1]);
+            if (c + 2 * nsl < nc) acc[2] = mac(pb[2 * sb], px[2 * nsl], acc[2]);
         }
         __syncthreads();                                // stage st fully read
         if (tid == 0 && i + stages < my_tiles) {
