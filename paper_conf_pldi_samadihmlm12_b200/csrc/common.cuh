@@ -45,6 +45,17 @@ template <class V> __device__ __forceinline__ auto vsum(const V& a) -> decltype(
     return (a.x + a.y) + (a.z + a.w);
 }
 
+// elements s .. s+3 of the 8-element concatenation (lo, hi), s in 0..3 (a funnel shift
+// of two aligned 128-bit vectors; the misaligned TMV and MV kernels)
+template <class V> __device__ __forceinline__ V funnel4(const V& lo, const V& hi, int s) {
+    V r;
+    r.x = s == 0 ? lo.x : s == 1 ? lo.y : s == 2 ? lo.z : lo.w;
+    r.y = s == 0 ? lo.y : s == 1 ? lo.z : s == 2 ? lo.w : hi.x;
+    r.z = s == 0 ? lo.z : s == 1 ? lo.w : s == 2 ? hi.x : hi.y;
+    r.w = s == 0 ? lo.w : s == 1 ? hi.x : s == 2 ? hi.y : hi.z;
+    return r;
+}
+
 // ---------------------------------------------------------------- loads
 // Matrix stream: read exactly once -> non-coherent path, no L1 allocation, and a
 // 256-byte L2 fetch granule (each warp-wide 128-bit load covers 512 contiguous

@@ -19,15 +19,6 @@
 
 namespace adaptic {
 
-// elements s .. s+3 of the 8-element concatenation (lo, hi), s in 0..3
-template <class V> __device__ __forceinline__ V funnel4(const V& lo, const V& hi, int s) {
-    V r;
-    r.x = s == 0 ? lo.x : s == 1 ? lo.y : s == 2 ? lo.z : lo.w;
-    r.y = s == 0 ? lo.y : s == 1 ? lo.z : s == 2 ? lo.w : hi.x;
-    r.z = s == 0 ? lo.z : s == 1 ? lo.w : s == 2 ? hi.x : hi.y;
-    r.w = s == 0 ? lo.w : s == 1 ? hi.x : s == 2 ? hi.y : hi.z;
-    return r;
-}
 
 // Aligned vector q of the aligned view (element e of B is element b0 + e of the view):
 // one 128-bit load when all four words lie inside B, else the words inside B one by one

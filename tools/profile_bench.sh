@@ -7,7 +7,7 @@
 set -u
 tag=${1:-r1}
 mkdir -p gpurun_out
-python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu-baseline --detail gpurun_out/detail_prof.jsonl \
+python bench.py --steps 20 --warmup 3 --no-e2e --no-cpu-baseline --detail gpurun_out/detail_prof.jsonl \
     > gpurun_out/bench_forprof.json 2> gpurun_out/bench_forprof.err
 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"mv_|tmv_" --csv \
     --log-file gpurun_out/launches_${tag}.csv \

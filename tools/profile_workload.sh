@@ -7,7 +7,7 @@
 set -u
 w=$1; n=$2; tag=${3:-r1}
 mkdir -p gpurun_out
-python bench.py --workload $w --steps 2 --warmup 3 --streams 1 --no-e2e --no-cpu-baseline \
+python bench.py --workload $w --steps 20 --warmup 3 --streams 1 --no-e2e --no-cpu-baseline \
     --detail gpurun_out/detail_${w}_${tag}.jsonl > gpurun_out/bench_${w}_forprof.json 2>/dev/null
 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"b1_|mv_|bicg_|st_direct|st_tile" --csv \
     --log-file gpurun_out/launches_${w}_${tag}.csv \
