@@ -208,6 +208,10 @@ typedef enum {
  *                      tile, [ADAPTIC_P_BLOCK] 256 / 512 / 1024 >= rows threads;
  *                      16-byte-aligned B and x, else the direct kernel.  A tile
  *                      height is capped so that two ring stages fit.
+ *                      MV (not DOT) with cols % 4 != 0, MV_SUBWARP / MV_WPR /
+ *                      MV_CPR / MV_SPLIT: 5 = x copied first (same stream, same
+ *                      call) into four shifted 16-byte-aligned copies in the
+ *                      workspace, so every row reads x with 128-bit loads.
  *   [ADAPTIC_P_BLOCK]  TMV_*: threads per CTA, 256 or 1024 (unroll <= 4 at 1024).
  *   [ADAPTIC_P_ROWS]   MV_CPR / MV_SPLIT: rows per CTA step sharing each x load,
  *                      (rows, unroll) in {(1,2),(1,4),(1,8),(2,2),(2,4),(4,2)}.

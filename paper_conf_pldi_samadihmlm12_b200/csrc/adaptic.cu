@@ -56,6 +56,7 @@ struct adaptic_plan_s {
     // workspace
     size_t ws_bytes, cnt_off;
     size_t fb_ws_off;      // staged-tile plans: the direct-kernel fallback's workspace starts here
+    size_t xsh_off;        // xmode 3 (misaligned MV): the four shifted copies of x start here
     void* ws;
     size_t ws_cap;
 };
@@ -734,6 +735,12 @@ adaptic_status derive_b1(adaptic_plan_s* p, const int32_t* params, const DevInfo
 
 adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& dev);
 
+// xmode 3: the four shifted copies of x (pitch round_up(C, 4)) after the plan's own workspace
+void add_xshift_workspace(adaptic_plan_s* p) {
+    p->xsh_off = (p->ws_bytes + 255) / 256 * 256;
+    p->ws_bytes = p->xsh_off + size_t(4) * size_t((p->C + 3) / 4 * 4) * 4;
+}
+
 // MV / DOT lane groups on TMA-staged row tiles (rowtile_kernel.cuh): MV_SUBWARP / MV_WPR
 // with [ADAPTIC_P_XSMEM] = 4.  [LANES] G (WPR: 32), [BLOCK] threads 256 | 512, [ROWS]
 // rows per tile k, [UNROLL] ring stages, [CTAS_PER_SM] resident CTAs the ring is sized
@@ -903,7 +910,10 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
         if (v == ADAPTIC_V_MV_TPR) { p->fb_lanes = G; p->fb_unroll = U; }
         else { p->lanes = G; p->unroll = U; p->rb = 8 / U; p->block = GROUP_NT; }
         const int rows_per_cta = (8 / U) * (32 / G) * (GROUP_NT / 32);
-        const int xm = (v == ADAPTIC_V_MV_TPR) ? (px ? 2 : 0) : pick_xmode(px, par(ADAPTIC_P_XSMEM), C, true);
+        const bool want_shift = v != ADAPTIC_V_MV_TPR && par(ADAPTIC_P_XSMEM) == 5;
+        if (want_shift && (px || !mis)) return ADAPTIC_ERR_UNSUPPORTED;   // shifted x: misaligned MV rows only
+        const int xm = (v == ADAPTIC_V_MV_TPR) ? (px ? 2 : 0)
+                       : want_shift ? XM_SHIFT_MODE : pick_xmode(px, par(ADAPTIC_P_XSMEM), C, true);
         if (xm < 0) return ADAPTIC_ERR_UNSUPPORTED;
         const size_t xsm = xm == 1 ? size_t((C * 4 + 15) / 16 * 16) : 0;
         int cps = par(ADAPTIC_P_CTAS_PER_SM);
@@ -924,6 +934,7 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
         }
         if (v != ADAPTIC_V_MV_TPR) {
             if (!p->path_ok[(p->vec_shape || mis) ? 1 : 0]) return ADAPTIC_ERR_UNSUPPORTED;
+            if (xm == XM_SHIFT_MODE) add_xshift_workspace(p);
             return ADAPTIC_OK;
         }
         // ---- MV_TPR proper: index 1 = the TMA-staged kernel (128-bit shared reads, or 32-bit
@@ -975,7 +986,9 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
                               (RB == 4 && U == 2);
         if (!combo_ok || (NT == 1024 && RB * U > 4)) return ADAPTIC_ERR_INVALID_ARG;
         // x staged in smem only for CPR (a split CTA reads a different x chunk per block)
-        const int xm = pick_xmode(px, par(ADAPTIC_P_XSMEM), C, v == ADAPTIC_V_MV_CPR);
+        const bool want_shift = par(ADAPTIC_P_XSMEM) == 5;
+        if (want_shift && (px || !mis)) return ADAPTIC_ERR_UNSUPPORTED;   // shifted x: misaligned MV rows only
+        const int xm = want_shift ? XM_SHIFT_MODE : pick_xmode(px, par(ADAPTIC_P_XSMEM), C, v == ADAPTIC_V_MV_CPR);
         if (xm < 0) return ADAPTIC_ERR_UNSUPPORTED;
         const size_t xsm = xm == 1 ? size_t((C * 4 + 15) / 16 * 16) : 0;
         int cps = par(ADAPTIC_P_CTAS_PER_SM);
@@ -1025,6 +1038,7 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
             p->cnt_off = part;
             p->ws_bytes = part + size_t(groups) * 4;
         }
+        if (xm == XM_SHIFT_MODE) add_xshift_workspace(p);
         return ADAPTIC_OK;
     }
 
@@ -1144,7 +1158,7 @@ adaptic_status make_plan(int op, int64_t rows, int64_t cols, int dtype, int vari
     adaptic_plan_s* p = new (std::nothrow) adaptic_plan_s();
     if (!p) return ADAPTIC_ERR_INVALID_ARG;
     p->op = op; p->dtype = dtype; p->R = rows; p->C = cols; p->sms = dev.sms; p->nvec = nvec;
-    p->ws = nullptr; p->ws_cap = 0; p->fb_ws_off = 0;
+    p->ws = nullptr; p->ws_cap = 0; p->fb_ws_off = 0; p->xsh_off = 0;
 
     if (variant != ADAPTIC_V_AUTO) {
         p->variant = variant; p->source = 0;
@@ -1280,6 +1294,27 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
     int stages = p->stages;
 
     void* args7[7];
+    if (mis && p->xmode == XM_SHIFT_MODE && p->op == ADAPTIC_OP_MV && p->nvec == 1 &&
+        p->variant >= ADAPTIC_V_MV_SUBWARP && p->variant <= ADAPTIC_V_MV_SPLIT) {
+        // shifted copies of x for the aligned 128-bit x loads (mv_mis_kernels.cuh XM_SHIFT)
+        void* xs = static_cast<char*>(p->ws) + p->xsh_off;
+        void* sfn = dt == DT_F32 ? mis_shift_fn_f32() : mis_shift_fn_i32();
+        const int64_t n4 = 4 * ((C + 3) / 4 * 4);
+        const unsigned sgrid = unsigned(std::max<int64_t>(1, std::min<int64_t>(ceil_div(n4, 256), int64_t(p->sms) * 8)));
+        void* sargs[3] = {&X, &xs, &C};
+        cudaLaunchConfig_t scfg = {};
+        scfg.gridDim = dim3(sgrid);
+        scfg.blockDim = dim3(256);
+        scfg.stream = stream;
+        cudaLaunchAttribute sattr[1];
+        sattr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+        sattr[0].val.programmaticStreamSerializationAllowed = 1;
+        scfg.attrs = sattr;
+        scfg.numAttrs = pdl_enabled() ? 1 : 0;
+        cudaError_t es = cudaLaunchKernelExC(&scfg, sfn, sargs);
+        if (es != cudaSuccess) return cuda_fail(es);
+        X = xs;
+    }
     if (p->op == ADAPTIC_OP_STENCIL5) {
         if (p->variant == ADAPTIC_V_ST_TILE && vec) {
             fn = st_tile_fn(p->rb, p->lanes);

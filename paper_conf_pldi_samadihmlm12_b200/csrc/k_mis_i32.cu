@@ -1,4 +1,5 @@
 #define KT uint32_t
 #define MIS_GROUP_FN mis_group_fn_i32
 #define MIS_CTA_FN mis_cta_fn_i32
+#define MIS_SHIFT_FN mis_shift_fn_i32
 #include "k_mis.inc"

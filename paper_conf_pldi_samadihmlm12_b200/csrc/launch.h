@@ -42,6 +42,11 @@ void* mis_group_fn_f32(int G, int U, int xmode);
 void* mis_group_fn_i32(int G, int U, int xmode);
 void* mis_cta_fn_f32(int NT, int U, int xmode);
 void* mis_cta_fn_i32(int NT, int U, int xmode);
+// x_shift_kernel (xmode 3 = XM_SHIFT): (const T* X, T* out, int64_t C), 256 threads; out holds
+// four copies of pitch round_up(C, 4), copy h = x shifted left by h elements
+void* mis_shift_fn_f32();
+void* mis_shift_fn_i32();
+constexpr int XM_SHIFT_MODE = 3;
 // Misaligned-row TMV (tmv_mis_kernel.cuh; R % 4 != 0, two aligned loads + funnel shift), NT = 256:
 //   (const T* B, const T* X, T* y, int64_t R, int64_t C, int S, T* part, unsigned* cnt)
 void* tmv_mis_fn_f32(int LR, int U);

@@ -50,6 +50,31 @@ template <int XM, class T> __device__ __forceinline__ vec4_t<T> ld_x4(const T* p
     return v;
 }
 
+// XM_SHIFT: x arrives as four shifted copies X_h[i] = x[i + h] (h = 0..3, each P =
+// round_up(C, 4) elements, 16-byte aligned; written by x_shift_kernel in the same stream
+// just before), so the x chunk of a row with head h is ONE aligned 128-bit load,
+// X_h[4v .. 4v+3] -- instead of four 32-bit loads at a misaligned offset, which made these
+// kernels L1-bound (ncu l1tex 80-87 % of peak on the C+1 shapes).  Copy 0 is x itself.
+constexpr int XM_SHIFT = 3;
+__host__ __device__ constexpr int64_t xshift_pitch(int64_t C) { return (C + 3) / 4 * 4; }
+
+template <class T>
+__global__ void __launch_bounds__(256) x_shift_kernel(const T* __restrict__ X, T* __restrict__ out, int64_t C)
+{
+    pdl_prologue();
+    const int64_t P = xshift_pitch(C);
+    for (int64_t i = int64_t(blockIdx.x) * 256 + threadIdx.x; i < 4 * P; i += int64_t(gridDim.x) * 256) {
+        const int64_t h = i / P, e = i - h * P + h;
+        out[i] = e < C ? X[e] : T(0);
+    }
+}
+
+// four consecutive x values at element offset h + 4v (the body of a row with head h)
+template <int XM, class T> __device__ __forceinline__ vec4_t<T> x_body(const T* Xs, int h, int64_t v, int64_t P) {
+    if constexpr (XM == XM_SHIFT) return ld_x(reinterpret_cast<const vec4_t<T>*>(Xs + h * P) + v);
+    else return ld_x4<XM>(Xs + h + 4 * v);
+}
+
 // ------------------------------------------------------------------ lane groups (MV_SUBWARP / MV_WPR)
 template <class T, int G, int RB, int U, int XM, int NT>
 __global__ void __launch_bounds__(NT, 2)
@@ -61,6 +86,7 @@ mv_group_mis_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restr
     constexpr int NG = 32 / G;
     constexpr bool PERROWX = (XM == XM_ROW);
     const T* __restrict__ Xs = stage_x_scalar<T, XM, NT>(X, C);
+    const int64_t P = xshift_pitch(C);
     const int lane = threadIdx.x & 31;
     const int g = lane / G, li = lane % G;
     const int64_t warp = (int64_t(blockIdx.x) * NT + threadIdx.x) >> 5;
@@ -103,7 +129,7 @@ mv_group_mis_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restr
                     const int64_t v = j0 + int64_t(G) * u;
                     a[i][u] = ld_stream(av[i] + v);
                     if constexpr (PERROWX) b[i][u] = ld_stream(bv[i] + v);
-                    else b[i][u] = ld_x4<XM>(Xs + h[i] + 4 * v);
+                    else b[i][u] = x_body<XM>(Xs, h[i], v, P);
                 }
 #pragma unroll
             for (int i = 0; i < RB; ++i)
@@ -122,7 +148,7 @@ mv_group_mis_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restr
 #pragma unroll
         for (int i = 0; i < RB; ++i) {
             for (int64_t v = j0; v < nb[i]; v += G) {     // body tail: < U vectors for this lane
-                const E b = PERROWX ? ld_stream(bv[i] + v) : ld_x4<XM>(Xs + h[i] + 4 * v);
+                const E b = PERROWX ? ld_stream(bv[i] + v) : x_body<XM>(Xs, h[i], v, P);
                 emac(acc[i][0], ld_stream(av[i] + v), b);
             }
             // scalar head [0, h) and tail [h + 4 nb, C): at most 3 + 3 elements per row
@@ -158,6 +184,7 @@ mv_cta_mis_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restric
     __shared__ T red[NT / 32];
     __shared__ unsigned int flag;
     const T* __restrict__ Xs = stage_x_scalar<T, XM, NT>(X, C);
+    const int64_t P = xshift_pitch(C);
     const int tid = threadIdx.x;
     const int64_t nblk = R * S;
 
@@ -187,7 +214,7 @@ mv_cta_mis_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restric
                 const int64_t v = b + tid + int64_t(NT) * u;
                 a[u] = ld_stream(av + v);
                 if constexpr (PERROWX) x[u] = ld_stream(bv + v);
-                else x[u] = ld_x4<XM>(Xs + h + 4 * v);
+                else x[u] = x_body<XM>(Xs, h, v, P);
             }
 #pragma unroll
             for (int u = 0; u < U; ++u) emac(acc[u], a[u], x[u]);
@@ -200,7 +227,7 @@ mv_cta_mis_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restric
         }
         const int64_t tail_end = min(end, b + BV);
         for (int64_t v = b + tid; v < tail_end; v += NT) {
-            const E x = PERROWX ? ld_stream(bv + v) : ld_x4<XM>(Xs + h + 4 * v);
+            const E x = PERROWX ? ld_stream(bv + v) : x_body<XM>(Xs, h, v, P);
             emac(acc[0], ld_stream(av + v), x);
         }
         if (s == 0) {                                    // scalar head and tail of the row

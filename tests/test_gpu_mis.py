@@ -26,7 +26,10 @@ FORCED = [("AUTO", None)] + [("MV_SUBWARP", [g, 0, 0, u]) for g in (1, 4, 16) fo
          [("MV_WPR", [0, 0, 0, u, xm]) for u in (1, 2, 4, 8) for xm in (1, 2)] + \
          [("MV_CPR", [nt, 0, 0, u, xm]) for nt, u in ((256, 2), (256, 4), (256, 8), (1024, 2), (1024, 4))
           for xm in (1, 2)] + \
-         [("MV_SPLIT", [nt, s, 0, u, 0, 0, 0, o]) for nt, u in ((256, 4), (1024, 2)) for s in (2, 5) for o in (1, 2)]
+         [("MV_SPLIT", [nt, s, 0, u, 0, 0, 0, o]) for nt, u in ((256, 4), (1024, 2)) for s in (2, 5) for o in (1, 2)] + \
+         [("MV_SUBWARP", [g, 0, 0, u, 5]) for g, u in ((1, 4), (4, 2), (16, 1))] + \
+         [("MV_WPR", [0, 0, 0, u, 5]) for u in (1, 8)] + [("MV_CPR", [256, 0, 0, 4, 5]), ("MV_CPR", [1024, 0, 0, 2, 5])] + \
+         [("MV_SPLIT", [256, s, 0, 4, 5, 0, 0, o]) for s in (2, 5) for o in (1, 2)]
 
 
 def check(y, ref, dt, what):
@@ -187,3 +190,19 @@ def test_tpr_rows_off_the_16_byte_grid(dt):
                 y = fn(torch.from_numpy(A).to(DEV), torch.from_numpy(X).to(DEV), variant="MV_TPR", params=p)
                 ref = oracle.mv(A, X) if op == "mv" else oracle.dot(A, X)
                 check(y.cpu().numpy(), ref, dt, f"tpr {op} {dt} {R}x{C} {p}")
+
+
+def test_shifted_x_copies_any_x_alignment():
+    """[ADAPTIC_P_XSMEM] = 5 (misaligned MV rows): x is first copied into four shifted,
+    16-byte-aligned copies in the workspace, so x may sit at any 4-byte offset."""
+    for R, C in [(37, 1001), (5, 100003), (3000, 77)]:
+        A = synth.matrix(R, C, "mv", np.float32, "uniform", 61 + C)
+        x = synth.vector(C, np.float32, "uniform", 62 + C)
+        Ad = torch.from_numpy(A).to(DEV)
+        for off in (0, 1, 2, 3):
+            xb = torch.zeros(C + 8, dtype=torch.float32, device=DEV)
+            xb[off:off + C] = torch.from_numpy(x).to(DEV)
+            for v, p in (("MV_WPR", [0, 0, 0, 2, 5]), ("MV_CPR", [256, 0, 0, 4, 5]),
+                         ("MV_SPLIT", [256, 3, 0, 4, 5])):
+                y = adaptic.mv(Ad, xb[off:off + C], variant=v, params=p).cpu().numpy()
+                check(y, oracle.mv(A, x), "f32", f"shift x off {off} {R}x{C} {v}")

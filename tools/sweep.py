@@ -62,6 +62,23 @@ def rowtile_grid(op, R, C):
     return out
 
 
+def shift_grid(op, R, C):
+    """Misaligned MV rows (C % 4 != 0) with x read from four shifted aligned copies (XSMEM 5)."""
+    if op != "mv" or C % 4 == 0 or C < 16:
+        return []
+    out = []
+    nv = C
+    if nv <= 256:
+        out += [("MV_SUBWARP", [g, 0, 0, u, 5]) for g in (2, 4, 8, 16) for u in (1, 2, 4) if g * u * 4 <= 2 * C]
+    if nv <= 16384:
+        out += [("MV_WPR", [0, 0, 0, u, 5]) for u in (1, 2, 4, 8) if 32 * u * 4 <= 2 * C]
+    if C >= 512:
+        out += [("MV_CPR", [nt, 0, 0, u, 5]) for nt, u in ((256, 2), (256, 4), (256, 8), (1024, 2), (1024, 4))]
+    if R <= 8192:
+        out += [("MV_SPLIT", [nt, 0, 0, u, 5, 0, 0, o]) for nt, u in ((256, 4), (256, 8), (1024, 4)) for o in (1, 2)]
+    return out
+
+
 def grids(op, R, C, dtype="f32"):
     """(variant, params) candidates; params = [lanes, splits, ctas_per_sm, unroll, xsmem, block, rows], 0 = auto."""
     out = [("AUTO", None)] + tile_grid(op, R, C, dtype) + rowtile_grid(op, R, C)
@@ -102,6 +119,7 @@ def grids(op, R, C, dtype="f32"):
             for nt, rb, u, pp in CTA_GRID:
                 for order in (1, 2):
                     out.append(("MV_SPLIT", [nt, 0, 0, u, 0, 0, rb, order, pp]))
+        out += shift_grid(op, R, C)
         if C <= 256:
             for nt in (128, 256):
                 for st in (2, 4, 8):
@@ -161,6 +179,7 @@ def main():
     ap.add_argument("--tile-only", action="store_true", help="time only the x-tile stream-K candidates (+ AUTO)")
     ap.add_argument("--rowtile-only", action="store_true", help="time only the staged row-tile candidates (+ AUTO)")
     ap.add_argument("--flat-only", action="store_true", help="time only the flat-stream TMV candidates (+ AUTO)")
+    ap.add_argument("--shift-only", action="store_true", help="time only the shifted-x MV candidates (+ AUTO)")
     a = ap.parse_args()
     dev = torch.device("cuda:0")
     tdt = torch.float32 if a.dtype == "f32" else torch.int32
@@ -198,6 +217,8 @@ def main():
                     cands = [("AUTO", None)] + tile_grid(op, R, C, a.dtype)
                 elif a.rowtile_only:
                     cands = [("AUTO", None)] + rowtile_grid(op, R, C)
+                elif a.shift_only:
+                    cands = [("AUTO", None)] + shift_grid(op, R, C)
                 elif a.flat_only:
                     cands = [("AUTO", None)] + [("TMV_REGTILE", [0, 0, 0, u]) for u in (2, 4, 8)] + \
                         rowtile_grid(op, R, C)
