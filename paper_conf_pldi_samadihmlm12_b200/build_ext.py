@@ -23,7 +23,8 @@ LIB = os.path.join(HERE, "libadaptic.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ARCH + ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O2",
-                "-Xptxas", "-warn-spills", "-I" + INCLUDE, "-I" + CSRC]
+                "-Xptxas", "-warn-spills", "-I" + INCLUDE, "-I" + CSRC] + \
+    os.environ.get("ADAPTIC_NVCC_EXTRA", "").split()        # experiments only (e.g. -DADAPTIC_REFILL_FENCE=1)
 
 
 def _deps():

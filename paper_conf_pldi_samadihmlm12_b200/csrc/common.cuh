@@ -115,6 +115,9 @@ template <class T> __device__ __forceinline__ T ld_partial_any(const T* p) { ret
 // therefore wait for that grid (and its memory) before touching inputs, and it
 // immediately allows the NEXT kernel to be scheduled into SMs its own CTAs free.
 // Without PDL both instructions are no-ops.
+#ifndef ADAPTIC_REFILL_FENCE
+#define ADAPTIC_REFILL_FENCE 1
+#endif
 #ifndef ADAPTIC_PDL_EARLY_TRIGGER
 #define ADAPTIC_PDL_EARLY_TRIGGER 0
 #endif
@@ -137,6 +140,15 @@ __device__ __forceinline__ void fence_mbar_init() {
 }
 __device__ __forceinline__ void fence_proxy_async() {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+// Before a TMA refill of a ring stage the CTA has read through the generic proxy (after a
+// __syncthreads).  A barrier alone orders the reads (CUTLASS's consumer-release pipelines issue
+// no proxy fence), and dropping the fence measured no difference (the staged kernels' ~1 us
+// per-tile cost is elsewhere), so the conservative fence stays on by default.
+__device__ __forceinline__ void refill_fence() {
+#if ADAPTIC_REFILL_FENCE
+    fence_proxy_async();
+#endif
 }
 __device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
     asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;"

@@ -127,7 +127,7 @@ mv_rowtile_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restric
         }
         __syncthreads();                                // every thread is done with stage st
         if (tid == 0 && i + stages < my_tiles) {
-            fence_proxy_async();                        // generic-proxy reads before the async refill
+            refill_fence();                        // generic-proxy reads before the async refill
             issue(i + stages);
         }
     }

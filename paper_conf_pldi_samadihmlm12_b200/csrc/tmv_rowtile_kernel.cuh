@@ -122,7 +122,7 @@ tmv_rowtile_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restri
         }
         __syncthreads();                                // stage st fully read
         if (tid == 0 && i + stages < my_tiles) {
-            fence_proxy_async();
+            refill_fence();
             issue(i + stages);
         }
     }

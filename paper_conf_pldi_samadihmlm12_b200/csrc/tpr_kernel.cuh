@@ -117,7 +117,7 @@ mv_tpr_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restrict__ 
             }
             __syncthreads();
             if (tid == 0 && i + stages < my_tiles) {
-                fence_proxy_async();
+                refill_fence();
                 issue(i + stages);
             }
             continue;
@@ -140,7 +140,7 @@ mv_tpr_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restrict__ 
         }
         __syncthreads();                      // every thread is done with stage st
         if (tid == 0 && i + stages < my_tiles) {
-            fence_proxy_async();              // generic-proxy reads before async-proxy refill
+            refill_fence();              // generic-proxy reads before async-proxy refill
             issue(i + stages);
         }
     }
