@@ -214,3 +214,32 @@ def test_tmv_rowtile_unaligned_bases_fall_back():
                            (torch.from_numpy(B).to(DEV), xb[off:off + C])):
                 y = adaptic.tmv(Bv, xv, variant="TMV_REGTILE", params=trt_params())
                 check(y.cpu().numpy(), oracle.tmv(B, x), "f32", f"tmv off {off} {R}x{C}")
+
+
+def test_batch_with_exclusive_staged_plans():
+    """adaptic_run_batch runs staged-tile plans (>= 64 KB of dynamic shared memory per CTA)
+    alone between the other lanes' work: results equal single runs bit for bit on 1..3
+    streams, with staged and direct plans interleaved."""
+    dev = torch.device(DEV)
+    stream = torch.cuda.current_stream().cuda_stream
+    cases = [("mv", 20000, 257, "MV_WPR", rt_params(32)), ("mv", 512, 3000, "AUTO", None),
+             ("tmv", 9, 300001, "TMV_REGTILE", trt_params()), ("dot", 7, 50000, "AUTO", None),
+             ("dot", 30000, 129, "MV_SUBWARP", rt_params(16)), ("tmv", 1000, 999, "AUTO", None)]
+    items, refs = [], []
+    for op, R, C, v, p in cases:
+        M = synth.matrix(R, C, "tmv" if op == "tmv" else "mv", np.float32, "uniform", 71 + R)
+        X = (synth.matrix(R, C, "mv", np.float32, "uniform", 72 + R) if op == "dot"
+             else synth.vector(C, np.float32, "uniform", 73 + C))
+        Md, Xd = torch.from_numpy(M).to(dev), torch.from_numpy(X).to(dev)
+        plan = adaptic.get_plan({"mv": L.OP_MV, "tmv": L.OP_TMV, "dot": L.OP_DOT}[op], R, C, L.F32, dev, v, p, stream)
+        y = torch.empty(R, device=dev)
+        items.append((plan, Md.data_ptr(), Xd.data_ptr(), y.data_ptr(), Md, Xd, y))
+        plan.run(Md.data_ptr(), Xd.data_ptr(), y.data_ptr(), stream)
+        refs.append(y.clone())
+    assert any(it[0].describe()["smem"] >= 64 * 1024 for it in items)
+    for k in (1, 2, 3):
+        for it in items:
+            it[6].fill_(float("nan"))
+        L.Batch([it[:4] for it in items]).run(k, stream)
+        for it, ref in zip(items, refs):
+            assert torch.equal(it[6], ref), k
