@@ -761,9 +761,10 @@ adaptic_status derive_rowtile(adaptic_plan_s* p, const int32_t* params, const De
     const int ngr = NT / G;
     const int64_t opb = int64_t(px ? 2 : 1) * 4;             // staged bytes per element
     int64_t k = par(ADAPTIC_P_ROWS);
-    if (k <= 0) {          // 0: ~24 KB of matrix per tile; -n: ~n KB (fitted tables); whole warps of rows
-        const int64_t kb = k < 0 ? -k : 24;
-        k = std::max<int64_t>(1, (kb * 1024) / (C * opb));
+    if (k < 0) {           // -n: the rows of ~n KB (fitted tables store a size; the sweep's height)
+        k = std::max<int64_t>(1, (int64_t(-k) * 1024) / (C * opb));
+    } else if (k == 0) {   // ~24 KB of matrix per tile, whole warps of rows
+        k = std::max<int64_t>(1, (24 * 1024) / (C * opb));
         if (k >= ngr) k = k / ngr * ngr;
     }
     k = std::min<int64_t>(k, std::max<int64_t>(1, R));
@@ -807,7 +808,8 @@ adaptic_status derive_tmv_rowtile(adaptic_plan_s* p, const int32_t* params, cons
     if (R > 1024) return ADAPTIC_ERR_UNSUPPORTED;
     int NT = par(ADAPTIC_P_BLOCK);
     if (NT <= 0) NT = R <= 64 ? 256 : 1024;
-    if ((NT != 256 && NT != 512 && NT != 1024) || R > NT) return ADAPTIC_ERR_INVALID_ARG;
+    if ((NT != 256 && NT != 512 && NT != 1024) || R > 2 * NT || (R > NT && NT == 1024)) return ADAPTIC_ERR_INVALID_ARG;
+    const int rpt = R > NT ? 2 : 1;                            // outputs per thread
     int cps = par(ADAPTIC_P_CTAS_PER_SM);
     if (cps <= 0) cps = 1024 / NT;
     int64_t k = par(ADAPTIC_P_ROWS);
@@ -829,14 +831,14 @@ adaptic_status derive_tmv_rowtile(adaptic_plan_s* p, const int32_t* params, cons
     if (par(ADAPTIC_P_UNROLL) > 0) stages = std::min(stages, par(ADAPTIC_P_UNROLL));
     if (stages < 2) return ADAPTIC_ERR_UNSUPPORTED;
     p->smem = size_t(stages) * stage_bytes;
-    void* fn = tmv_rowtile_fn(p->dtype, NT);
+    void* fn = tmv_rowtile_fn(p->dtype, NT, rpt);
     const int occ = occupancy(fn, NT, p->smem, dev.present, cps);
     if (occ < 1) return ADAPTIC_ERR_UNSUPPORTED;
     p->ctas_per_sm = std::min(cps, occ);
     const int64_t ntiles = ceil_div(C, k);
     const int64_t G = std::max<int64_t>(1, std::min<int64_t>(ntiles, int64_t(dev.sms) * p->ctas_per_sm));
-    const int64_t nsl = NT / R;
-    p->lanes = int(R); p->block = NT; p->rb = int(k); p->stages = stages; p->unroll = stages;
+    const int64_t nsl = int64_t(NT) * rpt / R;
+    p->lanes = int(R); p->block = NT; p->rb = int(k); p->stages = stages; p->unroll = rpt;
     p->xmode = 4; p->splits = 1; p->mis = !p->vec_shape;
     p->grid[1] = G;
     const int64_t rows_per_thread = ceil_div(ceil_div(ntiles, G) * k, nsl);
@@ -1415,7 +1417,7 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
             break;
         default:
             if (p->xmode == 4) {                          // TMV on staged tiles of B
-                fn = tmv_rowtile_fn(dt, p->block);
+                fn = tmv_rowtile_fn(dt, p->block, p->unroll);
                 smem = p->smem;
                 args9[0] = &A; args9[1] = &X; args9[2] = &y; args9[3] = &R; args9[4] = &C;
                 args9[5] = &tile_mb; args9[6] = &stages; args9[7] = &part; args9[8] = &cnt;

@@ -39,16 +39,20 @@ size_t rowtile_tile_words(int64_t k, int64_t C) { return size_t((k * C + 6 + 3) 
 }  // namespace adaptic
 
 namespace adaptic {
-// TMV on staged tiles of B (tmv_rowtile_kernel.cuh): 256, 512 or 1024 threads
-void* tmv_rowtile_fn(int dtype, int NT) {
-    switch (NT) {
-        case 256: return dtype == DT_F32 ? reinterpret_cast<void*>(&tmv_rowtile_kernel<float, 256>)
-                                         : reinterpret_cast<void*>(&tmv_rowtile_kernel<uint32_t, 256>);
-        case 512: return dtype == DT_F32 ? reinterpret_cast<void*>(&tmv_rowtile_kernel<float, 512>)
-                                         : reinterpret_cast<void*>(&tmv_rowtile_kernel<uint32_t, 512>);
-        case 1024: return dtype == DT_F32 ? reinterpret_cast<void*>(&tmv_rowtile_kernel<float, 1024>)
-                                          : reinterpret_cast<void*>(&tmv_rowtile_kernel<uint32_t, 1024>);
+// TMV on staged tiles of B (tmv_rowtile_kernel.cuh): 256, 512 or 1024 threads, one or two
+// outputs per thread (rpt = 2 for NT < R <= 2 NT)
+template <class T>
+static void* trt(int NT, int rpt) {
+    switch (NT * 4 + rpt) {
+        case 256 * 4 + 1: return reinterpret_cast<void*>(&tmv_rowtile_kernel<T, 256, 1>);
+        case 512 * 4 + 1: return reinterpret_cast<void*>(&tmv_rowtile_kernel<T, 512, 1>);
+        case 1024 * 4 + 1: return reinterpret_cast<void*>(&tmv_rowtile_kernel<T, 1024, 1>);
+        case 256 * 4 + 2: return reinterpret_cast<void*>(&tmv_rowtile_kernel<T, 256, 2>);
+        case 512 * 4 + 2: return reinterpret_cast<void*>(&tmv_rowtile_kernel<T, 512, 2>);
         default: return nullptr;
     }
+}
+void* tmv_rowtile_fn(int dtype, int NT, int rpt) {
+    return dtype == DT_F32 ? trt<float>(NT, rpt) : trt<uint32_t>(NT, rpt);
 }
 }  // namespace adaptic

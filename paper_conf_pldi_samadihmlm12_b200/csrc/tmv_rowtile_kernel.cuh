@@ -29,7 +29,7 @@ namespace adaptic {
 constexpr int TRT_MAX_STAGES = 8;
 constexpr int TRT_GROUP = 16;       // CTAs per first-level merge group
 
-template <class T, int NT>
+template <class T, int NT, int RPT>
 __global__ void __launch_bounds__(NT)
 tmv_rowtile_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restrict__ y,
                    int64_t R64, int64_t C, int k, int stages,
@@ -38,15 +38,21 @@ tmv_rowtile_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restri
     pdl_prologue();
     extern __shared__ __align__(128) unsigned char smem_raw[];
     __shared__ __align__(8) uint64_t full[TRT_MAX_STAGES];
-    __shared__ T P[NT];
+    constexpr int VT = NT * RPT;                        // virtual threads: tid + j NT, j < RPT
+    __shared__ T P[VT];
     __shared__ unsigned int flag;
 
     const int R = int(R64);
-    const int nsl = NT / R;                             // row slices (R <= NT)
+    const int nsl = VT / R;                             // row slices (R <= VT)
     const int NTa = nsl * R;
     const int tid = threadIdx.x;
-    const int r = tid % R, s = tid / R;
-    const bool active = tid < NTa;
+    int rj[RPT], sj[RPT];
+    bool act[RPT];
+#pragma unroll
+    for (int j = 0; j < RPT; ++j) {
+        const int vt = tid + j * NT;
+        rj[j] = vt % R; sj[j] = vt / R; act[j] = vt < NTa;
+    }
     const int64_t total = R64 * C;
     const int64_t ntiles = (C + k - 1) / k;
     const int64_t tile_w = ((int64_t(k) * R + 6 + 3) / 4) * 4;   // B words per stage (16-byte multiple)
@@ -80,9 +86,12 @@ tmv_rowtile_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restri
         for (int64_t i = 0; i < pre; ++i) issue(i);
     }
 
-    T acc[4] = {T(0), T(0), T(0), T(0)};
-    T outer = T(0);
-    int steps = 0;
+    T acc[RPT][4], outer[RPT];
+#pragma unroll
+    for (int j = 0; j < RPT; ++j) { acc[j][0] = acc[j][1] = acc[j][2] = acc[j][3] = T(0); outer[j] = T(0); }
+    int steps[RPT];
+#pragma unroll
+    for (int j = 0; j < RPT; ++j) steps[j] = 0;
     for (int64_t i = 0; i < my_tiles; ++i) {
         const int st = int(i % stages);
         const int64_t c0 = (blockIdx.x + i * gridDim.x) * int64_t(k);
@@ -98,27 +107,30 @@ tmv_rowtile_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restri
             for (int c = (nc & ~3) + tid; c < nc; c += NT) stg[tile_w + c] = X[c0 + c];
             __syncthreads();
         }
-        if (active) {
+#pragma unroll
+        for (int j = 0; j < RPT; ++j) {
+            if (!act[j]) continue;
             // running 32-bit smem offsets (a stage is < 256 KB): one add per row, no multiplies
-            const T* pb = stg + (w0 & 3) + r + s * R;
-            const T* px = stg + tile_w + s;
+            const T* pb = stg + (w0 & 3) + rj[j] + sj[j] * R;
+            const T* px = stg + tile_w + sj[j];
             const int sb = nsl * R;                     // words between a thread's rows
-            int c = s;
+            T* a = acc[j];
+            int c = sj[j];
             for (; c + 3 * nsl < nc; c += 4 * nsl) {
-                acc[0] = mac(pb[0], px[0], acc[0]);
-                acc[1] = mac(pb[sb], px[nsl], acc[1]);
-                acc[2] = mac(pb[2 * sb], px[2 * nsl], acc[2]);
-                acc[3] = mac(pb[3 * sb], px[3 * nsl], acc[3]);
+                a[0] = mac(pb[0], px[0], a[0]);
+                a[1] = mac(pb[sb], px[nsl], a[1]);
+                a[2] = mac(pb[2 * sb], px[2 * nsl], a[2]);
+                a[3] = mac(pb[3 * sb], px[3 * nsl], a[3]);
                 pb += 4 * sb; px += 4 * nsl;
-                if (++steps == FOLD) {
-                    steps = 0;
-                    outer += (acc[0] + acc[1]) + (acc[2] + acc[3]);
-                    acc[0] = acc[1] = acc[2] = acc[3] = T(0);
+                if (++steps[j] == FOLD) {
+                    steps[j] = 0;
+                    outer[j] += (a[0] + a[1]) + (a[2] + a[3]);
+                    a[0] = a[1] = a[2] = a[3] = T(0);
                 }
             }
-            if (c < nc) acc[0] = mac(pb[0], px[0], acc[0]);                            // < 4 rows left
-            if (c + nsl < nc) acc[1] = mac(pb[sb], px[nsl], acc[1]);
-            if (c + 2 * nsl < nc) acc[2] = mac(pb[2 * sb], px[2 * nsl], acc[2]);
+            if (c < nc) a[0] = mac(pb[0], px[0], a[0]);                                // < 4 rows left
+            if (c + nsl < nc) a[1] = mac(pb[sb], px[nsl], a[1]);
+            if (c + 2 * nsl < nc) a[2] = mac(pb[2 * sb], px[2 * nsl], a[2]);
         }
         __syncthreads();                                // stage st fully read
         if (tid == 0 && i + stages < my_tiles) {
@@ -128,12 +140,14 @@ tmv_rowtile_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restri
     }
 
     // slices of this CTA -> one partial per output, in slice order
-    P[tid] = active ? outer + ((acc[0] + acc[1]) + (acc[2] + acc[3])) : T(0);
+#pragma unroll
+    for (int j = 0; j < RPT; ++j)
+        P[tid + j * NT] = act[j] ? outer[j] + ((acc[j][0] + acc[j][1]) + (acc[j][2] + acc[j][3])) : T(0);
     __syncthreads();
-    if (tid < R) {
+    for (int rr = tid; rr < R; rr += NT) {
         T v = T(0);
-        for (int q = 0; q < nsl; ++q) v += P[q * R + tid];
-        ws_part[int64_t(blockIdx.x) * R + tid] = v;
+        for (int q = 0; q < nsl; ++q) v += P[q * R + rr];
+        ws_part[int64_t(blockIdx.x) * R + rr] = v;
     }
     // Two-level merge (fixed order at both levels): the last CTA of each group of
     // TRT_GROUP consecutive CTAs sums the group's partials, the last group finisher sums
@@ -141,26 +155,38 @@ tmv_rowtile_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restri
     // n partials of R values at src -> P[0 .. R) (thread (r, q) sums rows q, q + nsl, ...
     // eight loads in flight, then the nsl sums per output in q order)
     auto merge = [&](const T* src, int n) {
-        T v = T(0);
-        if (active) {
-            int g = s;
+        T v[RPT];
+#pragma unroll
+        for (int j = 0; j < RPT; ++j) {
+            v[j] = T(0);
+            if (!act[j]) continue;
+            int g = sj[j];
             for (; g + 7 * nsl < n; g += 8 * nsl) {
                 T p[8];
 #pragma unroll
-                for (int u = 0; u < 8; ++u) p[u] = ld_partial(src + int64_t(g + u * nsl) * R + r);
+                for (int u = 0; u < 8; ++u) p[u] = ld_partial(src + int64_t(g + u * nsl) * R + rj[j]);
 #pragma unroll
-                for (int u = 0; u < 8; ++u) v += p[u];
+                for (int u = 0; u < 8; ++u) v[j] += p[u];
             }
-            for (; g < n; g += nsl) v += ld_partial(src + int64_t(g) * R + r);
+            for (; g < n; g += nsl) v[j] += ld_partial(src + int64_t(g) * R + rj[j]);
         }
         __syncthreads();
-        P[tid] = v;
+#pragma unroll
+        for (int j = 0; j < RPT; ++j) P[tid + j * NT] = v[j];
         __syncthreads();
-        if (tid < R) {
-            T tot = T(0);
-            for (int q = 0; q < nsl; ++q) tot += P[q * R + tid];
-            P[tid] = tot;       // only thread tid reads it back
+        T tot[RPT];
+#pragma unroll
+        for (int j = 0; j < RPT; ++j) {
+            tot[j] = T(0);
+            const int rr = tid + j * NT;
+            if (rr < R)
+                for (int q = 0; q < nsl; ++q) tot[j] += P[q * R + rr];
         }
+        __syncthreads();
+#pragma unroll
+        for (int j = 0; j < RPT; ++j)
+            if (tid + j * NT < R) P[tid + j * NT] = tot[j];   // output rr's total at P[rr]
+        __syncthreads();
     };
     const int G = int(gridDim.x);
     const int ngroups = (G + TRT_GROUP - 1) / TRT_GROUP;
@@ -169,10 +195,10 @@ tmv_rowtile_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restri
     T* gpart = ws_part + int64_t(G) * R;                // group partials: ngroups x R
     if (ticket_is_last(ws_cnt + 1 + grp, unsigned(gsz), &flag)) {
         merge(ws_part + int64_t(grp) * TRT_GROUP * R, gsz);
-        if (tid < R) gpart[int64_t(grp) * R + tid] = P[tid];
+        for (int rr = tid; rr < R; rr += NT) gpart[int64_t(grp) * R + rr] = P[rr];
         if (ticket_is_last(ws_cnt, unsigned(ngroups), &flag)) {
             merge(gpart, ngroups);
-            if (tid < R) y[tid] = P[tid];
+            for (int rr = tid; rr < R; rr += NT) y[rr] = P[rr];
         }
     }
 }

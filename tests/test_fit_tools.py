@@ -19,11 +19,11 @@ def run(op, R, C, variant, params, gbps, grid=100, vec=False, mis=True, req=None
 
 
 def test_staged_tile_height_becomes_a_size():
-    # 47 rows of 257 words = 47 KB -> -48 KB (rounded to 4 KB); DOT stages two operands
+    # 47 rows of 257 words = 47.2 KB -> -48 KB (whole KB, rounded up); DOT stages two operands
     assert ft.norm_params(run("mv", 262144, 257, "MV_SUBWARP", [16, 0, 0, 0, 4, 256, 47], 1))[6] == -48
-    assert ft.norm_params(run("dot", 262144, 257, "MV_SUBWARP", [16, 0, 0, 0, 4, 256, 47], 1))[6] == -96
+    assert ft.norm_params(run("dot", 262144, 257, "MV_SUBWARP", [16, 0, 0, 0, 4, 256, 47], 1))[6] == -95
     # TMV: rows of B plus their x value
-    assert ft.norm_params(run("tmv", 9, 8388608, "TMV_REGTILE", [0, 0, 0, 0, 4, 512, 1364], 1))[6] == -52
+    assert ft.norm_params(run("tmv", 9, 8388608, "TMV_REGTILE", [0, 0, 0, 0, 4, 512, 1364], 1))[6] == -54
     # other plans keep their parameters
     assert ft.norm_params(run("mv", 8192, 8192, "MV_CPR", [256, 0, 0, 4, 1], 1))[:5] == [256, 0, 0, 4, 1]
 

@@ -88,8 +88,10 @@ def test_staged_tmv_tiles():
     assert p["xmode"] == 4 and p["block"] == 256 and p["rows_per_group"] % 4 == 0 and p["stages"] >= 3
     assert p["workspace_bytes"] > 0 and p["path_ok"][1]
     assert d("tmv", 513, 131072, variant="TMV_REGTILE", params=[0, 0, 0, 0, 4])["block"] == 1024
-    with pytest.raises(adaptic.AdapticError):                          # more outputs than threads
-        d("tmv", 300, 1000, variant="TMV_REGTILE", params=[0, 0, 0, 0, 4, 256])
+    two = d("tmv", 300, 1000, variant="TMV_REGTILE", params=[0, 0, 0, 0, 4, 256])
+    assert two["block"] == 256 and two["unroll"] == 2                  # two outputs per thread
+    with pytest.raises(adaptic.AdapticError):                          # more than 2 outputs per thread
+        d("tmv", 600, 1000, variant="TMV_REGTILE", params=[0, 0, 0, 0, 4, 256])
     with pytest.raises(adaptic.AdapticError):                          # R > 1024
         d("tmv", 1025, 1000, variant="TMV_REGTILE", params=[0, 0, 0, 0, 4])
     with pytest.raises(adaptic.AdapticError):                          # tile height not a multiple of 4

@@ -45,7 +45,7 @@ def rowtile_grid(op, R, C):
     if op == "tmv":
         if R > 1024:
             return []
-        return [("TMV_REGTILE", [0, 0, 0, 0, 4, nt, k]) for nt in (256, 512, 1024) if nt >= R
+        return [("TMV_REGTILE", [0, 0, 0, 0, 4, nt, k]) for nt in (256, 512, 1024) if 2 * nt >= R and (nt < 1024 or nt >= R)
                 for k in sorted({0, max(4, 12 * 1024 // (4 * R) // 4 * 4), max(4, 48 * 1024 // (4 * R) // 4 * 4)})]
     if op not in ("mv", "dot") or C > 1024:
         return []
