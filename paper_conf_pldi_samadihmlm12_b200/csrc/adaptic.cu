@@ -805,11 +805,12 @@ adaptic_status derive_rowtile(adaptic_plan_s* p, const int32_t* params, const De
 adaptic_status derive_tmv_rowtile(adaptic_plan_s* p, const int32_t* params, const DevInfo& dev) {
     auto par = [&](int i) -> int { return params ? params[i] : 0; };
     const int64_t R = p->R, C = p->C;
-    if (R > 1024) return ADAPTIC_ERR_UNSUPPORTED;
+    if (R > 4096) return ADAPTIC_ERR_UNSUPPORTED;
     int NT = par(ADAPTIC_P_BLOCK);
-    if (NT <= 0) NT = R <= 64 ? 256 : 1024;
-    if ((NT != 256 && NT != 512 && NT != 1024) || R > 2 * NT || (R > NT && NT == 1024)) return ADAPTIC_ERR_INVALID_ARG;
-    const int rpt = R > NT ? 2 : 1;                            // outputs per thread
+    if (NT <= 0) NT = R <= 64 ? 256 : R <= 1024 ? 1024 : 1024;
+    if (NT != 256 && NT != 512 && NT != 1024) return ADAPTIC_ERR_INVALID_ARG;
+    const int rpt = R <= NT ? 1 : R <= 2 * NT ? 2 : R <= 4 * NT ? 4 : 0;   // outputs per thread
+    if (rpt == 0 || !tmv_rowtile_fn(p->dtype, NT, rpt)) return ADAPTIC_ERR_INVALID_ARG;
     int cps = par(ADAPTIC_P_CTAS_PER_SM);
     if (cps <= 0) cps = 1024 / NT;
     int64_t k = par(ADAPTIC_P_ROWS);

@@ -39,8 +39,8 @@ size_t rowtile_tile_words(int64_t k, int64_t C) { return size_t((k * C + 6 + 3) 
 }  // namespace adaptic
 
 namespace adaptic {
-// TMV on staged tiles of B (tmv_rowtile_kernel.cuh): 256, 512 or 1024 threads, one or two
-// outputs per thread (rpt = 2 for NT < R <= 2 NT)
+// TMV on staged tiles of B (tmv_rowtile_kernel.cuh): 256, 512 or 1024 threads, 1, 2 or 4
+// outputs per thread (rpt = the power of two >= R / NT)
 template <class T>
 static void* trt(int NT, int rpt) {
     switch (NT * 4 + rpt) {
@@ -49,6 +49,9 @@ static void* trt(int NT, int rpt) {
         case 1024 * 4 + 1: return reinterpret_cast<void*>(&tmv_rowtile_kernel<T, 1024, 1>);
         case 256 * 4 + 2: return reinterpret_cast<void*>(&tmv_rowtile_kernel<T, 256, 2>);
         case 512 * 4 + 2: return reinterpret_cast<void*>(&tmv_rowtile_kernel<T, 512, 2>);
+        case 1024 * 4 + 2: return reinterpret_cast<void*>(&tmv_rowtile_kernel<T, 1024, 2>);
+        case 512 * 4 + 4: return reinterpret_cast<void*>(&tmv_rowtile_kernel<T, 512, 4>);
+        case 1024 * 4 + 4: return reinterpret_cast<void*>(&tmv_rowtile_kernel<T, 1024, 4>);
         default: return nullptr;
     }
 }

@@ -68,7 +68,7 @@ size_t rowtile_tile_words(int64_t k, int64_t C);
 // TMV with R <= NT outputs on staged tiles of B (tmv_rowtile_kernel.cuh; TMV_REGTILE with
 // [ADAPTIC_P_XSMEM] = 4), 16-byte-aligned B and x, k % 4 == 0, NT in {256, 512, 1024}:
 //   (const T* B, const T* X, T* y, int64_t R, int64_t C, int k, int stages, T* part, unsigned* cnt)
-void* tmv_rowtile_fn(int dtype, int NT, int rpt);   // rpt = ceil(R / NT) in {1, 2}
+void* tmv_rowtile_fn(int dtype, int NT, int rpt);   // rpt: power of two >= R / NT, in {1, 2, 4}
 
 // Multi-vector MV / TMV (mmv_kernels.cuh), fp32, K in {2, 4, 8}; X is K x C, Y is K x R:
 //   group: (const float* A, const float* X, float* Y, int64_t R, int64_t C), rows of <= G*U vectors

@@ -92,8 +92,10 @@ def test_staged_tmv_tiles():
     assert two["block"] == 256 and two["unroll"] == 2                  # two outputs per thread
     with pytest.raises(adaptic.AdapticError):                          # more than 2 outputs per thread
         d("tmv", 600, 1000, variant="TMV_REGTILE", params=[0, 0, 0, 0, 4, 256])
-    with pytest.raises(adaptic.AdapticError):                          # R > 1024
-        d("tmv", 1025, 1000, variant="TMV_REGTILE", params=[0, 0, 0, 0, 4])
+    four = d("tmv", 4000, 1000, variant="TMV_REGTILE", params=[0, 0, 0, 0, 4])
+    assert four["block"] == 1024 and four["unroll"] == 4               # four outputs per thread
+    with pytest.raises(adaptic.AdapticError):                          # R > 4096
+        d("tmv", 4097, 1000, variant="TMV_REGTILE", params=[0, 0, 0, 0, 4])
     with pytest.raises(adaptic.AdapticError):                          # tile height not a multiple of 4
         d("tmv", 9, 1000, variant="TMV_REGTILE", params=[0, 0, 0, 0, 4, 256, 6])
     for R, C in ((9, 8388608), (129, 524288), (14, 5162220)):

@@ -43,9 +43,10 @@ def rowtile_grid(op, R, C):
     """Lane groups on TMA-staged row tiles (XSMEM 4; MV/DOT, C <= 32*G): lanes per row G,
     threads per CTA and tile height (rows per ~12 / 24 (auto) / 48 KB of staged data)."""
     if op == "tmv":
-        if R > 1024:
+        if R > 4096:
             return []
-        return [("TMV_REGTILE", [0, 0, 0, 0, 4, nt, k]) for nt in (256, 512, 1024) if 2 * nt >= R and (nt < 1024 or nt >= R)
+        ok = lambda nt: R <= nt or (R <= 2 * nt and nt >= 256) or (R <= 4 * nt and nt >= 512)  # noqa: E731
+        return [("TMV_REGTILE", [0, 0, 0, 0, 4, nt, k]) for nt in (256, 512, 1024) if ok(nt)
                 for k in sorted({0, max(4, 12 * 1024 // (4 * R) // 4 * 4), max(4, 48 * 1024 // (4 * R) // 4 * 4)})]
     if op not in ("mv", "dot") or C > 1024:
         return []
