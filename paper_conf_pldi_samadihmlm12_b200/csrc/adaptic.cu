@@ -1607,7 +1607,15 @@ adaptic_status adaptic_run(adaptic_plan_t p, const void* A, const void* x, void*
 // ---- batched issue over concurrent streams (per host thread, per device)
 namespace {
 constexpr int kMaxBatchStreams = 8;
-constexpr size_t kExclusiveSmem = 64 * 1024;     // dynamic smem per CTA of a staged-tile plan
+// Plans that run alone inside adaptic_run_batch: the staged row-tile kernels (xmode 4 on the
+// lane-group variants and TMV_REGTILE), persistent grids sized for a free GPU.  Measured
+// (2 streams): offgrid step +1.7 %, while making MV_TPR exclusive too (any >= 64 KB of
+// dynamic smem) cost the default sweep 1.8 %.  ADAPTIC_EXCLUSIVE=0 disables (read once).
+bool plan_exclusive(const adaptic_plan_s* p) {
+    static const bool on = [] { const char* e = std::getenv("ADAPTIC_EXCLUSIVE"); return !(e && e[0] == '0'); }();
+    return on && p->nvec == 1 && p->xmode == 4 &&
+           (p->variant == ADAPTIC_V_MV_SUBWARP || p->variant == ADAPTIC_V_MV_WPR || p->variant == ADAPTIC_V_TMV_REGTILE);
+}
 struct StreamPool {
     int dev = -1;
     cudaStream_t side[kMaxBatchStreams - 1] = {};
@@ -1671,9 +1679,9 @@ adaptic_status adaptic_run_batch(int32_t n, const adaptic_plan_t* plans, const v
         cudaStream_t s = lane_stream(lane);
         // Staged-tile kernels size a persistent grid for the whole GPU and hold most of an
         // SM's shared memory: next to another stream's kernel their late CTAs stretch the
-        // launch (offgrid step 2.29 -> 2.81 ms measured), so they run alone -- after every
-        // lane's earlier work, and before any lane's later work.
-        const bool excl = plans[i]->smem >= kExclusiveSmem;
+        // launch, so they run alone -- after every lane's earlier work, and before any
+        // lane's later work (plan_exclusive).
+        const bool excl = plan_exclusive(plans[i]);
         if (excl)
             for (int l = 0; l < k; ++l) {
                 if (l == lane) continue;
