@@ -828,7 +828,7 @@ adaptic_status derive_tmv_rowtile(adaptic_plan_s* p, const int32_t* params, cons
     k = std::min(k, kmax2);
     const size_t stage_bytes = (rowtile_tile_words(k, R) + size_t(k)) * 4;
     if (stage_bytes > 200 * 1024) return ADAPTIC_ERR_UNSUPPORTED;
-    int stages = int(std::min<size_t>(8, (size_t(220) * 1024 / size_t(cps)) / stage_bytes));
+    int stages = int(std::min<size_t>(RT_MAX_STAGES_H, (size_t(220) * 1024 / size_t(cps)) / stage_bytes));
     if (par(ADAPTIC_P_UNROLL) > 0) stages = std::min(stages, par(ADAPTIC_P_UNROLL));
     if (stages < 2) return ADAPTIC_ERR_UNSUPPORTED;
     p->smem = size_t(stages) * stage_bytes;

@@ -6,6 +6,10 @@
 
 namespace adaptic {
 
+// the planner (adaptic.cu) sizes rings with the launch.h constants
+static_assert(RT_MAX_STAGES == RT_MAX_STAGES_H, "row-tile ring depth: kernel vs planner");
+static_assert(TRT_MAX_STAGES == RT_MAX_STAGES_H, "TMV tile ring depth: kernel vs planner");
+
 template <class T, int NT, bool PX>
 static void* rt_g(int G) {
     switch (G) {

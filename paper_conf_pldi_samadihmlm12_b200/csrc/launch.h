@@ -62,7 +62,7 @@ void* tmv_flat_fn(int dtype, int U, int NT);
 // [ADAPTIC_P_XSMEM] = 4), C <= 32*G, 16-byte-aligned A (and DOT's b), NT in {256, 512}:
 //   (const T* A, const T* X, T* y, int64_t R, int64_t C, int k, int stages)   [dynamic smem]
 constexpr int RT_MAX_C_PER_LANE = 32;
-constexpr int RT_MAX_STAGES_H = 8;          // == RT_MAX_STAGES (mbarriers per CTA)
+constexpr int RT_MAX_STAGES_H = 8;          // == RT_MAX_STAGES, TRT_MAX_STAGES (mbarriers per CTA; static_assert in k_rowtile.cu)
 void* rowtile_fn(int dtype, int NT, int G, bool px);
 size_t rowtile_tile_words(int64_t k, int64_t C);
 // TMV with R <= NT outputs on staged tiles of B (tmv_rowtile_kernel.cuh; TMV_REGTILE with
