@@ -163,6 +163,14 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
         "@!p bra WAIT_%=;\n"
         "}\n" :: "r"(smem_u32(bar)), "r"(parity) : "memory");
 }
+// Ring position of a staged pipeline, advanced once per tile: the stage index and the
+// mbarrier parity to wait for.  (Deriving them as i % stages and i / stages with a 64-bit
+// tile counter costs two software 64-bit divisions per thread per tile -- ~1 us per tile
+// per CTA measured on the staged kernels, the whole time of a small tile.)
+__device__ __forceinline__ void ring_advance(int& st, uint32_t& ph, int stages) {
+    if (++st == stages) { st = 0; ph ^= 1u; }
+}
+
 // 1-D bulk copy global -> shared, completion counted on the mbarrier (TMA engine;
 // SASS UBLKCP).  dst, src 16-byte aligned; bytes a multiple of 16.
 __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {

@@ -58,16 +58,16 @@ mv_rowtile_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restric
     }
     __syncthreads();
 
-    // local tile i -> stage i % stages (thread 0 only)
-    auto issue = [&](int64_t i) {
+    // local tile i -> ring stage `slot` (thread 0 only)
+    auto issue = [&](int64_t i, int slot) {
         const int64_t r0 = (blockIdx.x + i * gridDim.x) * int64_t(k);
         const int64_t w0 = r0 * C, w1 = min(R, r0 + k) * C;
         const int64_t a0 = w0 & ~int64_t(3);
         int64_t a1 = (w1 + 3) & ~int64_t(3);
         if (a1 > total) a1 = w1 & ~int64_t(3);          // last tile: never read past the matrix
         const uint32_t bytes = uint32_t((a1 - a0) * int64_t(sizeof(T)));
-        T* dst = ring + (i % stages) * stage_w;
-        uint64_t* bar = &full[i % stages];
+        T* dst = ring + slot * stage_w;
+        uint64_t* bar = &full[slot];
         mbar_arrive_expect_tx(bar, PERROWX ? 2 * bytes : bytes);
         if (bytes) {
             bulk_g2s(dst, A + a0, bytes, bar);
@@ -77,7 +77,7 @@ mv_rowtile_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restric
 
     if (tid == 0) {
         const int64_t pre = min(int64_t(stages), my_tiles);
-        for (int64_t i = 0; i < pre; ++i) issue(i);
+        for (int64_t i = 0; i < pre; ++i) issue(i, int(i));
     }
 
     // x slice of this lane, kept in registers across all rows (MV only)
@@ -90,14 +90,15 @@ mv_rowtile_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restric
         }
     }
 
-    for (int64_t i = 0; i < my_tiles; ++i) {
-        const int st = int(i % stages);
+    int st = 0;
+    uint32_t ph = 0;
+    for (int64_t i = 0; i < my_tiles; ++i, ring_advance(st, ph, stages)) {
         const int64_t r0 = (blockIdx.x + i * gridDim.x) * int64_t(k);
         const int nrows = int(min(int64_t(k), R - r0));
         const int64_t w0 = r0 * C;
         const int head = int(w0 & 3);
         T* stg = ring + st * stage_w;
-        mbar_wait(&full[st], uint32_t((i / stages) & 1));
+        mbar_wait(&full[st], ph);
         const int64_t w1 = w0 + int64_t(nrows) * C;
         if (((w1 + 3) & ~int64_t(3)) > total && (w1 & 3)) {  // the matrix's last < 4 words
             const int64_t a0 = w0 & ~int64_t(3);
@@ -128,7 +129,7 @@ mv_rowtile_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restric
         __syncthreads();                                // every thread is done with stage st
         if (tid == 0 && i + stages < my_tiles) {
             refill_fence();                        // generic-proxy reads before the async refill
-            issue(i + stages);
+            issue(i + stages, st);
         }
     }
 }

@@ -66,7 +66,7 @@ tmv_rowtile_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restri
     }
     __syncthreads();
 
-    auto issue = [&](int64_t i) {                       // thread 0 only
+    auto issue = [&](int64_t i, int slot) {             // thread 0 only; tile i -> ring stage slot
         const int64_t c0 = (blockIdx.x + i * gridDim.x) * int64_t(k);
         const int64_t nc = min(int64_t(k), C - c0);
         const int64_t w0 = c0 * R64, w1 = (c0 + nc) * R64;
@@ -75,15 +75,15 @@ tmv_rowtile_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restri
         if (a1 > total) a1 = w1 & ~int64_t(3);          // last tile: never read past B
         const uint32_t bb = uint32_t((a1 - a0) * int64_t(sizeof(T)));
         const uint32_t xb = uint32_t((nc & ~int64_t(3)) * int64_t(sizeof(T)));
-        T* dst = ring + (i % stages) * stage_w;
-        uint64_t* bar = &full[i % stages];
+        T* dst = ring + slot * stage_w;
+        uint64_t* bar = &full[slot];
         mbar_arrive_expect_tx(bar, bb + xb);
         if (bb) bulk_g2s(dst, B + a0, bb, bar);
         if (xb) bulk_g2s_keep(dst + tile_w, X + c0, xb, bar);
     };
     if (tid == 0) {
         const int64_t pre = min(int64_t(stages), my_tiles);
-        for (int64_t i = 0; i < pre; ++i) issue(i);
+        for (int64_t i = 0; i < pre; ++i) issue(i, int(i));
     }
 
     T acc[RPT][4], outer[RPT];
@@ -92,13 +92,14 @@ tmv_rowtile_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restri
     int steps[RPT];
 #pragma unroll
     for (int j = 0; j < RPT; ++j) steps[j] = 0;
-    for (int64_t i = 0; i < my_tiles; ++i) {
-        const int st = int(i % stages);
+    int st = 0;
+    uint32_t ph = 0;
+    for (int64_t i = 0; i < my_tiles; ++i, ring_advance(st, ph, stages)) {
         const int64_t c0 = (blockIdx.x + i * gridDim.x) * int64_t(k);
         const int nc = int(min(int64_t(k), C - c0));
         const int64_t w0 = c0 * R64, w1 = w0 + int64_t(nc) * R64;
         T* stg = ring + st * stage_w;
-        mbar_wait(&full[st], uint32_t((i / stages) & 1));
+        mbar_wait(&full[st], ph);
         const bool btail = ((w1 + 3) & ~int64_t(3)) > total && (w1 & 3);
         if (btail || (nc & 3)) {                        // last tile only (uniform over the CTA)
             const int64_t a0 = w0 & ~int64_t(3);
@@ -135,7 +136,7 @@ tmv_rowtile_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restri
         __syncthreads();                                // stage st fully read
         if (tid == 0 && i + stages < my_tiles) {
             refill_fence();
-            issue(i + stages);
+            issue(i + stages, st);
         }
     }
 

@@ -55,13 +55,13 @@ mv_tpr_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restrict__ 
     }
     __syncthreads();
 
-    auto issue = [&](int64_t i) {  // local tile i -> stage i % stages (thread 0 only)
+    auto issue = [&](int64_t i, int slot) {  // local tile i -> ring stage slot (thread 0 only)
         const int64_t tile = blockIdx.x + i * gridDim.x;
         const int64_t r0 = tile * NT;
         const int64_t nrows = min(int64_t(NT), R - r0);
         const uint32_t bytes = uint32_t(nrows * C * sizeof(T)) & (SCAL ? ~15u : ~0u);
-        T* dst = ring + size_t(i % stages) * stage_elems;
-        uint64_t* bar = &full[i % stages];
+        T* dst = ring + size_t(slot) * stage_elems;
+        uint64_t* bar = &full[slot];
         mbar_arrive_expect_tx(bar, PERROWX ? 2 * bytes : bytes);
         if (bytes) {
             bulk_g2s(dst, A + r0 * C, bytes, bar);
@@ -75,7 +75,7 @@ mv_tpr_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restrict__ 
             bulk_g2s_keep(xs, X, uint32_t(C * sizeof(T)), &xbar);
         }
         const int64_t pre = min(int64_t(stages), my_tiles);
-        for (int64_t i = 0; i < pre; ++i) issue(i);
+        for (int64_t i = 0; i < pre; ++i) issue(i, int(i));
     }
     if (!PERROWX && !SCAL) mbar_wait(&xbar, 0);
     if (!PERROWX && SCAL) {
@@ -84,9 +84,10 @@ mv_tpr_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restrict__ 
     }
 
     const V* xv = reinterpret_cast<const V*>(xs);
-    for (int64_t i = 0; i < my_tiles; ++i) {
-        const int st = int(i % stages);
-        mbar_wait(&full[st], uint32_t((i / stages) & 1));
+    int st = 0;
+    uint32_t ph = 0;
+    for (int64_t i = 0; i < my_tiles; ++i, ring_advance(st, ph, stages)) {
+        mbar_wait(&full[st], ph);
         const int64_t r0 = (blockIdx.x + i * gridDim.x) * int64_t(NT);
         if constexpr (SCAL) {
             T* stg = ring + size_t(st) * stage_elems;
@@ -118,7 +119,7 @@ mv_tpr_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restrict__ 
             __syncthreads();
             if (tid == 0 && i + stages < my_tiles) {
                 refill_fence();
-                issue(i + stages);
+                issue(i + stages, st);
             }
             continue;
         }
@@ -141,7 +142,7 @@ mv_tpr_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restrict__ 
         __syncthreads();                      // every thread is done with stage st
         if (tid == 0 && i + stages < my_tiles) {
             refill_fence();              // generic-proxy reads before async-proxy refill
-            issue(i + stages);
+            issue(i + stages, st);
         }
     }
 }

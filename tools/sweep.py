@@ -181,6 +181,7 @@ def main():
     ap.add_argument("--rowtile-only", action="store_true", help="time only the staged row-tile candidates (+ AUTO)")
     ap.add_argument("--flat-only", action="store_true", help="time only the flat-stream TMV candidates (+ AUTO)")
     ap.add_argument("--shift-only", action="store_true", help="time only the shifted-x MV candidates (+ AUTO)")
+    ap.add_argument("--staged-only", action="store_true", help="time only the TMA-staged candidates (+ AUTO)")
     a = ap.parse_args()
     dev = torch.device("cuda:0")
     tdt = torch.float32 if a.dtype == "f32" else torch.int32
@@ -220,6 +221,9 @@ def main():
                     cands = [("AUTO", None)] + rowtile_grid(op, R, C)
                 elif a.shift_only:
                     cands = [("AUTO", None)] + shift_grid(op, R, C)
+                elif a.staged_only:           # every TMA-staged plan: row tiles, TMV tiles, MV_TPR
+                    cands = [("AUTO", None)] + rowtile_grid(op, R, C) + \
+                        [c for c in grids(op, R, C, a.dtype) if c[0] == "MV_TPR"]
                 elif a.flat_only:
                     cands = [("AUTO", None)] + [("TMV_REGTILE", [0, 0, 0, u]) for u in (2, 4, 8)] + \
                         rowtile_grid(op, R, C)
