@@ -201,11 +201,12 @@ typedef enum {
  *                      row reduced by [ADAPTIC_P_LANES] lanes with x held in
  *                      registers ([ADAPTIC_P_BLOCK] 256 or 512 threads).  A, and
  *                      DOT's b, must be 16-byte aligned for it; other pointers run
- *                      the variant's direct kernel.  TMV_REGTILE (rows <= 1024):
+ *                      the variant's direct kernel.  TMV_REGTILE (rows <= 4096):
  *                      4 = tiles of [ADAPTIC_P_ROWS] rows of B (a multiple of 4;
  *                      0 / -n as above) and their x values staged by TMA, thread
  *                      (r, slice) accumulating output r over its rows of every
- *                      tile, [ADAPTIC_P_BLOCK] 256 / 512 / 1024 >= rows threads;
+ *                      tile, [ADAPTIC_P_BLOCK] 256 / 512 / 1024 threads with 1, 2
+ *                      or 4 outputs each (rows <= 4 x threads, 4 needs >= 512);
  *                      16-byte-aligned B and x, else the direct kernel.  A tile
  *                      height is capped so that two ring stages fit.
  *                      MV (not DOT) with cols % 4 != 0, MV_SUBWARP / MV_WPR /
