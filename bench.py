@@ -63,7 +63,35 @@ def parse():
     ap.add_argument("--detail", default=None, help="write per-problem JSONL here")
     ap.add_argument("--kernel-events-in-timed", action="store_true",
                     help="record per-launch events inside the timed region (default: separate pass)")
+    ap.add_argument("--dry-run", action="store_true",
+                    help="no GPU: launch the ranks (gloo), build every rank's partition of the workload, "
+                         "exchange it and print the line without timing (tests the N>1 plumbing on CPU)")
+    ap.add_argument("--backend", choices=["nccl", "gloo"], default="nccl",
+                    help="N>1 process-group backend (gloo + --share-gpu: exercise the N-rank path on one GPU)")
+    ap.add_argument("--share-gpu", action="store_true",
+                    help="every rank on cuda:0 (plumbing checks on a 1-GPU box; timings meaningless)")
+    ap.add_argument("--replicas", action="store_true",
+                    help="N>1: every rank runs the FULL workload (independent replicas, weak scaling) "
+                         "instead of partitioning each problem over the ranks")
     return ap.parse_args()
+
+
+def self_launch(args) -> bool:
+    """`--gpus N` without a launcher: re-exec under torch.distributed.run with N ranks on
+    127.0.0.1 (one process per GPU).  Returns True if this process only launched."""
+    if args.gpus <= 1 or "WORLD_SIZE" in os.environ:
+        return False
+    import socket
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + sys.argv[1:]
+    rc = subprocess.call(cmd)
+    if rc:
+        sys.exit(rc)
+    return True
 
 
 # ------------------------------------------------------------------------------ helpers
@@ -129,17 +157,27 @@ class Clocks:
                 "reasons": sorted(reasons), "samples": len(sm)}
 
 
-def dist_setup():
+def dist_setup(args=None):
     import torch
     import torch.distributed as dist
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args is not None and world != args.gpus:
+        raise SystemExit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}; launch with "
+                         f"--nproc-per-node {args.gpus} (or without a launcher: bench.py re-execs itself)")
+    if args is not None and args.dry_run:
+        if world > 1:
+            dist.init_process_group("gloo")
+        return world, rank, local
+    dev = 0 if (args is not None and args.share_gpu) else local
+    torch.cuda.set_device(dev)
     if world > 1:
-        torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    else:
-        torch.cuda.set_device(0)
+        backend = args.backend if args is not None else "nccl"
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", dev))
+        else:
+            dist.init_process_group("gloo")
     return world, rank, local
 
 
@@ -154,7 +192,8 @@ def max_over_ranks(v: float, world: int) -> float:
         return v
     import torch
     import torch.distributed as dist
-    t = torch.tensor([v], dtype=torch.float64, device="cuda")
+    dev = "cuda" if dist.get_backend() == "nccl" else "cpu"
+    t = torch.tensor([v], dtype=torch.float64, device=dev)
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return float(t.item())
 
@@ -163,6 +202,17 @@ def max_over_ranks(v: float, world: int) -> float:
 B1_OPS = ("asum", "nrm2", "iamax", "iamin", "b1all")
 ST_SHAPES = [(1 << k, 1 << (26 - k)) for k in range(8, 19)]
 B1_SHAPES = [(1, 1 << 26), (64, 1 << 20), (4096, 1 << 14), (1 << 16, 1024), (1 << 20, 64), (1 << 22, 16)]
+
+
+SPEC_GBS = 8000.0          # B200 HBM3e spec (% of peak is reported vs spec and vs measured)
+
+
+def algo_flops(op, R, C, nvec=1):
+    """Algorithmic flop (reading D8): one multiply + one add per term of every reduction;
+    BLAS-1 / stencil count one op per element read."""
+    if op in ("mv", "tmv", "dot"):
+        return 2 * R * C * nvec
+    return R * C
 
 
 def algo_bytes(op, R, C, nvec=1):
@@ -178,16 +228,20 @@ def algo_bytes(op, R, C, nvec=1):
 
 
 class Problem:
-    """One (op, R, C) instance, resident in HBM, with its selected plan."""
+    """One (op, R, C) instance (a rank's share of a logical Rf x Cf problem), resident in
+    HBM, with its selected plan.  ``y`` may be a view supplied by the caller (a split-K
+    bucket slot)."""
 
-    def __init__(self, op, R, C, cfg, variant="AUTO", shard=None, full=None, nvec=1, dtype="f32"):
+    def __init__(self, op, R, C, cfg, variant="AUTO", shard=None, full=None, nvec=1, dtype="f32", y=None,
+                 kind="rows"):
         import torch
         import synth
         import paper_conf_pldi_samadihmlm12_b200 as adaptic
         from paper_conf_pldi_samadihmlm12_b200 import _lib as L
-        self.op, self.R, self.C, self.nvec = op, R, C, nvec
+        self.op, self.R, self.C, self.nvec, self.kind = op, R, C, nvec, kind
         dev = torch.device("cuda", torch.cuda.current_device())
         Rf, Cf = full if full else (R, C)           # logical full problem (shards are slices)
+        self.full = (Rf, Cf)
         rows, cols = shard if shard else ((0, R), (0, C))
         tdt = torch.int32 if dtype == "i32" else torch.float32
         self.dtype = dtype
@@ -204,13 +258,17 @@ class Problem:
         else:
             self.X = torch.empty(C * nvec, dtype=tdt, device=dev)
             synth.device_vector(self.X, "uniform", synth.seed(cfg, "x"), start=cols[0])
-        self.y = torch.empty(R * C if op == "stencil5" else R * (4 if op == "b1all" else nvec),
-                             dtype=torch.int32 if op in ("iamax", "iamin") else tdt, device=dev)
+        if y is not None:
+            self.y = y
+        else:
+            self.y = torch.empty(R * C if op == "stencil5" else R * (4 if op == "b1all" else nvec),
+                                 dtype=torch.int32 if op in ("iamax", "iamin") else tdt, device=dev)
         opc = L.OPS[op]
         self.stream = torch.cuda.current_stream().cuda_stream
         self.plan = adaptic.get_plan(opc, R, C, L.I32 if dtype == "i32" else L.F32, dev, variant, None, self.stream, nvec)
         self.desc = self.plan.describe()
-        self.bytes = algo_bytes(op, R, C, nvec)
+        self.bytes = algo_bytes(op, R, C, nvec)              # this rank's kernel
+        self.logical_bytes = algo_bytes(op, Rf, Cf, nvec)     # the unsharded problem
         self.ptrs = (self.M.data_ptr(), self.X.data_ptr(), self.y.data_ptr())
 
     def launch(self):
@@ -220,65 +278,142 @@ class Problem:
         return f"{self.op}{'' if self.nvec == 1 else 'x%d' % self.nvec}:{self.R}x{self.C}:{self.desc['variant']}"
 
 
-def build_problems(args, world, rank):
+PARTITIONED = ("sweep", "offgrid", "rowshard", "splitk", "dot")
+
+
+def logical_problems(args):
+    """The workload's logical problems (op, R, C, cfg, nvec) and its config dict.  No GPU."""
     if args.workload == "sweep":
-        return [Problem(op, 1 << k, 1 << (26 - k), 1, args.variant, dtype=args.dtype)
+        return [("mv" if op == "mv" else "tmv", 1 << k, 1 << (26 - k), 1, 1)
                 for k in range(3, 24) for op in ("mv", "tmv")], \
             {"workload": "configs[1]: TMV/MV fp32 shape sweep at 256 MiB, 8Mx8 .. 8192x8192 .. 8x8M, "
-                         "both layouts, variant selector", "shapes": 42, "per_gpu": "full sweep (weak)"}
+                         "both layouts, variant selector", "shapes": 42}
     if args.workload == "offgrid":
-        return [Problem(op, (1 << k) + (op == "tmv"), (1 << (26 - k)) + (op == "mv"), 1, args.variant,
-                        dtype=args.dtype) for k in range(3, 24) for op in ("mv", "tmv")], \
+        return [(op, (1 << k) + (op == "tmv"), (1 << (26 - k)) + (op == "mv"), 1, 1)
+                for k in range(3, 24) for op in ("mv", "tmv")], \
             {"workload": "configs[1] off the 16-byte grid: the sweep's 21 shapes with C+1 (MV) / R+1 (TMV), "
-                         "256 MiB each, rows not 16-byte aligned, variant selector", "shapes": 42,
-             "per_gpu": "full sweep (weak)"}
+                         "256 MiB each, rows not 16-byte aligned, variant selector", "shapes": 42}
     if args.workload == "multi":
         shapes = [(8192, 8192), (65536, 1024), (1 << 20, 64), (64, 1 << 20)]
-        return [Problem(op, R, C, 8, args.variant, nvec=4) for R, C in shapes for op in ("mv", "tmv")], \
+        return [(op, R, C, 8, 4) for R, C in shapes for op in ("mv", "tmv")], \
             {"workload": "SURVEY 8(f)#2: multi-vector MV/TMV fp32, K=4 vectors per pass, 256 MiB matrices "
                          "(8192^2, 65536x1024, 1Mx64, 64x1M)", "shapes": 8, "nvec": 4}
     if args.workload == "config0":
-        return [Problem("tmv", 256, 256, 0, args.variant)], \
+        return [("tmv", 256, 256, 0, 1)], \
             {"workload": "configs[0]: TMV fp32 256x256 (L2-resident; latency-bound)", "shapes": 1}
     if args.workload == "blas1":
-        return [Problem(op, R, C, 7, args.variant) for R, C in B1_SHAPES for op in B1_OPS], \
+        return [(op, R, C, 7, 1) for R, C in B1_SHAPES for op in B1_OPS], \
             {"workload": "SURVEY 8(f)#1-2: BLAS-1 Sasum/Snrm2/Isamax/Isamin + the four fused in one pass "
                          "(B1ALL, horizontal actor integration) fp32 at 256 MiB, N x L = 1x2^26 .. 2^22x16",
              "shapes": len(B1_SHAPES) * len(B1_OPS)}
     if args.workload == "stencil":
-        return [Problem("stencil5", H, W, 9, args.variant) for H, W in ST_SHAPES], \
+        return [("stencil5", H, W, 9, 1) for H, W in ST_SHAPES], \
             {"workload": "SURVEY 8(f)#4: five-point stencil fp32 with input-adaptive super tiles, 256 MiB grids "
                          "H x W = 256x256K .. 8192^2 .. 256Kx256 (the paper's Convolution Separable aspect "
                          "ratios, P:796-874, scaled to B200)", "shapes": len(ST_SHAPES)}
     if args.workload == "dot":
-        return [Problem("dot", 1, 1 << k, 2, args.variant, dtype=args.dtype) for k in range(10, 31)], \
+        return [("dot", 1, 1 << k, 2, 1) for k in range(10, 31)], \
             {"workload": f"configs[2]: scalar product {args.dtype} N=1, L=2^10..2^30", "shapes": 21}
-    from paper_conf_pldi_samadihmlm12_b200.dist import shard_range
     if args.workload == "rowshard":
-        R, C = 131072, 32768
-        r0, r1 = shard_range(R, world, rank)
-        return [Problem("mv", r1 - r0, C, 3, args.variant, shard=((r0, r1), (0, C)), full=(R, C))], \
-            {"workload": "configs[3]: MV fp32 131072x32768 row-sharded, no collective", "rows_per_rank": r1 - r0}
-    R, C = 1024, 1 << 24
-    c0, c1 = shard_range(C, world, rank)
-    return [Problem("tmv", R, c1 - c0, 4, args.variant, shard=((0, R), (c0, c1)), full=(R, C))], \
-        {"workload": "configs[4]: TMV fp32 1024x16M split-K + NCCL all_reduce", "cols_per_rank": c1 - c0}
+        return [("mv", 131072, 32768, 3, 1)], \
+            {"workload": "configs[3]: MV fp32 131072x32768 row-sharded, no collective", "shapes": 1}
+    return [("tmv", 1024, 1 << 24, 4, 1)], \
+        {"workload": "configs[4]: TMV fp32 1024x16M split-K + NCCL all_reduce", "shapes": 1}
+
+
+def partition_plan(args, world, rank):
+    """Per logical problem: (op, R, C, cfg, nvec, kind, rows, cols) of THIS rank's share.
+    N = 1, --replicas and the non-MV/TMV/DOT workloads: every rank holds the whole problem."""
+    from paper_conf_pldi_samadihmlm12_b200.dist import partition
+    logical, config = logical_problems(args)
+    partitioned = world > 1 and not args.replicas and args.workload in PARTITIONED
+    out = []
+    for op, R, C, cfg, nvec in logical:
+        if partitioned:
+            kind, rows, cols = partition(R, C, world, rank)
+        else:
+            kind, rows, cols = "rows", (0, R), (0, C)
+        out.append((op, R, C, cfg, nvec, kind, rows, cols))
+    config = dict(config, partition=("dist.partition: row blocks when R >= G*1024 (no collective), "
+                                     "else split-K + one bucketed collective per step") if partitioned
+                  else ("replicas: every rank runs the full workload" if world > 1 else "single GPU"))
+    return out, config, partitioned
+
+
+def build_problems(args, world, rank):
+    """This rank's Problems (+ the split-K bucket, or None) and the config dict."""
+    import torch
+    from paper_conf_pldi_samadihmlm12_b200.dist import SplitKBucket
+    shares, config, partitioned = partition_plan(args, world, rank)
+    splitk = [sh for sh in shares if sh[5] == "splitk"]
+    bucket = None
+    if splitk:
+        tdt = torch.int32 if args.dtype == "i32" else torch.float32
+        bucket = SplitKBucket([sh[1] for sh in splitk], tdt, torch.device("cuda", torch.cuda.current_device()))
+    probs, j = [], 0
+    for op, R, C, cfg, nvec, kind, rows, cols in shares:
+        y = None
+        if kind == "splitk":
+            y = bucket.views[j]
+            j += 1
+        probs.append(Problem(op, rows[1] - rows[0], cols[1] - cols[0], cfg, args.variant,
+                             shard=(rows, cols), full=(R, C), nvec=nvec, dtype=args.dtype, y=y, kind=kind))
+    config["shares"] = {"rows": sum(1 for sh in shares if sh[5] == "rows"), "splitk": len(splitk)}
+    if bucket is not None:
+        config["collective_bytes_per_step"] = bucket.nbytes
+    if args.workload == "rowshard":
+        config["rows_per_rank"] = probs[0].R
+    if args.workload == "splitk":
+        config["cols_per_rank"] = probs[0].C
+    return probs, config, bucket, partitioned
 
 
 # ------------------------------------------------------------------------------ adaptic arm
+def run_dry(args):
+    """--dry-run: the N-rank plumbing without a GPU (gloo): every rank builds its share of
+    every logical problem; rank 0 checks that the shares tile each problem exactly once and
+    prints the line (value null)."""
+    import torch.distributed as dist
+    world, rank, _ = dist_setup(args)
+    shares, config, partitioned = partition_plan(args, world, rank)
+    mine = [(sh[5], sh[6], sh[7]) for sh in shares]
+    every = [None] * world
+    if world > 1:
+        dist.all_gather_object(every, mine)
+    else:
+        every = [mine]
+    elapsed = max_over_ranks(float(rank), world)       # exercises the max-over-ranks reduction
+    if rank == 0:
+        ok = True
+        for i, (op, R, C, *_rest) in enumerate(shares):
+            covered = sum((r[1] - r[0]) * (c[1] - c[0]) for _, r, c in (every[g][i] for g in range(world)))
+            ok &= covered == (R * C if partitioned else world * R * C)
+        print(json.dumps({
+            "metric": METRIC, "value": None, "unit": UNIT, "n_gpus": world, "steps": 0, "warmup": 0,
+            "dry_run": True, "shares_tile_problems": bool(ok), "max_rank_probe": elapsed,
+            "scaling": "strong" if args.workload in PARTITIONED and not args.replicas else "weak",
+            "config": dict(config, shares={"rows": sum(1 for k, _, _ in every[0] if k == "rows"),
+                                           "splitk": sum(1 for k, _, _ in every[0] if k == "splitk")})}),
+              flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
 def run_adaptic(args):
     import torch
     import torch.distributed as dist
-    world, rank, local = dist_setup()
-    probs, config = build_problems(args, world, rank)
-    splitk = args.workload == "splitk" and world > 1
+    world, rank, local = dist_setup(args)
+    probs, config, bucket, partitioned = build_problems(args, world, rank)
     torch.cuda.synchronize()
     n = len(probs)
-    step_bytes = sum(p.bytes for p in probs)
+    step_bytes = sum(p.bytes for p in probs)                       # this rank's kernels
+    job_bytes = (sum(p.logical_bytes for p in probs) if partitioned   # the whole job, all ranks
+                 else world * step_bytes)
 
     # the step: every problem through the C ABI's batched entry (adaptic_run_batch), which
     # issues them round-robin on `--streams` concurrent streams forked from / joined to the
-    # current stream; per-launch events (--kernel-events-in-timed) need one stream
+    # current stream; per-launch events (--kernel-events-in-timed) need one stream; then ONE
+    # collective for all split-K partials of the step (dist.SplitKBucket)
     from paper_conf_pldi_samadihmlm12_b200 import _lib as L
     main = torch.cuda.current_stream()
     nstreams = max(1, args.streams) if not args.kernel_events_in_timed else 1
@@ -292,8 +427,8 @@ def run_adaptic(args):
                 evs[i].record()
                 p.launch()
             evs[n].record()
-        if splitk:
-            dist.all_reduce(probs[0].y, op=dist.ReduceOp.SUM)
+        if bucket is not None:
+            bucket.combine()
 
     for _ in range(max(3, args.warmup)):
         one_step()
@@ -317,7 +452,32 @@ def run_adaptic(args):
     barrier(world)
     clk = clocks.stop()
     elapsed_ms = max_over_ranks(t0.elapsed_time(t1), world)
-    value = world * step_bytes * args.steps / (elapsed_ms / 1e3) / 1e9
+    value = job_bytes * args.steps / (elapsed_ms / 1e3) / 1e9
+
+    # compute / collective split of a step (SURVEY 8(d) configs[4]): events around the
+    # batch and around the bucket's collective, kev_steps samples after the timed region
+    split = None
+    if bucket is not None or args.workload == "splitk":
+        e = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(kev_steps)]
+        barrier(world)
+        for s in range(kev_steps):
+            e[s][0].record()
+            batch.run(nstreams, main.cuda_stream)
+            e[s][1].record()
+            if bucket is not None:
+                bucket.combine()
+            e[s][2].record()
+        torch.cuda.synchronize()
+        comp = [e[s][0].elapsed_time(e[s][1]) * 1e3 for s in range(kev_steps)]
+        comb = [e[s][1].elapsed_time(e[s][2]) * 1e3 for s in range(kev_steps)]
+        split = {"compute_us": max_over_ranks(statistics.median(comp), world),
+                 "collective_us": max_over_ranks(statistics.median(comb), world),
+                 "total_us": max_over_ranks(statistics.median([a + b for a, b in zip(comp, comb)]), world),
+                 "collective": (("all_reduce(SUM) fp32" if args.dtype == "f32" else
+                                 "all_gather int32 + fixed-order TMV merge kernel")
+                                + f" of {bucket.nbytes} B over {dist.get_backend()}") if bucket is not None
+                 else "none (N = 1: the whole reduction is local)",
+                 "samples": kev_steps}
 
     # per-kernel durations: CUDA events on the launching stream around every launch,
     # in a separate pass of kev_steps steps right after the timed region
@@ -328,19 +488,19 @@ def run_adaptic(args):
         # events, kev_steps samples -> the duration it sustains inside a stream of calls
         # (an event between every launch would add its launch latency to each sample
         # and cut the programmatic-dependent-launch overlap)
-        batch = 5
+        reps = 5
         torch.cuda.synchronize()
         dur = []
         for i, p in enumerate(probs):
             ds = []
             for s in range(kev_steps):
                 evs[s][0].record()
-                for _ in range(batch):       # on the events' (main) stream, whatever --streams says
+                for _ in range(reps):        # on the events' (main) stream, whatever --streams says
                     p.plan.run(*p.ptrs, main.cuda_stream)
                 evs[s][1].record()
             torch.cuda.synchronize()
             for s in range(kev_steps):
-                ds.append(evs[s][0].elapsed_time(evs[s][1]) / batch)
+                ds.append(evs[s][0].elapsed_time(evs[s][1]) / reps)
             dur.append(ds)
     mean_ms = [statistics.mean(d) for d in dur]
     kernel_sum_ms = sum(mean_ms)
@@ -348,9 +508,12 @@ def run_adaptic(args):
     per = []
     for i, p in enumerate(probs):
         gbs = p.bytes / (mean_ms[i] / 1e3) / 1e9
+        q = sorted(dur[i])
         per.append({"op": p.op, "R": p.R, "C": p.C, "variant": p.desc["variant"], "us": mean_ms[i] * 1e3,
-                    "us_median": statistics.median(dur[i]) * 1e3, "GBps": gbs, "frac": gbs / peak,
-                    "bytes": p.bytes, "share": mean_ms[i] / sum(mean_ms), "plan": p.desc})
+                    "us_median": statistics.median(q) * 1e3, "us_p10": q[int(0.1 * (len(q) - 1))] * 1e3,
+                    "us_p90": q[int(round(0.9 * (len(q) - 1)))] * 1e3, "GBps": gbs, "frac": gbs / peak,
+                    "frac_spec": gbs / SPEC_GBS, "GFLOPs": algo_flops(p.op, p.R, p.C, p.nvec) / (mean_ms[i] / 1e3) / 1e9,
+                    "bytes": p.bytes, "share": mean_ms[i] / sum(mean_ms), "kind": p.kind, "plan": p.desc})
     dom = max(range(n), key=lambda i: mean_ms[i])
     traffic = None
     tpath = os.path.join(ROOT, "profiles", "ncu_traffic.json")
@@ -360,7 +523,8 @@ def run_adaptic(args):
     roofline = {"bound": "hbm", "achieved": per[dom]["GBps"], "peak": peak, "unit": "GB/s",
                 "frac": per[dom]["GBps"] / peak, "traffic": traffic,
                 "kernel": probs[dom].key(), "peak_source": peak_src,
-                "step_frac": value / world / peak,
+                "step_frac": value / world / peak, "step_frac_spec": value / world / SPEC_GBS,
+                "p10_p90_us": [per[dom]["us_p10"], per[dom]["us_p90"]],
                 "min_frac": min(q["frac"] for q in per), "min_kernel": min(per, key=lambda q: q["frac"])["variant"]
                 + f" {min(per, key=lambda q: q['frac'])['op']} {min(per, key=lambda q: q['frac'])['R']}x"
                 f"{min(per, key=lambda q: q['frac'])['C']}",
@@ -371,7 +535,7 @@ def run_adaptic(args):
         latency = measure_latency(probs[0])
     e2e = None
     if not args.no_e2e and args.e2e_steps > 0:
-        e2e = measure_e2e(args, probs, world)
+        e2e = measure_e2e(args, probs, world, bucket, partitioned)
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cpu = cpu_baseline(probs, args)
@@ -380,9 +544,12 @@ def run_adaptic(args):
             for q in per:
                 f.write(json.dumps(q) + "\n")
     if rank == 0:
+        job_flops = sum(algo_flops(p.op, *p.full, p.nvec) for p in probs) * (1 if partitioned else world)
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": elapsed_ms / args.steps, "higher_is_better": True,
-                "scaling": "strong" if args.workload in ("rowshard", "splitk") else "weak",
+                "scaling": "strong" if args.workload in PARTITIONED and not args.replicas else "weak",
+                "gflops": job_flops * args.steps / (elapsed_ms / 1e3) / 1e9,
+                "frac_spec": value / world / SPEC_GBS, "spec_peak_gbs": SPEC_GBS,
                 "vs_baseline": None, "dtype": args.dtype,
                 "data": "synthetic (seeded splitmix64; fp32 U[-1,1), int32 U{-128..127})",
                 "config": dict(config, bytes_per_step_per_gpu=step_bytes, variant=args.variant,
@@ -398,7 +565,8 @@ def run_adaptic(args):
                                   f"{kev_steps} samples (the timed region itself has events only at its ends)"),
                 "kernel_sum_ms": kernel_sum_ms, "latency_us": latency, "streams": nstreams,
                 "issue": f"adaptic_run_batch over {nstreams} stream(s) per step",
-                "gpu_launches": n * args.steps, "clocks": clk,
+                "gpu_launches": (n + (1 if bucket is not None and args.dtype == "i32" else 0)) * args.steps,
+                "split": split, "clocks": clk,
                 "selected": {q["op"] + f" {q['R']}x{q['C']}": [q["variant"], round(q["frac"], 3)] for q in per}}
         print(json.dumps(line), flush=True)
     if world > 1:
@@ -453,16 +621,22 @@ def measure_latency(p, reps=200):
             "variant": p.desc["variant"]}
 
 
-def measure_e2e(args, probs, world):
+def measure_e2e(args, probs, world, bucket=None, partitioned=False):
     """Same metric through the C ABI with HOST buffers: every step copies each problem's
-    inputs host->device (pinned), runs the kernel, and reads y back."""
+    inputs host->device (pinned), runs the kernel, and reads y back.  At N > 1 with a
+    split-K bucket the step also runs the bucket's collective and reads the COMBINED
+    partials back (the per-problem D2H of a split-K share is its partial sum)."""
     import torch
     import psutil
     need = sum(p.M.numel() * 4 + p.X.numel() * 4 for p in probs)
-    sel = probs
+    k = len(probs)
     if need > 0.5 * psutil.virtual_memory().available:
         k = max(1, int(len(probs) * 0.5 * psutil.virtual_memory().available / need))
-        sel = probs[:: max(1, len(probs) // k)]
+    k = int(-max_over_ranks(-float(k), world))           # every rank takes the same subset
+    sel = probs if k >= len(probs) else probs[:: max(1, len(probs) // k)]
+    flat_h = None
+    if bucket is not None:
+        flat_h = torch.empty(bucket.flat.numel(), dtype=bucket.flat.dtype, pin_memory=True)
     hosts = []
     for p in sel:
         Mh = torch.empty(p.M.numel(), dtype=p.M.dtype, pin_memory=True)
@@ -486,6 +660,9 @@ def measure_e2e(args, probs, world):
             p.plan.run_host(h[0], h[1], h[2], p.ptrs[0], p.ptrs[1], p.ptrs[2], st.cuda_stream)
         for s in side[1:]:
             main.wait_stream(s)
+        if bucket is not None:
+            bucket.combine()
+            flat_h.copy_(bucket.flat, non_blocking=True)
 
     step()
     torch.cuda.synchronize()
@@ -499,10 +676,10 @@ def measure_e2e(args, probs, world):
     torch.cuda.synchronize()
     barrier(world)
     ms = max_over_ranks(t0.elapsed_time(t1), world)
-    b = sum(p.bytes for p in sel)
+    b = sum(p.logical_bytes for p in sel) if partitioned else world * sum(p.bytes for p in sel)
     h2d = sum(p.M.numel() * 4 + p.X.numel() * 4 for p in sel)
-    d2h = sum(p.y.numel() * 4 for p in sel)
-    return {"value": world * b * args.e2e_steps / (ms / 1e3) / 1e9, "unit": UNIT,
+    d2h = sum(p.y.numel() * 4 for p in sel) + (bucket.nbytes if bucket is not None else 0)
+    return {"value": b * args.e2e_steps / (ms / 1e3) / 1e9, "unit": UNIT,
             "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h, "steps": args.e2e_steps,
             "problems": len(sel), "streams": len(side),
             "api": "adaptic_run_host (C ABI, pinned host buffers), problems alternating over the streams"}
@@ -682,7 +859,11 @@ def run_bicgstab(args):
 
 if __name__ == "__main__":
     a = parse()
-    if a.impl == "reference":
+    if a.impl != "reference" and self_launch(a):
+        sys.exit(0)
+    if a.dry_run:
+        run_dry(a)
+    elif a.impl == "reference":
         run_reference(a)
     elif a.workload == "bicgstab":
         run_bicgstab(a)

@@ -125,3 +125,24 @@ def test_gloo_world2_partitions_and_collectives():
     for r in range(world):
         assert np.all(np.abs(results[r]["dot"] - yd) <= 1e-4 * Sd)
         assert results[r]["dtype_error"]
+
+
+def test_partition_rule_is_rows_or_splitk():
+    """Row blocks when every rank gets >= ROW_MIN outputs (no collective), else the
+    reduction is split (P:480's merge across GPUs); the shares tile the problem."""
+    from paper_conf_pldi_samadihmlm12_b200.dist import ROW_MIN, partition
+    assert partition(8192, 8192, 8, 3)[0] == "rows"
+    assert partition(1024, 1 << 24, 8, 3) == ("splitk", (0, 1024), (3 << 21, 4 << 21))
+    assert partition(131072, 32768, 8, 7) == ("rows", (7 * 16384, 8 * 16384), (0, 32768))
+    assert partition(5, 7, 1, 0) == ("rows", (0, 5), (0, 7))
+    for R, C in [(8, 1 << 23), (1 << 23, 8), (4096, 16384), (2048, 32768), (1000, 1001)]:
+        for G in (2, 3, 4, 8):
+            kinds = {partition(R, C, G, g)[0] for g in range(G)}
+            assert len(kinds) == 1
+            kind = kinds.pop()
+            assert kind == ("rows" if R >= G * ROW_MIN else "splitk")
+            covered = sum((r1 - r0) * (c1 - c0) for _, (r0, r1), (c0, c1) in
+                          (partition(R, C, G, g) for g in range(G)))
+            assert covered == R * C
+    with pytest.raises(ValueError):
+        partition(4, 4, 2, 2)

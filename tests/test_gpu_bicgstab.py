@@ -101,3 +101,57 @@ def test_paper_sizes_8192_device_generated():
     assert np.linalg.norm(b - A64 @ xg) / np.linalg.norm(b) <= 1e-4
     xo, ito, _ = oracle_bicgstab(A64, b.astype(np.float64), tol=1e-5, max_iters=100)
     assert abs(it - ito) <= 2 and np.linalg.norm(xg - xo) <= 1e-4 * np.linalg.norm(xo)
+
+
+def convection_diffusion(m: int, beta: float) -> np.ndarray:
+    """The classic nonsymmetric BiCGSTAB test system (van der Vorst 1992): -Δu + β ∂u/∂x on
+    an m x m interior grid, 5-point Laplacian, central convection differences, Dirichlet
+    boundary; n = m^2, scaled by h^2 (diagonal 4).  kappa ~ 10^3 at m = 64 (computed in the
+    test), so the method needs tens to hundreds of iterations -- unlike the diagonally
+    dominant `diagdom` systems above (kappa ~ 1, two iterations)."""
+    n, h = m * m, 1.0 / (m + 1)
+    A = np.zeros((n, n), dtype=np.float32)
+    i, j = np.divmod(np.arange(n), m)
+    k = np.arange(n)
+    A[k, k] = 4.0
+    for di, dj, w in ((1, 0, -1.0 + beta * h / 2), (-1, 0, -1.0 - beta * h / 2), (0, 1, -1.0), (0, -1, -1.0)):
+        ii, jj = i + di, j + dj
+        ok = (ii >= 0) & (ii < m) & (jj >= 0) & (jj < m)
+        A[k[ok], (ii * m + jj)[ok]] = w
+    return A
+
+
+@pytest.mark.parametrize("m,beta,tol,count", [(64, 5.0, 1e-3, True), (64, 5.0, 1e-4, True), (64, 20.0, 1e-4, True),
+                                              (64, 5.0, 1e-5, False), (64, 20.0, 1e-5, False)])
+def test_ill_conditioned_nonsymmetric_system(m, beta, tol, count):
+    """P:1252-1304 (nonsymmetric systems): a kappa ~ 10^3 system that needs >= 30 iterations.
+    fp32 iterates vs the fp64 oracle (reading R18): convergence with the true residual within
+    10 x tol, and the first 8 iterations' residual history within 1e-3 relative (step-by-step
+    agreement before fp32 drift).  The iteration count must be within max(3, 15 %) of the
+    oracle's only while tol is above fp32's attainable accuracy on this system (tol >= 1e-4):
+    near kappa * u32 ~ 1e-5..1e-4 the fp32 recurrence is driven by rounding (measured: 103
+    GPU vs 80 oracle iterations for 1e-5 at beta = 20), so there only convergence is checked."""
+    A = convection_diffusion(m, beta)
+    n = m * m
+    b = synth.vector(n, np.float32, "uniform", synth.seed(23, "b"))
+    A64, b64 = A.astype(np.float64), b.astype(np.float64)
+    assert np.linalg.cond(A64) > 500 and not np.allclose(A64, A64.T)
+    xo, ito, hist = oracle_bicgstab(A64, b64, tol=tol, max_iters=2000)
+    assert ito >= 30
+    Ad, bd = torch.from_numpy(A).to(DEV), torch.from_numpy(b).to(DEV)
+    x, it, rel = adaptic.bicgstab(Ad, bd, tol=tol, max_iters=2000, check_every=4)
+    xg = x.cpu().numpy().astype(np.float64)
+    assert rel < tol
+    assert np.linalg.norm(b64 - A64 @ xg) / np.linalg.norm(b64) <= 10 * tol
+    if count:
+        assert abs(it - ito) <= max(3, 0.15 * ito), (it, ito)
+    # step-by-step: one iteration at a time, the recurrence residual after each
+    xs = torch.empty(n, device=DEV)
+    S = adaptic.bicgstab_solver(n, torch.device(DEV))
+    stream = torch.cuda.current_stream().cuda_stream
+    S.start(bd.data_ptr(), xs.data_ptr(), stream)
+    for k in range(8):
+        S.iterate(Ad.data_ptr(), xs.data_ptr(), 1, 0.0, stream)
+        itk, relk, done = S.state(stream)
+        assert itk == k + 1 and not done
+        assert abs(relk - hist[k]["relres"]) <= 1e-3 * hist[k]["relres"], (k, relk, hist[k]["relres"])

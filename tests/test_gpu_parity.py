@@ -435,6 +435,21 @@ def test_config2_scalar_product_lengths(dt):
         check(y, ref, dt, f"dot L=2^{k}")
 
 
+@pytest.mark.parametrize("k", [29, 30])
+def test_config2_fp32_longest_lengths(k):
+    """configs[2]'s two longest fp32 lengths (2 and 4 GiB per operand), the ones the bench
+    times beyond 2^28: every term through the plan's split/fold tree, tolerance 1e-4 * S."""
+    L_ = 1 << k
+    a = torch.empty(L_, dtype=torch.float32, device=DEV)
+    b = torch.empty(L_, dtype=torch.float32, device=DEV)
+    synth.device_matrix(a, 1, L_, "mv", "uniform", synth.seed(2, "A"))
+    synth.device_matrix(b, 1, L_, "mv", "uniform", synth.seed(2, "b"))
+    y = adaptic.dot(a, b).cpu().numpy()
+    ah, bh = a.cpu().numpy(), b.cpu().numpy()
+    del a, b
+    check(y, oracle.dot(ah[None, :], bh[None, :]), "f32", f"dot L=2^{k}")
+
+
 def test_config2_int32_wrap_at_2pow30():
     L_ = 1 << 30
     a = torch.empty(L_, dtype=torch.int32, device=DEV)
