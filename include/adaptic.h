@@ -241,8 +241,13 @@ typedef enum {
 typedef struct adaptic_plan_s* adaptic_plan_t;   /* opaque; owned by the caller */
 
 /* Selector (host only, O(1), no device work): picks the variant and its launch
- * parameters for (op, rows, cols, dtype) from the fitted threshold table.
- * *out receives a new plan (free with adaptic_plan_destroy). */
+ * parameters for (op, rows, cols, dtype) from the fitted threshold table (P:230-236:
+ * the runtime kernel management unit picks the kernel and its launch shape from the
+ * actual input).  The table's nearest-cell answer is memoised per (op, dtype, load
+ * class, floor(log2 R), floor(log2 C)) cell and the derived plan per (op, dtype, R, C,
+ * device), so a repeated shape costs one hash lookup and a struct copy
+ * (tools/plan_latency.c measures it).  Thread-safe.  *out receives a new plan (free
+ * with adaptic_plan_destroy). */
 adaptic_status adaptic_plan(adaptic_op op, int64_t rows, int64_t cols, adaptic_dtype dtype,
                             adaptic_plan_t* out);
 
@@ -265,8 +270,11 @@ adaptic_status adaptic_plan_forced(adaptic_op op, int64_t rows, int64_t cols,
  * every FOLD/U steps).  Variants: MV_SUBWARP / MV_WPR (rows of at most G*U loads,
  * x held in registers), MV_CPR / MV_SPLIT (8/K rows per CTA share each x load),
  * TMV_COL / TMV_SPLITK / TMV_REGTILE; variant = ADAPTIC_V_AUTO selects (params
- * ignored).  A 128-bit-shape lane-group plan run on pointers that are not 16-byte
- * aligned returns ADAPTIC_ERR_MISALIGNED. */
+ * ignored).  A 128-bit-shape plan run on pointers that are 4-byte but not 16-byte
+ * aligned runs a fallback planned with it (MV_CPR / MV_SPLIT or register-fed TMV_SPLITK
+ * on 4-byte loads: correct, slower; its workspace is included in
+ * adaptic_plan_workspace_bytes); only pointers that are not 4-byte aligned return
+ * ADAPTIC_ERR_MISALIGNED. */
 adaptic_status adaptic_plan_multi(adaptic_op op, int64_t rows, int64_t cols, int32_t nvec,
                                   adaptic_dtype dtype, adaptic_variant variant,
                                   const int32_t* params, adaptic_plan_t* out);
@@ -307,10 +315,14 @@ adaptic_status adaptic_run_batch(int32_t n, const adaptic_plan_t* plans, const v
 
 /* End-to-end form with HOST buffers: enqueue on `stream` the host->device copy
  * of A and x into the caller's device buffers dA, dx (sizes as for
- * adaptic_run), the kernel into dy, and the device->host copy of dy into y_host.
- * For MV/DOT the copy of A is split into row blocks so that each block's
- * reduction overlaps the next block's transfer.  Host buffers should be
- * page-locked for the copies to be asynchronous.  Returns after enqueueing;
+ * adaptic_run), the kernel into dy, and the device->host copy of dy into y_host,
+ * in that order on the one stream (x, then A as ONE copy, then the kernel: the
+ * transfer is PCIe-bound, ~55 GB/s against the kernel's ~7 TB/s, so a row-block
+ * pipeline would hide at most ~1 % of the call; callers overlap problems instead by
+ * issuing them on several streams).  Host buffers should be page-locked for the
+ * copies to be asynchronous.  Sizes are the plan's (R, C, nvec): the caller guarantees
+ * A_host/dA hold R*C elements, x_host/dx C*nvec (DOT: R*C), y_host/dy R*nvec (B1ALL:
+ * 4*R; STENCIL5: R*C) -- the Python binding checks them.  Returns after enqueueing;
  * the caller synchronises the stream before reading y_host. */
 adaptic_status adaptic_run_host(adaptic_plan_t plan, const void* A_host, const void* x_host,
                                 void* y_host, void* dA, void* dx, void* dy, void* stream);

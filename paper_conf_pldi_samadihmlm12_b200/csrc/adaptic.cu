@@ -21,6 +21,7 @@
 #include <cstring>
 #include <mutex>
 #include <string>
+#include <unordered_map>
 
 using namespace adaptic;
 
@@ -57,6 +58,8 @@ struct adaptic_plan_s {
     size_t ws_bytes, cnt_off;
     size_t fb_ws_off;      // staged-tile plans: the direct-kernel fallback's workspace starts here
     size_t xsh_off;        // xmode 3 (misaligned MV): the four shifted copies of x start here
+    bool multi_fb_ok;      // multi-vector 128-bit-shape plan: a 4-byte-path fallback is planned
+                           // (its workspace slice starts at fb_ws_off)
     void* ws;
     size_t ws_cap;
 };
@@ -254,7 +257,7 @@ int heuristic_variant(int op, int64_t R, int64_t C, int sms) {
 // path needs C % 4 == 0, for TMV R % 4 == 0 -- the two paths have different optima).
 constexpr int kBeyondL2Log2 = 26;   // 2^26 elements = 256 MiB of fp32, 2x the 126 MB L2
 
-const TableEntry* table_lookup(int op, int dtype, int64_t R, int64_t C, bool* projected) {
+const TableEntry* table_lookup_scan(int op, int dtype, int64_t R, int64_t C, bool* projected) {
     const int lr = ilog2_floor(R), lc = ilog2_floor(C);
     *projected = false;
     const int vec = (op == ADAPTIC_OP_TMV) ? (R % 4 == 0) : (C % 4 == 0);
@@ -291,8 +294,34 @@ const TableEntry* table_lookup(int op, int dtype, int64_t R, int64_t C, bool* pr
         if (pb && pd <= 2) { *projected = true; return pb; }
     }
     // int32 moves the same bytes as fp32: use the fp32 cells when int32 was not swept
-    if (dtype != ADAPTIC_F32) return table_lookup(op, ADAPTIC_F32, R, C, projected);
+    if (dtype != ADAPTIC_F32) return table_lookup_scan(op, ADAPTIC_F32, R, C, projected);
     return nullptr;
+}
+
+// O(1) selector: the scan above depends on (op, dtype, vec, lr, lc) only, so its answer is
+// memoised per cell in a dense index (0 = not computed yet, -1 = no cell, else entry index
+// + 1 with bit 30 = projected).  Filling a cell is idempotent, so concurrent planners may
+// race on it harmlessly (relaxed atomics); every later plan of that cell is one load.
+constexpr int kOpsN = ADAPTIC_OP_STENCIL5 + 1;
+std::atomic<int32_t> g_cell[kOpsN][2][2][64][64];
+
+const TableEntry* table_lookup(int op, int dtype, int64_t R, int64_t C, bool* projected) {
+    const int lr = ilog2_floor(R), lc = ilog2_floor(C);
+    const int vec = (op == ADAPTIC_OP_TMV) ? (R % 4 == 0) : (C % 4 == 0);
+    *projected = false;
+    if (op < 0 || op >= kOpsN || dtype < 0 || dtype > 1 || lr < 0 || lc < 0 || lr > 63 || lc > 63)
+        return table_lookup_scan(op, dtype, R, C, projected);
+    std::atomic<int32_t>& cell = g_cell[op][dtype][vec][lr][lc];
+    int32_t v = cell.load(std::memory_order_relaxed);
+    if (v == 0) {
+        bool pj = false;
+        const TableEntry* e = table_lookup_scan(op, dtype, R, C, &pj);
+        v = e ? int32_t(e - kTable + 1) | (pj ? (1 << 30) : 0) : -1;
+        cell.store(v, std::memory_order_relaxed);
+    }
+    if (v < 0) return nullptr;
+    *projected = (v >> 30) & 1;
+    return &kTable[(v & ((1 << 30) - 1)) - 1];
 }
 
 // Five-point stencil: ST_DIRECT (no shared memory) or ST_TILE (TMA-staged super tiles,
@@ -860,6 +889,25 @@ adaptic_status derive_tmv_rowtile(adaptic_plan_s* p, const int32_t* params, cons
     return ADAPTIC_OK;
 }
 
+// A multi-vector plan with a 128-bit shape run on pointers that are not 16-byte aligned
+// (the x-tile / TMA / register-x kernels need aligned rows): the generic CTA kernels'
+// 4-byte path of the same K -- MV_CPR (no workspace) when its error bound holds, else
+// MV_SPLIT; TMV: the register-fed SPLITK tiles.  Only 4-byte misalignment is an error (8(b)).
+bool multi_fallback(const adaptic_plan_s& p, adaptic_plan_s* fb, const DevInfo& dev) {
+    int32_t prm[ADAPTIC_NPARAMS] = {0};
+    prm[ADAPTIC_P_XSMEM] = 1;                    // x through L1 (MV), register-fed tiles (TMV)
+    const int mv_cands[2] = {ADAPTIC_V_MV_CPR, ADAPTIC_V_MV_SPLIT};
+    const int tmv_cands[1] = {ADAPTIC_V_TMV_SPLITK};
+    const int* cands = p.op == ADAPTIC_OP_TMV ? tmv_cands : mv_cands;
+    const int n = p.op == ADAPTIC_OP_TMV ? 1 : 2;
+    for (int i = 0; i < n; ++i) {
+        *fb = p;
+        fb->variant = cands[i]; fb->ws = nullptr; fb->ws_cap = 0; fb->multi_fb_ok = false;
+        if (derive_multi(fb, prm, dev) == ADAPTIC_OK && fb->path_ok[0]) return true;
+    }
+    return false;
+}
+
 // Fill the kernel parameters of `p` for p->variant.  params: user overrides or nullptr.
 adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& dev) {
     const int op = p->op, dt = p->dtype;
@@ -868,7 +916,19 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
     auto par = [&](int i) -> int { return params ? params[i] : 0; };
     const int v = p->variant;
     if (!op_has_variant(op, v)) return ADAPTIC_ERR_UNSUPPORTED;
-    if (p->nvec > 1) return derive_multi(p, params, dev);
+    if (p->nvec > 1) {
+        p->multi_fb_ok = false;
+        const adaptic_status st = derive_multi(p, params, dev);
+        if (st == ADAPTIC_OK && p->vec_shape) {
+            adaptic_plan_s fb;
+            if (multi_fallback(*p, &fb, dev)) {
+                p->multi_fb_ok = true;
+                p->fb_ws_off = ((p->ws_bytes + 255) / 256) * 256;
+                if (fb.ws_bytes > 0) p->ws_bytes = p->fb_ws_off + fb.ws_bytes;
+            }
+        }
+        return st;
+    }
     // single-vector MV (fp32 or int32) on the x-tile stream-K kernel (param XSMEM 3)
     if (op == ADAPTIC_OP_MV && (v == ADAPTIC_V_MV_CPR || v == ADAPTIC_V_MV_SPLIT) &&
         par(ADAPTIC_P_XSMEM) == 3 && C % 4 == 0)
@@ -1479,6 +1539,54 @@ adaptic_status check_run(const adaptic_plan_s* p, const void* A, const void* x, 
     return ADAPTIC_OK;
 }
 
+// Plan cache (SURVEY 8(a) a1 "plan caching"; selection must add no visible time):
+// a selector plan depends only on (op, dtype, R, C, nvec) and the device it is made on,
+// so the derived struct is memoised and later calls copy it (no workspace attached).
+struct PlanKey {
+    int op, dtype, nvec, dev;
+    int64_t R, C;
+    bool operator==(const PlanKey& o) const {
+        return op == o.op && dtype == o.dtype && nvec == o.nvec && dev == o.dev && R == o.R && C == o.C;
+    }
+};
+struct PlanKeyHash {
+    size_t operator()(const PlanKey& k) const {
+        uint64_t h = uint64_t(k.R) * 0x9E3779B97F4A7C15ull ^ (uint64_t(k.C) + 0x632BE59BD9B4E019ull);
+        h ^= uint64_t(k.op | (k.dtype << 8) | (k.nvec << 16)) * 0xBF58476D1CE4E5B9ull + uint64_t(k.dev + 1);
+        return size_t(h ^ (h >> 31));
+    }
+};
+std::mutex g_plan_cache_mu;
+std::unordered_map<PlanKey, adaptic_plan_s, PlanKeyHash> g_plan_cache;
+constexpr size_t kPlanCacheMax = 4096;
+
+adaptic_status cached_plan(int op, int64_t rows, int64_t cols, int dtype, int nvec, adaptic_plan_t* out) {
+    if (!out) return ADAPTIC_ERR_INVALID_ARG;
+    int dev = -1;
+    if (cudaGetDevice(&dev) != cudaSuccess) { (void)cudaGetLastError(); dev = -1; }
+    const PlanKey key{op, dtype, nvec, dev, rows, cols};
+    {
+        std::lock_guard<std::mutex> lk(g_plan_cache_mu);
+        auto it = g_plan_cache.find(key);
+        if (it != g_plan_cache.end()) {
+            adaptic_plan_s* p = new (std::nothrow) adaptic_plan_s(it->second);
+            if (!p) return ADAPTIC_ERR_INVALID_ARG;
+            *out = p;
+            return ADAPTIC_OK;
+        }
+    }
+    const adaptic_status st = make_plan(op, rows, cols, dtype, ADAPTIC_V_AUTO, nullptr, out, nvec);
+    if (st == ADAPTIC_OK) {
+        adaptic_plan_s tmpl = **out;
+        tmpl.ws = nullptr;
+        tmpl.ws_cap = 0;
+        std::lock_guard<std::mutex> lk(g_plan_cache_mu);
+        if (g_plan_cache.size() >= kPlanCacheMax) g_plan_cache.clear();
+        g_plan_cache.emplace(key, tmpl);
+    }
+    return st;
+}
+
 }  // namespace
 
 // =================================================================== C ABI
@@ -1486,18 +1594,19 @@ extern "C" {
 
 adaptic_status adaptic_plan(adaptic_op op, int64_t rows, int64_t cols, adaptic_dtype dtype,
                             adaptic_plan_t* out) {
-    return make_plan(op, rows, cols, dtype, ADAPTIC_V_AUTO, nullptr, out);
+    return cached_plan(op, rows, cols, dtype, 1, out);
 }
 
 adaptic_status adaptic_plan_forced(adaptic_op op, int64_t rows, int64_t cols, adaptic_dtype dtype,
                                    adaptic_variant variant, const int32_t* params, adaptic_plan_t* out) {
-    if (variant == ADAPTIC_V_AUTO) return make_plan(op, rows, cols, dtype, ADAPTIC_V_AUTO, nullptr, out);
+    if (variant == ADAPTIC_V_AUTO) return cached_plan(op, rows, cols, dtype, 1, out);
     return make_plan(op, rows, cols, dtype, variant, params, out);
 }
 
 adaptic_status adaptic_plan_multi(adaptic_op op, int64_t rows, int64_t cols, int32_t nvec, adaptic_dtype dtype,
                                   adaptic_variant variant, const int32_t* params, adaptic_plan_t* out) {
-    return make_plan(op, rows, cols, dtype, variant, variant == ADAPTIC_V_AUTO ? nullptr : params, out, nvec);
+    if (variant == ADAPTIC_V_AUTO) return cached_plan(op, rows, cols, dtype, nvec, out);
+    return make_plan(op, rows, cols, dtype, variant, params, out, nvec);
 }
 
 adaptic_variant adaptic_plan_variant(adaptic_plan_t plan) {
@@ -1561,6 +1670,16 @@ adaptic_status adaptic_run(adaptic_plan_t p, const void* A, const void* x, void*
         vec = aligned(A, 16) && aligned(y, 16);
     } else if (vec && p->nvec > 1) {
         vec = aligned(A, 16) && aligned(x, 16) && aligned(y, 16);
+        if (!vec) {                               // 4-byte-aligned pointers: the planned fallback
+            adaptic_plan_s fb;
+            if (!p->multi_fb_ok || !multi_fallback(*p, &fb, device_info())) return ADAPTIC_ERR_MISALIGNED;
+            if (fb.ws_bytes > 0) {                // its own zeroed slice of p's workspace
+                if (!p->ws || p->fb_ws_off + fb.ws_bytes > p->ws_cap) return ADAPTIC_ERR_NO_WORKSPACE;
+                fb.ws = static_cast<char*>(p->ws) + p->fb_ws_off;
+                fb.ws_cap = p->ws_cap - p->fb_ws_off;
+            }
+            return launch(&fb, A, x, y, stream, false, false);
+        }
     } else if (vec) {
         if (p->op == ADAPTIC_OP_TMV) vec = aligned(A, 16) && aligned(y, 16);
         else if (is_b1_op(p->op)) vec = aligned(A, 16);

@@ -218,6 +218,10 @@ def run_host(op: str, M_host: torch.Tensor, X_host: torch.Tensor, y_host: torch.
     enqueues H2D copies of M and X into dM/dX, the kernel, and the D2H copy of y
     on the current stream.  The caller synchronises before reading y_host."""
     opc = L.OPS[op]
+    if opc not in (L.OP_MV, L.OP_TMV, L.OP_DOT, L.OP_STENCIL5):
+        raise ValueError(f"run_host supports mv, tmv, dot and stencil5, got {op!r}")
+    if M_host.dim() not in (1, 2) or (opc != L.OP_DOT and M_host.dim() != 2):
+        raise ValueError(f"run_host: bad matrix shape {tuple(M_host.shape)}")
     if opc == L.OP_TMV:
         C, R = M_host.shape
     elif M_host.dim() == 1:
@@ -225,11 +229,22 @@ def run_host(op: str, M_host: torch.Tensor, X_host: torch.Tensor, y_host: torch.
     else:
         R, C = M_host.shape
     dev = _check_dev(dM, dX, dy)
+    dt = _dtype_code(M_host)
     for t in (M_host, X_host, y_host):
         if t.device.type != "cpu" or not t.is_contiguous():
             raise ValueError("host buffers must be contiguous CPU tensors")
+    # every buffer the library copies blindly must have the plan's size and dtype
+    nx = R * C if opc == L.OP_DOT else 2 if opc == L.OP_STENCIL5 else C     # stencil: {c, n}
+    ny = R * C if opc == L.OP_STENCIL5 else R
+    want = {"M_host": (M_host, R * C), "X_host": (X_host, nx), "y_host": (y_host, ny),
+            "dM": (dM, R * C), "dX": (dX, nx), "dy": (dy, ny)}
+    for name, (t, n) in want.items():
+        if t.dtype != M_host.dtype:
+            raise TypeError(f"run_host: {name} is {t.dtype}, expected {M_host.dtype}")
+        if t.numel() != n:
+            raise ValueError(f"run_host: {name} has {t.numel()} elements, expected {n}")
     stream = torch.cuda.current_stream(dev).cuda_stream
-    plan = get_plan(opc, R, C, _dtype_code(dM), dev, variant, None, stream)
+    plan = get_plan(opc, R, C, dt, dev, variant, None, stream)
     plan.run_host(M_host.data_ptr(), X_host.data_ptr(), y_host.data_ptr(),
                   dM.data_ptr(), dX.data_ptr(), dy.data_ptr(), stream)
     return y_host
@@ -238,9 +253,13 @@ def run_host(op: str, M_host: torch.Tensor, X_host: torch.Tensor, y_host: torch.
 _solvers: dict = {}
 
 
-def bicgstab_solver(n: int, device: torch.device) -> "L.BiCGSTAB":
-    """Cached solver for n x n systems on `device` with its zero-filled workspace."""
-    key = (int(n), device.index)
+def bicgstab_solver(n: int, device: torch.device, stream: int | None = None) -> "L.BiCGSTAB":
+    """Cached solver for n x n systems on `device` with its zero-filled workspace.  The
+    solver's vectors, MV workspace and device state are per solver, so the cache is keyed
+    by the stream too (two streams never share one: their solves would race)."""
+    if stream is None:
+        stream = torch.cuda.current_stream(device).cuda_stream
+    key = (int(n), device.index, int(stream or 0))
     with _cache_lock:
         ent = _solvers.get(key)
         if ent is not None:
@@ -262,9 +281,18 @@ def bicgstab(A: torch.Tensor, b: torch.Tensor, *, tol: float = 1e-6, max_iters: 
     dev = _check_dev(A, b)
     if A.dtype != torch.float32:
         raise TypeError("bicgstab takes float32")
-    x = torch.empty_like(b) if out is None else out
-    S = bicgstab_solver(A.shape[0], dev)
+    if out is None:
+        x = torch.empty_like(b)
+    else:
+        x = out
+        if (x.dtype != torch.float32 or x.device != dev or not x.is_contiguous() or x.shape != b.shape):
+            raise ValueError(f"out must be a contiguous float32 [{b.shape[0]}] tensor on {dev}")
+        n4 = 4 * b.shape[0]
+        for t, nb in ((b, n4), (A, n4 * A.shape[0])):
+            if x.data_ptr() < t.data_ptr() + nb and t.data_ptr() < x.data_ptr() + n4:
+                raise ValueError("out must not overlap A or b")
     stream = torch.cuda.current_stream(dev).cuda_stream
+    S = bicgstab_solver(A.shape[0], dev, stream)
     it, rel = S.solve(A.data_ptr(), b.data_ptr(), x.data_ptr(), max_iters, tol, check_every, stream)
     return x, it, rel
 

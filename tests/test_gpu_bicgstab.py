@@ -155,3 +155,24 @@ def test_ill_conditioned_nonsymmetric_system(m, beta, tol, count):
         itk, relk, done = S.state(stream)
         assert itk == k + 1 and not done
         assert abs(relk - hist[k]["relres"]) <= 1e-3 * hist[k]["relres"], (k, relk, hist[k]["relres"])
+
+
+def test_out_is_validated_and_solvers_are_per_stream():
+    """`out` is checked (dtype, device, shape, no overlap with A or b), and two
+    streams get two solvers (their vectors and state would race otherwise)."""
+    n = 256
+    A, b = system(n)
+    Ad, bd = torch.from_numpy(A).to(DEV), torch.from_numpy(b).to(DEV)
+    for out in (torch.empty(n, dtype=torch.float64, device=DEV), torch.empty(n + 1, device=DEV), bd,
+                Ad.view(-1)[:n]):
+        with pytest.raises(ValueError):
+            adaptic.bicgstab(Ad, bd, out=out)
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+    assert adaptic.bicgstab_solver(n, torch.device(DEV), s1.cuda_stream) is not \
+        adaptic.bicgstab_solver(n, torch.device(DEV), s2.cuda_stream)
+    xs = []
+    for s in (s1, s2):
+        with torch.cuda.stream(s):
+            xs.append(adaptic.bicgstab(Ad, bd, tol=1e-6)[0])
+    torch.cuda.synchronize()
+    assert torch.equal(xs[0], xs[1])

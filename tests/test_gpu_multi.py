@@ -104,3 +104,31 @@ def test_device_generated_256MiB():
         fn = adaptic.mv_multi if op == "mv" else adaptic.tmv_multi
         Y = fn(t.view(M.shape), torch.from_numpy(X).to(DEV)).cpu().numpy()
         check(Y, M, X, op, f"{op} {R}x{C} K={K} 256MiB")
+
+
+@pytest.mark.parametrize("op", ["mv", "tmv"])
+@pytest.mark.parametrize("K", [2, 4, 8])
+def test_4byte_aligned_pointers_fall_back(op, K):
+    """only non-4-byte-aligned pointers are errors.  A 128-bit-shape multi plan
+    (AUTO: x tiles / TMA tiles / register-x lane groups) run on 4-byte-aligned views of the
+    same data takes its planned 4-byte fallback and matches the oracle."""
+    fails = []
+    for R, C in [(64, 1 << 16), (1 << 15, 64), (8192, 1024), (8, 1 << 18), (4096, 16), (256, 4096)]:
+        M = synth.matrix(R, C, op, np.float32, "uniform", synth.seed(14, "A") + R)
+        X = synth.matrix(K, C, "mv", np.float32, "uniform", synth.seed(14, "x") + C)
+        for off in (1, 2, 3):
+            Mb = torch.empty(M.size + off, dtype=torch.float32, device=DEV)
+            Xb = torch.empty(X.size + off, dtype=torch.float32, device=DEV)
+            Yb = torch.empty(K * R + off, dtype=torch.float32, device=DEV)
+            Md = Mb[off:].view(M.shape)
+            Xd = Xb[off:].view(X.shape)
+            Md.copy_(torch.from_numpy(M))
+            Xd.copy_(torch.from_numpy(X))
+            Yd = Yb[off:].view(K, R)
+            try:
+                fn = adaptic.mv_multi if op == "mv" else adaptic.tmv_multi
+                fn(Md, Xd, out=Yd)
+                check(Yd.cpu().numpy(), M, X, op, f"{op} {R}x{C} K={K} off={off}")
+            except Exception as e:  # noqa: BLE001
+                fails.append(f"{op} {R}x{C} K={K} off={off}: {type(e).__name__}: {str(e)[:160]}")
+    assert not fails, "\n".join(fails)

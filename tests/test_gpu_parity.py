@@ -513,3 +513,28 @@ def test_run_batch_equals_single_runs():
     assert e.value.status == L.ERR_ALIAS
     torch.cuda.synchronize()
     assert (items[0][6] == 7.0).all()                    # nothing was issued
+
+
+def test_run_host_validates_every_buffer():
+    """adaptic_run_host copies R*C, C and R elements blindly, so the binding must
+    reject short, mistyped or misplaced buffers before calling it."""
+    R, C = 300, 257
+    M = torch.ones(R, C, dtype=torch.float32).pin_memory()
+    X = torch.ones(C, dtype=torch.float32).pin_memory()
+    y = torch.empty(R, dtype=torch.float32).pin_memory()
+    dM = torch.empty(R * C, device=DEV)
+    dX = torch.empty(C, device=DEV)
+    dy = torch.empty(R, device=DEV)
+    adaptic.run_host("mv", M, X, y, dM, dX, dy)
+    torch.cuda.synchronize()
+    assert (y == C).all()                         # P1
+    bad = [
+        dict(y=torch.empty(R - 1)), dict(X=torch.ones(C - 1)), dict(dy=torch.empty(R - 1, device=DEV)),
+        dict(dM=torch.empty(R * C - 1, device=DEV)), dict(dX=torch.empty(C + 1, device=DEV)),
+        dict(X=torch.ones(C, dtype=torch.float64)), dict(dy=torch.empty(R, dtype=torch.int32, device=DEV)),
+    ]
+    for over in bad:
+        args = dict(M=M, X=X, y=y, dM=dM, dX=dX, dy=dy)
+        args.update(over)
+        with pytest.raises((ValueError, TypeError)):
+            adaptic.run_host("mv", args["M"], args["X"], args["y"], args["dM"], args["dX"], args["dy"])
