@@ -60,6 +60,7 @@ def parse():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-cublas", action="store_true", help="skip the cuBLAS sgemv context leg")
     ap.add_argument("--detail", default=None, help="write per-problem JSONL here")
     ap.add_argument("--kernel-events-in-timed", action="store_true",
                     help="record per-launch events inside the timed region (default: separate pass)")
@@ -539,6 +540,10 @@ def run_adaptic(args):
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cpu = cpu_baseline(probs, args)
+    cublas = None
+    if rank == 0 and world == 1 and args.workload in ("sweep", "offgrid", "rowshard", "splitk", "dot") \
+            and args.dtype == "f32" and not args.no_cublas:
+        cublas = cublas_context(probs, per)
     if args.detail and rank == 0:
         with open(args.detail, "w") as f:
             for q in per:
@@ -559,7 +564,7 @@ def run_adaptic(args):
                                    if args.workload == "config0" else
                                    "dot: lengths 2^10..2^30 back to back; the >= 2^25 ones exceed L2"
                                    if args.workload == "dot" else "inputs > L2; no flush needed")),
-                "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
+                "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "cublas_context": cublas,
                 "kernel_timing": ("per-launch CUDA events inside the timed region" if inner else
                                   f"per-kernel CUDA events after the timed region: each kernel 5x back to back, "
                                   f"{kev_steps} samples (the timed region itself has events only at its ends)"),
@@ -571,6 +576,44 @@ def run_adaptic(args):
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()
+
+
+def cublas_context(probs, per, reps=5, samples=5):
+    """The paper's Fig. 10 comparator (CUBLAS Sgemv; Fig. 1) on B200: torch.mv
+    (cuBLAS sgemv / dot) on the SAME resident inputs, outside the timed region; MV = A x,
+    TMV = B^T x (the transposed operand).  Context only -- not the metric."""
+    import torch
+    out, tot_b, tot_t = {}, 0, 0.0
+    ev = [torch.cuda.Event(enable_timing=True) for _ in range(2)]
+    for p, q in zip(probs, per):
+        if p.op == "mv":
+            f = (lambda M=p.M.view(p.R, p.C), x=p.X: torch.mv(M, x))
+        elif p.op == "tmv":
+            f = (lambda M=p.M.view(p.C, p.R), x=p.X: torch.mv(M.t(), x))
+        elif p.op == "dot" and p.R == 1:
+            f = (lambda a=p.M, b=p.X: torch.dot(a, b))
+        else:
+            continue
+        f()
+        torch.cuda.synchronize()
+        ts = []
+        for _ in range(samples):
+            ev[0].record()
+            for _ in range(reps):
+                f()
+            ev[1].record()
+            torch.cuda.synchronize()
+            ts.append(ev[0].elapsed_time(ev[1]) / reps)
+        t = statistics.median(ts)
+        out[f"{p.op} {p.R}x{p.C}"] = [round(p.bytes / (t / 1e3) / 1e9, 1), round(q["GBps"] / (p.bytes / (t / 1e3) / 1e9), 3)]
+        tot_b += p.bytes
+        tot_t += t
+    if not out:
+        return None
+    return {"value": tot_b / (tot_t / 1e3) / 1e9, "unit": UNIT, "api": "torch.mv / torch.dot (cuBLAS), same inputs",
+            "per_shape_GBps_and_adaptic_speedup": out,
+            "adaptic_speedup_min": min(v[1] for v in out.values()),
+            "adaptic_speedup_median": statistics.median(v[1] for v in out.values())}
 
 
 def measure_latency(p, reps=200):
@@ -615,7 +658,23 @@ def measure_latency(p, reps=200):
             evs[1].record(stream)
             evs[1].synchronize()
             cold.append(evs[0].elapsed_time(evs[1]) * 1e3)
-    return {"single_launch_median": statistics.median(single), "single_launch_min": min(single),
+    # plan latency (selection must add no visible time): through the Python binding
+    # (ctypes call + plan cache) and, when built, the C-level microbenchmark over 93 shapes
+    import paper_conf_pldi_samadihmlm12_b200 as adaptic
+    pl = []
+    for _ in range(2000):
+        t = time.perf_counter()
+        adaptic.plan("tmv", p.R, p.C)
+        pl.append(time.perf_counter() - t)
+    c_level = None
+    exe = os.path.join(ROOT, "tools", "plan_latency")
+    if os.path.exists(exe):
+        try:
+            c_level = json.loads(subprocess.check_output([exe, "2000"], text=True, timeout=60))
+        except Exception as e:  # noqa: BLE001 -- report, do not fail the bench
+            c_level = {"error": str(e)[:200]}
+    return {"plan_us_python_median": statistics.median(pl) * 1e6, "plan_c_abi": c_level,
+            "single_launch_median": statistics.median(single), "single_launch_min": min(single),
             "graph_amortized": amort, "graph_launches": reps,
             "l2_cold_median": statistics.median(cold), "l2_cold_note": "2x L2 scratch write before each launch",
             "variant": p.desc["variant"]}

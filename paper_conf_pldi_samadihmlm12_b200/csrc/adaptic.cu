@@ -414,6 +414,69 @@ adaptic_status derive_stencil(adaptic_plan_s* p, const int32_t* params, const De
 // Multi-vector MV / TMV (adaptic_plan_multi): K = nvec vectors share one pass over the
 // matrix (horizontal actor integration; mmv_kernels.cuh).  fp32, 128-bit path
 // shapes and scalar shapes alike (aligned pointers take the 128-bit instances).
+// TMV (any K, any alignment, any R) with B staged by TMA (tmv_ring_kernel.cuh): tiles of TW
+// outputs = WPT column groups of 32 OPT words, LC = 8 / WPT row lanes; one tile covering all
+// outputs streams whole rows (one contiguous copy per stage of ~32 KB), else CR row segments.
+// params: LANES = OPT, PIPE = stages (default 4: the measured optimum of a bare TMA stream)
+adaptic_status derive_tmv_ring(adaptic_plan_s* p, const int32_t* params, const DevInfo& dev) {
+    auto par = [&](int i) -> int { return params ? params[i] : 0; };
+    const int K = p->nvec;
+    const int64_t R = p->R, C = p->C;
+    const int opt_max = std::min(8, 32 / K);
+    const bool flat = R <= int64_t(256);                     // one tile, output per thread
+    int OPT = par(ADAPTIC_P_LANES);
+    if (OPT <= 0) OPT = flat ? 1 : clampi(pow2_floor(std::max<int64_t>(1, R / 256)), 1, opt_max);
+    if (OPT > opt_max || (OPT & (OPT - 1))) return ADAPTIC_ERR_INVALID_ARG;
+    if (!tmv_ring_fn(p->dtype, K, OPT)) return ADAPTIC_ERR_UNSUPPORTED;
+    const int WW = 32 * OPT;
+    // tile width: as wide as possible (long bulk copies), but the last CTA of a tile merges
+    // TW K outputs x (CTAs per tile ~ sms TW / R) partials -- keep that <= ~24 loads of
+    // 16 bytes per thread (measured: one 2048-word tile over 148 CTAs cost ~150 us to merge)
+    int WPT = flat ? 1 : clampi(pow2_ceil(ceil_div(R, int64_t(WW))), 1, 8);
+    if (par(ADAPTIC_P_ROWS) > 0) WPT = clampi(par(ADAPTIC_P_ROWS), 1, 8);
+    else
+        while (!flat && WPT > 1) {
+            const int64_t tw = int64_t(WW) * WPT;
+            const int64_t per_tile = ceil_div(int64_t(dev.sms) * tw, R) + 1;
+            if (tw * K * per_tile / 4 <= 24 * 256) break;
+            WPT /= 2;
+        }
+    const int TW = flat ? int(R) : WW * WPT, LC = 8 / WPT;
+    const bool contig = TW >= R;
+    // ~32 KB stages (B rows + their x chunks); row-segment stages take one producer lane per
+    // row, the x chunks the last K lanes
+    const int CR = contig ? int(std::max<int64_t>(1, std::min<int64_t>(C, (int64_t(8192) - 40 - 40 * int64_t(K)) / (R + K))))
+                          : std::max(1, std::min(32 - K, 8704 / (TW + 8 + K)));
+    const int64_t sw = tring_stage_words_h(R, TW, CR, K);
+    const int64_t red = (flat ? int64_t(int64_t(256) / R) * K * R : int64_t(LC - 1) * K * TW) * 4;
+    const int64_t fit = (MRING_SMEM_BUDGET - red) / (sw * 4);
+    const int stages = int(std::min<int64_t>(par(ADAPTIC_P_PIPE) > 0 ? std::min(8, par(ADAPTIC_P_PIPE)) : 4, fit));
+    if (stages < 2) return ADAPTIC_ERR_UNSUPPORTED;
+    const int64_t ntiles = ceil_div(R, int64_t(TW)), Tw = ntiles * C;
+    if (Tw > (int64_t(1) << 62) / 256) return ADAPTIC_ERR_UNSUPPORTED;
+    const int64_t grid = std::max<int64_t>(1, std::min<int64_t>(dev.sms, Tw));
+    const int64_t per = std::max<int64_t>(1, Tw / grid);
+    const int64_t maxs = C / per + 2;
+    if (maxs > int64_t(INT_MAX) / 64) return ADAPTIC_ERR_UNSUPPORTED;
+    const int64_t lanes = flat ? int64_t(256) / R : int64_t(LC);      // row lanes per output
+    const int64_t P = ceil_div(std::min(C, ceil_div(Tw, grid)), lanes);   // rows per thread per segment
+    p->xmode = 6; p->block = MRING_BLOCK; p->ctas_per_sm = 1;
+    p->ilv = par(ADAPTIC_P_ORDER) >= 8 ? par(ADAPTIC_P_ORDER) - 8 : 0;
+    p->lanes = TW; p->unroll = OPT; p->splits = CR; p->stages = stages; p->rb = int(maxs);
+    p->smem = size_t(int64_t(stages) * sw * 4 + red);
+    p->mis = false; p->flat = false; p->vec_shape = R % 4 == 0; p->xsh_off = 0; p->fb_ws_off = 0;
+    for (int w = 0; w < 2; ++w) {
+        p->grid[w] = grid;
+        p->chain[w] = std::min<int64_t>(P, FOLD) + P / FOLD;
+        p->depth[w] = lanes + ceil_div(maxs, 2) + 2;
+        p->path_ok[w] = bound_ok(p->chain[w] + p->depth[w]);
+    }
+    const size_t part = ((size_t(ntiles) * size_t(maxs) * size_t(K) * size_t(TW) * 4 + 255) / 256) * 256;
+    p->cnt_off = part;
+    p->ws_bytes = part + size_t(ntiles) * 4;
+    return p->path_ok[1] ? ADAPTIC_OK : ADAPTIC_ERR_UNSUPPORTED;
+}
+
 adaptic_status derive_multi(adaptic_plan_s* p, const int32_t* params, const DevInfo& dev) {
     const int op = p->op, v = p->variant, K = p->nvec;
     const int64_t R = p->R, C = p->C;
@@ -467,6 +530,45 @@ adaptic_status derive_multi(adaptic_plan_s* p, const int32_t* params, const DevI
             p->path_ok[w] = bound_ok(p->chain[w] + p->depth[w]);
         }
         return p->path_ok[p->vec_shape ? 1 : 0] ? ADAPTIC_OK : ADAPTIC_ERR_UNSUPPORTED;
+    }
+    // AUTO multi-vector MV_SPLIT with long rows (C >= 8192): the matrix through the TMA ring
+    // (measured, scratch r2f: 64 x 1M K = 4 0.66 -> 0.85 of the copy peak, K = 8 0.36 -> 0.67;
+    // 16384 x 4096 and shorter rows: the x-tile kernel is as fast or faster)
+    const bool ring_rule = K > 1 && v == ADAPTIC_V_MV_SPLIT && par(ADAPTIC_P_XSMEM) <= 0 && C >= 8192;
+    if (op == ADAPTIC_OP_MV && (v == ADAPTIC_V_MV_CPR || v == ADAPTIC_V_MV_SPLIT) && p->vec_shape &&
+        (par(ADAPTIC_P_XSMEM) == 6 || ring_rule)) {
+        // the matrix through a TMA ring (mmv_ring_kernel.cuh): groups of 8 rows, 256-float4
+        // stages, stream-K over the (group, column) positions of one CTA per SM
+        constexpr int RT = 8, CH = 256, FOLDP = 128, NT = 256;
+        const int64_t nv = C / 4, ngroups = ceil_div(R, RT), Tw = ngroups * nv;
+        const int cps = std::max(1, std::min(2, par(ADAPTIC_P_CTAS_PER_SM)));     // CTAs per SM
+        const int64_t grid = std::max<int64_t>(1, std::min<int64_t>(int64_t(dev.sms) * cps, Tw));
+        const int64_t xbytes = int64_t(K) * C * 4;
+        const bool xres = xbytes <= 64 * 1024 / cps;
+        const int64_t stage = int64_t(RT + (xres ? 0 : K)) * CH * 16;
+        // 4 stages of 32 KB of A in flight per SM is the measured optimum of a bare TMA
+        // stream (7.1 TB/s; 6 stages: 6.5 TB/s -- too many requests in flight, scratch r2h)
+        const int64_t fit = (MRING_SMEM_BUDGET / cps - (xres ? xbytes : 0)) / stage;
+        int stages = int(std::min<int64_t>(par(ADAPTIC_P_PIPE) > 0 ? std::min(8, par(ADAPTIC_P_PIPE)) : 4, fit));
+        if (stages < 2 || !mmv_ring_fn(p->dtype, K)) return ADAPTIC_ERR_UNSUPPORTED;
+        if (Tw > (int64_t(1) << 62) / 256) return ADAPTIC_ERR_UNSUPPORTED;
+        const int64_t per = std::max<int64_t>(1, Tw / grid);     // shortest CTA range
+        const int64_t maxs = nv / per + 2;                       // CTAs touching one group
+        if (maxs > int64_t(INT_MAX) / 64) return ADAPTIC_ERR_UNSUPPORTED;
+        const int N = RT * K, NG = NT / N;
+        const int64_t P = ceil_div(std::min(nv, ceil_div(Tw, grid)), int64_t(CH));   // positions / segment
+        p->smem = size_t((xres ? xbytes : 0) + int64_t(stages) * stage);
+        p->xmode = 6;
+        p->block = MRING_BLOCK; p->ctas_per_sm = cps; p->splits = 1; p->unroll = 1;
+        p->stages = stages; p->lanes = (xres ? 1 : 0) | (par(ADAPTIC_P_ORDER) == 9 ? 2 : 0); p->rb = int(maxs);
+        p->grid[1] = grid;
+        p->chain[1] = 4 * std::min<int64_t>(P, FOLDP) + P / FOLDP;
+        p->depth[1] = 5 + (NT / 32) + ceil_div(maxs, NG) + NG + 1;
+        p->path_ok[1] = bound_ok(p->chain[1] + p->depth[1]);
+        const size_t part = ((size_t(ngroups) * size_t(maxs) * size_t(N) * 4 + 255) / 256) * 256;
+        p->cnt_off = part;
+        p->ws_bytes = part + size_t(ngroups) * 4;
+        return p->path_ok[1] ? ADAPTIC_OK : ADAPTIC_ERR_UNSUPPORTED;
     }
     if (op == ADAPTIC_OP_MV && (v == ADAPTIC_V_MV_CPR || v == ADAPTIC_V_MV_SPLIT) && p->vec_shape &&
         (par(ADAPTIC_P_XSMEM) == 3 ||
@@ -563,6 +665,7 @@ adaptic_status derive_multi(adaptic_plan_s* p, const int32_t* params, const DevI
         return ADAPTIC_OK;
     }
     if (op != ADAPTIC_OP_TMV || !is_tmv_family(v)) return ADAPTIC_ERR_UNSUPPORTED;
+    if (par(ADAPTIC_P_XSMEM) == 6) return derive_tmv_ring(p, params, dev);
     // TMV tiles: LR output vectors x (256 / LR) c-lanes, S c-ranges
     const int NT = 256;
     int U = par(ADAPTIC_P_UNROLL);
@@ -931,8 +1034,9 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
     }
     // single-vector MV (fp32 or int32) on the x-tile stream-K kernel (param XSMEM 3)
     if (op == ADAPTIC_OP_MV && (v == ADAPTIC_V_MV_CPR || v == ADAPTIC_V_MV_SPLIT) &&
-        par(ADAPTIC_P_XSMEM) == 3 && C % 4 == 0)
+        (par(ADAPTIC_P_XSMEM) == 3 || par(ADAPTIC_P_XSMEM) == 6) && C % 4 == 0)
         return derive_multi(p, params, dev);
+    if (op == ADAPTIC_OP_TMV && par(ADAPTIC_P_XSMEM) == 6) return derive_tmv_ring(p, params, dev);
     if (op == ADAPTIC_OP_STENCIL5) return derive_stencil(p, params, dev);
     if (is_b1_op(op)) return derive_b1(p, params, dev);
 
@@ -1355,6 +1459,12 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
     void* args6[6];
     void** args = nullptr;
     int stages = p->stages;
+    int ring_xres = p->lanes, ring_maxs = p->rb;   // mmv_ring_kernel: x resident, partial slots
+    void* args10[10];
+    int tr_tw = p->lanes, tr_cr = p->splits;       // tmv_ring_kernel: tile width, rows per stage
+    int tr_sw = p->xmode == 6 && p->op == ADAPTIC_OP_TMV ? int(tring_stage_words_h(p->R, p->lanes, p->splits, p->nvec)) : 0;
+    void* args12[13];
+    int tr_dbg = p->ilv;                           // experiments only (param ORDER 8 + d)
 
     void* args7[7];
     if (mis && p->xmode == XM_SHIFT_MODE && p->op == ADAPTIC_OP_MV && p->nvec == 1 &&
@@ -1399,13 +1509,24 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
         }
     } else if (p->nvec > 1) {
         const int K = p->nvec;
-        if (p->op == ADAPTIC_OP_TMV && p->xmode == 5) { fn = vec ? tmmv_tma_fn(K, p->lanes) : nullptr; smem = p->smem; }
+        if (p->op == ADAPTIC_OP_TMV && p->xmode == 6) { fn = tmv_ring_fn(ADAPTIC_F32, K, p->unroll); smem = p->smem; }
+        else if (p->op == ADAPTIC_OP_TMV && p->xmode == 5) { fn = vec ? tmmv_tma_fn(K, p->lanes) : nullptr; smem = p->smem; }
         else if (p->op == ADAPTIC_OP_TMV) fn = tmmv_fn(K, p->lanes, p->unroll, vec);
         else if (p->xmode == 4) { fn = vec ? mmv_tile_fn(ADAPTIC_F32, K) : nullptr; smem = p->smem; }
+        else if (p->xmode == 6) { fn = vec ? mmv_ring_fn(ADAPTIC_F32, K) : nullptr; smem = p->smem; }
         else if (p->xmode == 3) { fn = mmv_warp_fn(K); smem = p->smem; }
         else if (p->variant == ADAPTIC_V_MV_SUBWARP || p->variant == ADAPTIC_V_MV_WPR) fn = mmv_group_fn(K, p->lanes, p->unroll, vec);
         else { fn = mmv_cta_fn(K, p->unroll, vec, p->xmode == 1); smem = p->smem; }
-        if (p->op == ADAPTIC_OP_MV && p->xmode == 4) {
+        if (p->op == ADAPTIC_OP_TMV && p->xmode == 6) {
+            args12[0] = &A; args12[1] = &X; args12[2] = &y; args12[3] = &R; args12[4] = &C;
+            args12[5] = &tr_tw; args12[6] = &tr_cr; args12[7] = &stages; args12[8] = &tr_sw; args12[9] = &ring_maxs;
+            args12[10] = &part; args12[11] = &cnt; args12[12] = &tr_dbg;
+            args = args12;
+        } else if (p->op == ADAPTIC_OP_MV && p->xmode == 6) {
+            args10[0] = &A; args10[1] = &X; args10[2] = &y; args10[3] = &R; args10[4] = &C;
+            args10[5] = &stages; args10[6] = &ring_xres; args10[7] = &ring_maxs; args10[8] = &part; args10[9] = &cnt;
+            args = args10;
+        } else if (p->op == ADAPTIC_OP_MV && p->xmode == 4) {
             args9[0] = &A; args9[1] = &X; args9[2] = &y; args9[3] = &R; args9[4] = &C;
             args9[5] = &tile_cw; args9[6] = &tile_mb; args9[7] = &part; args9[8] = &cnt;
             args = args9;
@@ -1461,6 +1582,14 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
             break;
         case ADAPTIC_V_MV_CPR:
         case ADAPTIC_V_MV_SPLIT:
+            if (p->xmode == 6) {                          // TMA-ring kernel, K = 1
+                fn = vec ? mmv_ring_fn(dt, 1) : nullptr;
+                smem = p->smem;
+                args10[0] = &A; args10[1] = &X; args10[2] = &y; args10[3] = &R; args10[4] = &C;
+                args10[5] = &stages; args10[6] = &ring_xres; args10[7] = &ring_maxs; args10[8] = &part; args10[9] = &cnt;
+                args = args10;
+                break;
+            }
             if (p->xmode == 4) {                          // x-tile stream-K kernel, K = 1
                 fn = vec ? mmv_tile_fn(dt, 1) : nullptr;
                 smem = p->smem;
@@ -1477,6 +1606,15 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
             args = args9;
             break;
         default:
+            if (p->xmode == 6) {                          // TMV with B through the TMA ring
+                fn = tmv_ring_fn(dt, 1, p->unroll);
+                smem = p->smem;
+                args12[0] = &A; args12[1] = &X; args12[2] = &y; args12[3] = &R; args12[4] = &C;
+                args12[5] = &tr_tw; args12[6] = &tr_cr; args12[7] = &stages; args12[8] = &tr_sw; args12[9] = &ring_maxs;
+                args12[10] = &part; args12[11] = &cnt; args12[12] = &tr_dbg;
+                args = args12;
+                break;
+            }
             if (p->xmode == 4) {                          // TMV on staged tiles of B
                 fn = tmv_rowtile_fn(dt, p->block, p->unroll);
                 smem = p->smem;
@@ -1670,6 +1808,8 @@ adaptic_status adaptic_run(adaptic_plan_t p, const void* A, const void* x, void*
         vec = aligned(A, 16) && aligned(y, 16);
     } else if (vec && p->nvec > 1) {
         vec = aligned(A, 16) && aligned(x, 16) && aligned(y, 16);
+        if (!vec && p->op == ADAPTIC_OP_TMV && p->xmode == 6)          // the TMV ring takes any alignment
+            return launch(p, A, x, y, stream, false, false);
         if (!vec) {                               // 4-byte-aligned pointers: the planned fallback
             adaptic_plan_s fb;
             if (!p->multi_fb_ok || !multi_fallback(*p, &fb, device_info())) return ADAPTIC_ERR_MISALIGNED;
@@ -1708,7 +1848,7 @@ adaptic_status adaptic_run(adaptic_plan_t p, const void* A, const void* x, void*
         }
         return adaptic_run(&fb, A, x, y, stream_);
     }
-    if (!vec && p->nvec == 1 && p->xmode == 4) {
+    if (!vec && p->nvec == 1 && (p->xmode == 4 || (p->xmode == 6 && p->op == ADAPTIC_OP_MV))) {
         // the x-tile kernel needs 16-byte rows and bases (TMA): a single-vector plan run on
         // 4-byte-aligned pointers takes the CTA-per-row kernel of the same shape instead
         adaptic_plan_s fb = *p;

@@ -86,6 +86,19 @@ void* mmv_tile_fn(int dt, int K);
 //   tmma : tmmv arguments; B rows staged by TMA in TMMV_TMA_STAGES stages of
 //          TMMV_TMA_STAGE_V4 float4 (CR = STAGE_V4 / LR rows of LR float4), NT = 256, LR in {16..256}
 void* tmmv_tma_fn(int K, int LR);
+//   ring : (A, X, Y, R, C, int stages, int xres, int maxs, T* part, unsigned* cnt): the MATRIX
+//          staged by TMA in an mbarrier ring (producer warp + 8 consumer warps, NT = 288),
+//          groups of 8 rows x 256-float4 stages, stream-K over (group, column) positions;
+//          K in {1, 2, 4, 8} (fp32), K = 1 also int32 (mmv_ring_kernel.cuh)
+void* mmv_ring_fn(int dt, int K);
+constexpr int MRING_BLOCK = 288;
+//   tring: (B, X, Y, R, C, int TW, int CR, int stages, int stage_words, int maxs, T* part,
+//          unsigned* cnt): TMV with B staged by TMA (tiles of TW outputs, CR rows per stage,
+//          16-byte covers of any alignment), NT = 288; fp32 K in {1,2,4,8}, int32 K = 1;
+//          opt = words per lane per row (tmv_ring_kernel.cuh)
+void* tmv_ring_fn(int dt, int K, int opt);
+int64_t tring_stage_words_h(int64_t R, int TW, int CR, int K);
+constexpr int64_t MRING_SMEM_BUDGET = 220 * 1024;
 constexpr int TMMV_TMA_STAGE_V4 = 2048;              // 32 KB per stage
 constexpr int TMMV_TMA_STAGES = 3;
 constexpr int64_t MMV_TILE_XBYTES = 32 * 1024;       // x bytes per piece (all K vectors)
