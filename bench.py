@@ -745,40 +745,60 @@ def measure_e2e(args, probs, world, bucket=None, partitioned=False):
 
 
 def cpu_baseline(probs, args, budget_s: float = 20.0):
-    """The fp64 oracle as it stands, single-threaded, on the box's host cores, over a
-    bounded sample of the workload's problems (inputs copied from HBM)."""
+    """The fp64 oracle as it stands, single-threaded and PINNED to one host core
+    (os.sched_setaffinity), best of 3 per problem, over a bounded
+    sample of the workload's problems (inputs copied from HBM first)."""
     import numpy as np
     import oracle
     t_total, b_total, names = 0.0, 0, []
     order = sorted(range(len(probs)), key=lambda i: (i * 7) % len(probs))
-    for i in order:
-        p = probs[i]
-        M = p.M.cpu().numpy()
-        X = p.X.cpu().numpy()
-        t = time.perf_counter()
-        if p.op == "mv":
-            for j in range(p.nvec):
-                oracle.mv(M.reshape(p.R, p.C), X[j * p.C:(j + 1) * p.C])
-        elif p.op == "tmv":
-            for j in range(p.nvec):
-                oracle.tmv(M.reshape(p.C, p.R), X[j * p.C:(j + 1) * p.C])
-        elif p.op == "stencil5":
-            oracle.stencil5(M.reshape(p.R, p.C), float(X[0]), float(X[1]))
-        elif p.op in B1_OPS:
-            for f in (("asum", "nrm2", "iamax", "iamin") if p.op == "b1all" else (p.op,)):
-                getattr(oracle, f)(M.reshape(p.R, p.C))
-        else:
-            oracle.dot(M.reshape(p.R, p.C), X.reshape(p.R, p.C))
-        t_total += time.perf_counter() - t
-        b_total += p.bytes
-        names.append(f"{p.op} {p.R}x{p.C}")
-        del M, X
-        if t_total > budget_s:
-            break
+    old_aff = os.sched_getaffinity(0)
+    core = min(old_aff)
+    os.sched_setaffinity(0, {core})
+    spent = 0.0
+    try:
+        for i in order:
+            p = probs[i]
+            M = p.M.cpu().numpy()
+            X = p.X.cpu().numpy()
+
+            def run():
+                if p.op == "mv":
+                    for j in range(p.nvec):
+                        oracle.mv(M.reshape(p.R, p.C), X[j * p.C:(j + 1) * p.C])
+                elif p.op == "tmv":
+                    for j in range(p.nvec):
+                        oracle.tmv(M.reshape(p.C, p.R), X[j * p.C:(j + 1) * p.C])
+                elif p.op == "stencil5":
+                    oracle.stencil5(M.reshape(p.R, p.C), float(X[0]), float(X[1]))
+                elif p.op in B1_OPS:
+                    for fn in (("asum", "nrm2", "iamax", "iamin") if p.op == "b1all" else (p.op,)):
+                        getattr(oracle, fn)(M.reshape(p.R, p.C))
+                else:
+                    oracle.dot(M.reshape(p.R, p.C), X.reshape(p.R, p.C))
+            best = None
+            for _ in range(3):
+                t = time.perf_counter()
+                run()
+                dt = time.perf_counter() - t
+                spent += dt
+                best = dt if best is None else min(best, dt)
+                if spent > budget_s:
+                    break
+            t_total += best
+            b_total += p.bytes
+            names.append(f"{p.op} {p.R}x{p.C}")
+            del M, X
+            if spent > budget_s:
+                break
+    finally:
+        os.sched_setaffinity(0, old_aff)
+    import platform
     return {"value": b_total / t_total / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
-            "seconds": t_total, "host_cores_available": os.cpu_count(),
-            "sample": f"{len(names)} of {len(probs)} problems, full size: " + ", ".join(names[:6])
-                      + (" ..." if len(names) > 6 else "")}
+            "seconds": t_total, "host_cores_available": os.cpu_count(), "pinned_core": core, "best_of": 3,
+            "cpu": platform.processor() or platform.machine(),
+            "sample": f"{len(names)} of {len(probs)} problems, full size, best of 3 each on one pinned core: "
+                      + ", ".join(names[:6]) + (" ..." if len(names) > 6 else "")}
 
 
 # ------------------------------------------------------------------------------ reference arm
