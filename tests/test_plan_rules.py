@@ -39,8 +39,10 @@ def test_tile_kernel_cells_fp32_and_int32():
 
 
 def test_multi_vector_rules():
-    assert d("mv", 8192, 8192, nvec=4)["xmode"] == 4               # x-tile stream-K
-    assert d("mv", 8, 1 << 23, nvec=4)["xmode"] != 4               # R <= 16: interleaved splits
+    assert d("mv", 16384, 4096, nvec=4)["xmode"] == 4              # x-tile stream-K (C < 8192)
+    assert d("mv", 8192, 8192, nvec=4)["xmode"] == 6               # long rows: the matrix via the TMA ring
+    assert d("mv", 64, 1 << 20, nvec=8)["xmode"] == 6
+    assert d("mv", 8, 1 << 23, nvec=4)["xmode"] == 6                # (round 1: interleaved splits)
     assert d("mv", 1 << 20, 64, nvec=4)["variant"] == "MV_SUBWARP"  # short rows: x in registers
     few = d("tmv", 64, 1 << 20, nvec=4)
     assert few["xmode"] == 5 and few["lanes"] == 16                 # one contiguous TMA tile
