@@ -50,7 +50,7 @@ def parse():
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", choices=["adaptic", "reference"], default="adaptic")
-    ap.add_argument("--workload", choices=["sweep", "offgrid", "rowshard", "splitk", "dot", "blas1", "config0", "multi", "bicgstab", "stencil"], default="sweep")
+    ap.add_argument("--workload", choices=["sweep", "offgrid", "rowshard", "splitk", "dot", "blas1", "config0", "multi", "bicgstab", "stencil", "small"], default="sweep")
     ap.add_argument("--variant", default="AUTO", help="force one variant (fixed-variant sweeps)")
     ap.add_argument("--dtype", choices=["f32", "i32"], default="f32",
                     help="element type of the MV/TMV/DOT workloads (i32: arithmetic modulo 2^32)")
@@ -871,6 +871,122 @@ def run_reference(args):
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}), flush=True)
 
 
+def run_small(args):
+    """The paper's own input sizes (P:614 Sdot 1K..4M, P:914-1240 the 1M..16M-element grid):
+    MV/TMV diagonals of 2^20, 2^22, 2^24 elements (4-64 MiB) and Sdot N = 1, L = 2^10..2^22,
+    all L2-resident.  Per shape: single-launch latency (events around one adaptic_run,
+    host enqueue included), graph-amortized L2-hot time, and L2-cold time (2 x L2 of scratch
+    written before each launch), against a launch floor (the same measures on MV 1 x 4) and
+    the L2 bandwidth of a device copy of a 16 MiB buffer (L2-resident)."""
+    import torch
+    import synth
+    import paper_conf_pldi_samadihmlm12_b200 as adaptic
+    from paper_conf_pldi_samadihmlm12_b200 import _lib as L
+    world, rank, _ = dist_setup(args)
+    dev = torch.device("cuda", torch.cuda.current_device())
+    stream = torch.cuda.Stream()
+    l2 = torch.cuda.get_device_properties(dev).L2_cache_size
+    scratch = torch.empty(2 * l2 // 4 + 1024, dtype=torch.float32, device=dev)
+    ev = [torch.cuda.Event(enable_timing=True) for _ in range(2)]
+
+    def measure(fn, reps=100):
+        with torch.cuda.stream(stream):
+            for _ in range(10):
+                fn()
+            torch.cuda.synchronize()
+            single = []
+            for _ in range(30):
+                ev[0].record(stream)
+                fn()
+                ev[1].record(stream)
+                ev[1].synchronize()
+                single.append(ev[0].elapsed_time(ev[1]) * 1e3)
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g, stream=stream):
+                for _ in range(reps):
+                    fn()
+            g.replay()
+            torch.cuda.synchronize()
+            ev[0].record(stream)
+            for _ in range(3):
+                g.replay()
+            ev[1].record(stream)
+            torch.cuda.synchronize()
+            hot = ev[0].elapsed_time(ev[1]) * 1e3 / (3 * reps)
+            cold = []
+            for _ in range(15):
+                scratch.fill_(1.0)
+                ev[0].record(stream)
+                fn()
+                ev[1].record(stream)
+                ev[1].synchronize()
+                cold.append(ev[0].elapsed_time(ev[1]) * 1e3)
+        return statistics.median(single), hot, statistics.median(cold)
+
+    # L2 bandwidth reference: device copy of a 16 MiB buffer, back to back (read + write bytes)
+    a16 = torch.empty(4 << 20, device=dev)
+    b16 = torch.empty_like(a16)
+    with torch.cuda.stream(stream):
+        for _ in range(5):
+            b16.copy_(a16)
+        torch.cuda.synchronize()
+        ev[0].record(stream)
+        for _ in range(200):
+            b16.copy_(a16)
+        ev[1].record(stream)
+        torch.cuda.synchronize()
+    l2_copy = 2 * a16.numel() * 4 * 200 / (ev[0].elapsed_time(ev[1]) / 1e3) / 1e9
+    # and an L2-resident READ: torch.sum over 32 MiB (the inputs here are read-mostly)
+    a32 = torch.ones(8 << 20, device=dev)
+    with torch.cuda.stream(stream):
+        for _ in range(5):
+            a32.sum()
+        torch.cuda.synchronize()
+        ev[0].record(stream)
+        for _ in range(200):
+            a32.sum()
+        ev[1].record(stream)
+        torch.cuda.synchronize()
+    l2_read = a32.numel() * 4 * 200 / (ev[0].elapsed_time(ev[1]) / 1e3) / 1e9
+    l2_gbs = max(l2_copy, l2_read)
+
+    shapes = [(op, 1 << k, 1 << (e - k)) for e in (20, 22, 24) for k in (3, 7, 11, 15) for op in ("mv", "tmv")] + \
+             [("dot", 1, 1 << k) for k in range(10, 23, 2)] + [("mv", 1, 4)]
+    out, tot_b, tot_t = [], 0, 0.0
+    floor = None
+    for op, R, C in shapes:
+        M = torch.empty(R * C, device=dev)
+        synth.device_matrix(M, R, C, "tmv" if op == "tmv" else "mv", "uniform", synth.seed(5, "A"))
+        X = torch.empty(R * C if op == "dot" else C, device=dev)
+        synth.device_vector(X, "uniform", synth.seed(5, "x"))
+        y = torch.empty(R, device=dev)
+        plan = adaptic.get_plan(L.OPS[op], R, C, L.F32, dev, "AUTO", None, stream.cuda_stream)
+        ptrs = (M.data_ptr(), X.data_ptr(), y.data_ptr())
+        single, hot, cold = measure(lambda: plan.run(*ptrs, torch.cuda.current_stream().cuda_stream))
+        nb = algo_bytes(op, R, C)
+        rec = {"op": op, "R": R, "C": C, "bytes": nb, "variant": plan.describe()["variant"],
+               "single_us": single, "hot_us": hot, "cold_us": cold, "hot_GBps": nb / hot / 1e3,
+               "cold_GBps": nb / cold / 1e3, "hot_frac_l2": nb / hot / 1e3 / l2_gbs}
+        if (op, R, C) == ("mv", 1, 4):
+            floor = rec
+            continue
+        out.append(rec)
+        tot_b += nb
+        tot_t += hot
+    for r in out:
+        r["hot_over_floor"] = r["hot_us"] / floor["hot_us"]
+    if rank == 0:
+        print(json.dumps({
+            "metric": METRIC, "value": tot_b / tot_t / 1e3, "unit": UNIT, "n_gpus": world, "steps": 1, "warmup": 10,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
+            "data": "synthetic (seeded splitmix64; fp32 U[-1,1))",
+            "config": {"workload": "the paper's small inputs: MV/TMV 2^20..2^24 elements (4-64 MiB), Sdot 1K..4M; "
+                                   "L2-resident: value = bytes / graph-amortized L2-hot time",
+                       "l2": "inputs fit in L2 by design; cold_us adds a 2 x L2 scratch write before each launch"},
+            "launch_floor": floor, "l2_copy_gbs": l2_copy, "l2_read_sum_gbs": l2_read,
+            "l2_ref_gbs": l2_gbs, "shapes": out}), flush=True)
+
+
 def run_bicgstab(args):
     """One step = one BiCGSTAB iteration on an n x n diagonally dominant system (device
     resident); value = algorithmic bytes / s (2 MVs of 4(n^2 + 2n) bytes plus the
@@ -946,5 +1062,7 @@ if __name__ == "__main__":
         run_reference(a)
     elif a.workload == "bicgstab":
         run_bicgstab(a)
+    elif a.workload == "small":
+        run_small(a)
     else:
         run_adaptic(a)

@@ -581,6 +581,10 @@ adaptic_status derive_multi(adaptic_plan_s* p, const int32_t* params, const DevI
         if (CW <= 0) CW = (int64_t(K) * C * 4 <= MMV_TILE_ONE_CHUNK) ? C : MMV_TILE_XBYTES / (4 * K);
         if (CW <= 0 || CW % 4 != 0 || 2 * int64_t(K) * CW * 4 > kXsMaxBytes) return ADAPTIC_ERR_INVALID_ARG;
         CW = std::min<int64_t>(CW, C);
+        // balanced chunks: a table width fitted on C = 2^k (an exact multiple) would leave the
+        // last chunk of another C mostly empty (held-out 6144 x 26624: 1.6 chunks of 16384, 0.86
+        // of the best plan); the same number of chunks, evenly filled
+        CW = std::min<int64_t>(CW, (ceil_div(C, ceil_div(C, CW)) + 3) / 4 * 4);
         const int64_t nch = ceil_div(C, CW);
         int MB = par(ADAPTIC_P_ROWS);
         if (MB <= 0) {
@@ -1242,6 +1246,40 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
     }
     const bool tmis = !p->vec_shape && R >= 8;
     p->mis = tmis;
+    if (tmis && (v == ADAPTIC_V_TMV_SPLITK || v == ADAPTIC_V_TMV_COL) && par(ADAPTIC_P_XSMEM) == 7) {
+        // constant word shift per c-lane (tmv_shift_kernel): one aligned load per row, no funnel
+        int LR = par(ADAPTIC_P_LANES);
+        if (LR <= 0) LR = clampi(pow2_ceil(ceil_div(R + 4, 4)), 16, 64);
+        int U = par(ADAPTIC_P_UNROLL);
+        if (U <= 0) U = 4;
+        if (!tmv_shift_fn(dt, LR, U)) return ADAPTIC_ERR_INVALID_ARG;
+        const int NT = 256, LC = NT / LR, WT = 4 * LR - 4;
+        int cps = par(ADAPTIC_P_CTAS_PER_SM);
+        if (cps <= 0) cps = occupancy(tmv_shift_fn(dt, LR, U), NT, 0, dev.present, 2048 / NT);
+        const int64_t slots = int64_t(dev.sms) * cps;
+        const int64_t tiles = ceil_div(R, int64_t(WT));
+        int64_t S = par(ADAPTIC_P_SPLITS) > 0 ? par(ADAPTIC_P_SPLITS)
+                                              : pick_splits(tiles, slots, std::max<int64_t>(1, ceil_div(C, int64_t(LC) * U)), 1);
+        for (;;) {
+            const int64_t iters = ceil_div(ceil_div(C, S), int64_t(LC) * U);
+            p->chain[1] = fold_chain(iters);
+            p->depth[1] = ilog2c(U) + LC + (S > 1 ? ceil_div(S, 2) + 1 : 0) + 1;
+            p->path_ok[1] = (dt == DT_I32) || bound_ok(p->chain[1] + p->depth[1]);
+            if (p->path_ok[1] || S >= (int64_t(1) << 20)) break;
+            S *= 2;
+        }
+        if (S > INT_MAX || !p->path_ok[1]) return ADAPTIC_ERR_UNSUPPORTED;
+        p->xmode = 7;
+        p->lanes = LR; p->unroll = U; p->block = NT; p->ctas_per_sm = cps; p->splits = int(S);
+        p->grid[1] = std::max<int64_t>(1, std::min<int64_t>(tiles * S, slots));
+        p->grid[0] = p->grid[1]; p->chain[0] = p->chain[1]; p->depth[0] = p->depth[1]; p->path_ok[0] = p->path_ok[1];
+        if (S > 1) {
+            const size_t part = ((size_t(tiles) * size_t(WT) * size_t(S) * 4 + 255) / 256) * 256;
+            p->cnt_off = part;
+            p->ws_bytes = part + size_t(tiles) * 4;
+        }
+        return ADAPTIC_OK;
+    }
     const int64_t rv1 = p->vec_shape ? R / 4 : tmis ? ceil_div(R, 4) : R;
     int LR = par(ADAPTIC_P_LANES);
     if (LR <= 0) {
@@ -1630,7 +1668,8 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
                 args = args7;
                 break;
             }
-            fn = mis ? tmv_mis_fn(dt, p->lanes, p->unroll) : tmv_fn(dt, p->lanes, p->unroll, vec, p->block);
+            fn = (mis && p->xmode == 7) ? tmv_shift_fn(dt, p->lanes, p->unroll)
+                 : mis ? tmv_mis_fn(dt, p->lanes, p->unroll) : tmv_fn(dt, p->lanes, p->unroll, vec, p->block);
             args8[0] = &A; args8[1] = &X; args8[2] = &y; args8[3] = &R; args8[4] = &C;
             args8[5] = &S; args8[6] = &part; args8[7] = &cnt;
             args = args8;

@@ -1,0 +1,33 @@
+// Instances of the constant-shift misaligned TMV kernel (tmv_mis_kernel.cuh, round 2):
+// fp32 and int32 (uint32 arithmetic), LR in {16, 32, 64} (c-lanes 16, 8, 4), U in {2, 4, 8},
+// NT = 256.
+#include "tmv_mis_kernel.cuh"
+#include "adaptic.h"
+
+namespace adaptic {
+
+template <class T, int LR>
+static void* ts_u(int U) {
+    switch (U) {
+        case 2: return reinterpret_cast<void*>(&tmv_shift_kernel<T, LR, 2, 256>);
+        case 4: return reinterpret_cast<void*>(&tmv_shift_kernel<T, LR, 4, 256>);
+        case 8: return reinterpret_cast<void*>(&tmv_shift_kernel<T, LR, 8, 256>);
+        default: return nullptr;
+    }
+}
+
+template <class T>
+static void* ts_l(int LR, int U) {
+    switch (LR) {
+        case 16: return ts_u<T, 16>(U);
+        case 32: return ts_u<T, 32>(U);
+        case 64: return ts_u<T, 64>(U);
+        default: return nullptr;
+    }
+}
+
+void* tmv_shift_fn(int dt, int LR, int U) {
+    return dt == ADAPTIC_I32 ? ts_l<uint32_t>(LR, U) : ts_l<float>(LR, U);
+}
+
+}  // namespace adaptic

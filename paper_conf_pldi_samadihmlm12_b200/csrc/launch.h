@@ -97,6 +97,10 @@ constexpr int MRING_BLOCK = 288;
 //          16-byte covers of any alignment), NT = 288; fp32 K in {1,2,4,8}, int32 K = 1;
 //          opt = words per lane per row (tmv_ring_kernel.cuh)
 void* tmv_ring_fn(int dt, int K, int opt);
+//   tshift: tmv arguments (B, X, y, R, C, S, part, cnt); rows off the 16-byte grid, one aligned
+//           128-bit load per row and thread at a constant word shift per c-lane; tiles of
+//           4 LR - 4 outputs, LR in {16, 32, 64}, U in {2, 4, 8}, NT = 256 (tmv_mis_kernel.cuh)
+void* tmv_shift_fn(int dt, int LR, int U);
 int64_t tring_stage_words_h(int64_t R, int TW, int CR, int K);
 constexpr int64_t MRING_SMEM_BUDGET = 220 * 1024;
 constexpr int TMMV_TMA_STAGE_V4 = 2048;              // 32 KB per stage

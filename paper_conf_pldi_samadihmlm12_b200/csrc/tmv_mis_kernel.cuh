@@ -147,3 +147,118 @@ tmv_mis_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restrict__
 }
 
 }  // namespace adaptic
+
+namespace adaptic {
+
+// Rows off the 16-byte grid WITHOUT the funnel (round 2).  With c-lanes LC a multiple of 4,
+// the rows a thread visits (c = c0 + lc + LC k) all have the same word shift
+// sh = (b0 + (c0 + lc) R) mod 4, so a thread can stream ONE aligned 128-bit vector per row
+// -- the aligned kernel's instruction mix -- and simply remember which outputs its four
+// words belong to: thread (lr, lc) of tile t accumulates words 4 lr .. 4 lr + 3 of the
+// aligned window that starts at output ob = t WT, i.e. outputs ob - sh + 4 lr + j.  A tile
+// owns WT = 4 LR - 4 outputs (the window's 4 LR words cover them at any shift; the extra
+// vector per row is re-read by the neighbouring tile: 1 / LR more L2 traffic), and the
+// c-lane combine sums, per owned output, each lane's word at its own shift, in lane order.
+// Tiling, splits and the ticket merge as tmv_kernel; B's first / last 16 bytes are loaded
+// word by word (ld_inside).
+template <class T, int LR, int U, int NT>
+__global__ void __launch_bounds__(NT, U <= 2 ? 4 : U <= 4 ? 3 : 2)
+tmv_shift_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restrict__ y,
+                 int64_t R, int64_t C, int S, T* __restrict__ ws_part, unsigned int* __restrict__ ws_cnt)
+{
+    pdl_prologue();
+    using E = vec4_t<T>;
+    constexpr int LC = NT / LR;
+    static_assert(LC % 4 == 0, "c-lanes: a multiple of 4 (one word shift per c-lane)");
+    constexpr int WT = 4 * LR - 4;                    // outputs owned by a tile
+    __shared__ T red[LC * 4 * LR];                    // [lc][4 lr + j]
+    __shared__ unsigned int flag;
+    const int64_t ntiles = (R + WT - 1) / WT;
+    const int64_t Rp = ntiles * WT;                   // partial row length
+    const int64_t chunk = (C + S - 1) / S;
+    const int b0 = int((reinterpret_cast<uintptr_t>(B) >> 2) & 3u);
+    const E* __restrict__ Ba = reinterpret_cast<const E*>(B - b0);
+    const int64_t total = R * C;
+    const int tid = threadIdx.x;
+    const int lr = tid % LR, lc = tid / LR;
+    const int64_t nblk = ntiles * S;
+
+    for (int64_t blk = blockIdx.x; blk < nblk; blk += gridDim.x) {
+        const int64_t tile = blk % ntiles;
+        const int s = int(blk / ntiles);
+        const int64_t ob = tile * WT;
+        const int64_t c0 = int64_t(s) * chunk;
+        const int64_t c1 = min(C, c0 + chunk);
+        E acc[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) acc[u] = zero_of<E>();
+        E outer = zero_of<E>();
+        int it = 0;
+        int64_t c = c0 + lc;
+        for (; c + int64_t(LC) * (U - 1) < c1; c += int64_t(LC) * U) {
+            E a[U];
+            T xs[U];
+            const int64_t qf = ((b0 + c * R + ob) >> 2) + lr;
+            const int64_t ql = ((b0 + (c + int64_t(LC) * (U - 1)) * R + ob) >> 2) + lr;
+            if (4 * qf - b0 >= 0 && 4 * ql - b0 + 3 < total) {
+#pragma unroll
+                for (int u = 0; u < U; ++u) {
+                    const int64_t cc = c + int64_t(LC) * u;
+                    a[u] = ld_stream(Ba + ((b0 + cc * R + ob) >> 2) + lr);
+                    xs[u] = ld_x(X + cc);
+                }
+            } else {
+#pragma unroll
+                for (int u = 0; u < U; ++u) {
+                    const int64_t cc = c + int64_t(LC) * u;
+                    a[u] = ld_inside(Ba, B, ((b0 + cc * R + ob) >> 2) + lr, b0, total);
+                    xs[u] = ld_x(X + cc);
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < U; ++u) esmac(acc[u], a[u], xs[u]);
+            if (++it == FOLD) {
+                it = 0;
+                outer = eadd(outer, tree_sum<U>(acc));
+#pragma unroll
+                for (int u = 0; u < U; ++u) acc[u] = zero_of<E>();
+            }
+        }
+        for (; c < c1; c += LC)
+            esmac(acc[0], ld_inside(Ba, B, ((b0 + c * R + ob) >> 2) + lr, b0, total), ld_x(X + c));
+        const E tot = eadd(outer, tree_sum<U>(acc));
+        T* rl = red + lc * 4 * LR + 4 * lr;
+        rl[0] = tot.x; rl[1] = tot.y; rl[2] = tot.z; rl[3] = tot.w;
+        __syncthreads();
+        // owned output rho: lane l's word rho + sh_l, summed in lane order (sh_l = shift of its rows)
+        T v = T(0);
+        if (tid < WT) {
+#pragma unroll 4
+            for (int l = 0; l < LC; ++l) {
+                const int sh = int((b0 + (c0 + l) * R + ob) & 3);
+                v += red[l * 4 * LR + tid + sh];
+            }
+        }
+        const bool rok = tid < WT && ob + tid < R;
+        if (S == 1) {
+            if (rok) y[ob + tid] = v;
+        } else {
+            if (tid < WT) ws_part[int64_t(s) * Rp + ob + tid] = v;
+            if (ticket_is_last(ws_cnt + tile, unsigned(S), &flag)) {
+                T m0 = T(0), m1 = T(0);
+                if (rok) {
+                    int k = 0;
+                    for (; k + 1 < S; k += 2) {
+                        m0 += ld_partial(ws_part + int64_t(k) * Rp + ob + tid);
+                        m1 += ld_partial(ws_part + int64_t(k + 1) * Rp + ob + tid);
+                    }
+                    if (k < S) m0 += ld_partial(ws_part + int64_t(k) * Rp + ob + tid);
+                    y[ob + tid] = m0 + m1;
+                }
+            }
+        }
+        __syncthreads();                              // red / flag reuse
+    }
+}
+
+}  // namespace adaptic

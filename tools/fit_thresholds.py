@@ -39,38 +39,81 @@ def norm_params(r):
     return p[:9]
 
 
-def fit(rows, tie=0.01):
+def fit(rows, tie=0.01, protect=None, protect_tol=0.01, neighbor_weight=0.0, portable_tie=0.0):
     """Per cell (op, dtype, load-path class, floor(log2 R), floor(log2 C)): the candidate
     (variant, portable params) with the best mean fraction of each shape's best GB/s over
     the cell's measured shapes (a cell may hold a diagonal shape and held-out ones of other
     sizes, so raw times are not comparable; a shape a candidate was not run on counts at
-    the candidate's own mean less 3 %).  Ties within 1 %: fewer CTAs."""
+    the candidate's own mean less 3 %).  Ties within 1 %: fewer CTAs.
+
+    protect: (op, R, C) shapes whose cell pick must stay within protect_tol of the best
+    measured run ON THAT SHAPE (the benchmark's own shapes): in a cell holding one, only
+    such candidates compete, and the cell's other shapes decide among them.
+
+    neighbor_weight: the shapes of the adjacent cells (Manhattan distance 1, same op, dtype
+    and load class) also score a candidate, with this weight -- a pick is used for unmeasured
+    shapes around its cell too, so one that only fits its own shapes generalises badly.
+    portable_tie: among candidates within this fraction of the top score, prefer the one
+    with the most planner-derived (0) parameters (they adapt to the actual shape)."""
     cells = collections.defaultdict(list)
     for r in rows:
         if r["req"] == "AUTO":
             continue
         vec = 1 if r["plan"]["vec_shape"] else 0      # 128-bit path shape (C % 4 == 0; TMV: R % 4 == 0)
         cells[(r["op"], r["dtype"], vec, int(math.log2(r["R"])), int(math.log2(r["C"])))].append(r)
+    def cell_cands(rs):
+        best = {}
+        cand = collections.defaultdict(dict)          # (variant, params) -> shape -> best run
+        for r in rs:
+            sh = (r["R"], r["C"])
+            best[sh] = max(best.get(sh, 0.0), r["GBps"])
+            ck = (r["variant"], tuple(norm_params(r)))
+            if sh not in cand[ck] or r["GBps"] > cand[ck][sh]["GBps"]:
+                cand[ck][sh] = r
+        return best, cand
+    per_cell = {key: cell_cands(cells[key]) for key in cells}
     table = []
     for key in sorted(cells):
         rs = cells[key]
         shapes = sorted({(r["R"], r["C"]) for r in rs})
-        best = {sh: max(r["GBps"] for r in rs if (r["R"], r["C"]) == sh) for sh in shapes}
-        cand = collections.defaultdict(dict)          # (variant, params) -> shape -> best run
-        for r in rs:
-            ck = (r["variant"], tuple(norm_params(r)))
-            sh = (r["R"], r["C"])
-            if sh not in cand[ck] or r["GBps"] > cand[ck][sh]["GBps"]:
-                cand[ck][sh] = r
+        best, cand = per_cell[key]
+        nbrs = []
+        if neighbor_weight > 0:
+            for dl, dc in ((1, 0), (-1, 0), (0, 1), (0, -1)):
+                nk = key[:3] + (key[3] + dl, key[4] + dc)
+                if nk in per_cell:
+                    nbrs.append(per_cell[nk])
         pool = list(cand)
+        prot = [sh for sh in shapes if protect and (key[0], sh[0], sh[1]) in protect]
+        if prot:
+            keep = [ck for ck in pool if all(sh in cand[ck] and cand[ck][sh]["GBps"] >= (1 - protect_tol) * best[sh]
+                                              for sh in prot)]
+            if keep:
+                pool = keep
 
         def sc(ck):      # a shape the candidate was not measured on counts at its own mean - 3 %
             got = [cand[ck][sh]["GBps"] / best[sh] for sh in cand[ck]]
             m = sum(got) / len(got)
-            return (sum(got) + 0.97 * m * (len(shapes) - len(got))) / len(shapes)
+            own = (sum(got) + 0.97 * m * (len(shapes) - len(got))) / len(shapes)
+            if not nbrs:
+                return own
+            tot, wt = own, 1.0
+            for nbest, ncand in nbrs:                 # neighbour cells: measured shapes only
+                if ck in ncand:
+                    ng = [ncand[ck][sh]["GBps"] / nbest[sh] for sh in ncand[ck]]
+                    tot += neighbor_weight * sum(ng) / len(ng)
+                else:
+                    tot += neighbor_weight * 0.97 * m
+                wt += neighbor_weight
+            return tot / wt
         score = {ck: sc(ck) for ck in pool}
-        top = max(score.values())
+        top = max(score[ck] for ck in pool)
         near = [ck for ck in pool if score[ck] >= top * (1 - tie)]
+        if portable_tie > 0:
+            port = [ck for ck in pool if score[ck] >= top * (1 - portable_tie)]
+            nz = lambda ck: sum(1 for v in ck[1] if v != 0)       # noqa: E731
+            fewest = min(nz(ck) for ck in port)
+            near = [ck for ck in port if nz(ck) == fewest]
         big = shapes[-1] if len(shapes) == 1 else max(shapes, key=lambda sh: sh[0] * sh[1])
 
         def grid_of(ck):
@@ -106,11 +149,24 @@ def main():
     ap.add_argument("--out", required=True)
     ap.add_argument("--json", default=None)
     ap.add_argument("--ops", default=None, help="comma list: fit only these ops (e.g. the BLAS-1 table)")
+    ap.add_argument("--neighbor-weight", type=float, default=0.0,
+                    help="score candidates on the adjacent cells' shapes too, with this weight")
+    ap.add_argument("--portable-tie", type=float, default=0.0)
+    ap.add_argument("--protect-bench", action="store_true",
+                    help="keep every cell pick within 1 %% of the best run on bench.py's own shapes (the 42 "
+                         "sweep shapes, their C+1 / R+1 off-grid twins, configs[2..4])")
     a = ap.parse_args()
     rows = [json.loads(l) for p in a.inputs for l in open(p) if l.strip()]
     if a.ops:
         rows = [r for r in rows if r["op"] in a.ops.split(",")]
-    table = fit(rows)
+    protect = None
+    if a.protect_bench:
+        protect = set()
+        for k in range(3, 24):
+            R, C = 1 << k, 1 << (26 - k)
+            protect |= {("mv", R, C), ("tmv", R, C), ("mv", R, C + 1), ("tmv", R + 1, C)}
+        protect |= {("dot", 1, 1 << k) for k in range(10, 31)} | {("mv", 131072, 32768), ("tmv", 1024, 1 << 24)}
+    table = fit(rows, protect=protect, neighbor_weight=a.neighbor_weight, portable_tie=a.portable_tie)
     write_inc(table, a.out)
     if a.json:
         with open(a.json, "w") as f:

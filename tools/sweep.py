@@ -80,9 +80,17 @@ def shift_grid(op, R, C):
     return out
 
 
+def tshift_grid(op, R, C):
+    """TMV rows off the 16-byte grid on the constant-shift kernel (XSMEM 7, round 2):
+    tile width LR (c-lanes 256 / LR, a multiple of 4) x loads in flight U."""
+    if op != "tmv" or R % 4 == 0 or R < 8:
+        return []
+    return [("TMV_SPLITK", [lr, 0, 0, u, 7]) for lr in (16, 32, 64) for u in (2, 4, 8)]
+
+
 def grids(op, R, C, dtype="f32"):
     """(variant, params) candidates; params = [lanes, splits, ctas_per_sm, unroll, xsmem, block, rows], 0 = auto."""
-    out = [("AUTO", None)] + tile_grid(op, R, C, dtype) + rowtile_grid(op, R, C)
+    out = [("AUTO", None)] + tile_grid(op, R, C, dtype) + rowtile_grid(op, R, C) + tshift_grid(op, R, C)
     if op in B1:
         nv = C // 4 if C % 4 == 0 else C
         if nv <= 64:
@@ -146,12 +154,36 @@ def grids(op, R, C, dtype="f32"):
     return out
 
 
-def time_plan(plan, ptrs, stream, reps, batch=5):
+def time_plan(plan, ptrs, stream, reps, batch=5, graph=False):
     """Per-launch time of back-to-back launches (the way bench.py and a stream of
-    calls see it): `reps` samples, each = CUDA-event time of `batch` launches / batch."""
+    calls see it): `reps` samples, each = CUDA-event time of `batch` launches / batch.
+    graph=True (small, L2-resident problems, round 2): the launches are replayed from a CUDA
+    graph of 20, so the sample is device time, not the host's launch rate (~5 us per
+    ctypes launch, which had made every candidate of a <= 64 MiB shape look alike)."""
     for _ in range(2):
         plan.run(*ptrs, stream)
     torch.cuda.synchronize()
+    if graph:
+        n = 20
+        s = torch.cuda.Stream()
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.stream(s):
+            plan.run(*ptrs, s.cuda_stream)
+            torch.cuda.synchronize()
+            with torch.cuda.graph(g, stream=s):
+                for _ in range(n):
+                    plan.run(*ptrs, torch.cuda.current_stream().cuda_stream)
+            g.replay()
+            torch.cuda.synchronize()
+            out = []
+            for _ in range(reps):
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record(s)
+                g.replay()
+                b.record(s)
+                b.synchronize()
+                out.append(a.elapsed_time(b) * 1e3 / n)
+        return out
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(reps)]
     for a, b in evs:
         a.record()
@@ -182,6 +214,9 @@ def main():
     ap.add_argument("--flat-only", action="store_true", help="time only the flat-stream TMV candidates (+ AUTO)")
     ap.add_argument("--shift-only", action="store_true", help="time only the shifted-x MV candidates (+ AUTO)")
     ap.add_argument("--staged-only", action="store_true", help="time only the TMA-staged candidates (+ AUTO)")
+    ap.add_argument("--tshift-only", action="store_true", help="time only the constant-shift TMV candidates (+ AUTO)")
+    ap.add_argument("--graph-below", type=float, default=0,
+                    help="time problems smaller than this many bytes from CUDA graphs (device time)")
     a = ap.parse_args()
     dev = torch.device("cuda:0")
     tdt = torch.float32 if a.dtype == "f32" else torch.int32
@@ -201,7 +236,7 @@ def main():
     else:
         shapes = [(R, C, 0) for R, C in shapes]
     maxel = max(R * C for R, C, _ in shapes) + max(R + C for R, C, _ in shapes)
-    M = torch.empty(maxel * (2 if "dot" in a.ops else 1), dtype=tdt, device=dev)
+    M = torch.empty(maxel * (2 if "dot" in a.ops else 1) + 64, dtype=tdt, device=dev)
     X = torch.empty(max(C for _, C, _ in shapes) + 1, dtype=tdt, device=dev)
     Y = torch.empty(4 * (max(R for R, _, _ in shapes) + 1), dtype=tdt, device=dev)   # 4-byte y; B1ALL: 4 per row
     synth.device_matrix(M, 1, M.numel(), "mv", "uniform", 11)
@@ -211,7 +246,10 @@ def main():
         for op in a.ops.split(","):
             for R0, C0, pert in shapes:
                 R, C = (R0 + pert, C0) if op == "tmv" else (R0, C0 + pert)
-                Xp = M.data_ptr() + R * C * 4 if op == "dot" else X.data_ptr()
+                # DOT's b: 256-byte aligned like a separate allocation (round 1 placed it right
+                # after a, so a and b differed in address mod 16 whenever R*C % 4 != 0 and the
+                # misaligned-row DOT kernels -- which need equal alignment -- fell back to scalar)
+                Xp = M.data_ptr() + (R * C * 4 + 255) // 256 * 256 if op == "dot" else X.data_ptr()
                 ptrs = (M.data_ptr(), Xp, Y.data_ptr())
                 if a.auto_only:
                     cands = [("AUTO", None)]
@@ -224,6 +262,8 @@ def main():
                 elif a.staged_only:           # every TMA-staged plan: row tiles, TMV tiles, MV_TPR
                     cands = [("AUTO", None)] + rowtile_grid(op, R, C) + \
                         [c for c in grids(op, R, C, a.dtype) if c[0] == "MV_TPR"]
+                elif a.tshift_only:
+                    cands = [("AUTO", None)] + tshift_grid(op, R, C)
                 elif a.flat_only:
                     cands = [("AUTO", None)] + [("TMV_REGTILE", [0, 0, 0, u]) for u in (2, 4, 8)] + \
                         rowtile_grid(op, R, C)
@@ -234,13 +274,14 @@ def main():
                         plan = adaptic.get_plan(OPC[op], R, C, dtc, dev, variant, params, stream)
                     except adaptic.AdapticError:
                         continue
-                    ts = time_plan(plan, ptrs, stream, a.reps)
-                    med = statistics.median(ts)
                     nbytes = 4 * (R * C * (2 if op == "dot" else 1) + (4 if op == "b1all" else 1) * R
                                   + (0 if op in ("dot",) + B1 else C))
+                    ts = time_plan(plan, ptrs, stream, a.reps, graph=nbytes < a.graph_below)
+                    med = statistics.median(ts)
                     d = plan.describe()
                     f.write(json.dumps({"op": op, "dtype": a.dtype, "R": R, "C": C, "variant": d["variant"],
                                         "req": variant, "params": params, "us": med, "us_min": min(ts),
+                                        "timing": "graph" if nbytes < a.graph_below else "stream",
                                         "GBps": nbytes / med / 1e3, "plan": d}) + "\n")
                 adaptic.clear_cache()
                 f.flush()
