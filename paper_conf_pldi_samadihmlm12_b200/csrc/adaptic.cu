@@ -179,6 +179,23 @@ int occupancy(void* fn, int block, size_t smem, bool present, int fallback) {
     return n;
 }
 
+// Does `dyn` bytes of dynamic shared memory fit beside the kernel's static shared memory?
+// (the opt-in per-block maximum; without a device: 227 KB and an assumed 16 KB static)
+bool smem_fits(void* fn, size_t dyn, bool present) {
+    size_t stat = 16 * 1024, cap = 227 * 1024;
+    if (present && fn) {
+        cudaFuncAttributes fa;
+        int dev = 0, optin = 0;
+        if (cudaFuncGetAttributes(&fa, fn) == cudaSuccess) stat = fa.sharedSizeBytes;
+        else (void)cudaGetLastError();
+        if (cudaGetDevice(&dev) == cudaSuccess &&
+            cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev) == cudaSuccess && optin > 0)
+            cap = size_t(optin);
+        else (void)cudaGetLastError();
+    }
+    return dyn + stat <= cap;
+}
+
 // Error bound of a tree whose longest path has `m` roundings (Higham eq. 4.4).
 bool bound_ok(int64_t m) {
     const double mu = double(m) * kUnitRoundoff;
@@ -414,6 +431,15 @@ adaptic_status derive_stencil(adaptic_plan_s* p, const int32_t* params, const De
 // Multi-vector MV / TMV (adaptic_plan_multi): K = nvec vectors share one pass over the
 // matrix (horizontal actor integration; mmv_kernels.cuh).  fp32, 128-bit path
 // shapes and scalar shapes alike (aligned pointers take the 128-bit instances).
+// Multi-vector TMV rows in groups of 4 (tmmv4_kernel) where it measured > 2 % faster than
+// round 1's choice on the 256 MiB diagonals (profiles/r2_exp/r2z_t4_cmp.jsonl; bit
+// floor(log2 R) of the mask)
+bool tmmv4_rule(int K, int64_t R, int64_t C) {
+    const uint32_t mask = K == 2 ? 0x13FF00u : K == 4 ? 0x17FF00u : K == 8 ? 0x3FFFC0u : 0u;
+    const int lr = ilog2_floor(R);
+    return R % 4 == 0 && C % 4 == 0 && lr >= 0 && lr < 32 && ((mask >> lr) & 1u);
+}
+
 // TMV (any K, any alignment, any R) with B staged by TMA (tmv_ring_kernel.cuh): tiles of TW
 // outputs = WPT column groups of 32 OPT words, LC = 8 / WPT row lanes; one tile covering all
 // outputs streams whole rows (one contiguous copy per stage of ~32 KB), else CR row segments.
@@ -670,6 +696,50 @@ adaptic_status derive_multi(adaptic_plan_s* p, const int32_t* params, const DevI
     }
     if (op != ADAPTIC_OP_TMV || !is_tmv_family(v)) return ADAPTIC_ERR_UNSUPPORTED;
     if (par(ADAPTIC_P_XSMEM) == 6) return derive_tmv_ring(p, params, dev);
+    // AUTO: where the row-group kernel measured > 2 % faster than round 1's choice on the
+    // 256 MiB diagonals (profiles/r2_exp/r2z_t4_cmp.jsonl; bit lr of the mask = floor(log2 R)):
+    // tiles of 16 / 64 / 128 output vectors, L2 prefetch 2 groups ahead except at K = 8
+    const int lr_r = ilog2_floor(R);
+    const bool t4_rule = !params && v == ADAPTIC_V_TMV_SPLITK && tmmv4_rule(K, R, C);
+    if (par(ADAPTIC_P_XSMEM) == 8 || t4_rule) {
+        // rows in groups of 4: x_j as one float4 per group, L2 prefetch (tmmv4_kernel)
+        if (!p->vec_shape || C % 4 != 0) return ADAPTIC_ERR_UNSUPPORTED;
+        const int NT = 256;
+        const int64_t rv = R / 4;
+        int LR = par(ADAPTIC_P_LANES);
+        if (LR <= 0) LR = t4_rule ? (lr_r <= 11 ? 16 : lr_r <= 16 ? 64 : 128) : clampi(pow2_ceil(rv), 16, 64);
+        int PF = par(ADAPTIC_P_UNROLL);
+        if (PF < 0) PF = 0;
+        if (par(ADAPTIC_P_UNROLL) == 0) PF = (K == 8 || (K == 4 && lr_r <= 11)) ? 1 : 2;
+        void* fn = tmmv4_fn(K, LR, PF == 1 ? 0 : PF);
+        if (!fn) return ADAPTIC_ERR_INVALID_ARG;
+        int cps = par(ADAPTIC_P_CTAS_PER_SM);
+        if (cps <= 0) cps = occupancy(fn, NT, 0, dev.present, 2);
+        const int LC = NT / LR;
+        const int64_t slots = int64_t(dev.sms) * cps;
+        const int64_t tiles = ceil_div(rv, int64_t(LR));
+        const int64_t ngr = C / 4;
+        int64_t S = par(ADAPTIC_P_SPLITS) > 0 ? par(ADAPTIC_P_SPLITS)
+                                              : pick_splits_wave(tiles, slots, std::max<int64_t>(1, ceil_div(ngr, int64_t(LC))));
+        for (;;) {
+            const int64_t gpt = ceil_div(ceil_div(ngr, S), int64_t(LC));          // groups per thread
+            p->chain[1] = 4 * std::min<int64_t>(gpt, FOLD / 4) + gpt / (FOLD / 4);
+            p->depth[1] = ilog2c(LC) + (S > 1 ? ceil_div(S, LC) + ilog2c(LC) : 0) + 1;
+            p->path_ok[1] = bound_ok(p->chain[1] + p->depth[1]);
+            if (p->path_ok[1] || S >= (int64_t(1) << 20)) break;
+            S *= 2;
+        }
+        if (S > INT_MAX || !p->path_ok[1]) return ADAPTIC_ERR_UNSUPPORTED;
+        p->xmode = 8;
+        p->lanes = LR; p->unroll = PF == 1 ? 0 : PF; p->block = NT; p->ctas_per_sm = cps; p->splits = int(S);
+        p->grid[1] = std::max<int64_t>(1, std::min<int64_t>(tiles * S, slots));
+        if (S > 1) {
+            const size_t part = ((size_t(R) * size_t(K) * size_t(S) * 4 + 255) / 256) * 256;
+            p->cnt_off = part;
+            p->ws_bytes = part + size_t(tiles) * 4;
+        }
+        return ADAPTIC_OK;
+    }
     // TMV tiles: LR output vectors x (256 / LR) c-lanes, S c-ranges
     const int NT = 256;
     int U = par(ADAPTIC_P_UNROLL);
@@ -915,10 +985,11 @@ adaptic_status derive_rowtile(adaptic_plan_s* p, const int32_t* params, const De
     if (stage_bytes > 200 * 1024) return ADAPTIC_ERR_UNSUPPORTED;
     int stages = int(std::min<size_t>(RT_MAX_STAGES_H, (size_t(220) * 1024 / size_t(cps)) / stage_bytes));
     if (par(ADAPTIC_P_UNROLL) > 0) stages = std::min(stages, par(ADAPTIC_P_UNROLL));
-    if (stages < 2) return ADAPTIC_ERR_UNSUPPORTED;
-    p->smem = size_t(stages) * stage_bytes;
     void* fn = rowtile_fn(p->dtype, NT, G, px);
     if (!fn) return ADAPTIC_ERR_UNSUPPORTED;
+    while (stages >= 2 && !smem_fits(fn, size_t(stages) * stage_bytes, dev.present)) --stages;   // + static smem
+    if (stages < 2) return ADAPTIC_ERR_UNSUPPORTED;
+    p->smem = size_t(stages) * stage_bytes;
     const int occ = occupancy(fn, NT, p->smem, dev.present, cps);
     if (occ < 1) return ADAPTIC_ERR_UNSUPPORTED;
     p->ctas_per_sm = std::min(cps, occ);
@@ -966,9 +1037,10 @@ adaptic_status derive_tmv_rowtile(adaptic_plan_s* p, const int32_t* params, cons
     if (stage_bytes > 200 * 1024) return ADAPTIC_ERR_UNSUPPORTED;
     int stages = int(std::min<size_t>(RT_MAX_STAGES_H, (size_t(220) * 1024 / size_t(cps)) / stage_bytes));
     if (par(ADAPTIC_P_UNROLL) > 0) stages = std::min(stages, par(ADAPTIC_P_UNROLL));
+    void* fn = tmv_rowtile_fn(p->dtype, NT, rpt);
+    while (stages >= 2 && !smem_fits(fn, size_t(stages) * stage_bytes, dev.present)) --stages;   // + static smem
     if (stages < 2) return ADAPTIC_ERR_UNSUPPORTED;
     p->smem = size_t(stages) * stage_bytes;
-    void* fn = tmv_rowtile_fn(p->dtype, NT, rpt);
     const int occ = occupancy(fn, NT, p->smem, dev.present, cps);
     if (occ < 1) return ADAPTIC_ERR_UNSUPPORTED;
     p->ctas_per_sm = std::min(cps, occ);
@@ -1386,7 +1458,8 @@ adaptic_status make_plan(int op, int64_t rows, int64_t cols, int dtype, int vari
             // with C >= 128 (derive_multi's rule); register-fed SPLITK tiles with one wave of
             // splits elsewhere; TMV_COL for huge R with few rows of B
             const int64_t rv = rows / 4;
-            if (rows % 4 == 0 && rv >= 65536 && cols < 128) p->variant = ADAPTIC_V_TMV_COL;
+            if (tmmv4_rule(nvec, rows, cols)) p->variant = ADAPTIC_V_TMV_SPLITK;     // row groups of 4
+            else if (rows % 4 == 0 && rv >= 65536 && cols < 128) p->variant = ADAPTIC_V_TMV_COL;
             else if (rows % 4 == 0 && rv >= 16) p->variant = ADAPTIC_V_TMV_SPLITK;
             else p->variant = heuristic_variant(op, rows, cols, dev.sms);
         }
@@ -1411,6 +1484,19 @@ adaptic_status make_plan(int op, int64_t rows, int64_t cols, int dtype, int vari
         p->variant = e->variant; p->source = 1;
         if (derive(p, tp, dev) == ADAPTIC_OK) { *out = p; return ADAPTIC_OK; }
         if (derive(p, nullptr, dev) == ADAPTIC_OK) { *out = p; return ADAPTIC_OK; }
+    }
+    // short rows off the 16-byte grid whose cell entry does not fit this shape (e.g. a
+    // thread-per-row tile fitted on C = 33 that needs 248 KB at C = 61): the staged row tiles
+    // are the robust choice there (held-out DOT 3085902 x 61: heuristic MV_WPR 0.20 of the
+    // best fixed; staged lane groups at the best)
+    if ((op == ADAPTIC_OP_MV || op == ADAPTIC_OP_DOT) && cols % 4 != 0 && cols <= 1024) {
+        int32_t tp[ADAPTIC_NPARAMS] = {0};
+        tp[ADAPTIC_P_XSMEM] = 4;
+        const int order[2] = {ADAPTIC_V_MV_SUBWARP, ADAPTIC_V_MV_WPR};
+        for (int i = 0; i < 2; ++i) {
+            p->variant = order[i]; p->source = 2;
+            if (derive(p, tp, dev) == ADAPTIC_OK) { *out = p; return ADAPTIC_OK; }
+        }
     }
     p->variant = heuristic_variant(op, rows, cols, dev.sms);
     p->source = 2;
@@ -1548,6 +1634,7 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
     } else if (p->nvec > 1) {
         const int K = p->nvec;
         if (p->op == ADAPTIC_OP_TMV && p->xmode == 6) { fn = tmv_ring_fn(ADAPTIC_F32, K, p->unroll); smem = p->smem; }
+        else if (p->op == ADAPTIC_OP_TMV && p->xmode == 8) fn = vec ? tmmv4_fn(K, p->lanes, p->unroll) : nullptr;
         else if (p->op == ADAPTIC_OP_TMV && p->xmode == 5) { fn = vec ? tmmv_tma_fn(K, p->lanes) : nullptr; smem = p->smem; }
         else if (p->op == ADAPTIC_OP_TMV) fn = tmmv_fn(K, p->lanes, p->unroll, vec);
         else if (p->xmode == 4) { fn = vec ? mmv_tile_fn(ADAPTIC_F32, K) : nullptr; smem = p->smem; }

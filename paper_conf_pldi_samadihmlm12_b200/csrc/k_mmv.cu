@@ -109,6 +109,37 @@ void* tmmv_tma_fn(int K, int LR) {
     }
 }
 
+// TMV groups of 4 rows, x as float4 (+ L2 prefetch PF groups ahead): LR in {16, 32, 64, 128,
+// 256}, PF in {0, 2, 4}, NT = 256
+template <int K, int PF>
+static void* t4_l(int LR) {
+    switch (LR) {
+        case 16: return reinterpret_cast<void*>(&tmmv4_kernel<K, 16, PF, 256>);
+        case 32: return reinterpret_cast<void*>(&tmmv4_kernel<K, 32, PF, 256>);
+        case 64: return reinterpret_cast<void*>(&tmmv4_kernel<K, 64, PF, 256>);
+        case 128: return reinterpret_cast<void*>(&tmmv4_kernel<K, 128, PF, 256>);
+        case 256: return reinterpret_cast<void*>(&tmmv4_kernel<K, 256, PF, 256>);
+        default: return nullptr;
+    }
+}
+template <int K>
+static void* t4_p(int LR, int PF) {
+    switch (PF) {
+        case 0: return t4_l<K, 0>(LR);
+        case 2: return t4_l<K, 2>(LR);
+        case 4: return t4_l<K, 4>(LR);
+        default: return nullptr;
+    }
+}
+void* tmmv4_fn(int K, int LR, int PF) {
+    switch (K) {
+        case 2: return t4_p<2>(LR, PF);
+        case 4: return t4_p<4>(LR, PF);
+        case 8: return t4_p<8>(LR, PF);
+        default: return nullptr;
+    }
+}
+
 #define ADAPTIC_K(FN, ...)                                                       \
     switch (K) {                                                                 \
         case 2: return vec ? FN<2, true>(__VA_ARGS__) : FN<2, false>(__VA_ARGS__); \

@@ -78,6 +78,9 @@ constexpr int MMV_GROUP_RB = 2;
 void* mmv_group_fn(int K, int G, int U, bool vec);
 void* mmv_cta_fn(int K, int U, bool vec, bool xs);   // xs: K*C*4 bytes of x staged in smem
 void* tmmv_fn(int K, int LR, int U, bool vec);
+//   tmmv4: tmmv arguments; rows in groups of 4 (x_j as one float4 per group), L2 prefetch PF
+//          groups ahead; C % 4 == 0, 16-byte-aligned B, X, Y; NT = 256 (XSMEM 8, UNROLL = PF)
+void* tmmv4_fn(int K, int LR, int PF);
 //   warp : (A, X, Y, R, C), warp per row, all K x-vectors in smem (K * C * 4 <= MMV_WARP_SMEM)
 void* mmv_warp_fn(int K);
 //   tile : (A, X, Y, R, C, int CW, int MB, float* part, unsigned* cnt), x chunks of CW values

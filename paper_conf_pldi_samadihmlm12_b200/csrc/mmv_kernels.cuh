@@ -605,6 +605,100 @@ tmmv_kernel(const float* __restrict__ B, const float* __restrict__ X, float* __r
     }
 }
 
+// ------------------------------------------------------------------ TMV tiles, rows in groups of 4 (round 2)
+// tmmv_kernel reads x_j[c] as K scalar loads per row (K U loads of x next to U of B per
+// iteration: 20 load instructions for 64 FMA at K = U = 4) and keeps U B-vectors in flight in
+// registers beside 2K accumulators (ncu: 118-128 registers, 22-25 % occupancy, 0.73-0.76 of
+// the copy peak).  Here a c-lane walks GROUPS of 4 consecutive rows, so x_j[4g .. 4g+3] is
+// ONE 128-bit load per vector (K loads per 4 rows, 4x fewer), and (PF > 0) every thread
+// prefetches its B vectors PF groups ahead into L2 (prefetch.global.L2: no register holds
+// the bytes in flight, the later load waits for an L2 hit instead of DRAM).  Needs C % 4 == 0
+// and a 16-byte-aligned X (planner); splits cut C at multiples of 4 rows.
+__device__ __forceinline__ void prefetch_l2(const void* p) {
+    asm volatile("prefetch.global.L2::evict_last [%0];" :: "l"(p));
+}
+
+template <int K, int LR, int PF, int NT>
+__global__ void __launch_bounds__(NT, 2)
+tmmv4_kernel(const float* __restrict__ B, const float* __restrict__ X, float* __restrict__ Y,
+             int64_t R, int64_t C, int S, float* __restrict__ ws_part, unsigned int* __restrict__ ws_cnt)
+{
+    pdl_prologue();
+    constexpr int LC = NT / LR;
+    __shared__ float4 red[LC > 1 ? NT : 1];
+    __shared__ unsigned int flag;
+    const int64_t rv = R / 4;
+    const int64_t ntiles = (rv + LR - 1) / LR;
+    const int64_t ngr = C / 4;                        // groups of 4 rows of B
+    const int64_t gchunk = (ngr + S - 1) / S;
+    const float4* __restrict__ Bv = reinterpret_cast<const float4*>(B);
+    const float4* __restrict__ Xv = reinterpret_cast<const float4*>(X);
+    const int tid = threadIdx.x;
+    const int lr = tid % LR, lc = tid / LR;
+    const int64_t nblk = ntiles * S;
+
+    for (int64_t blk = blockIdx.x; blk < nblk; blk += gridDim.x) {
+        const int64_t tile = blk % ntiles;
+        const int s = int(blk / ntiles);
+        const int64_t r4 = tile * LR + lr;
+        const bool rok = r4 < rv;
+        const int64_t g0 = int64_t(s) * gchunk;
+        const int64_t g1 = min(ngr, g0 + gchunk);
+        float4 acc[K], outer[K];
+#pragma unroll
+        for (int j = 0; j < K; ++j) { acc[j] = make_float4(0.f, 0.f, 0.f, 0.f); outer[j] = acc[j]; }
+        int it = 0;
+        const float4* __restrict__ Bc = Bv + (rok ? r4 : 0);
+        for (int64_t g = g0 + lc; g < g1; g += LC) {
+            if (PF > 0 && g + int64_t(PF) * LC < g1) {
+#pragma unroll
+                for (int u = 0; u < 4; ++u) prefetch_l2(Bc + (4 * (g + int64_t(PF) * LC) + u) * rv);
+            }
+            float4 b[4];
+#pragma unroll
+            for (int u = 0; u < 4; ++u) b[u] = ld_stream(Bc + (4 * g + u) * rv);
+            float4 xv[K];
+#pragma unroll
+            for (int j = 0; j < K; ++j) xv[j] = ld_x(Xv + (int64_t(j) * C) / 4 + g);
+#pragma unroll
+            for (int j = 0; j < K; ++j) {
+                vmacs(acc[j], b[0], xv[j].x);
+                vmacs(acc[j], b[1], xv[j].y);
+                vmacs(acc[j], b[2], xv[j].z);
+                vmacs(acc[j], b[3], xv[j].w);
+            }
+            if (++it == FOLD / 4) {
+                it = 0;
+#pragma unroll
+                for (int j = 0; j < K; ++j) { outer[j] = eadd(outer[j], acc[j]); acc[j] = make_float4(0.f, 0.f, 0.f, 0.f); }
+            }
+        }
+        float4* yv = reinterpret_cast<float4*>(Y);
+        float4* pv = reinterpret_cast<float4*>(ws_part);
+#pragma unroll
+        for (int j = 0; j < K; ++j) {
+            float4 tot = lc_combine<NT, LR>(eadd(outer[j], acc[j]), red);
+            if (S == 1) {
+                if (tid < LR && rok) yv[j * rv + r4] = tot;
+            } else if (tid < LR && rok) {
+                pv[(int64_t(s) * K + j) * rv + r4] = tot;
+            }
+            __syncthreads();                              // red[] reuse by the next vector
+        }
+        if (S > 1 && ticket_is_last(ws_cnt + tile, unsigned(S), &flag)) {
+#pragma unroll
+            for (int j = 0; j < K; ++j) {
+                float4 m = make_float4(0.f, 0.f, 0.f, 0.f);
+                if (rok) m = merge_partials<LC>(pv + int64_t(j) * rv + r4, int64_t(K) * rv, lc, S);
+                m = lc_combine<NT, LR>(m, red);
+                if (tid < LR && rok) yv[j * rv + r4] = m;
+                __syncthreads();
+            }
+        }
+        __syncthreads();
+    }
+}
+
 // ------------------------------------------------------------------ TMV tiles, TMA-staged
 // Same tiling and split/merge as tmmv_kernel, but the B rows of a (tile, split) block
 // arrive in shared memory by TMA bulk copies (one per B row segment of 16 LR bytes,

@@ -132,3 +132,22 @@ def test_4byte_aligned_pointers_fall_back(op, K):
             except Exception as e:  # noqa: BLE001
                 fails.append(f"{op} {R}x{C} K={K} off={off}: {type(e).__name__}: {str(e)[:160]}")
     assert not fails, "\n".join(fails)
+
+
+@pytest.mark.parametrize("K", [2, 4, 8])
+def test_tmv_row_groups_of_four(K):
+    """tmmv4_kernel (XSMEM 8): x_j read as one float4 per 4 rows, optional L2 prefetch; tiles,
+    splits (ticket merge) and ragged tiles against the oracle."""
+    fails = []
+    for (R, C), p in itertools.product([(4, 4), (64, 4096), (1028, 1000), (8192, 64), (260, 40000), (4096, 1 << 16)],
+                                       [[0, 0, 0, 0, 8], [16, 0, 0, 2, 8], [64, 7, 0, 4, 8], [256, 0, 0, 1, 8]]):
+        B = synth.matrix(R, C, "tmv", np.float32, "uniform", synth.seed(15, "A") + R)
+        X = synth.matrix(K, C, "mv", np.float32, "uniform", synth.seed(15, "x") + C)
+        try:
+            assert adaptic.plan("tmv", R, C, variant="TMV_SPLITK", params=p, nvec=K).describe()["xmode"] == 8
+            Y = adaptic.tmv_multi(torch.from_numpy(B).to(DEV), torch.from_numpy(X).to(DEV), variant="TMV_SPLITK",
+                                  params=p).cpu().numpy()
+            check(Y, B, X, "tmv", f"tmmv4 {R}x{C} {p}")
+        except Exception as e:  # noqa: BLE001
+            fails.append(f"{R}x{C} {p}: {type(e).__name__}: {str(e)[:160]}")
+    assert not fails, "\n".join(fails)

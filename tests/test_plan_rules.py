@@ -46,11 +46,14 @@ def test_multi_vector_rules():
     assert d("mv", 1 << 20, 64, nvec=4)["variant"] == "MV_SUBWARP"  # short rows: x in registers
     few = d("tmv", 64, 1 << 20, nvec=4)
     assert few["xmode"] == 5 and few["lanes"] == 16                 # one contiguous TMA tile
-    huge = d("tmv", 262144, 256, nvec=4)
+    huge = d("tmv", 262144, 256, nvec=2)
     assert huge["xmode"] == 5 and huge["lanes"] == 256 and huge["splits"] == 1
+    assert d("tmv", 262144, 256, nvec=4)["xmode"] == 8                # row groups of 4 (measured +2 %)
     mid = d("tmv", 8192, 8192, nvec=4)
-    assert mid["xmode"] == 0 and mid["variant"] == "TMV_SPLITK"     # register-fed tiles
-    assert d("tmv", 1 << 20, 64, nvec=4)["variant"] == "TMV_COL"
+    assert mid["xmode"] == 8 and mid["variant"] == "TMV_SPLITK"     # rows in groups of 4, x as float4
+    assert d("tmv", 1 << 20, 64, nvec=4)["xmode"] == 8
+    assert d("tmv", 1 << 21, 32, nvec=4)["variant"] == "TMV_COL"
+    assert d("tmv", 8192, 8190, nvec=4)["xmode"] != 8               # C % 4 != 0: register-fed tiles
     forced = d("tmv", 8192, 8192, variant="TMV_SPLITK", params=[128, 9, 0, 0, 3], nvec=8)
     assert forced["xmode"] == 5 and forced["splits"] == 9
 

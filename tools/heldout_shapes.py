@@ -33,6 +33,18 @@ def shapes(which="A"):
 
 
 def small_shapes(which="Bs"):
+    if which == "As":                 # small TRAINING shapes (5 / 7 multipliers, own seed)
+        out = []
+        for a in range(1, 14):
+            s = (14, 15, 17)[a % 3]
+            if s - a >= 1:
+                out.append((5 << a, 7 << (s - a)))
+                out.append((7 << a, 5 << (s - a)))
+        rng = random.Random(20261020)
+        for _ in range(12):
+            R = int(round(math.exp(rng.uniform(math.log(8), math.log(1 << 20)))))
+            out.append((R, max(1, int(round(rng.uniform(1 << 20, 1 << 24) / R)))))
+        return out
     """Held-out shapes of the paper's small-input regime (4-64 MiB, L2-resident): 3*2^a x
     13*2^b with a + b in {15, 16, 18} (5, 10, 41 MB), and 12 seeded random shapes with R*C
     uniform in [2^20, 2^24] elements.  Never fitted."""
@@ -53,4 +65,4 @@ def small_shapes(which="Bs"):
 if __name__ == "__main__":
     import sys
     w = sys.argv[1] if len(sys.argv) > 1 else "B"
-    print(",".join(f"{R}x{C}" for R, C in (small_shapes(w) if w == "Bs" else shapes(w))))
+    print(",".join(f"{R}x{C}" for R, C in (small_shapes(w) if w in ("As", "Bs") else shapes(w))))

@@ -19,6 +19,8 @@ def main():
     ap.add_argument("--peak", type=float, default=None, help="HBM GB/s (default MEASURED_PEAKS.json)")
     ap.add_argument("--md", default=None)
     ap.add_argument("--min-bytes", type=float, default=256 * 2 ** 20, help="gate applies at >= this many bytes")
+    ap.add_argument("--no-peak-gate", action="store_true",
+                    help="small (L2-resident) shapes: gate only on AUTO >= 0.95 x best fixed")
     ap.add_argument("--best-from", nargs="*", default=[],
                     help="sweeps whose fixed-variant runs give 'best fixed' (AUTO is taken from the inputs)")
     a = ap.parse_args()
@@ -43,7 +45,7 @@ def main():
         by[(r["op"], r["dtype"], r["R"], r["C"])].append(r)
     out = ["| op | R x C | bytes | AUTO variant | AUTO GB/s | best fixed | best GB/s | AUTO/best | AUTO/peak | gates |",
            "|---|---|---|---|---|---|---|---|---|---|"]
-    n_gate = n_pass = 0
+    n_gate = n_pass = n_10 = n_peak = 0
     worst = []
     for key in sorted(by, key=lambda k: (k[0], k[1], k[2] * k[3], k[2])):
         rs = by[key]
@@ -59,16 +61,19 @@ def main():
         frac = au["GBps"] / peak
         gate = ""
         if nbytes >= a.min_bytes:
-            ok = ratio >= 0.95 and frac >= 0.70
+            ok = ratio >= 0.95 and (a.no_peak_gate or frac >= 0.70)
             n_gate += 1
             n_pass += ok
+            n_10 += ratio >= 0.90
+            n_peak += frac >= 0.70
             gate = "PASS" if ok else "FAIL"
             worst.append((ratio, f"{opn} {R}x{C}"))
         out.append(f"| {opn} {dt} | {R}x{C} | {nbytes / 2**20:.0f} MiB | {au['variant']} | {au['GBps']:.0f} | "
                    f"{be['variant']} {be['params']} | {be['GBps']:.0f} | {ratio:.3f} | {frac:.3f} | {gate} |")
     out.append("")
+    gate_txt = "AUTO >= 0.95 x best fixed" + ("" if a.no_peak_gate else " and >= 0.70 x peak")
     out.append(f"peak = {peak:.1f} GB/s; gated shapes (>= {a.min_bytes / 2**20:.0f} MiB): {n_pass}/{n_gate} pass "
-               f"(AUTO >= 0.95 x best fixed and >= 0.70 x peak).")
+               f"({gate_txt}); {n_10}/{n_gate} within 10 % of the best fixed; {n_peak}/{n_gate} >= 0.70 of peak.")
     if worst:
         worst.sort()
         out.append("lowest AUTO/best: " + ", ".join(f"{w[1]} {w[0]:.3f}" for w in worst[:5]))
