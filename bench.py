@@ -489,20 +489,32 @@ def run_adaptic(args):
         # events, kev_steps samples -> the duration it sustains inside a stream of calls
         # (an event between every launch would add its launch latency to each sample
         # and cut the programmatic-dependent-launch overlap)
-        reps = 5
+        # each problem's launch x10 captured in a CUDA graph, replayed kev_steps times between
+        # two events on the capture stream: device time per launch, back to back as in the step
+        # (no host launch rate in it); median / p10 / p90 over the samples
+        reps = 10
         torch.cuda.synchronize()
         dur = []
+        gs = torch.cuda.Stream()
         for i, p in enumerate(probs):
             ds = []
-            for s in range(kev_steps):
-                evs[s][0].record()
-                for _ in range(reps):        # on the events' (main) stream, whatever --streams says
-                    p.plan.run(*p.ptrs, main.cuda_stream)
-                evs[s][1].record()
-            torch.cuda.synchronize()
+            with torch.cuda.stream(gs):
+                p.plan.run(*p.ptrs, gs.cuda_stream)
+                torch.cuda.synchronize()
+                g = torch.cuda.CUDAGraph()
+                with torch.cuda.graph(g, stream=gs):
+                    for _ in range(reps):
+                        p.plan.run(*p.ptrs, torch.cuda.current_stream().cuda_stream)
+                g.replay()
+                for s in range(kev_steps):
+                    evs[s][0].record(gs)
+                    g.replay()
+                    evs[s][1].record(gs)
+                torch.cuda.synchronize()
             for s in range(kev_steps):
                 ds.append(evs[s][0].elapsed_time(evs[s][1]) / reps)
             dur.append(ds)
+            del g
     mean_ms = [statistics.mean(d) for d in dur]
     kernel_sum_ms = sum(mean_ms)
     peak, peak_src = peaks()
@@ -566,8 +578,9 @@ def run_adaptic(args):
                                    if args.workload == "dot" else "inputs > L2; no flush needed")),
                 "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "cublas_context": cublas,
                 "kernel_timing": ("per-launch CUDA events inside the timed region" if inner else
-                                  f"per-kernel CUDA events after the timed region: each kernel 5x back to back, "
-                                  f"{kev_steps} samples (the timed region itself has events only at its ends)"),
+                                  f"per-kernel: a CUDA graph of 10 launches per problem after the timed region, "
+                                  f"{kev_steps} replays between events (the timed region itself has events only at "
+                                  f"its ends)"),
                 "kernel_sum_ms": kernel_sum_ms, "latency_us": latency, "streams": nstreams,
                 "issue": f"adaptic_run_batch over {nstreams} stream(s) per step",
                 "gpu_launches": (n + (1 if bucket is not None and args.dtype == "i32" else 0)) * args.steps,

@@ -161,6 +161,9 @@ void* mis_group_fn(int dtype, int G, int U, int xm) {
 void* mis_cta_fn(int dtype, int NT, int U, int xm) {
     return dtype == DT_F32 ? mis_cta_fn_f32(NT, U, xm) : mis_cta_fn_i32(NT, U, xm);
 }
+void* mis_cta_rb_fn(int dtype, int NT, int U, int RB) {
+    return dtype == DT_F32 ? mis_cta_rb_fn_f32(NT, U, RB) : mis_cta_rb_fn_i32(NT, U, RB);
+}
 constexpr int64_t kMisMinCols = 16;   // below this a row is one or two vectors: scalar path
 void* tmv_mis_fn(int dtype, int LR, int U) {
     return dtype == DT_F32 ? tmv_mis_fn_f32(LR, U) : tmv_mis_fn_i32(LR, U);
@@ -1221,15 +1224,19 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
         int NT = par(ADAPTIC_P_LANES);
         if (NT <= 0) NT = (v == ADAPTIC_V_MV_CPR && nv1 >= 8192) ? 1024 : 256;
         if (NT != 256 && NT != 1024) return ADAPTIC_ERR_INVALID_ARG;
-        int RB = par(ADAPTIC_P_ROWS);
-        if (RB <= 0 || mis) RB = 1;                        // misaligned kernels: one row per CTA step
-        int U = par(ADAPTIC_P_UNROLL);
-        if (U <= 0) U = RB == 4 ? 2 : 4;
-        const bool combo_ok = (RB == 1 && (U == 2 || U == 4 || U == 8)) || (RB == 2 && (U == 2 || U == 4)) ||
-                              (RB == 4 && U == 2);
-        if (!combo_ok || (NT == 1024 && RB * U > 4)) return ADAPTIC_ERR_INVALID_ARG;
         // x staged in smem only for CPR (a split CTA reads a different x chunk per block)
         const bool want_shift = par(ADAPTIC_P_XSMEM) == 5;
+        int RB = par(ADAPTIC_P_ROWS);
+        // misaligned kernels: one row per CTA step, except the shifted-x kernel with RB rows of
+        // one residue class (mv_cta_mis_rb_kernel, RB in {2, 4}, NT 256)
+        const bool mis_rb = mis && want_shift && (RB == 2 || RB == 4) && NT == 256;
+        if (RB <= 0 || (mis && !mis_rb)) RB = 1;
+        int U = par(ADAPTIC_P_UNROLL);
+        if (U <= 0) U = (RB == 4 && !mis_rb) ? 2 : 4;
+        const bool combo_ok = mis_rb ? (U == 2 || U == 4)
+                                     : ((RB == 1 && (U == 2 || U == 4 || U == 8)) || (RB == 2 && (U == 2 || U == 4)) ||
+                                        (RB == 4 && U == 2));
+        if (!combo_ok || (NT == 1024 && RB * U > 4)) return ADAPTIC_ERR_INVALID_ARG;
         if (want_shift && (px || !mis)) return ADAPTIC_ERR_UNSUPPORTED;   // shifted x: misaligned MV rows only
         const int xm = want_shift ? XM_SHIFT_MODE : pick_xmode(px, par(ADAPTIC_P_XSMEM), C, v == ADAPTIC_V_MV_CPR);
         if (xm < 0) return ADAPTIC_ERR_UNSUPPORTED;
@@ -1240,14 +1247,15 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
         if (pipe_req < 0 || pipe_req > 2 || (pipe_req == 2 && NT != 256)) return ADAPTIC_ERR_INVALID_ARG;
         p->pipe = (pipe_req == 2 && !mis) ? 1 : 0;
         p->mis = mis;
-        if (cps <= 0) cps = occupancy(mis ? mis_cta_fn(dt, NT, U, xm) : cta_fn(dt, NT, RB, U, p->vec_shape, xm, p->pipe),
+        if (cps <= 0) cps = occupancy(mis_rb ? mis_cta_rb_fn(dt, NT, U, RB)
+                                      : mis ? mis_cta_fn(dt, NT, U, xm) : cta_fn(dt, NT, RB, U, p->vec_shape, xm, p->pipe),
                                       NT, xsm, dev.present, 2048 / NT);
         p->lanes = NT; p->unroll = U; p->rb = RB; p->block = NT; p->ctas_per_sm = cps; p->xmode = xm; p->smem = xsm;
         // split order: 1 contiguous chunks, 2 interleaved steps (default for S > 1)
         const int order = par(ADAPTIC_P_ORDER);
         if (order < 0 || order > 2) return ADAPTIC_ERR_INVALID_ARG;
         const int64_t slots = int64_t(dev.sms) * cps;
-        const int64_t groups = ceil_div(R, RB);
+        const int64_t groups = mis_rb ? 4 * ceil_div(R, 4 * int64_t(RB)) : ceil_div(R, RB);   // residue-class groups
         int64_t S = 1;
         if (v == ADAPTIC_V_MV_SPLIT) {
             if (par(ADAPTIC_P_SPLITS) > 0) S = par(ADAPTIC_P_SPLITS);
@@ -1723,7 +1731,8 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
                 args = args9;
                 break;
             }
-            fn = mis ? mis_cta_fn(dt, p->lanes, p->unroll, p->xmode)
+            fn = (mis && p->xmode == XM_SHIFT_MODE && p->rb > 1) ? mis_cta_rb_fn(dt, p->lanes, p->unroll, p->rb)
+               : mis ? mis_cta_fn(dt, p->lanes, p->unroll, p->xmode)
                      : cta_fn(dt, p->lanes, p->rb, p->unroll, vec, p->xmode, p->pipe != 0);
             smem = p->smem;
             args9[0] = &A; args9[1] = &X; args9[2] = &y; args9[3] = &R; args9[4] = &C;

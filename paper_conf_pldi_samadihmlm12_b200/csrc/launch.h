@@ -46,6 +46,10 @@ void* mis_cta_fn_i32(int NT, int U, int xmode);
 // four copies of pitch round_up(C, 4), copy h = x shifted left by h elements
 void* mis_shift_fn_f32();
 void* mis_shift_fn_i32();
+// shifted-x CTA kernel, RB rows of one residue class (r mod 4) per step sharing x: the
+// mis_cta arguments; NT = 256, U in {2, 4}, RB in {2, 4} (MV_CPR / MV_SPLIT, XSMEM 5, ROWS RB)
+void* mis_cta_rb_fn_f32(int NT, int U, int RB);
+void* mis_cta_rb_fn_i32(int NT, int U, int RB);
 constexpr int XM_SHIFT_MODE = 3;
 // Misaligned-row TMV (tmv_mis_kernel.cuh; R % 4 != 0, two aligned loads + funnel shift), NT = 256:
 //   (const T* B, const T* X, T* y, int64_t R, int64_t C, int S, T* part, unsigned* cnt)

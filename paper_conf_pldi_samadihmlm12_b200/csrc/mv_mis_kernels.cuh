@@ -258,3 +258,125 @@ mv_cta_mis_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restric
 }
 
 }  // namespace adaptic
+
+namespace adaptic {
+
+// Misaligned MV rows, RB rows per CTA step that SHARE their x loads (round 2).  A row's
+// head h = (a0 + r C) mod 4 depends on r mod 4 only, so rows r, r + 4, r + 8, ... have the
+// same head and read the same shifted copy X_h (XM_SHIFT): a group of RB rows of one residue
+// class loads each x vector once for RB rows, where the one-row kernel streamed one x
+// vector per A vector (L2 -> SM traffic 2x the matrix bytes).  Groups: g -> class g % 4,
+// rows class + 4 (g / 4 * RB + i); splits S per group as in mv_cta_mis_kernel (interleaved
+// or contiguous), the same-launch ticket merge per group, scalar head / tail per row by
+// split 0.  x is the four shifted copies (x_shift_kernel, same stream, just before).
+template <class T, int NT, int U, int RB>
+__global__ void __launch_bounds__(NT)
+mv_cta_mis_rb_kernel(const T* __restrict__ A, const T* __restrict__ Xs, T* __restrict__ y,
+                     int64_t R, int64_t C, int S, int ilv, T* __restrict__ ws_part, unsigned int* __restrict__ ws_cnt)
+{
+    pdl_prologue();
+    using E = vec4_t<T>;
+    constexpr int64_t BV = int64_t(NT) * U;
+    __shared__ T red[RB * (NT / 32)];
+    __shared__ unsigned int flag;
+    const int64_t P = xshift_pitch(C);
+    const int tid = threadIdx.x;
+    const int64_t nb4 = (R + 4 * RB - 1) / (4 * RB);         // groups per residue class
+    const int64_t nblk = 4 * nb4 * S;
+
+    for (int64_t blk = blockIdx.x; blk < nblk; blk += gridDim.x) {
+        const int64_t g = blk / S;
+        const int s = int(blk - g * S);
+        const int64_t row0 = (g & 3) + 4 * ((g >> 2) * RB);
+        if (row0 >= R) continue;                             // uniform over the group's CTAs
+        int64_t rows[RB];
+        const E* av[RB];
+#pragma unroll
+        for (int i = 0; i < RB; ++i) rows[i] = row0 + 4 * i;
+        const int h = head_elems(A + row0 * C);
+#pragma unroll
+        for (int i = 0; i < RB; ++i)
+            av[i] = reinterpret_cast<const E*>(A + (rows[i] < R ? rows[i] : row0) * C + h);
+        const E* xv = reinterpret_cast<const E*>(Xs + h * P);
+        const int64_t nb = (C - h) >> 2;
+        const int64_t chunk = (nb + S - 1) / S;
+        const int64_t start = ilv ? int64_t(s) * BV : int64_t(s) * chunk;
+        const int64_t stride = ilv ? int64_t(S) * BV : BV;
+        const int64_t end = ilv ? nb : min(nb, start + chunk);
+
+        E acc[RB][U];
+#pragma unroll
+        for (int i = 0; i < RB; ++i)
+#pragma unroll
+            for (int u = 0; u < U; ++u) acc[i][u] = zero_of<E>();
+        T outer[RB], edge[RB];
+#pragma unroll
+        for (int i = 0; i < RB; ++i) { outer[i] = T(0); edge[i] = T(0); }
+        int it = 0;
+        int64_t b = start;
+        for (; b + tid + int64_t(NT) * (U - 1) < end; b += stride) {
+            E a[RB][U], x[U];
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                const int64_t v = b + tid + int64_t(NT) * u;
+                x[u] = ld_x(xv + v);
+#pragma unroll
+                for (int i = 0; i < RB; ++i) a[i][u] = ld_stream(av[i] + v);
+            }
+#pragma unroll
+            for (int i = 0; i < RB; ++i)
+#pragma unroll
+                for (int u = 0; u < U; ++u) emac(acc[i][u], a[i][u], x[u]);
+            if (++it == FOLD) {
+                it = 0;
+#pragma unroll
+                for (int i = 0; i < RB; ++i) {
+                    outer[i] += esum(tree_sum<U>(acc[i]));
+#pragma unroll
+                    for (int u = 0; u < U; ++u) acc[i][u] = zero_of<E>();
+                }
+            }
+        }
+        const int64_t tail_end = min(end, b + BV);
+        for (int64_t v = b + tid; v < tail_end; v += NT) {
+            const E x = ld_x(xv + v);
+#pragma unroll
+            for (int i = 0; i < RB; ++i) emac(acc[i][0], ld_stream(av[i] + v), x);
+        }
+        if (s == 0) {                                        // scalar head and tail of every row
+            const int64_t t0 = h + 4 * nb;
+            if (tid < h + int(C - t0)) {
+                const int64_t c = tid < h ? tid : t0 + (tid - h);
+                const T xs = ld_x(Xs + c);                   // copy 0 is x itself
+#pragma unroll
+                for (int i = 0; i < RB; ++i)
+                    if (rows[i] < R) edge[i] = mac(ld_stream(A + rows[i] * C + c), xs, edge[i]);
+            }
+        }
+        T val[RB];
+#pragma unroll
+        for (int i = 0; i < RB; ++i) val[i] = (outer[i] + esum(tree_sum<U>(acc[i]))) + edge[i];
+        cta_sum_rows<NT, RB>(val, red);                      // thread i < RB holds row i
+
+        if (S == 1) {
+            if (tid < RB && rows[tid] < R) y[rows[tid]] = val[0];
+        } else {
+            if (tid < RB && rows[tid] < R) ws_part[rows[tid] * S + s] = val[0];
+            if (ticket_is_last(ws_cnt + g, unsigned(S), &flag)) {
+                __syncthreads();
+                T m[RB];
+#pragma unroll
+                for (int i = 0; i < RB; ++i) {
+                    m[i] = T(0);
+                    if (rows[i] < R)
+                        for (int k = tid; k < S; k += NT) m[i] += ld_partial(ws_part + rows[i] * S + k);
+                }
+                cta_sum_rows<NT, RB>(m, red);
+                if (tid < RB && rows[tid] < R) y[rows[tid]] = m[0];
+            }
+        }
+        __syncthreads();
+    }
+}
+
+}  // namespace adaptic

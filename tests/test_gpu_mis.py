@@ -206,3 +206,37 @@ def test_shifted_x_copies_any_x_alignment():
                          ("MV_SPLIT", [256, 3, 0, 4, 5])):
                 y = adaptic.mv(Ad, xb[off:off + C], variant=v, params=p).cpu().numpy()
                 check(y, oracle.mv(A, x), "f32", f"shift x off {off} {R}x{C} {v}")
+
+
+def test_shifted_x_row_groups_share_x():
+    """mv_cta_mis_rb_kernel (MV_SPLIT / MV_CPR, XSMEM 5, ROWS 2 or 4): RB rows of one residue
+    class (r mod 4: same head, same shifted copy of x) per CTA step; ragged groups (R not a
+    multiple of 4 RB), splits (ticket merge per group), every base alignment; fp32 within
+    1e-4 S_r, int32 exact."""
+    import itertools
+    fails = []
+    for (R, C), off, p in itertools.product([(1, 1001), (7, 40001), (64, 65537), (130, 3003), (517, 1025)],
+                                            (0, 1, 3),
+                                            [[256, 0, 0, 4, 5, 0, 2], [256, 0, 0, 2, 5, 0, 4], [256, 5, 0, 4, 5, 0, 4, 1],
+                                             [256, 0, 0, 2, 5, 0, 2, 2]]):
+        for dt in ("f32", "i32"):
+            np_dt = np.float32 if dt == "f32" else np.int32
+            tdt = torch.float32 if dt == "f32" else torch.int32
+            A = synth.matrix(R, C, "mv", np_dt, "uniform", 31 + R)
+            x = synth.vector(C, np_dt, "uniform", 32 + C)
+            buf = torch.zeros(A.size + 8, dtype=tdt, device=DEV)
+            buf[off:off + A.size] = torch.from_numpy(A.reshape(-1)).to(DEV)
+            try:
+                for v in ("MV_SPLIT", "MV_CPR"):
+                    d = adaptic.plan("mv", R, C, dt, variant=v, params=p).describe()
+                    assert d["xmode"] == 3, d
+                    y = adaptic.mv(buf[off:off + A.size].view(R, C), torch.from_numpy(x).to(DEV), variant=v,
+                                   params=p).cpu().numpy()
+                    if dt == "i32":
+                        assert np.array_equal(y, oracle.mv(A, x)), "int32 mismatch"
+                    else:
+                        yr, S = oracle.mv(A, x)
+                        assert np.all(np.abs(y.astype(np.float64) - yr) <= 1e-4 * S), "out of tolerance"
+            except Exception as e:  # noqa: BLE001
+                fails.append(f"{dt} {R}x{C} off={off} {p}: {type(e).__name__}: {str(e)[:160]}")
+    assert not fails, f"{len(fails)} failures\n" + "\n".join(fails[:20])

@@ -69,9 +69,26 @@ def main():
     ap.add_argument("--json", default=None)
     ap.add_argument("--md", default=None)
     ap.add_argument("--traffic", default=None)
+    ap.add_argument("--detail", default=None,
+                    help="bench.py --detail JSONL of the captured step: keys op:RxC:VARIANT in launch order; a "
+                         "plan's pre-kernel (x_shift_kernel) is folded into the next problem's DRAM bytes")
     a = ap.parse_args()
     rows = [r for rep in a.reps for r in read(rep)]
     keys = json.load(open(a.keys)) if a.keys else [None] * len(rows)
+    if a.detail:
+        det = [json.loads(l) for l in open(a.detail) if l.strip()]
+        dk = iter(f"{q['op']}:{q['R']}x{q['C']}:{q['variant']}" for q in det)
+        keys, extra = [], 0.0
+        for r in rows:
+            if "x_shift" in r["kernel"]:
+                keys.append(None)
+                extra += r.get("dram_bytes", 0.0)
+                continue
+            keys.append(next(dk, None))
+            if extra and "dram_bytes" in r:
+                r["dram_bytes"] += extra
+                r["prekernel_bytes"] = extra
+            extra = 0.0
     for r, k in zip(rows, keys):
         r["key"] = k
     if a.json:

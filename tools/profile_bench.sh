@@ -9,12 +9,12 @@ tag=${1:-r1}
 mkdir -p gpurun_out
 python bench.py --steps 20 --warmup 3 --no-e2e --no-cpu-baseline --detail gpurun_out/detail_prof.jsonl \
     > gpurun_out/bench_forprof.json 2> gpurun_out/bench_forprof.err
-ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"mv_|tmv_" --csv \
+ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"mv_|tmv_|mv4_|ring" --csv \
     --log-file gpurun_out/launches_${tag}.csv \
     python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu-baseline > /dev/null 2>&1
 # the full report of 42 kernels exceeds gpurun's 64 MiB copy-back: keep it in /tmp, bring back
 # the raw-page CSV (all metrics, one row per kernel) and the source page of the first kernel
-ncu --set full --clock-control none --import-source on -k regex:"mv_|tmv_" -c 42 \
+ncu --set full --clock-control none --import-source on -k regex:"mv_|tmv_|mv4_|ring" -c 42 \
     -o /tmp/bench_full_${tag} -f \
     python bench.py --steps 1 --warmup 3 --no-e2e --no-cpu-baseline > gpurun_out/ncu_full_${tag}.log 2>&1
 ncu -i /tmp/bench_full_${tag}.ncu-rep --page raw --csv > gpurun_out/bench_full_${tag}_raw.csv 2>/dev/null
