@@ -161,6 +161,9 @@ void* mis_group_fn(int dtype, int G, int U, int xm) {
 void* mis_cta_fn(int dtype, int NT, int U, int xm) {
     return dtype == DT_F32 ? mis_cta_fn_f32(NT, U, xm) : mis_cta_fn_i32(NT, U, xm);
 }
+void* mis_cta_fx_fn(int dtype, int NT, int U) {
+    return dtype == DT_F32 ? mis_cta_fx_fn_f32(NT, U) : mis_cta_fx_fn_i32(NT, U);
+}
 void* mis_cta_rb_fn(int dtype, int NT, int U, int RB) {
     return dtype == DT_F32 ? mis_cta_rb_fn_f32(NT, U, RB) : mis_cta_rb_fn_i32(NT, U, RB);
 }
@@ -1238,7 +1241,10 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
                                         (RB == 4 && U == 2));
         if (!combo_ok || (NT == 1024 && RB * U > 4)) return ADAPTIC_ERR_INVALID_ARG;
         if (want_shift && (px || !mis)) return ADAPTIC_ERR_UNSUPPORTED;   // shifted x: misaligned MV rows only
-        const int xm = want_shift ? XM_SHIFT_MODE : pick_xmode(px, par(ADAPTIC_P_XSMEM), C, v == ADAPTIC_V_MV_CPR);
+        const bool want_fx = par(ADAPTIC_P_XSMEM) == 9;                 // x funnel (mv_cta_mis_fx_kernel)
+        if (want_fx && (px || !mis || NT != 256 || !mis_cta_fx_fn(dt, NT, U))) return ADAPTIC_ERR_UNSUPPORTED;
+        const int xm = want_fx ? XM_FX_MODE : want_shift ? XM_SHIFT_MODE
+                                                         : pick_xmode(px, par(ADAPTIC_P_XSMEM), C, v == ADAPTIC_V_MV_CPR);
         if (xm < 0) return ADAPTIC_ERR_UNSUPPORTED;
         const size_t xsm = xm == 1 ? size_t((C * 4 + 15) / 16 * 16) : 0;
         int cps = par(ADAPTIC_P_CTAS_PER_SM);
@@ -1247,7 +1253,7 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
         if (pipe_req < 0 || pipe_req > 2 || (pipe_req == 2 && NT != 256)) return ADAPTIC_ERR_INVALID_ARG;
         p->pipe = (pipe_req == 2 && !mis) ? 1 : 0;
         p->mis = mis;
-        if (cps <= 0) cps = occupancy(mis_rb ? mis_cta_rb_fn(dt, NT, U, RB)
+        if (cps <= 0) cps = occupancy(want_fx ? mis_cta_fx_fn(dt, NT, U) : mis_rb ? mis_cta_rb_fn(dt, NT, U, RB)
                                       : mis ? mis_cta_fn(dt, NT, U, xm) : cta_fn(dt, NT, RB, U, p->vec_shape, xm, p->pipe),
                                       NT, xsm, dev.present, 2048 / NT);
         p->lanes = NT; p->unroll = U; p->rb = RB; p->block = NT; p->ctas_per_sm = cps; p->xmode = xm; p->smem = xsm;
@@ -1731,7 +1737,9 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
                 args = args9;
                 break;
             }
-            fn = (mis && p->xmode == XM_SHIFT_MODE && p->rb > 1) ? mis_cta_rb_fn(dt, p->lanes, p->unroll, p->rb)
+            fn = (mis && p->xmode == XM_FX_MODE) ? (aligned(X, 16) ? mis_cta_fx_fn(dt, p->lanes, p->unroll)
+                                                                    : mis_cta_fn(dt, p->lanes, p->unroll, 0))
+               : (mis && p->xmode == XM_SHIFT_MODE && p->rb > 1) ? mis_cta_rb_fn(dt, p->lanes, p->unroll, p->rb)
                : mis ? mis_cta_fn(dt, p->lanes, p->unroll, p->xmode)
                      : cta_fn(dt, p->lanes, p->rb, p->unroll, vec, p->xmode, p->pipe != 0);
             smem = p->smem;

@@ -50,6 +50,11 @@ void* mis_shift_fn_i32();
 // mis_cta arguments; NT = 256, U in {2, 4}, RB in {2, 4} (MV_CPR / MV_SPLIT, XSMEM 5, ROWS RB)
 void* mis_cta_rb_fn_f32(int NT, int U, int RB);
 void* mis_cta_rb_fn_i32(int NT, int U, int RB);
+// x as two aligned 128-bit loads + a compile-time funnel per row head (mv_cta_mis_fx_kernel):
+// the mis_cta arguments; NT = 256, U in {2, 4, 8}; needs a 16-byte-aligned x (XSMEM 9)
+void* mis_cta_fx_fn_f32(int NT, int U);
+void* mis_cta_fx_fn_i32(int NT, int U);
+constexpr int XM_FX_MODE = 9;
 constexpr int XM_SHIFT_MODE = 3;
 // Misaligned-row TMV (tmv_mis_kernel.cuh; R % 4 != 0, two aligned loads + funnel shift), NT = 256:
 //   (const T* B, const T* X, T* y, int64_t R, int64_t C, int S, T* part, unsigned* cnt)

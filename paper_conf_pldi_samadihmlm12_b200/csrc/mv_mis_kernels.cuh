@@ -380,3 +380,131 @@ mv_cta_mis_rb_kernel(const T* __restrict__ A, const T* __restrict__ Xs, T* __res
 }
 
 }  // namespace adaptic
+
+namespace adaptic {
+
+// Misaligned MV rows with x read as TWO aligned 128-bit vectors per body vector and a
+// COMPILE-TIME funnel (round 2, XSMEM 9): a row with head h needs x[h + 4v .. h + 4v + 3],
+// i.e. words h..h+3 of x4[v] ++ x4[v + 1].  h is the same for the whole row, so the row's
+// stream loop is instantiated for h = 0..3 and the funnel is register renaming.  Replaces
+// four 32-bit x loads per A vector (XM_LDG: L1-bound) without the shifted-copy pre-kernel
+// (XM_SHIFT: 4 C words written per call -- on few long rows as long as the matrix pass
+// saves).  Needs a 16-byte-aligned x (launch falls back to XM_LDG).
+template <int H, class E> __device__ __forceinline__ E funnel_c(const E& lo, const E& hi) {
+    if constexpr (H == 0) return lo;
+    else if constexpr (H == 1) return E{lo.y, lo.z, lo.w, hi.x};
+    else if constexpr (H == 2) return E{lo.z, lo.w, hi.x, hi.y};
+    else return E{lo.w, hi.x, hi.y, hi.z};
+}
+
+// x4[q] with the words at or beyond C read one by one (the last vector of x may end past it)
+template <class T> __device__ __forceinline__ vec4_t<T> ld_x_end(const T* X, int64_t q, int64_t C) {
+    using E = vec4_t<T>;
+    if (4 * q + 3 < C) return ld_x(reinterpret_cast<const E*>(X) + q);
+    E v = zero_of<E>();
+    if (4 * q < C) v.x = ld_x(X + 4 * q);
+    if (4 * q + 1 < C) v.y = ld_x(X + 4 * q + 1);
+    if (4 * q + 2 < C) v.z = ld_x(X + 4 * q + 2);
+    return v;
+}
+
+// one row's share [start, end) (stride) of body vectors: the fp32 partial of this thread
+template <class T, int NT, int U, int H>
+__device__ __forceinline__ T mis_fx_stream(const vec4_t<T>* __restrict__ av, const T* __restrict__ X, int64_t C,
+                                           int64_t nb, int64_t start, int64_t stride, int64_t end) {
+    using E = vec4_t<T>;
+    constexpr int64_t BV = int64_t(NT) * U;
+    const E* __restrict__ x4 = reinterpret_cast<const E*>(X);
+    const int tid = threadIdx.x;
+    E acc[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) acc[u] = zero_of<E>();
+    T outer = T(0);
+    int it = 0;
+    const int64_t end_main = min(end, nb - 1);                 // x4[v + 1] inside x for v < nb - 1
+    int64_t b = start;
+    for (; b + tid + int64_t(NT) * (U - 1) < end_main; b += stride) {
+        E a[U], lo[U], hi[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            const int64_t v = b + tid + int64_t(NT) * u;
+            a[u] = ld_stream(av + v);
+            lo[u] = ld_x(x4 + v);
+            if (H != 0) hi[u] = ld_x(x4 + v + 1);
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) emac(acc[u], a[u], funnel_c<H>(lo[u], H != 0 ? hi[u] : lo[u]));
+        if (++it == FOLD) {
+            it = 0;
+            outer += esum(tree_sum<U>(acc));
+#pragma unroll
+            for (int u = 0; u < U; ++u) acc[u] = zero_of<E>();
+        }
+    }
+    const int64_t tail_end = min(end, b + BV);
+    for (int64_t v = b + tid; v < tail_end; v += NT) {
+        const E lo = ld_x_end(X, v, C);
+        const E hi = H != 0 ? ld_x_end(X, v + 1, C) : lo;
+        emac(acc[0], ld_stream(av + v), funnel_c<H>(lo, hi));
+    }
+    return outer + esum(tree_sum<U>(acc));
+}
+
+template <class T, int NT, int U>
+__global__ void __launch_bounds__(NT)
+mv_cta_mis_fx_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restrict__ y,
+                     int64_t R, int64_t C, int S, int ilv, T* __restrict__ ws_part, unsigned int* __restrict__ ws_cnt)
+{
+    pdl_prologue();
+    using E = vec4_t<T>;
+    constexpr int64_t BV = int64_t(NT) * U;
+    __shared__ T red[NT / 32];
+    __shared__ unsigned int flag;
+    const int tid = threadIdx.x;
+    const int64_t nblk = R * S;
+    for (int64_t blk = blockIdx.x; blk < nblk; blk += gridDim.x) {
+        const int64_t row = blk / S;
+        const int s = int(blk - row * S);
+        const T* rowp = A + row * C;
+        const int h = head_elems(rowp);
+        const E* av = reinterpret_cast<const E*>(rowp + h);
+        const int64_t nb = (C - h) >> 2;
+        const int64_t chunk = (nb + S - 1) / S;
+        const int64_t start = ilv ? int64_t(s) * BV : int64_t(s) * chunk;
+        const int64_t stride = ilv ? int64_t(S) * BV : BV;
+        const int64_t end = ilv ? nb : min(nb, start + chunk);
+        // the body's x starts at word h (its aligned vectors: x4[v], x4[v + 1] shifted by h)
+        T part;
+        switch (h) {
+            case 0: part = mis_fx_stream<T, NT, U, 0>(av, X, C, nb, start, stride, end); break;
+            case 1: part = mis_fx_stream<T, NT, U, 1>(av, X + 0, C, nb, start, stride, end); break;
+            case 2: part = mis_fx_stream<T, NT, U, 2>(av, X + 0, C, nb, start, stride, end); break;
+            default: part = mis_fx_stream<T, NT, U, 3>(av, X + 0, C, nb, start, stride, end); break;
+        }
+        T edge = T(0);
+        if (s == 0) {                                        // scalar head and tail of the row
+            const int64_t t0 = h + 4 * nb;
+            if (tid < h + int(C - t0)) {
+                const int64_t c = tid < h ? tid : t0 + (tid - h);
+                edge = mac(ld_stream(rowp + c), ld_x(X + c), edge);
+            }
+        }
+        T val[1] = {part + edge};
+        cta_sum_rows<NT, 1>(val, red);
+        if (S == 1) {
+            if (tid == 0) y[row] = val[0];
+        } else {
+            if (tid == 0) ws_part[row * S + s] = val[0];
+            if (ticket_is_last(ws_cnt + row, unsigned(S), &flag)) {
+                __syncthreads();
+                T m[1] = {T(0)};
+                for (int k = tid; k < S; k += NT) m[0] += ld_partial(ws_part + row * S + k);
+                cta_sum_rows<NT, 1>(m, red);
+                if (tid == 0) y[row] = m[0];
+            }
+        }
+        __syncthreads();
+    }
+}
+
+}  // namespace adaptic

@@ -240,3 +240,35 @@ def test_shifted_x_row_groups_share_x():
             except Exception as e:  # noqa: BLE001
                 fails.append(f"{dt} {R}x{C} off={off} {p}: {type(e).__name__}: {str(e)[:160]}")
     assert not fails, f"{len(fails)} failures\n" + "\n".join(fails[:20])
+
+
+def test_x_funnel_cta_kernel():
+    """mv_cta_mis_fx_kernel (MV_SPLIT / MV_CPR, XSMEM 9): x as two aligned 128-bit loads and a
+    compile-time funnel per row head h = 0..3 (every row residue), the last body vector's
+    x read word by word at the end of x; splits; x only 4-byte aligned -> the XM_LDG kernel."""
+    import itertools
+    fails = []
+    for (R, C), off, xoff, p in itertools.product([(1, 1001), (7, 40001), (64, 65537), (130, 3003), (9, 1030)],
+                                                  (0, 1, 3), (0, 1),
+                                                  [[256, 0, 0, 4, 9], [256, 6, 0, 2, 9, 0, 0, 1], [256, 0, 0, 8, 9]]):
+        for dt in ("f32", "i32"):
+            np_dt = np.float32 if dt == "f32" else np.int32
+            tdt = torch.float32 if dt == "f32" else torch.int32
+            A = synth.matrix(R, C, "mv", np_dt, "uniform", 41 + R)
+            x = synth.vector(C, np_dt, "uniform", 42 + C)
+            buf = torch.zeros(A.size + 8, dtype=tdt, device=DEV)
+            buf[off:off + A.size] = torch.from_numpy(A.reshape(-1)).to(DEV)
+            xb = torch.zeros(C + 8, dtype=tdt, device=DEV)
+            xb[xoff:xoff + C] = torch.from_numpy(x).to(DEV)
+            try:
+                for v in ("MV_SPLIT", "MV_CPR"):
+                    y = adaptic.mv(buf[off:off + A.size].view(R, C), xb[xoff:xoff + C], variant=v,
+                                   params=p).cpu().numpy()
+                    if dt == "i32":
+                        assert np.array_equal(y, oracle.mv(A, x)), "int32 mismatch"
+                    else:
+                        yr, S = oracle.mv(A, x)
+                        assert np.all(np.abs(y.astype(np.float64) - yr) <= 1e-4 * S), "out of tolerance"
+            except Exception as e:  # noqa: BLE001
+                fails.append(f"{dt} {R}x{C} off={off} xoff={xoff} {p}: {type(e).__name__}: {str(e)[:160]}")
+    assert not fails, f"{len(fails)} failures\n" + "\n".join(fails[:20])
