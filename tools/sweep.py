@@ -80,6 +80,19 @@ def shift_grid(op, R, C):
     return out
 
 
+def misx_grid(op, R, C):
+    """Misaligned MV rows, round-2 kernels: x as two aligned loads + a compile-time funnel
+    (XSMEM 9) and the shifted-x kernel with RB rows of one residue class (XSMEM 5, ROWS 2/4)."""
+    if op != "mv" or C % 4 == 0 or C < 512:
+        return []
+    out = [("MV_CPR", [256, 0, 0, u, 9]) for u in (2, 4, 8)]
+    out += [("MV_CPR", [256, 0, 0, u, 5, 0, rb]) for u in (2, 4) for rb in (2, 4)]
+    if R <= 8192:
+        out += [("MV_SPLIT", [256, 0, 0, u, 9, 0, 0, o]) for u in (2, 4) for o in (1, 2)]
+        out += [("MV_SPLIT", [256, 0, 0, u, 5, 0, rb, o]) for u in (2, 4) for rb in (2, 4) for o in (1, 2)]
+    return out
+
+
 def tshift_grid(op, R, C):
     """TMV rows off the 16-byte grid on the constant-shift kernel (XSMEM 7, round 2):
     tile width LR (c-lanes 256 / LR, a multiple of 4) x loads in flight U."""
@@ -90,7 +103,8 @@ def tshift_grid(op, R, C):
 
 def grids(op, R, C, dtype="f32"):
     """(variant, params) candidates; params = [lanes, splits, ctas_per_sm, unroll, xsmem, block, rows], 0 = auto."""
-    out = [("AUTO", None)] + tile_grid(op, R, C, dtype) + rowtile_grid(op, R, C) + tshift_grid(op, R, C)
+    out = [("AUTO", None)] + tile_grid(op, R, C, dtype) + rowtile_grid(op, R, C) + tshift_grid(op, R, C) + \
+        misx_grid(op, R, C)
     if op in B1:
         nv = C // 4 if C % 4 == 0 else C
         if nv <= 64:
@@ -215,6 +229,7 @@ def main():
     ap.add_argument("--shift-only", action="store_true", help="time only the shifted-x MV candidates (+ AUTO)")
     ap.add_argument("--staged-only", action="store_true", help="time only the TMA-staged candidates (+ AUTO)")
     ap.add_argument("--tshift-only", action="store_true", help="time only the constant-shift TMV candidates (+ AUTO)")
+    ap.add_argument("--misx-only", action="store_true", help="time only the round-2 misaligned-MV candidates (+ AUTO)")
     ap.add_argument("--graph-below", type=float, default=0,
                     help="time problems smaller than this many bytes from CUDA graphs (device time)")
     a = ap.parse_args()
@@ -262,6 +277,8 @@ def main():
                 elif a.staged_only:           # every TMA-staged plan: row tiles, TMV tiles, MV_TPR
                     cands = [("AUTO", None)] + rowtile_grid(op, R, C) + \
                         [c for c in grids(op, R, C, a.dtype) if c[0] == "MV_TPR"]
+                elif a.misx_only:
+                    cands = [("AUTO", None)] + misx_grid(op, R, C)
                 elif a.tshift_only:
                     cands = [("AUTO", None)] + tshift_grid(op, R, C)
                 elif a.flat_only:
