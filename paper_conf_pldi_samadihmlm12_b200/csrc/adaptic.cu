@@ -1332,6 +1332,41 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
     }
     const bool tmis = !p->vec_shape && R >= 8;
     p->mis = tmis;
+    if (tmis && (v == ADAPTIC_V_TMV_SPLITK || v == ADAPTIC_V_TMV_COL) && par(ADAPTIC_P_XSMEM) == 10) {
+        // sliding window (tmv_window_kernel): one aligned load per row and thread, no c-lanes
+        int G8 = par(ADAPTIC_P_UNROLL) == 4 ? 1 : 2;
+        void* fn = tmv_window_fn(dt, G8);
+        if (!fn) return ADAPTIC_ERR_INVALID_ARG;
+        const int NT = 256;
+        int cps = par(ADAPTIC_P_CTAS_PER_SM);
+        if (cps <= 0) cps = occupancy(fn, NT, 0, dev.present, 2);
+        const int64_t slots = int64_t(dev.sms) * cps;
+        const int64_t tiles = ceil_div(ceil_div(R, 4), int64_t(NT - 1));
+        // splits only when the tiles cannot fill the GPU (the per-output merge costs more than a
+        // partly idle last wave: 1048577 x 64 at S = 2 ran 0.69 of peak, S = 1 shapes 0.93)
+        int64_t S = par(ADAPTIC_P_SPLITS) > 0 ? par(ADAPTIC_P_SPLITS)
+                  : tiles * 2 >= slots ? 1
+                  : pick_splits(tiles, slots, std::max<int64_t>(1, ceil_div(C, int64_t(8 * G8))), 1);
+        for (;;) {
+            const int64_t rows = ceil_div(C, S);
+            p->chain[1] = std::min<int64_t>(rows, FOLD) + rows / FOLD;
+            p->depth[1] = (S > 1 ? ceil_div(S, 2) + 1 : 0) + 2;
+            p->path_ok[1] = (dt == DT_I32) || bound_ok(p->chain[1] + p->depth[1]);
+            if (p->path_ok[1] || S >= (int64_t(1) << 20)) break;
+            S *= 2;
+        }
+        if (S > INT_MAX || !p->path_ok[1]) return ADAPTIC_ERR_UNSUPPORTED;
+        p->xmode = 10;
+        p->lanes = NT - 1; p->unroll = 4 * G8; p->block = NT; p->ctas_per_sm = cps; p->splits = int(S);
+        p->grid[1] = std::max<int64_t>(1, std::min<int64_t>(tiles * S, slots));
+        p->grid[0] = p->grid[1]; p->chain[0] = p->chain[1]; p->depth[0] = p->depth[1]; p->path_ok[0] = p->path_ok[1];
+        if (S > 1) {
+            const size_t part = ((size_t(R) * size_t(S) * 4 + 255) / 256) * 256;
+            p->cnt_off = part;
+            p->ws_bytes = part + size_t(tiles) * 4;
+        }
+        return ADAPTIC_OK;
+    }
     if (tmis && (v == ADAPTIC_V_TMV_SPLITK || v == ADAPTIC_V_TMV_COL) && par(ADAPTIC_P_XSMEM) == 7) {
         // constant word shift per c-lane (tmv_shift_kernel): one aligned load per row, no funnel
         int LR = par(ADAPTIC_P_LANES);
@@ -1772,7 +1807,8 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
                 args = args7;
                 break;
             }
-            fn = (mis && p->xmode == 7) ? tmv_shift_fn(dt, p->lanes, p->unroll)
+            fn = (mis && p->xmode == 10) ? tmv_window_fn(dt, p->unroll / 4)
+                 : (mis && p->xmode == 7) ? tmv_shift_fn(dt, p->lanes, p->unroll)
                  : mis ? tmv_mis_fn(dt, p->lanes, p->unroll) : tmv_fn(dt, p->lanes, p->unroll, vec, p->block);
             args8[0] = &A; args8[1] = &X; args8[2] = &y; args8[3] = &R; args8[4] = &C;
             args8[5] = &S; args8[6] = &part; args8[7] = &cnt;
@@ -2009,12 +2045,13 @@ adaptic_status adaptic_run(adaptic_plan_t p, const void* A, const void* x, void*
 // ---- batched issue over concurrent streams (per host thread, per device)
 namespace {
 constexpr int kMaxBatchStreams = 8;
-// Plans that run alone inside adaptic_run_batch: the staged row-tile kernels (xmode 4 on the
-// lane-group variants and TMV_REGTILE), persistent grids sized for a free GPU.  Measured
-// (2 streams): offgrid step +1.7 %, while making MV_TPR exclusive too (any >= 64 KB of
-// dynamic smem) cost the default sweep 1.8 %.  ADAPTIC_EXCLUSIVE=0 disables (read once).
+// Plans that may run alone inside adaptic_run_batch: the staged row-tile kernels (xmode 4 on the
+// lane-group variants and TMV_REGTILE), persistent grids sized for a free GPU.  Round 1
+// measured +1.7 % on the offgrid step with them exclusive; with round 2's kernels the same step
+// is 4 % FASTER without it (5689 -> 5901 GB/s, 2 streams; 3 streams without it: 5106), so it is
+// off by default.  ADAPTIC_EXCLUSIVE=1 enables it (read once).
 bool plan_exclusive(const adaptic_plan_s* p) {
-    static const bool on = [] { const char* e = std::getenv("ADAPTIC_EXCLUSIVE"); return !(e && e[0] == '0'); }();
+    static const bool on = [] { const char* e = std::getenv("ADAPTIC_EXCLUSIVE"); return e && e[0] == '1'; }();
     return on && p->nvec == 1 && p->xmode == 4 &&
            (p->variant == ADAPTIC_V_MV_SUBWARP || p->variant == ADAPTIC_V_MV_WPR || p->variant == ADAPTIC_V_TMV_REGTILE);
 }

@@ -30,4 +30,13 @@ void* tmv_shift_fn(int dt, int LR, int U) {
     return dt == ADAPTIC_I32 ? ts_l<uint32_t>(LR, U) : ts_l<float>(LR, U);
 }
 
+// sliding-window misaligned TMV (tmv_window_kernel): G8 groups of 4 rows in flight, NT = 256
+void* tmv_window_fn(int dt, int G8) {
+    if (dt == ADAPTIC_I32)
+        return G8 == 1 ? reinterpret_cast<void*>(&tmv_window_kernel<uint32_t, 1, 256>)
+             : G8 == 2 ? reinterpret_cast<void*>(&tmv_window_kernel<uint32_t, 2, 256>) : nullptr;
+    return G8 == 1 ? reinterpret_cast<void*>(&tmv_window_kernel<float, 1, 256>)
+         : G8 == 2 ? reinterpret_cast<void*>(&tmv_window_kernel<float, 2, 256>) : nullptr;
+}
+
 }  // namespace adaptic

@@ -113,6 +113,10 @@ void* tmv_ring_fn(int dt, int K, int opt);
 //           128-bit load per row and thread at a constant word shift per c-lane; tiles of
 //           4 LR - 4 outputs, LR in {16, 32, 64}, U in {2, 4, 8}, NT = 256 (tmv_mis_kernel.cuh)
 void* tmv_shift_fn(int dt, int LR, int U);
+//   twin: tmv arguments; rows off the 16-byte grid, one aligned load per row per thread, 7
+//         accumulators and a compile-time shift pattern per 4 rows (tmv_window_kernel), tiles of
+//         NT - 1 owned windows, G8 in {1, 2} groups of 4 rows in flight, NT = 256 (XSMEM 10)
+void* tmv_window_fn(int dt, int G8);
 int64_t tring_stage_words_h(int64_t R, int TW, int CR, int K);
 constexpr int64_t MRING_SMEM_BUDGET = 220 * 1024;
 constexpr int TMMV_TMA_STAGE_V4 = 2048;              // 32 KB per stage

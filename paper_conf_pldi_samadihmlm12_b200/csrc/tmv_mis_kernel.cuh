@@ -262,3 +262,175 @@ tmv_shift_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restrict
 }
 
 }  // namespace adaptic
+
+namespace adaptic {
+
+// Rows off the 16-byte grid with ONE aligned 128-bit load per row and thread and no c-lanes
+// (round 2, "sliding window"): thread w of the aligned view streams window w (words 4w..4w+3
+// of every row's aligned base); in row c, word j is output 4w + j - s_c (s_c = (b0 + c R)
+// mod 4), so over all rows a thread touches outputs 4w - 3 .. 4w + 3 and keeps 7
+// accumulators.  s_c has period 4 in c, so rows are taken in groups of 4 whose shift
+// pattern (s0, R mod 4) is a template argument: every accumulator index is a compile-time
+// constant.  At the end output 4w + k = acc_w[k + 3] + acc_{w+1}[k - 1] (k >= 1): a shuffle
+// from the next lane; the last thread of a tile only supplies that halo (tiles of NT - 1
+// owned windows).  Splits over c, the ticket merge per tile as tmv_kernel.
+template <class T, int S0, int RM, int G8>
+__device__ __forceinline__ void win_rows(T (&acc)[7], const vec4_t<T>* __restrict__ Ba, const T* __restrict__ B,
+                                         const T* __restrict__ X, int b0, int64_t R, int64_t C, int64_t total,
+                                         int64_t w, int64_t c, int64_t c1) {
+    using E = vec4_t<T>;
+    constexpr int RMN = RM & 3;
+    // G8 groups of 4 rows per iteration (4 G8 loads in flight)
+    for (; c + 4 * G8 - 1 < c1; c += 4 * G8) {
+        E a[4 * G8];
+        T xs[4 * G8];
+        const int64_t qf = ((b0 + c * R) >> 2) + w;
+        const int64_t ql = ((b0 + (c + 4 * G8 - 1) * R) >> 2) + w;
+        if (4 * qf - b0 >= 0 && 4 * ql - b0 + 3 < total) {
+#pragma unroll
+            for (int u = 0; u < 4 * G8; ++u) {
+                a[u] = ld_stream(Ba + ((b0 + (c + u) * R) >> 2) + w);
+                xs[u] = ld_x(X + c + u);
+            }
+        } else {
+#pragma unroll
+            for (int u = 0; u < 4 * G8; ++u) {
+                a[u] = ld_inside(Ba, B, ((b0 + (c + u) * R) >> 2) + w, b0, total);
+                xs[u] = ld_x(X + c + u);
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < 4 * G8; ++u) {
+            const int s = (S0 + (u & 3) * RMN) & 3;          // compile-time after unrolling
+            // word j -> accumulator j - s + 3
+            switch (s) {
+                case 0: acc[3] = mac(a[u].x, xs[u], acc[3]); acc[4] = mac(a[u].y, xs[u], acc[4]);
+                        acc[5] = mac(a[u].z, xs[u], acc[5]); acc[6] = mac(a[u].w, xs[u], acc[6]); break;
+                case 1: acc[2] = mac(a[u].x, xs[u], acc[2]); acc[3] = mac(a[u].y, xs[u], acc[3]);
+                        acc[4] = mac(a[u].z, xs[u], acc[4]); acc[5] = mac(a[u].w, xs[u], acc[5]); break;
+                case 2: acc[1] = mac(a[u].x, xs[u], acc[1]); acc[2] = mac(a[u].y, xs[u], acc[2]);
+                        acc[3] = mac(a[u].z, xs[u], acc[3]); acc[4] = mac(a[u].w, xs[u], acc[4]); break;
+                default: acc[0] = mac(a[u].x, xs[u], acc[0]); acc[1] = mac(a[u].y, xs[u], acc[1]);
+                         acc[2] = mac(a[u].z, xs[u], acc[2]); acc[3] = mac(a[u].w, xs[u], acc[3]); break;
+            }
+        }
+    }
+    for (; c < c1; ++c) {                                   // rows left: runtime shift
+        const int64_t f = b0 + c * R;
+        const E a = ld_inside(Ba, B, (f >> 2) + w, b0, total);
+        const T xv = ld_x(X + c);
+        const int s = int(f & 3);
+        const T v[4] = {a.x, a.y, a.z, a.w};
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            const int k = j - s + 3;
+#pragma unroll
+            for (int q = 0; q < 7; ++q)
+                if (q == k) acc[q] = mac(v[j], xv, acc[q]);
+        }
+    }
+}
+
+template <class T, int G8, int S0, int RM>
+__device__ __forceinline__ void win_dispatch_rm(T (&acc)[7], const vec4_t<T>* Ba, const T* B, const T* X, int b0,
+                                                int64_t R, int64_t C, int64_t total, int64_t w, int64_t c, int64_t c1) {
+    win_rows<T, S0, RM, G8>(acc, Ba, B, X, b0, R, C, total, w, c, c1);
+}
+
+template <class T, int G8>
+__device__ __forceinline__ void win_dispatch(T (&acc)[7], const vec4_t<T>* Ba, const T* B, const T* X, int b0,
+                                             int64_t R, int64_t C, int64_t total, int64_t w, int64_t c, int64_t c1) {
+    const int s0 = int((b0 + c * R) & 3), rm = int(R & 3);
+    switch (s0 * 4 + rm) {
+#define ADAPTIC_WIN(S, M) case S * 4 + M: win_rows<T, S, M, G8>(acc, Ba, B, X, b0, R, C, total, w, c, c1); break;
+        ADAPTIC_WIN(0, 0) ADAPTIC_WIN(0, 1) ADAPTIC_WIN(0, 2) ADAPTIC_WIN(0, 3)
+        ADAPTIC_WIN(1, 0) ADAPTIC_WIN(1, 1) ADAPTIC_WIN(1, 2) ADAPTIC_WIN(1, 3)
+        ADAPTIC_WIN(2, 0) ADAPTIC_WIN(2, 1) ADAPTIC_WIN(2, 2) ADAPTIC_WIN(2, 3)
+        ADAPTIC_WIN(3, 0) ADAPTIC_WIN(3, 1) ADAPTIC_WIN(3, 2) ADAPTIC_WIN(3, 3)
+#undef ADAPTIC_WIN
+        default: break;
+    }
+}
+
+template <class T, int G8, int NT>
+__global__ void __launch_bounds__(NT, 2)
+tmv_window_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restrict__ y,
+                  int64_t R, int64_t C, int S, T* __restrict__ ws_part, unsigned int* __restrict__ ws_cnt)
+{
+    pdl_prologue();
+    using E = vec4_t<T>;
+    __shared__ T halo[NT][3];
+    __shared__ unsigned int flag;
+    const int b0 = int((reinterpret_cast<uintptr_t>(B) >> 2) & 3u);
+    const E* __restrict__ Ba = reinterpret_cast<const E*>(B - b0);
+    const int64_t total = R * C;
+    const int64_t own = (R + 3) / 4;                       // windows that own outputs (4w < R)
+    const int64_t ntiles = (own + NT - 2) / (NT - 1);
+    const int64_t chunk = (C + S - 1) / S;
+    const int tid = threadIdx.x;
+    const int64_t nblk = ntiles * S;
+    for (int64_t blk = blockIdx.x; blk < nblk; blk += gridDim.x) {
+        const int64_t tile = blk % ntiles;
+        const int s = int(blk / ntiles);
+        const int64_t w = tile * (NT - 1) + tid;             // this thread's window
+        const int64_t c0 = min(C, int64_t(s) * chunk), c1 = min(C, c0 + chunk);
+        T acc[7];
+#pragma unroll
+        for (int q = 0; q < 7; ++q) acc[q] = T(0);
+        if (4 * w < R + 3) {                                 // windows past the data hold nothing
+            // fp32 chains: fold every FOLD rows into a second level
+            T outer[7];
+#pragma unroll
+            for (int q = 0; q < 7; ++q) outer[q] = T(0);
+            for (int64_t cb = c0; cb < c1; cb += FOLD) {
+                const int64_t ce = min(c1, cb + int64_t(FOLD));
+                T a2[7];
+#pragma unroll
+                for (int q = 0; q < 7; ++q) a2[q] = T(0);
+                win_dispatch<T, G8>(a2, Ba, B, X, b0, R, C, total, w, cb, ce);
+#pragma unroll
+                for (int q = 0; q < 7; ++q) outer[q] += a2[q];
+            }
+#pragma unroll
+            for (int q = 0; q < 7; ++q) acc[q] = outer[q];
+        }
+        halo[tid][0] = acc[0]; halo[tid][1] = acc[1]; halo[tid][2] = acc[2];
+        __syncthreads();
+        T out[4];
+        out[0] = acc[3];
+#pragma unroll
+        for (int k = 1; k < 4; ++k) out[k] = acc[3 + k] + (tid + 1 < NT ? halo[tid + 1][k - 1] : T(0));
+        const bool owner = tid < NT - 1 && w < own;
+        if (S == 1) {
+            if (owner)
+#pragma unroll
+                for (int k = 0; k < 4; ++k)
+                    if (4 * w + k < R) y[4 * w + k] = out[k];
+        } else {
+            if (owner)
+#pragma unroll
+                for (int k = 0; k < 4; ++k)
+                    if (4 * w + k < R) ws_part[int64_t(s) * R + 4 * w + k] = out[k];
+            if (ticket_is_last(ws_cnt + tile, unsigned(S), &flag)) {
+                if (owner)
+#pragma unroll
+                    for (int k = 0; k < 4; ++k) {
+                        const int64_t o = 4 * w + k;
+                        if (o < R) {
+                            T m0 = T(0), m1 = T(0);
+                            int q = 0;
+                            for (; q + 1 < S; q += 2) {
+                                m0 += ld_partial(ws_part + int64_t(q) * R + o);
+                                m1 += ld_partial(ws_part + int64_t(q + 1) * R + o);
+                            }
+                            if (q < S) m0 += ld_partial(ws_part + int64_t(q) * R + o);
+                            y[o] = m0 + m1;
+                        }
+                    }
+            }
+        }
+        __syncthreads();
+    }
+}
+
+}  // namespace adaptic

@@ -218,9 +218,9 @@ def test_tmv_rowtile_unaligned_bases_fall_back():
 
 
 def test_batch_with_exclusive_staged_plans():
-    """adaptic_run_batch runs staged-tile plans (>= 64 KB of dynamic shared memory per CTA)
-    alone between the other lanes' work: results equal single runs bit for bit on 1..3
-    streams, with staged and direct plans interleaved."""
+    """adaptic_run_batch with staged-tile plans (>= 64 KB of dynamic shared memory per CTA;
+    run alone between the other lanes' work when ADAPTIC_EXCLUSIVE=1, interleaved by default):
+    results equal single runs bit for bit on 1..3 streams, staged and direct plans mixed."""
     dev = torch.device(DEV)
     stream = torch.cuda.current_stream().cuda_stream
     cases = [("mv", 20000, 257, "MV_WPR", rt_params(32)), ("mv", 512, 3000, "AUTO", None),

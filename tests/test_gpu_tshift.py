@@ -61,3 +61,35 @@ def test_tshift_int32_and_p5_exact():
         yf = adaptic.tmv(placed(Bf, off, torch.float32), torch.from_numpy(xf).to(DEV), variant="TMV_SPLITK",
                          params=[32, 5, 0, 4, 7]).cpu().numpy()
         assert np.array_equal(yf.astype(np.float64), oracle.tmv(Bf, xf)[0]), (R, C, off)
+
+
+def test_window_kernel_every_shape_alignment_and_split():
+    """tmv_window_kernel (TMV_SPLITK with XSMEM 10): one aligned 128-bit load per row and
+    thread, 7 accumulators with a compile-time shift pattern per 4 rows (every R mod 4 and B
+    base alignment), the halo shuffle between windows and tiles, rows left over after the
+    groups of 4 / 8, splits with the ticket merge; fp32 within 1e-4 S_r, int32 exact."""
+    fails = []
+    shapes = SHAPES + [(1021, 3), (1022, 13), (1023, 300), (250000, 9), (8193, 1)]
+    for (R, C), off, p in itertools.product(shapes, (0, 1, 2, 3),
+                                            [[0, 0, 0, 0, 10], [0, 0, 0, 4, 10], [0, 7, 0, 8, 10]]):
+        for dt in ("f32", "i32"):
+            np_dt = np.float32 if dt == "f32" else np.int32
+            tdt = torch.float32 if dt == "f32" else torch.int32
+            B = synth.matrix(R, C, "tmv", np_dt, "uniform", 71 + R)
+            x = synth.vector(C, np_dt, "uniform", 72 + C)
+            try:
+                d = adaptic.plan("tmv", R, C, dt, variant="TMV_SPLITK", params=p).describe()
+                if R % 4 == 0 or R < 8:
+                    continue
+                assert d["xmode"] == 10, d
+                y = adaptic.tmv(placed(B, off, tdt), placed(x, (off + 2) % 4, tdt), variant="TMV_SPLITK",
+                                params=p).cpu().numpy()
+                if dt == "i32":
+                    assert np.array_equal(y, oracle.tmv(B, x)), "int32 mismatch"
+                else:
+                    yr, S = oracle.tmv(B, x)
+                    bad = ~(np.abs(y.astype(np.float64) - yr) <= 1e-4 * S)
+                    assert not bad.any(), f"{bad.sum()} out of tolerance, first {np.argwhere(bad)[:4].ravel()}"
+            except Exception as e:  # noqa: BLE001
+                fails.append(f"{dt} {R}x{C} off={off} {p}: {type(e).__name__}: {str(e)[:160]}")
+    assert not fails, f"{len(fails)} failures\n" + "\n".join(fails[:30])

@@ -94,11 +94,13 @@ def misx_grid(op, R, C):
 
 
 def tshift_grid(op, R, C):
-    """TMV rows off the 16-byte grid on the constant-shift kernel (XSMEM 7, round 2):
-    tile width LR (c-lanes 256 / LR, a multiple of 4) x loads in flight U."""
+    """TMV rows off the 16-byte grid, round 2: the constant-shift kernel (XSMEM 7; tile width LR,
+    c-lanes 256 / LR a multiple of 4, x loads in flight U) and the sliding-window kernel (XSMEM
+    10; 4 or 8 rows in flight, splits auto or 1)."""
     if op != "tmv" or R % 4 == 0 or R < 8:
         return []
-    return [("TMV_SPLITK", [lr, 0, 0, u, 7]) for lr in (16, 32, 64) for u in (2, 4, 8)]
+    return [("TMV_SPLITK", [lr, 0, 0, u, 7]) for lr in (16, 32, 64) for u in (2, 4, 8)] + \
+        [("TMV_SPLITK", [0, 0, 0, u, 10]) for u in (4, 8)] + [("TMV_SPLITK", [0, 1, 0, 8, 10])]
 
 
 def grids(op, R, C, dtype="f32"):
