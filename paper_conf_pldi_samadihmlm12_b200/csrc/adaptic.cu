@@ -1011,6 +1011,56 @@ adaptic_status derive_rowtile(adaptic_plan_s* p, const int32_t* params, const De
     return ADAPTIC_OK;
 }
 
+// MV on TMA-staged tiles of k <= RTC_KMAX_H long rows, each tile reduced by the whole CTA with x
+// staged once in shared memory (rowtile_kernel.cuh mv_rowtile_cta_kernel): MV_CPR with
+// [ADAPTIC_P_XSMEM] = 11.  [BLOCK] 256 | 512, [ROWS] k (-n: ~n KB per tile), [UNROLL] ring
+// stages, [CTAS_PER_SM]; C <= 36 * NT (x in registers; describe()'s lanes = x values per
+// thread).  16-byte-aligned A at run time, else the variant's direct kernel.
+adaptic_status derive_rowtile_cta(adaptic_plan_s* p, const int32_t* params, const DevInfo& dev) {
+    auto par = [&](int i) -> int { return params ? params[i] : 0; };
+    const int64_t R = p->R, C = p->C;
+    int NT = par(ADAPTIC_P_BLOCK);
+    if (NT <= 0) NT = C <= 256 * 36 ? 256 : 512;
+    if (NT != 256 && NT != 512) return ADAPTIC_ERR_INVALID_ARG;
+    const int64_t mx_need = ceil_div(C, int64_t(NT));
+    const int MX = mx_need <= 4 ? 4 : mx_need <= 8 ? 8 : mx_need <= 16 ? 16 : mx_need <= 36 ? 36 : 0;
+    if (MX == 0) return ADAPTIC_ERR_UNSUPPORTED;              // x must fit the registers
+    int cps = par(ADAPTIC_P_CTAS_PER_SM);
+    if (cps <= 0) cps = C <= 4096 ? 2 : 1;
+    const size_t budget = size_t(220) * 1024 / size_t(cps);
+    const size_t xbytes = 0;
+    if (xbytes + 2 * rowtile_tile_words(1, C) * 4 > budget) return ADAPTIC_ERR_UNSUPPORTED;
+    int64_t k = par(ADAPTIC_P_ROWS);
+    if (k < 0) k = (int64_t(-k) * 1024) / (C * 4);
+    else if (k == 0) k = (int64_t(32) * 1024) / (C * 4);
+    k = std::max<int64_t>(1, std::min<int64_t>({k, int64_t(RTC_KMAX_H), std::max<int64_t>(1, R)}));
+    while (k > 1 && xbytes + 2 * rowtile_tile_words(k, C) * 4 > budget) --k;
+    const size_t stage_bytes = rowtile_tile_words(k, C) * 4;
+    int stages = int(std::min<size_t>(RT_MAX_STAGES_H, (budget - xbytes) / stage_bytes));
+    if (par(ADAPTIC_P_UNROLL) > 0) stages = std::min(stages, par(ADAPTIC_P_UNROLL));
+    void* fn = rowtile_cta_fn(p->dtype, NT, MX, int(k));
+    if (!fn) return ADAPTIC_ERR_UNSUPPORTED;
+    while (stages >= 2 && !smem_fits(fn, size_t(stages) * stage_bytes + xbytes, dev.present)) --stages;
+    if (stages < 2) return ADAPTIC_ERR_UNSUPPORTED;
+    p->smem = size_t(stages) * stage_bytes + xbytes;
+    const int occ = occupancy(fn, NT, p->smem, dev.present, cps);
+    if (occ < 1) return ADAPTIC_ERR_UNSUPPORTED;
+    p->ctas_per_sm = std::min(cps, occ);
+    p->lanes = MX; p->block = NT; p->rb = int(k); p->stages = stages; p->unroll = stages;
+    p->xmode = 11;
+    p->mis = !p->vec_shape;
+    p->grid[1] = std::max<int64_t>(1, std::min<int64_t>(ceil_div(R, k), int64_t(dev.sms) * p->ctas_per_sm));
+    p->chain[1] = mx_need;
+    p->depth[1] = 5 + NT / 64 + 1;                      // butterfly, two chains over the warps, their sum
+    p->path_ok[1] = (p->dtype == DT_I32) || bound_ok(p->chain[1] + p->depth[1]);
+    if (!p->path_ok[1]) return ADAPTIC_ERR_UNSUPPORTED;
+    p->ws_bytes = 0;
+    adaptic_plan_s fb = *p;                             // the direct kernel for unaligned A
+    p->fb_ws_off = 0;
+    if (derive(&fb, nullptr, dev) == ADAPTIC_OK) p->ws_bytes = fb.ws_bytes;
+    return ADAPTIC_OK;
+}
+
 // TMV with few outputs on TMA-staged tiles of B (tmv_rowtile_kernel.cuh): TMV_REGTILE with
 // [ADAPTIC_P_XSMEM] = 4.  [BLOCK] threads 256 | 512 | 1024 (>= R), [ROWS] rows of B per
 // tile k (a multiple of 4), [UNROLL] ring stages, [CTAS_PER_SM].  16-byte-aligned B and x
@@ -1139,6 +1189,8 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
     for (int w = 0; w < 2; ++w) { p->grid[w] = 0; p->chain[w] = 0; p->depth[w] = 0; p->path_ok[w] = false; }
     if ((v == ADAPTIC_V_MV_SUBWARP || v == ADAPTIC_V_MV_WPR) && par(ADAPTIC_P_XSMEM) == 4)
         return derive_rowtile(p, params, dev);
+    if (v == ADAPTIC_V_MV_CPR && op == ADAPTIC_OP_MV && par(ADAPTIC_P_XSMEM) == 11)
+        return derive_rowtile_cta(p, params, dev);
 
     // rows not 16-byte aligned (C % 4 != 0): the misaligned-row kernels keep the matrix
     // stream 128-bit; the plain scalar kernels (index 0) remain for DOT operands whose
@@ -1359,6 +1411,17 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
         p->xmode = 10;
         p->lanes = NT - 1; p->unroll = 4 * G8; p->block = NT; p->ctas_per_sm = cps; p->splits = int(S);
         p->grid[1] = std::max<int64_t>(1, std::min<int64_t>(tiles * S, slots));
+        if (S == 1) {
+            // warp tiles of 31 windows, halo by shuffle, no CTA barrier (tmv_window_warp_kernel)
+            const int minb = par(ADAPTIC_P_CTAS_PER_SM) >= 3 && G8 == 1 ? 3 : 2;
+            void* wf = tmv_window_warp_fn(dt, G8, minb);
+            if (!wf) return ADAPTIC_ERR_INVALID_ARG;
+            p->ctas_per_sm = occupancy(wf, NT, 0, dev.present, minb);
+            const int64_t wtiles = ceil_div(ceil_div(R, 4), int64_t(31));
+            p->lanes = 31;
+            p->grid[1] = std::max<int64_t>(1, std::min<int64_t>(ceil_div(wtiles, int64_t(NT / 32)),
+                                                                int64_t(dev.sms) * p->ctas_per_sm));
+        }
         p->grid[0] = p->grid[1]; p->chain[0] = p->chain[1]; p->depth[0] = p->depth[1]; p->path_ok[0] = p->path_ok[1];
         if (S > 1) {
             const size_t part = ((size_t(R) * size_t(S) * 4 + 255) / 256) * 256;
@@ -1756,6 +1819,14 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
             break;
         case ADAPTIC_V_MV_CPR:
         case ADAPTIC_V_MV_SPLIT:
+            if (p->xmode == 11) {                         // long rows on staged tiles, CTA-wide
+                fn = rowtile_cta_fn(dt, p->block, p->lanes, p->rb);
+                smem = p->smem;
+                args7[0] = &A; args7[1] = &X; args7[2] = &y; args7[3] = &R; args7[4] = &C;
+                args7[5] = &tile_mb; args7[6] = &stages;
+                args = args7;
+                break;
+            }
             if (p->xmode == 6) {                          // TMA-ring kernel, K = 1
                 fn = vec ? mmv_ring_fn(dt, 1) : nullptr;
                 smem = p->smem;
@@ -1805,6 +1876,12 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
                 args7[0] = &A; args7[1] = &X; args7[2] = &y; args7[3] = &R; args7[4] = &C;
                 args7[5] = &part; args7[6] = &cnt;
                 args = args7;
+                break;
+            }
+            if (mis && p->xmode == 10 && S == 1) {
+                fn = tmv_window_warp_fn(dt, p->unroll / 4, p->ctas_per_sm >= 3 ? 3 : 2);
+                args8[0] = &A; args8[1] = &X; args8[2] = &y; args8[3] = &R; args8[4] = &C;
+                args = args8;
                 break;
             }
             fn = (mis && p->xmode == 10) ? tmv_window_fn(dt, p->unroll / 4)
@@ -2010,8 +2087,8 @@ adaptic_status adaptic_run(adaptic_plan_t p, const void* A, const void* x, void*
                 ((reinterpret_cast<uintptr_t>(A) - reinterpret_cast<uintptr_t>(x)) & 15u) == 0);
     if (mis && p->variant == ADAPTIC_V_MV_TPR)   // bulk copies of row tiles: 16-byte aligned bases
         mis = aligned(A, 16) && (p->op != ADAPTIC_OP_DOT || aligned(x, 16));
-    if (p->nvec == 1 && p->xmode == 4 && (p->variant == ADAPTIC_V_MV_SUBWARP || p->variant == ADAPTIC_V_MV_WPR ||
-                                           p->variant == ADAPTIC_V_TMV_REGTILE)) {
+    if (p->nvec == 1 && ((p->xmode == 4 && (p->variant == ADAPTIC_V_MV_SUBWARP || p->variant == ADAPTIC_V_MV_WPR ||
+                                            p->variant == ADAPTIC_V_TMV_REGTILE)) || p->xmode == 11)) {
         // row tiles are bulk-copied from 16-byte-aligned bases; other pointers take the
         // direct kernel of the same variant and shape
         if (aligned(A, 16) && (p->op == ADAPTIC_OP_MV || aligned(x, 16)))

@@ -34,6 +34,42 @@ void* rowtile_fn(int dtype, int NT, int G, bool px) {
     return dtype == DT_F32 ? rt_t<float>(NT, G, px) : rt_t<uint32_t>(NT, G, px);
 }
 
+// whole-CTA reduction of k <= RTC_KMAX long rows per staged tile (MV_CPR, XSMEM 11): NT in
+// {256, 512}, MX x values per thread in {4, 8, 16, 36} (C <= NT * MX), KR rows bound in
+// {1, 2, 3, 4, 6, 8} (k <= KR)
+template <class T, int NT, int MX>
+static void* rtc_k(int KR) {
+    switch (KR) {
+        case 1: return reinterpret_cast<void*>(&mv_rowtile_cta_kernel<T, NT, MX, 1>);
+        case 2: return reinterpret_cast<void*>(&mv_rowtile_cta_kernel<T, NT, MX, 2>);
+        case 3: return reinterpret_cast<void*>(&mv_rowtile_cta_kernel<T, NT, MX, 3>);
+        case 4: return reinterpret_cast<void*>(&mv_rowtile_cta_kernel<T, NT, MX, 4>);
+        case 6: return reinterpret_cast<void*>(&mv_rowtile_cta_kernel<T, NT, MX, 6>);
+        case 8: return reinterpret_cast<void*>(&mv_rowtile_cta_kernel<T, NT, MX, 8>);
+        default: return nullptr;
+    }
+}
+template <class T, int NT>
+static void* rtc_m(int MX, int KR) {
+    switch (MX) {
+        case 4: return rtc_k<T, NT, 4>(KR);
+        case 8: return rtc_k<T, NT, 8>(KR);
+        case 16: return rtc_k<T, NT, 16>(KR);
+        case 36: return rtc_k<T, NT, 36>(KR);
+        default: return nullptr;
+    }
+}
+template <class T>
+static void* rtc_n(int NT, int MX, int KR) {
+    return NT == 256 ? rtc_m<T, 256>(MX, KR) : NT == 512 ? rtc_m<T, 512>(MX, KR) : nullptr;
+}
+int rowtile_cta_kr(int k) { return k <= 4 ? k : k <= 6 ? 6 : 8; }
+void* rowtile_cta_fn(int dtype, int NT, int MX, int k) {
+    const int KR = rowtile_cta_kr(k);
+    return dtype == DT_F32 ? rtc_n<float>(NT, MX, KR) : rtc_n<uint32_t>(NT, MX, KR);
+}
+static_assert(RTC_KMAX == RTC_KMAX_H, "long-row tile height: kernel vs planner");
+
 }  // namespace adaptic
 
 namespace adaptic {

@@ -39,4 +39,17 @@ void* tmv_window_fn(int dt, int G8) {
          : G8 == 2 ? reinterpret_cast<void*>(&tmv_window_kernel<float, 2, 256>) : nullptr;
 }
 
+// warp-tile form (S = 1): register cap for 2 resident CTAs of 256 (8 rows in flight) or 3
+// (4 rows; 8 rows at 3 CTAs spill)
+template <class T>
+static void* tww(int G8, int minb) {
+    if (G8 == 2 && minb <= 2) return reinterpret_cast<void*>(&tmv_window_warp_kernel<T, 2, 256, 2>);
+    if (G8 == 1 && minb <= 2) return reinterpret_cast<void*>(&tmv_window_warp_kernel<T, 1, 256, 2>);
+    if (G8 == 1 && minb == 3) return reinterpret_cast<void*>(&tmv_window_warp_kernel<T, 1, 256, 3>);
+    return nullptr;
+}
+void* tmv_window_warp_fn(int dt, int G8, int minb) {
+    return dt == ADAPTIC_I32 ? tww<uint32_t>(G8, minb) : tww<float>(G8, minb);
+}
+
 }  // namespace adaptic

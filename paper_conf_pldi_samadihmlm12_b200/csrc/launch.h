@@ -71,6 +71,7 @@ void* tmv_flat_fn(int dtype, int U, int NT);
 // [ADAPTIC_P_XSMEM] = 4), C <= 32*G, 16-byte-aligned A (and DOT's b), NT in {256, 512}:
 //   (const T* A, const T* X, T* y, int64_t R, int64_t C, int k, int stages)   [dynamic smem]
 constexpr int RT_MAX_C_PER_LANE = 32;
+constexpr int RTC_KMAX_H = 8;                // rows per long-row staged tile (rowtile_kernel.cuh RTC_KMAX)
 constexpr int RT_MAX_STAGES_H = 8;          // == RT_MAX_STAGES, TRT_MAX_STAGES (mbarriers per CTA; static_assert in k_rowtile.cu)
 void* rowtile_fn(int dtype, int NT, int G, bool px);
 size_t rowtile_tile_words(int64_t k, int64_t C);
@@ -117,6 +118,8 @@ void* tmv_shift_fn(int dt, int LR, int U);
 //         accumulators and a compile-time shift pattern per 4 rows (tmv_window_kernel), tiles of
 //         NT - 1 owned windows, G8 in {1, 2} groups of 4 rows in flight, NT = 256 (XSMEM 10)
 void* tmv_window_fn(int dt, int G8);
+void* rowtile_cta_fn(int dtype, int NT, int MX, int k);   // MX in {4, 8, 16, 36}: C <= NT * MX; k <= 8 rows
+void* tmv_window_warp_fn(int dt, int G8, int minb);
 int64_t tring_stage_words_h(int64_t R, int TW, int CR, int K);
 constexpr int64_t MRING_SMEM_BUDGET = 220 * 1024;
 constexpr int TMMV_TMA_STAGE_V4 = 2048;              // 32 KB per stage

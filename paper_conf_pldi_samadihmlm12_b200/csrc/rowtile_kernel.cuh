@@ -134,4 +134,126 @@ mv_rowtile_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restric
     }
 }
 
+// ---------------------------------------------------------------------------------------
+// Long rows off the 16-byte grid (round 2, MV_CPR with [ADAPTIC_P_XSMEM] = 11): C up to ~18K
+// elements, C % 4 != 0 -- 65536 x 1025 ran 0.72-0.74 of the copy peak on the direct
+// misaligned-row kernels (a warp per row has 8 vectors per lane: two round trips and a
+// butterfly per 4 KB row).  Loading is the row-tile ring above (k <= RTC_KMAX whole rows per
+// bulk copy); the reduction uses the WHOLE CTA on all k rows of a tile at once: thread t takes
+// columns t + NT*m (m < MX) of every row (k <= KR, a template bound so that absent rows
+// cost no predicated instructions) with x[t + NT*m] in registers for the whole kernel,
+// so each element costs one conflict-free 32-bit shared load and one FMA.  The k row sums
+// leave each warp through a transposing butterfly (offset 16 exchanges 4 of the 8 row
+// partials, 8 exchanges 2, 4 exchanges 1, then 2 and 1 finish: 9 shuffles for 8 rows instead
+// of 40), and one barrier per tile (per-warp partials double-buffered by tile parity, so the
+// same barrier frees the stage for its refill).  Fixed order throughout (P7).
+constexpr int RTC_KMAX = 8;
+
+template <class T, int NT, int MX, int KR>
+__global__ void __launch_bounds__(NT)
+mv_rowtile_cta_kernel(const T* __restrict__ A, const T* __restrict__ X, T* __restrict__ y,
+                      int64_t R, int64_t C, int k, int stages)
+{
+    pdl_prologue();
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    __shared__ __align__(8) uint64_t full[RT_MAX_STAGES];
+    __shared__ T red[2][NT / 32][RTC_KMAX];
+    constexpr int NW = NT / 32;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int Ci = int(C);
+    const int64_t total = R * C;
+    const int64_t ntiles = (R + k - 1) / k;
+    const int64_t tile_w = ((int64_t(k) * C + 6 + 3) / 4) * 4;
+    T* ring = reinterpret_cast<T*>(smem_raw);
+    const int64_t my_tiles = blockIdx.x < ntiles ? (ntiles - 1 - blockIdx.x) / gridDim.x + 1 : 0;
+
+    if (tid == 0) {
+        for (int s = 0; s < stages; ++s) mbar_init(&full[s], 1);
+        fence_mbar_init();
+    }
+    __syncthreads();
+    auto issue = [&](int64_t i, int slot) {
+        const int64_t r0 = (blockIdx.x + i * gridDim.x) * int64_t(k);
+        const int64_t w0 = r0 * C, w1 = min(R, r0 + k) * C;
+        const int64_t a0 = w0 & ~int64_t(3);
+        int64_t a1 = (w1 + 3) & ~int64_t(3);
+        if (a1 > total) a1 = w1 & ~int64_t(3);
+        const uint32_t bytes = uint32_t((a1 - a0) * int64_t(sizeof(T)));
+        mbar_arrive_expect_tx(&full[slot], bytes);
+        if (bytes) bulk_g2s(ring + slot * tile_w, A + a0, bytes, &full[slot]);
+    };
+    if (tid == 0) {
+        const int64_t pre = min(int64_t(stages), my_tiles);
+        for (int64_t i = 0; i < pre; ++i) issue(i, int(i));
+    }
+    T xr[MX];
+#pragma unroll
+    for (int m = 0; m < MX; ++m) xr[m] = tid + NT * m < Ci ? ld_x(X + tid + NT * m) : T(0);
+
+    int st = 0;
+    uint32_t ph = 0;
+    for (int64_t i = 0; i < my_tiles; ++i, ring_advance(st, ph, stages)) {
+        const int64_t r0 = (blockIdx.x + i * gridDim.x) * int64_t(k);
+        const int nrows = int(min(int64_t(k), R - r0));
+        const int64_t w0 = r0 * C;
+        T* stg = ring + st * tile_w;
+        mbar_wait(&full[st], ph);
+        const int64_t w1 = w0 + int64_t(nrows) * C;
+        if (((w1 + 3) & ~int64_t(3)) > total && (w1 & 3)) {   // the matrix's last < 4 words
+            const int64_t a0 = w0 & ~int64_t(3);
+            for (int64_t e = (w1 & ~int64_t(3)) + tid; e < w1; e += NT) stg[e - a0] = A[e];
+            __syncthreads();
+        }
+        const T* base = stg + (w0 & 3) + tid;
+        T v[RTC_KMAX];
+#pragma unroll
+        for (int r = 0; r < RTC_KMAX; ++r) v[r] = T(0);
+#pragma unroll
+        for (int m = 0; m < MX; ++m) {
+            if (tid + NT * m < Ci) {
+#pragma unroll
+                for (int r = 0; r < KR; ++r)          // KR >= k rows: no issue slots for absent rows
+                    if (r < nrows) v[r] = mac(base[r * Ci + NT * m], xr[m], v[r]);
+            }
+        }
+        // transposing butterfly: lane bit 4 keeps rows 4b4..4b4+3, bit 3 two of those, bit 2 one
+        {
+            const bool b4 = lane & 16, b3 = lane & 8, b2 = lane & 4;
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                const T send = b4 ? v[j] : v[j + 4];
+                const T keep = b4 ? v[j + 4] : v[j];
+                v[j] = keep + __shfl_xor_sync(0xffffffffu, send, 16);
+            }
+#pragma unroll
+            for (int j = 0; j < 2; ++j) {
+                const T send = b3 ? v[j] : v[j + 2];
+                const T keep = b3 ? v[j + 2] : v[j];
+                v[j] = keep + __shfl_xor_sync(0xffffffffu, send, 8);
+            }
+            {
+                const T send = b2 ? v[0] : v[1];
+                const T keep = b2 ? v[1] : v[0];
+                v[0] = keep + __shfl_xor_sync(0xffffffffu, send, 4);
+            }
+            v[0] += __shfl_xor_sync(0xffffffffu, v[0], 2);
+            v[0] += __shfl_xor_sync(0xffffffffu, v[0], 1);
+        }
+        const int par = int(i & 1);
+        if ((lane & 3) == 0) red[par][warp][lane >> 2] = v[0];    // row (b4 b3 b2) = lane / 4
+        __syncthreads();                       // partials written; stage st fully read
+        if (tid == 0 && i + stages < my_tiles) {
+            refill_fence();
+            issue(i + stages, st);
+        }
+        if (tid < nrows) {
+            T s0 = T(0), s1 = T(0);
+#pragma unroll
+            for (int w = 0; w + 1 < NW; w += 2) { s0 += red[par][w][tid]; s1 += red[par][w + 1][tid]; }
+            if (NW & 1) s0 += red[par][NW - 1][tid];
+            y[r0 + tid] = s0 + s1;
+        }
+    }
+}
+
 }  // namespace adaptic

@@ -271,9 +271,12 @@ namespace adaptic {
 // mod 4), so over all rows a thread touches outputs 4w - 3 .. 4w + 3 and keeps 7
 // accumulators.  s_c has period 4 in c, so rows are taken in groups of 4 whose shift
 // pattern (s0, R mod 4) is a template argument: every accumulator index is a compile-time
-// constant.  At the end output 4w + k = acc_w[k + 3] + acc_{w+1}[k - 1] (k >= 1): a shuffle
-// from the next lane; the last thread of a tile only supplies that halo (tiles of NT - 1
-// owned windows).  Splits over c, the ticket merge per tile as tmv_kernel.
+// constant.  At the end output 4w + k = acc_w[k + 3] + acc_{w+1}[k - 1] (k >= 1): read from
+// the next thread through shared memory; the last thread of a tile only supplies that halo
+// (tiles of NT - 1 owned windows).  Splits over c, the ticket merge per tile as tmv_kernel.
+// tmv_window_warp_kernel (S = 1): the same per thread, but each WARP owns a tile of 31
+// windows and takes the halo by shuffle -- no shared memory and no CTA barrier, so warps
+// move on to their next tile independently.
 template <class T, int S0, int RM, int G8>
 __device__ __forceinline__ void win_rows(T (&acc)[7], const vec4_t<T>* __restrict__ Ba, const T* __restrict__ B,
                                          const T* __restrict__ X, int b0, int64_t R, int64_t C, int64_t total,
@@ -430,6 +433,53 @@ tmv_window_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restric
             }
         }
         __syncthreads();
+    }
+}
+
+template <class T, int G8, int NT, int MINB>
+__global__ void __launch_bounds__(NT, MINB)
+tmv_window_warp_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restrict__ y, int64_t R, int64_t C)
+{
+    pdl_prologue();
+    const int b0 = int((reinterpret_cast<uintptr_t>(B) >> 2) & 3u);
+    const vec4_t<T>* __restrict__ Ba = reinterpret_cast<const vec4_t<T>*>(B - b0);
+    const int64_t total = R * C;
+    const int64_t own = (R + 3) / 4;
+    const int64_t ntiles = (own + 30) / 31;
+    const int lane = threadIdx.x & 31;
+    const int64_t nw = int64_t(gridDim.x) * (NT / 32);
+    const bool yv = (reinterpret_cast<uintptr_t>(y) & 15) == 0;
+    for (int64_t t = int64_t(blockIdx.x) * (NT / 32) + (threadIdx.x >> 5); t < ntiles; t += nw) {
+        const int64_t w = t * 31 + lane;
+        T acc[7];
+#pragma unroll
+        for (int q = 0; q < 7; ++q) acc[q] = T(0);
+        if (4 * w < R + 3) {
+            for (int64_t cb = 0; cb < C; cb += FOLD) {
+                const int64_t ce = min(C, cb + int64_t(FOLD));
+                T a2[7];
+#pragma unroll
+                for (int q = 0; q < 7; ++q) a2[q] = T(0);
+                win_dispatch<T, G8>(a2, Ba, B, X, b0, R, C, total, w, cb, ce);
+#pragma unroll
+                for (int q = 0; q < 7; ++q) acc[q] += a2[q];
+            }
+        }
+        T out[4];
+        out[0] = acc[3];
+#pragma unroll
+        for (int k = 1; k < 4; ++k) out[k] = acc[3 + k] + __shfl_down_sync(0xffffffffu, acc[k - 1], 1);
+        if (lane < 31 && w < own) {
+            if (yv && 4 * w + 3 < R) {
+                vec4_t<T> o;
+                o.x = out[0]; o.y = out[1]; o.z = out[2]; o.w = out[3];
+                *reinterpret_cast<vec4_t<T>*>(y + 4 * w) = o;
+            } else {
+#pragma unroll
+                for (int k = 0; k < 4; ++k)
+                    if (4 * w + k < R) y[4 * w + k] = out[k];
+            }
+        }
     }
 }
 

@@ -152,6 +152,82 @@ def test_rowtile_large_held_out_shape_sampled():
         assert np.all(err <= TOL * S), f"{v} {p}"
 
 
+# ---------------------------------------------------------------- long rows, CTA-wide (XSMEM 11)
+def rtc_params(nt=0, k=0, stages=0, cps=0):
+    """MV_CPR [lanes, splits, ctas_per_sm, unroll(stages), xsmem=11, block, rows]"""
+    return [0, 0, cps, stages, 11, nt, k]
+
+
+RTC_SHAPES = [(1, 1), (1, 4097), (2, 1025), (7, 3), (8, 999), (9, 1025), (33, 2049), (100, 77), (257, 1026),
+              (1000, 1027), (3, 5000), (17, 8193), (5, 16385), (4096, 1028), (12345, 129)]
+RTC_PLANS = [rtc_params()] + [rtc_params(nt, k, st, cps) for nt, k, st, cps in
+                              ((512, 0, 0, 0), (256, 1, 2, 0), (256, 8, 3, 2), (512, 3, 8, 1), (256, 5, 0, 2))]
+
+
+@pytest.mark.parametrize("dt", ["f32", "i32"])
+def test_rowtile_cta_long_rows(dt):
+    """mv_rowtile_cta_kernel: k <= 8 whole rows per bulk copy reduced by the whole CTA, x in
+    registers (4..36 values per thread), the transposing butterfly; every C % 4 phase, tiles of 1..8 rows, ragged last tiles, the matrix's
+    last < 4 words copied by the threads, 256/512 threads, 2..8 stages."""
+    npdt = np.float32 if dt == "f32" else np.int32
+
+    def case(R, C, p):
+        A = synth.matrix(R, C, "mv", npdt, "uniform", synth.seed(23, "A") + R + C)
+        x = synth.vector(C, npdt, "uniform", synth.seed(23, "x") + C)
+        try:
+            plan = adaptic.plan("mv", R, C, dt, variant="MV_CPR", params=p)
+        except adaptic.AdapticError as e:
+            # x lives in registers: C <= 36 threads' worth of columns per thread
+            assert e.status == L.ERR_UNSUPPORTED and C > 36 * (p[5] or 512), str(e)
+            return
+        d = plan.describe()
+        assert d["xmode"] == 11 and d["stages"] >= 2 and 1 <= d["rows_per_group"] <= 8, d
+        y = adaptic.mv(torch.from_numpy(A).to(DEV), torch.from_numpy(x).to(DEV), variant="MV_CPR", params=p)
+        check(y.cpu().numpy(), oracle.mv(A, x), dt, f"mv {dt} {R}x{C} {p}")
+    _collect([(f"{R}x{C} {p}", lambda R=R, C=C, p=p: case(R, C, p))
+              for (R, C), p in itertools.product(RTC_SHAPES, RTC_PLANS)])
+
+
+def test_rowtile_cta_exact_deterministic_and_unaligned():
+    """P5 exact on integer-valued fp32; P7 scaling / negation / rerun identity; an A that is
+    not 16-byte aligned takes MV_CPR's direct kernel with the same results."""
+    for R, C in [(4099, 1025), (333, 4097), (65, 8193)]:
+        A = synth.matrix(R, C, "mv", np.float32, "smallint", 91 + C)
+        x = synth.vector(C, np.float32, "smallint", 92 + C)
+        y = adaptic.mv(torch.from_numpy(A).to(DEV), torch.from_numpy(x).to(DEV), variant="MV_CPR",
+                       params=rtc_params()).cpu().numpy()
+        assert np.array_equal(y.astype(np.float64), oracle.mv(A, x)[0]), f"P5 {R}x{C}"
+    R, C = 3001, 1025
+    A = torch.from_numpy(synth.matrix(R, C, "mv", np.float32, "uniform", 93)).to(DEV)
+    x = torch.from_numpy(synth.vector(C, np.float32, "uniform", 94)).to(DEV)
+    p = rtc_params()
+    y = adaptic.mv(A, x, variant="MV_CPR", params=p)
+    assert torch.equal(adaptic.mv(A, x * 8, variant="MV_CPR", params=p), y * 8)
+    assert torch.equal(adaptic.mv(A, -x, variant="MV_CPR", params=p), -y)
+    assert torch.equal(adaptic.mv(A, x, variant="MV_CPR", params=p), y)
+    An = A.cpu().numpy()
+    for off in (1, 2, 3):
+        big = torch.zeros(R * C + 8, dtype=torch.float32, device=DEV)
+        big[off:off + R * C] = A.reshape(-1)
+        yo = adaptic.mv(big[off:off + R * C].view(R, C), x, variant="MV_CPR", params=p).cpu().numpy()
+        check(yo, oracle.mv(An, x.cpu().numpy()), "f32", f"A off by {4 * off} bytes")
+
+
+def test_rowtile_cta_full_size_sampled():
+    """The offgrid bench shapes at 256 MiB in the bench's configuration: sampled rows."""
+    for R, C in [(65536, 1025), (16384, 4097)]:
+        A = torch.empty(R * C, dtype=torch.float32, device=DEV)
+        synth.device_matrix(A, R, C, "mv", "uniform", 95)
+        x = torch.empty(C, dtype=torch.float32, device=DEV)
+        synth.device_vector(x, "uniform", 96)
+        rows = np.unique(np.concatenate([np.arange(0, 32), np.arange(R - 32, R),
+                                         np.random.default_rng(5).integers(0, R, 128)]))
+        y = adaptic.mv(A.view(R, C), x, variant="MV_CPR", params=rtc_params()).cpu().numpy()
+        Arows = A.view(R, C)[torch.from_numpy(rows).to(DEV)].cpu().numpy()
+        yr, S = oracle.mv(Arows, x.cpu().numpy())
+        assert np.all(np.abs(y[rows].astype(np.float64) - yr) <= TOL * S), f"{R}x{C}"
+
+
 # ---------------------------------------------------------------- TMV on staged tiles of B
 def trt_params(nt=0, k=0, stages=0, cps=0):
     """TMV_REGTILE [lanes, splits, ctas_per_sm, unroll(stages), xsmem=4, block, rows]"""

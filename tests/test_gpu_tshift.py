@@ -67,11 +67,14 @@ def test_window_kernel_every_shape_alignment_and_split():
     """tmv_window_kernel (TMV_SPLITK with XSMEM 10): one aligned 128-bit load per row and
     thread, 7 accumulators with a compile-time shift pattern per 4 rows (every R mod 4 and B
     base alignment), the halo shuffle between windows and tiles, rows left over after the
-    groups of 4 / 8, splits with the ticket merge; fp32 within 1e-4 S_r, int32 exact."""
+    groups of 4 / 8, splits with the ticket merge; with one split (S = 1) the warp-tile form
+    (31 windows per warp, halo by shuffle, 128-bit y stores when y is aligned) at 2 and 3
+    resident CTAs; fp32 within 1e-4 S_r, int32 exact."""
     fails = []
     shapes = SHAPES + [(1021, 3), (1022, 13), (1023, 300), (250000, 9), (8193, 1)]
     for (R, C), off, p in itertools.product(shapes, (0, 1, 2, 3),
-                                            [[0, 0, 0, 0, 10], [0, 0, 0, 4, 10], [0, 7, 0, 8, 10]]):
+                                            [[0, 0, 0, 0, 10], [0, 0, 0, 4, 10], [0, 7, 0, 8, 10],
+                                             [0, 1, 0, 4, 10], [0, 1, 0, 8, 10], [0, 1, 3, 4, 10]]):
         for dt in ("f32", "i32"):
             np_dt = np.float32 if dt == "f32" else np.int32
             tdt = torch.float32 if dt == "f32" else torch.int32
@@ -82,6 +85,7 @@ def test_window_kernel_every_shape_alignment_and_split():
                 if R % 4 == 0 or R < 8:
                     continue
                 assert d["xmode"] == 10, d
+                assert (d["lanes"] == 31) == (d["splits"] == 1), d
                 y = adaptic.tmv(placed(B, off, tdt), placed(x, (off + 2) % 4, tdt), variant="TMV_SPLITK",
                                 params=p).cpu().numpy()
                 if dt == "i32":

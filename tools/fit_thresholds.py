@@ -30,7 +30,7 @@ def norm_params(r):
     measured shape) becomes a tile SIZE, -KB (derive() reads ROWS < 0 as kilobytes), so the
     entry means the same thing for every shape of its cell."""
     p = list(r["params"] or []) + [0] * 9
-    if p[4] == 4 and p[6] > 0:
+    if p[4] in (4, 11) and p[6] > 0:
         if r["op"] == "tmv":
             row_bytes = 4 * (r["R"] + 1)
         else:

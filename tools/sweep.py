@@ -93,6 +93,15 @@ def misx_grid(op, R, C):
     return out
 
 
+def rtc_grid(op, R, C):
+    """Long misaligned MV rows, round 2: k <= 8 whole rows per TMA-staged tile reduced by the
+    whole CTA with x in registers (MV_CPR, XSMEM 11); [ctas_per_sm, block, rows (-KB)]."""
+    if op != "mv" or C % 4 == 0 or C < 512 or C > 36 * 512:
+        return []
+    return [("MV_CPR", [0, 0, cps, 0, 11, nt, k]) for nt, k, cps in
+            ((256, 0, 0), (256, -48, 0), (512, 0, 0), (512, -48, 0), (512, -48, 2), (256, -48, 2))]
+
+
 def tshift_grid(op, R, C):
     """TMV rows off the 16-byte grid, round 2: the constant-shift kernel (XSMEM 7; tile width LR,
     c-lanes 256 / LR a multiple of 4, x loads in flight U) and the sliding-window kernel (XSMEM
@@ -106,7 +115,7 @@ def tshift_grid(op, R, C):
 def grids(op, R, C, dtype="f32"):
     """(variant, params) candidates; params = [lanes, splits, ctas_per_sm, unroll, xsmem, block, rows], 0 = auto."""
     out = [("AUTO", None)] + tile_grid(op, R, C, dtype) + rowtile_grid(op, R, C) + tshift_grid(op, R, C) + \
-        misx_grid(op, R, C)
+        misx_grid(op, R, C) + rtc_grid(op, R, C)
     if op in B1:
         nv = C // 4 if C % 4 == 0 else C
         if nv <= 64:
@@ -232,6 +241,7 @@ def main():
     ap.add_argument("--staged-only", action="store_true", help="time only the TMA-staged candidates (+ AUTO)")
     ap.add_argument("--tshift-only", action="store_true", help="time only the constant-shift TMV candidates (+ AUTO)")
     ap.add_argument("--misx-only", action="store_true", help="time only the round-2 misaligned-MV candidates (+ AUTO)")
+    ap.add_argument("--rtc-only", action="store_true", help="time only the long-row staged MV candidates (+ AUTO)")
     ap.add_argument("--graph-below", type=float, default=0,
                     help="time problems smaller than this many bytes from CUDA graphs (device time)")
     a = ap.parse_args()
@@ -281,6 +291,8 @@ def main():
                         [c for c in grids(op, R, C, a.dtype) if c[0] == "MV_TPR"]
                 elif a.misx_only:
                     cands = [("AUTO", None)] + misx_grid(op, R, C)
+                elif a.rtc_only:
+                    cands = [("AUTO", None)] + rtc_grid(op, R, C)
                 elif a.tshift_only:
                     cands = [("AUTO", None)] + tshift_grid(op, R, C)
                 elif a.flat_only:
