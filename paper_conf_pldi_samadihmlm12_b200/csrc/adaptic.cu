@@ -1016,7 +1016,7 @@ adaptic_status derive_rowtile(adaptic_plan_s* p, const int32_t* params, const De
 // [ADAPTIC_P_XSMEM] = 11.  [BLOCK] 256 | 512, [ROWS] k (-n: ~n KB per tile), [UNROLL] ring
 // stages, [CTAS_PER_SM]; C <= 36 * NT (x in registers; describe()'s lanes = x values per
 // thread).  16-byte-aligned A at run time, else the variant's direct kernel.
-adaptic_status derive_rowtile_cta(adaptic_plan_s* p, const int32_t* params, const DevInfo& dev) {
+adaptic_status derive_rowtile_cta_staged(adaptic_plan_s* p, const int32_t* params, const DevInfo& dev) {
     auto par = [&](int i) -> int { return params ? params[i] : 0; };
     const int64_t R = p->R, C = p->C;
     int NT = par(ADAPTIC_P_BLOCK);
@@ -1059,6 +1059,23 @@ adaptic_status derive_rowtile_cta(adaptic_plan_s* p, const int32_t* params, cons
     p->fb_ws_off = 0;
     if (derive(&fb, nullptr, dev) == ADAPTIC_OK) p->ws_bytes = fb.ws_bytes;
     return ADAPTIC_OK;
+}
+
+// Rows too long for whole-row tiles (x in registers: C <= 36 * NT; two stages in the ring): the
+// direct CTA-per-row kernel with 256 lanes x 2 vectors in flight and shifted copies of x
+// (XSMEM 5), the best fixed plan measured on the held-out long misaligned rows (8460 x 20903
+// 0.96, 8348 x 29273 0.98 of peak; the planner's default 1024-lane CTA ran 0.38-0.47 there).
+// So a fitted XSMEM 11 entry is valid for every shape of its cell.
+adaptic_status derive_rowtile_cta(adaptic_plan_s* p, const int32_t* params, const DevInfo& dev) {
+    const adaptic_status st = derive_rowtile_cta_staged(p, params, dev);
+    if (st != ADAPTIC_ERR_UNSUPPORTED) return st;
+    int32_t tp[ADAPTIC_NPARAMS] = {0};
+    tp[ADAPTIC_P_LANES] = 256;
+    tp[ADAPTIC_P_UNROLL] = 2;
+    tp[ADAPTIC_P_XSMEM] = 5;
+    if (derive(p, tp, dev) == ADAPTIC_OK) return ADAPTIC_OK;
+    tp[ADAPTIC_P_XSMEM] = 0;
+    return derive(p, tp, dev);
 }
 
 // TMV with few outputs on TMA-staged tiles of B (tmv_rowtile_kernel.cuh): TMV_REGTILE with
@@ -2128,9 +2145,11 @@ constexpr int kMaxBatchStreams = 8;
 // is 4 % FASTER without it (5689 -> 5901 GB/s, 2 streams; 3 streams without it: 5106), so it is
 // off by default.  ADAPTIC_EXCLUSIVE=1 enables it (read once).
 bool plan_exclusive(const adaptic_plan_s* p) {
-    static const bool on = [] { const char* e = std::getenv("ADAPTIC_EXCLUSIVE"); return e && e[0] == '1'; }();
-    return on && p->nvec == 1 && p->xmode == 4 &&
+    static const int mode = [] { const char* e = std::getenv("ADAPTIC_EXCLUSIVE"); return e ? std::atoi(e) : 0; }();
+    const bool rt4 = p->nvec == 1 && p->xmode == 4 &&
            (p->variant == ADAPTIC_V_MV_SUBWARP || p->variant == ADAPTIC_V_MV_WPR || p->variant == ADAPTIC_V_TMV_REGTILE);
+    const bool rt11 = p->nvec == 1 && p->xmode == 11;
+    return (mode == 1 && (rt4 || rt11)) || (mode == 2 && rt11) || (mode == 3 && rt4);
 }
 struct StreamPool {
     int dev = -1;

@@ -8,6 +8,7 @@
 #   sweep_r2_small    the 4-64 MiB diagonals, AUTO and every candidate in one run
 #   sweep_r2_tshift_* the constant-shift TMV kernel on the R+1 shapes and set A's R % 4 != 0 shapes
 #   sweep_r2_misx_*   the misaligned-MV x-funnel / residue-class kernels on the C+1 shapes and set A
+#   sweep_r2_rtc_*    the long-row staged MV kernel (MV_CPR, XSMEM 11) on the C+1 shapes and set A
 #   sweep_r2_dot1     Sdot N = 1, L = 2^10 .. 2^24 (graph-timed, like sweep_r2_small)
 #   sweep_r2_trainAs  small training shapes (tools/heldout_shapes.py As, 4-64 MiB, graph-timed)
 # Set B (tools/heldout_shapes.py B / Bs) is NEVER fitted: profiles/val_r2_* only.
@@ -21,6 +22,6 @@ python tools/merge_sweeps.py "$OUT" \
   $P/sweep_r1f_tmvrt.jsonl.gz +$P/sweep_r1g_tmvmis.jsonl.gz $P/sweep_r1k_shift_restricted.jsonl.gz \
   $P/sweep_r1o_rowtile_vec_restricted.jsonl.gz $P/sweep_r1l_tmvrt.jsonl.gz +$P/sweep_r1s_offgrid_full.jsonl.gz \
   +$P/sweep_r2_trainA.jsonl.gz +$P/sweep_r2_dotA.jsonl.gz +$P/sweep_r2_small.jsonl.gz +$P/sweep_r2_trainAs.jsonl.gz \
-  $P/sweep_r2_tshift_fit.jsonl.gz $P/sweep_r2_tshift_A.jsonl.gz $P/sweep_r2_misx_fit.jsonl.gz $P/sweep_r2_misx_A.jsonl.gz $(ls $P/sweep_r2_dot1.jsonl.gz 2>/dev/null | sed 's/^/+/')
+  $P/sweep_r2_tshift_fit.jsonl.gz $P/sweep_r2_tshift_A.jsonl.gz $P/sweep_r2_misx_fit.jsonl.gz $P/sweep_r2_misx_A.jsonl.gz $P/sweep_r2_rtc_fit.jsonl.gz $P/sweep_r2_rtc_A.jsonl.gz $(ls $P/sweep_r2_dot1.jsonl.gz 2>/dev/null | sed 's/^/+/')
 python tools/fit_thresholds.py "$OUT" --ops mv,tmv,dot --protect-bench --neighbor-weight 0.5 \
   --out paper_conf_pldi_samadihmlm12_b200/csrc/table_data.inc --json $P/selector_table_r2.json > /dev/null
