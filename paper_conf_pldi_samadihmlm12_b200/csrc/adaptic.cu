@@ -1141,6 +1141,76 @@ adaptic_status derive_tmv_rowtile(adaptic_plan_s* p, const int32_t* params, cons
     return ADAPTIC_OK;
 }
 
+// TMV with rows off the 16-byte grid on groups of four rows (tmv_group_kernel.cuh):
+// TMV_REGTILE / TMV_SPLITK with [ADAPTIC_P_XSMEM] = 12, 4 <= R <= 2560.  [UNROLL] groups in
+// flight (R <= 1024: 4 or 8), [BLOCK] threads (0: the fewest idle slots), [CTAS_PER_SM],
+// [ORDER] 1 = contiguous group range per CTA (default), 2 = CTAs interleaved,
+// [ROWS] slots per thread S (0: S = 1 for R <= 1024 (KG = NT div R groups per CTA step), else the
+// smallest S in {2, 3, 4} with ceil(R / S) <= 640).  16-byte-aligned B at run time, else the
+// variant's direct kernel on its own slice of the workspace.
+adaptic_status derive_tmv_group(adaptic_plan_s* p, const int32_t* params, const DevInfo& dev) {
+    auto par = [&](int i) -> int { return params ? params[i] : 0; };
+    const int64_t R = p->R, C = p->C;
+    if (R < 4 || R > 2560) return ADAPTIC_ERR_UNSUPPORTED;
+    int S = par(ADAPTIC_P_ROWS);
+    if (S <= 0) { S = 1; if (R > 1024) { S = 2; while (S < 4 && ceil_div(R, S) > 640) ++S; } }
+    if (S > 4) return ADAPTIC_ERR_INVALID_ARG;
+    int U = par(ADAPTIC_P_UNROLL);
+    if (U <= 0) U = S == 1 ? 4 : S == 2 ? 4 : 2;
+    void* fn = tmv_group_fn(p->dtype, S, U);
+    if (!fn) return ADAPTIC_ERR_INVALID_ARG;
+    const int maxnt = tmv_group_maxnt(S, U);
+    int NT = par(ADAPTIC_P_BLOCK);
+    int KG = 1;
+    if (S == 1) {
+        if (R > maxnt) return ADAPTIC_ERR_UNSUPPORTED;
+        if (NT <= 0) {                  // the block size (multiple of 32) with the fewest idle threads
+            double best = -1.0;
+            for (int nt = 256; nt <= maxnt; nt += 32) {
+                if (nt < R) continue;
+                const int kg = nt / int(R);
+                const double use = double(kg * R) / double(nt);
+                if (use > best + 0.02) { best = use; NT = nt; }
+            }
+            if (NT <= 0) NT = int(ceil_div(R, 32) * 32);
+        }
+        if (NT < R || NT > maxnt) return ADAPTIC_ERR_INVALID_ARG;
+        KG = NT / int(R);
+    } else {
+        const int need = int(ceil_div(ceil_div(R, S), 32) * 32);
+        if (NT <= 0) NT = need;
+        if (NT < ceil_div(R, S) || NT > maxnt) return ADAPTIC_ERR_INVALID_ARG;
+    }
+    int cps = par(ADAPTIC_P_CTAS_PER_SM);
+    const int occ = occupancy(fn, NT, 0, dev.present, std::max(1, 1024 / NT));
+    if (occ < 1) return ADAPTIC_ERR_UNSUPPORTED;
+    cps = cps <= 0 ? occ : std::min(cps, occ);
+    const int64_t NG = C / 4;
+    const int64_t G = std::max<int64_t>(1, std::min<int64_t>(int64_t(dev.sms) * cps, ceil_div(NG, int64_t(KG) * U)));
+    const int64_t ngroups = ceil_div(G, TG_GROUP_H);
+    const int ord = par(ADAPTIC_P_ORDER);
+    if (ord < 0 || ord > 2) return ADAPTIC_ERR_INVALID_ARG;
+    p->ilv = ord == 2 ? 1 : 0;
+    p->xmode = 12; p->mis = true; p->splits = 1;
+    p->lanes = int(R); p->block = NT; p->rb = S; p->unroll = U; p->ctas_per_sm = cps;
+    p->grid[1] = G; p->grid[0] = G;
+    p->chain[1] = fold_chain(ceil_div(ceil_div(NG, G), KG)) + 1;
+    p->depth[1] = 4 * KG + TG_GROUP_H + ngroups + (C % 4) + 1;
+    p->chain[0] = p->chain[1]; p->depth[0] = p->depth[1];
+    p->path_ok[1] = (p->dtype == DT_I32) || bound_ok(p->chain[1] + p->depth[1]);
+    p->path_ok[0] = p->path_ok[1];
+    if (!p->path_ok[1]) return ADAPTIC_ERR_UNSUPPORTED;
+    // CTA partials (G x R), group partials (ngroups x R), then 1 + ngroups counters
+    const size_t part = ((size_t(G + ngroups) * size_t(R) * 4 + 255) / 256) * 256;
+    p->cnt_off = part;
+    p->ws_bytes = part + ((size_t(1 + ngroups) * 4 + 255) / 256) * 256;
+    adaptic_plan_s fb = *p;                     // B not 16-byte aligned: the direct kernel
+    fb.variant = ADAPTIC_V_TMV_SPLITK;
+    p->fb_ws_off = p->ws_bytes;
+    if (derive(&fb, nullptr, dev) == ADAPTIC_OK) p->ws_bytes += fb.ws_bytes;
+    return ADAPTIC_OK;
+}
+
 // A multi-vector plan with a 128-bit shape run on pointers that are not 16-byte aligned
 // (the x-tile / TMA / register-x kernels need aligned rows): the generic CTA kernels'
 // 4-byte path of the same K -- MV_CPR (no workspace) when its error bound holds, else
@@ -1374,6 +1444,8 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
     // scalar path is planned for these shapes
     p->flat = false;
     if (v == ADAPTIC_V_TMV_REGTILE && par(ADAPTIC_P_XSMEM) == 4) return derive_tmv_rowtile(p, params, dev);
+    if (!p->vec_shape && (v == ADAPTIC_V_TMV_REGTILE || v == ADAPTIC_V_TMV_SPLITK) && par(ADAPTIC_P_XSMEM) == 12)
+        return derive_tmv_group(p, params, dev);
     if (!p->vec_shape && v == ADAPTIC_V_TMV_REGTILE && R <= TMV_FLAT_MAX_R) {
         // few outputs off the 16-byte grid: stream B as one flat array (tmv_flat_kernel.cuh)
         const int FNT = R <= TMV_FLAT_NT_SMALL_R ? 256 : 1024;
@@ -1888,6 +1960,13 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
                 args = args9;
                 break;
             }
+            if (p->xmode == 12) {                         // groups of four rows (16-byte-aligned B)
+                fn = tmv_group_fn(dt, p->rb, p->unroll);
+                args8[0] = &A; args8[1] = &X; args8[2] = &y; args8[3] = &R; args8[4] = &C;
+                args8[5] = &ilv; args8[6] = &part; args8[7] = &cnt;
+                args = args8;
+                break;
+            }
             if (p->flat && mis) {
                 fn = tmv_flat_fn(dt, p->unroll, p->block);
                 args7[0] = &A; args7[1] = &X; args7[2] = &y; args7[3] = &R; args7[4] = &C;
@@ -2104,6 +2183,22 @@ adaptic_status adaptic_run(adaptic_plan_t p, const void* A, const void* x, void*
                 ((reinterpret_cast<uintptr_t>(A) - reinterpret_cast<uintptr_t>(x)) & 15u) == 0);
     if (mis && p->variant == ADAPTIC_V_MV_TPR)   // bulk copies of row tiles: 16-byte aligned bases
         mis = aligned(A, 16) && (p->op != ADAPTIC_OP_DOT || aligned(x, 16));
+    if (p->nvec == 1 && p->xmode == 12 && p->op == ADAPTIC_OP_TMV) {
+        // groups of four rows are 16-byte aligned only on a 16-byte-aligned B; other
+        // pointers take the TMV_SPLITK direct kernel of the same shape
+        if (aligned(A, 16)) return launch(p, A, x, y, stream, false, true);
+        adaptic_plan_s fb = *p;
+        fb.variant = ADAPTIC_V_TMV_SPLITK;
+        if (derive(&fb, nullptr, device_info()) != ADAPTIC_OK) return ADAPTIC_ERR_UNSUPPORTED;
+        if (fb.ws_bytes > 0) {
+            if (!p->ws || p->fb_ws_off + fb.ws_bytes > p->ws_cap) return ADAPTIC_ERR_NO_WORKSPACE;
+            fb.ws = static_cast<char*>(p->ws) + p->fb_ws_off;
+            fb.ws_cap = p->ws_cap - p->fb_ws_off;
+        } else {
+            fb.ws = nullptr; fb.ws_cap = 0;
+        }
+        return adaptic_run(&fb, A, x, y, stream_);
+    }
     if (p->nvec == 1 && ((p->xmode == 4 && (p->variant == ADAPTIC_V_MV_SUBWARP || p->variant == ADAPTIC_V_MV_WPR ||
                                             p->variant == ADAPTIC_V_TMV_REGTILE)) || p->xmode == 11)) {
         // row tiles are bulk-copied from 16-byte-aligned bases; other pointers take the

@@ -120,6 +120,13 @@ void* tmv_shift_fn(int dt, int LR, int U);
 void* tmv_window_fn(int dt, int G8);
 void* rowtile_cta_fn(int dtype, int NT, int MX, int k);   // MX in {4, 8, 16, 36}: C <= NT * MX; k <= 8 rows
 void* tmv_window_warp_fn(int dt, int G8, int minb);
+//   tgroup: (B, X, y, R, C, int ilv, T* part, unsigned* cnt): rows off the 16-byte grid on groups of four
+//           rows (4R words = R aligned vectors), S slots per thread with fixed outputs, U groups
+//           in flight, two-level ticket merge; 16-byte-aligned B, any x (tmv_group_kernel.cuh,
+//           XSMEM 12); (S, U) in {(1,4), (1,8), (2,4), (3,2), (4,2)}, blockDim <= tmv_group_maxnt
+void* tmv_group_fn(int dt, int S, int U);
+int tmv_group_maxnt(int S, int U);
+constexpr int TG_GROUP_H = 16;                      // == TG_GROUP (static_assert in k_tgroup.cu)
 int64_t tring_stage_words_h(int64_t R, int TW, int CR, int K);
 constexpr int64_t MRING_SMEM_BUDGET = 220 * 1024;
 constexpr int TMMV_TMA_STAGE_V4 = 2048;              // 32 KB per stage
