@@ -213,6 +213,23 @@ typedef enum {
  *                      MV_CPR / MV_SPLIT: 5 = x copied first (same stream, same
  *                      call) into four shifted 16-byte-aligned copies in the
  *                      workspace, so every row reads x with 128-bit loads.
+ *                      Further forced modes (round 2; the fitted table may select
+ *                      them, DESIGN.md section 4 describes each):
+ *                      7 = TMV_SPLITK / TMV_COL rows off the 16-byte grid at a constant
+ *                      word shift per c-lane; 9 = MV_CPR / MV_SPLIT misaligned rows with
+ *                      x read as two aligned 128-bit loads and a funnel (16-byte-aligned
+ *                      x, else the direct kernel); 10 = TMV sliding-window kernel (rows
+ *                      off the grid, one aligned load per row and thread); 11 = MV_CPR
+ *                      long rows (cols <= 36 x threads) on staged row tiles reduced by
+ *                      the whole CTA; 12 = TMV_REGTILE / TMV_SPLITK rows off the grid on
+ *                      groups of four rows (4 <= rows <= 2560, [ADAPTIC_P_ROWS] slots per
+ *                      thread, [ADAPTIC_P_ORDER] 2 = interleaved CTA ranges); 13 = MV_CPR /
+ *                      MV_SPLIT rows of any length and alignment on staged COLUMN CHUNKS
+ *                      ([ADAPTIC_P_LANES] x values per thread in {8, 16, 36},
+ *                      [ADAPTIC_P_BLOCK] 256 | 512 consumer threads plus one producer
+ *                      warp, [ADAPTIC_P_ROWS] row segments per tile <= 4).  Modes 11-13
+ *                      need a 16-byte-aligned matrix base; other pointers run the
+ *                      variant's direct kernel (same results, slower).
  *   [ADAPTIC_P_BLOCK]  TMV_*: threads per CTA, 256 or 1024 (unroll <= 4 at 1024).
  *   [ADAPTIC_P_ROWS]   MV_CPR / MV_SPLIT: rows per CTA step sharing each x load,
  *                      (rows, unroll) in {(1,2),(1,4),(1,8),(2,2),(2,4),(4,2)}.

@@ -1078,6 +1078,72 @@ adaptic_status derive_rowtile_cta(adaptic_plan_s* p, const int32_t* params, cons
     return derive(p, tp, dev);
 }
 
+// MV rows too long for x in registers on staged COLUMN CHUNKS (rowtile_kernel.cuh
+// mv_chunk_cta_kernel): MV_CPR / MV_SPLIT with [ADAPTIC_P_XSMEM] = 13, any C and any row
+// alignment.  [BLOCK] 256 | 512 (default 512), [LANES] x values per thread MX in {8, 16, 36}
+// (default 16; chunk width W = ceil(C / nch) <= NT MX, nch chunks), [ROWS] rows per tile k
+// (0: ~64 KB of segments per tile, -n: ~n KB; <= 4), [UNROLL] ring stages, [CTAS_PER_SM]
+// (default 1).  describe(): splits = nch, rows_per_group = k, lanes = MX.  16-byte-aligned A
+// at run time, else the variant's direct kernel.
+adaptic_status derive_chunk_cta(adaptic_plan_s* p, const int32_t* params, const DevInfo& dev) {
+    auto par = [&](int i) -> int { return params ? params[i] : 0; };
+    const int64_t R = p->R, C = p->C;
+    int NT = par(ADAPTIC_P_BLOCK);
+    if (NT <= 0) NT = 512;
+    if (NT != 256 && NT != 512) return ADAPTIC_ERR_INVALID_ARG;
+    int MX = par(ADAPTIC_P_LANES);
+    if (MX <= 0) MX = 16;
+    if (MX != 8 && MX != 16 && MX != 36) return ADAPTIC_ERR_INVALID_ARG;
+    const int64_t nch = ceil_div(C, int64_t(NT) * MX);
+    const int64_t W = ceil_div(C, nch);
+    if (W > INT_MAX / 2) return ADAPTIC_ERR_UNSUPPORTED;
+    int cps = par(ADAPTIC_P_CTAS_PER_SM);
+    if (cps <= 0) cps = 1;
+    const size_t budget = size_t(220) * 1024 / size_t(cps);
+    const size_t slot_bytes = size_t((W + 6 + 3) / 4 * 4) * 4;
+    int64_t k = par(ADAPTIC_P_ROWS);
+    if (k < 0) k = (int64_t(-k) * 1024) / int64_t(slot_bytes);
+    else if (k == 0) k = (int64_t(64) * 1024) / int64_t(slot_bytes);   // 32 KB tiles: 0.87 vs 0.91 (r2g)
+    k = std::max<int64_t>(1, std::min<int64_t>({k, int64_t(4), std::max<int64_t>(1, R)}));
+    while (k > 1 && 2 * size_t(k) * slot_bytes > budget) --k;
+    const size_t stage_bytes = size_t(k) * slot_bytes;
+    if (2 * stage_bytes > budget) return ADAPTIC_ERR_UNSUPPORTED;
+    int stages = int(std::min<size_t>(RT_MAX_STAGES_H, budget / stage_bytes));
+    if (par(ADAPTIC_P_UNROLL) > 0) stages = std::min(stages, par(ADAPTIC_P_UNROLL));
+    void* fn = chunk_cta_fn(p->dtype, NT, MX, int(k));
+    if (!fn) return ADAPTIC_ERR_UNSUPPORTED;
+    while (stages >= 2 && !smem_fits(fn, size_t(stages) * stage_bytes, dev.present)) --stages;
+    if (stages < 2) return ADAPTIC_ERR_UNSUPPORTED;
+    p->smem = size_t(stages) * stage_bytes;
+    const int occ = occupancy(fn, NT + 32, p->smem, dev.present, cps);
+    if (occ < 1) return ADAPTIC_ERR_UNSUPPORTED;
+    p->ctas_per_sm = std::min(cps, occ);
+    const int64_t units = nch * ceil_div(R, k);
+    p->lanes = MX; p->block = NT; p->rb = int(k); p->stages = stages; p->unroll = stages;
+    p->splits = int(nch);
+    p->xmode = 13;
+    p->mis = !p->vec_shape;
+    p->grid[1] = std::max<int64_t>(1, std::min<int64_t>(units, int64_t(dev.sms) * p->ctas_per_sm));
+    p->grid[0] = p->grid[1];
+    int L = 1;
+    while (L < 32 && 2 * L * R <= NT) L *= 2;
+    p->chain[1] = MX;
+    p->depth[1] = 5 + NT / 64 + 1 + (nch > 1 ? ceil_div(nch, L) + ilog2c(L) : 0);
+    p->chain[0] = p->chain[1]; p->depth[0] = p->depth[1];
+    p->path_ok[1] = (p->dtype == DT_I32) || bound_ok(p->chain[1] + p->depth[1]);
+    p->path_ok[0] = p->path_ok[1];
+    if (!p->path_ok[1]) return ADAPTIC_ERR_UNSUPPORTED;
+    p->ws_bytes = 0;
+    if (nch > 1) {
+        p->cnt_off = ((size_t(nch) * size_t(R) * 4 + 255) / 256) * 256;
+        p->ws_bytes = p->cnt_off + 256;
+    }
+    adaptic_plan_s fb = *p;                             // the direct kernel for unaligned A
+    p->fb_ws_off = p->ws_bytes;
+    if (derive(&fb, nullptr, dev) == ADAPTIC_OK) p->ws_bytes += fb.ws_bytes;
+    return ADAPTIC_OK;
+}
+
 // TMV with few outputs on TMA-staged tiles of B (tmv_rowtile_kernel.cuh): TMV_REGTILE with
 // [ADAPTIC_P_XSMEM] = 4.  [BLOCK] threads 256 | 512 | 1024 (>= R), [ROWS] rows of B per
 // tile k (a multiple of 4), [UNROLL] ring stages, [CTAS_PER_SM].  16-byte-aligned B and x
@@ -1278,6 +1344,8 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
         return derive_rowtile(p, params, dev);
     if (v == ADAPTIC_V_MV_CPR && op == ADAPTIC_OP_MV && par(ADAPTIC_P_XSMEM) == 11)
         return derive_rowtile_cta(p, params, dev);
+    if ((v == ADAPTIC_V_MV_CPR || v == ADAPTIC_V_MV_SPLIT) && op == ADAPTIC_OP_MV && par(ADAPTIC_P_XSMEM) == 13)
+        return derive_chunk_cta(p, params, dev);
 
     // rows not 16-byte aligned (C % 4 != 0): the misaligned-row kernels keep the matrix
     // stream 128-bit; the plain scalar kernels (index 0) remain for DOT operands whose
@@ -1790,6 +1858,7 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
     int tr_sw = p->xmode == 6 && p->op == ADAPTIC_OP_TMV ? int(tring_stage_words_h(p->R, p->lanes, p->splits, p->nvec)) : 0;
     void* args12[13];
     int tr_dbg = p->ilv;                           // experiments only (param ORDER 8 + d)
+    int chunk_w = 0;                               // mv_chunk_cta_kernel: columns per chunk
 
     void* args7[7];
     if (mis && p->xmode == XM_SHIFT_MODE && p->op == ADAPTIC_OP_MV && p->nvec == 1 &&
@@ -1908,6 +1977,16 @@ adaptic_status launch(const adaptic_plan_s* p, const void* A, const void* X, voi
             break;
         case ADAPTIC_V_MV_CPR:
         case ADAPTIC_V_MV_SPLIT:
+            if (p->xmode == 13) {                         // column chunks on staged tiles, CTA-wide
+                fn = chunk_cta_fn(dt, p->block, p->lanes, p->rb);
+                smem = p->smem;
+                block = p->block + 32;                    // + the producer warp
+                chunk_w = int(ceil_div(C, int64_t(p->splits)));
+                args10[0] = &A; args10[1] = &X; args10[2] = &y; args10[3] = &R; args10[4] = &C;
+                args10[5] = &tile_mb; args10[6] = &stages; args10[7] = &chunk_w; args10[8] = &part; args10[9] = &cnt;
+                args = args10;
+                break;
+            }
             if (p->xmode == 11) {                         // long rows on staged tiles, CTA-wide
                 fn = rowtile_cta_fn(dt, p->block, p->lanes, p->rb);
                 smem = p->smem;
@@ -2200,7 +2279,7 @@ adaptic_status adaptic_run(adaptic_plan_t p, const void* A, const void* x, void*
         return adaptic_run(&fb, A, x, y, stream_);
     }
     if (p->nvec == 1 && ((p->xmode == 4 && (p->variant == ADAPTIC_V_MV_SUBWARP || p->variant == ADAPTIC_V_MV_WPR ||
-                                            p->variant == ADAPTIC_V_TMV_REGTILE)) || p->xmode == 11)) {
+                                            p->variant == ADAPTIC_V_TMV_REGTILE)) || p->xmode == 11 || p->xmode == 13)) {
         // row tiles are bulk-copied from 16-byte-aligned bases; other pointers take the
         // direct kernel of the same variant and shape
         if (aligned(A, 16) && (p->op == ADAPTIC_OP_MV || aligned(x, 16)))

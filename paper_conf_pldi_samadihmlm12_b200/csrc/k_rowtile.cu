@@ -70,6 +70,34 @@ void* rowtile_cta_fn(int dtype, int NT, int MX, int k) {
 }
 static_assert(RTC_KMAX == RTC_KMAX_H, "long-row tile height: kernel vs planner");
 
+// column-chunk form (mv_chunk_cta_kernel, XSMEM 13): NT in {256, 512}, MX in {8, 16, 36},
+// KR in {1, 2, 4} (k <= KR row segments per tile)
+template <class T, int NT, int MX>
+static void* ck_k(int KR) {
+    switch (KR) {
+        case 1: return reinterpret_cast<void*>(&mv_chunk_cta_kernel<T, NT, MX, 1>);
+        case 2: return reinterpret_cast<void*>(&mv_chunk_cta_kernel<T, NT, MX, 2>);
+        case 4: return reinterpret_cast<void*>(&mv_chunk_cta_kernel<T, NT, MX, 4>);
+        default: return nullptr;
+    }
+}
+template <class T, int NT>
+static void* ck_m(int MX, int KR) {
+    switch (MX) {
+        case 8: return ck_k<T, NT, 8>(KR);
+        case 16: return ck_k<T, NT, 16>(KR);
+        case 36: return ck_k<T, NT, 36>(KR);
+        default: return nullptr;
+    }
+}
+void* chunk_cta_fn(int dtype, int NT, int MX, int k) {
+    const int KR = k <= 1 ? 1 : k <= 2 ? 2 : k <= 4 ? 4 : 0;
+    if (KR == 0) return nullptr;
+    if (NT == 256) return dtype == DT_F32 ? ck_m<float, 256>(MX, KR) : ck_m<uint32_t, 256>(MX, KR);
+    if (NT == 512) return dtype == DT_F32 ? ck_m<float, 512>(MX, KR) : ck_m<uint32_t, 512>(MX, KR);
+    return nullptr;
+}
+
 }  // namespace adaptic
 
 namespace adaptic {

@@ -119,6 +119,10 @@ void* tmv_shift_fn(int dt, int LR, int U);
 //         NT - 1 owned windows, G8 in {1, 2} groups of 4 rows in flight, NT = 256 (XSMEM 10)
 void* tmv_window_fn(int dt, int G8);
 void* rowtile_cta_fn(int dtype, int NT, int MX, int k);   // MX in {4, 8, 16, 36}: C <= NT * MX; k <= 8 rows
+//   chunk: (A, X, y, R, C, int k, int stages, int W, T* part, unsigned* cnt): the long-row staged
+//          CTA reduction on column chunks of W <= NT * MX (MX in {8, 16, 36}), k <= 4 row
+//          segments per tile, chunk partials merged by the last CTA (XSMEM 13)
+void* chunk_cta_fn(int dtype, int NT, int MX, int k);
 void* tmv_window_warp_fn(int dt, int G8, int minb);
 //   tgroup: (B, X, y, R, C, int ilv, T* part, unsigned* cnt): rows off the 16-byte grid on groups of four
 //           rows (4R words = R aligned vectors), S slots per thread with fixed outputs, U groups

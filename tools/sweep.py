@@ -154,6 +154,7 @@ def grids(op, R, C, dtype="f32"):
                 for order in (1, 2):
                     out.append(("MV_SPLIT", [nt, 0, 0, u, 0, 0, rb, order, pp]))
         out += shift_grid(op, R, C)
+        out += chunk_grid(op, R, C)
         if C <= 256:
             for nt in (128, 256):
                 for st in (2, 4, 8):
@@ -177,6 +178,15 @@ def grids(op, R, C, dtype="f32"):
         for u in (2, 4, 8):
             out.append(("TMV_REGTILE", [0, 0, 0, u]))
     return out
+
+
+def chunk_grid(op, R, C):
+    """MV rows on staged column chunks (XSMEM 13, round 2; any C, any alignment): x values per
+    thread MX and threads NT (chunk width <= NT MX), row segments per tile (0: ~64 KB)."""
+    if op != "mv" or C < 8192:
+        return []
+    return [("MV_SPLIT", [mx, 0, 0, 0, 13, nt, k]) for mx, nt in ((16, 512), (36, 512), (36, 256))
+            for k in (0, 1, 2, 4)]
 
 
 def time_plan(plan, ptrs, stream, reps, batch=5, graph=False):
@@ -242,6 +252,7 @@ def main():
     ap.add_argument("--tshift-only", action="store_true", help="time only the constant-shift TMV candidates (+ AUTO)")
     ap.add_argument("--misx-only", action="store_true", help="time only the round-2 misaligned-MV candidates (+ AUTO)")
     ap.add_argument("--rtc-only", action="store_true", help="time only the long-row staged MV candidates (+ AUTO)")
+    ap.add_argument("--chunk-only", action="store_true", help="time only the column-chunk staged MV candidates (+ AUTO)")
     ap.add_argument("--graph-below", type=float, default=0,
                     help="time problems smaller than this many bytes from CUDA graphs (device time)")
     a = ap.parse_args()
@@ -293,6 +304,8 @@ def main():
                     cands = [("AUTO", None)] + misx_grid(op, R, C)
                 elif a.rtc_only:
                     cands = [("AUTO", None)] + rtc_grid(op, R, C)
+                elif a.chunk_only:
+                    cands = [("AUTO", None)] + chunk_grid(op, R, C)
                 elif a.tshift_only:
                     cands = [("AUTO", None)] + tshift_grid(op, R, C)
                 elif a.flat_only:
