@@ -105,3 +105,48 @@ def test_staged_tmv_tiles():
         d("tmv", 9, 1000, variant="TMV_REGTILE", params=[0, 0, 0, 0, 4, 256, 6])
     for R, C in ((9, 8388608), (129, 524288), (14, 5162220)):
         assert d("tmv", R, C)["xmode"] == 4, (R, C)
+
+
+def _p(p):
+    return (list(p) + [0] * 9)[:9]
+
+
+def test_chunk_plan_geometry():
+    """XSMEM 13 (staged column chunks): nch = ceil(C / (NT MX)) chunks, k <= 4 row segments per
+    ~64 KB tile, >= 2 ring stages, partials nch x R (+ counter) only when nch > 1; the selector
+    takes it for the offgrid bench's long C + 1 rows (profiles/sweep_r2_offmv_full)."""
+    for R, C, MX, NT in ((512, 131073, 16, 512), (16, 4194305, 36, 512), (3, 5000, 8, 256), (1000, 8193, 36, 256)):
+        p = d("mv", R, C, variant="MV_SPLIT", params=_p([MX, 0, 0, 0, 13, NT]))
+        nch = -(-C // (NT * MX))
+        assert p["xmode"] == 13 and p["splits"] == nch and p["lanes"] == MX and p["block"] == NT, p
+        assert 1 <= p["rows_per_group"] <= min(4, R) and p["stages"] >= 2 and p["path_ok"][1]
+        W = -(-C // nch)
+        assert p["smem"] == p["stages"] * p["rows_per_group"] * ((W + 9) // 4 * 4) * 4
+        if nch > 1:
+            assert p["workspace_bytes"] >= nch * R * 4 + 4
+    for MX in (4, 12, 64):
+        with pytest.raises(adaptic.AdapticError):
+            d("mv", 100, 100000, variant="MV_SPLIT", params=_p([MX, 0, 0, 0, 13]))
+    for R in (32, 128, 512, 1024):
+        a = d("mv", R, (1 << 26) // R + 1)
+        assert a["xmode"] == 13, (R, a)
+
+
+def test_group_plan_geometry():
+    """XSMEM 12 (TMV on groups of four rows): KG = NT div R sub-groups with the fewest idle
+    threads for R <= 1024, S = 2..4 slots per thread above, R in [4, 2560]; two-level merge
+    workspace (G + ceil(G / 16)) x R partials."""
+    for R in (5, 17, 129, 513, 1023):
+        p = d("tmv", R, 100003, variant="TMV_SPLITK", params=_p([0, 0, 0, 0, 12]))
+        assert p["xmode"] == 12 and p["rows_per_group"] == 1 and p["block"] >= R and p["block"] % 32 == 0, p
+        assert (p["block"] // R) * R / p["block"] >= 0.75
+    for R, S in ((1025, 2), (1537, 3), (2049, 4), (2559, 4)):
+        p = d("tmv", R, 9999, variant="TMV_REGTILE", params=_p([0, 0, 0, 0, 12]))
+        assert p["rows_per_group"] == S and p["block"] * S >= R and p["block"] <= 640, (R, p)
+        G = p["grid"][1]
+        assert p["workspace_bytes"] >= (G + -(-G // 16)) * R * 4
+    for R in (3, 2561):
+        with pytest.raises(adaptic.AdapticError):
+            d("tmv", R, 1000, variant="TMV_SPLITK", params=_p([0, 0, 0, 0, 12]))
+    # interleaved order and forced slots
+    assert d("tmv", 129, 5000, variant="TMV_SPLITK", params=_p([0, 0, 0, 0, 12, 0, 2, 2]))["rows_per_group"] == 2
