@@ -613,6 +613,11 @@ adaptic_status derive_multi(adaptic_plan_s* p, const int32_t* params, const DevI
         if (CW <= 0) CW = (int64_t(K) * C * 4 <= MMV_TILE_ONE_CHUNK) ? C : MMV_TILE_XBYTES / (4 * K);
         if (CW <= 0 || CW % 4 != 0 || 2 * int64_t(K) * CW * 4 > kXsMaxBytes) return ADAPTIC_ERR_INVALID_ARG;
         CW = std::min<int64_t>(CW, C);
+        // a fitted width above the default that would still cut C into several chunks: the
+        // default.  Every such pair in the training sweeps measured the wider chunks slower
+        // (1 CTA per SM with the double-buffered 2 x 64 KB of x; 0.75-0.97, median 0.87 of the
+        // 8192 chunks over 57 shapes); a wider width only pays as ONE chunk (C <= width)
+        if (K == 1 && CW < C && CW > MMV_TILE_XBYTES / 4) CW = MMV_TILE_XBYTES / 4;
         // balanced chunks: a table width fitted on C = 2^k (an exact multiple) would leave the
         // last chunk of another C mostly empty (held-out 6144 x 26624: 1.6 chunks of 16384, 0.86
         // of the best plan); the same number of chunks, evenly filled
