@@ -34,16 +34,19 @@ def report(args):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--out", default=os.path.join(P, "r2_selector_report.md"))
-    ap.add_argument("--valB", default=os.path.join(P, "val_r2_valB_auto.jsonl.gz"))
-    ap.add_argument("--valBs", default=os.path.join(P, "val_r2_valBs_auto.jsonl.gz"))
+    ap.add_argument("--valB", default=os.path.join(P, "val_r2_valB3_auto.jsonl.gz"))
+    ap.add_argument("--valBs", default=os.path.join(P, "val_r2_valBs3_auto.jsonl.gz"))
     a = ap.parse_args()
     best_B = [os.path.join(P, f) for f in ("val_r2_heldoutB_nodot.jsonl.gz", "val_r2_dotB.jsonl.gz",
-                                             "val_r2_tshift_B.jsonl.gz")]
+                                             "val_r2_tshift_B.jsonl.gz", "val_r2_misx_B.jsonl.gz",
+                                             "val_r2_rtc_B.jsonl.gz", "val_r2_chunk_B.jsonl.gz")]
     parts = ["# Selector report (round 2): held-out generalisation\n",
              "Shapes: `tools/heldout_shapes.py` (A, B: 256 MiB - 2 GiB; As, Bs: 4-64 MiB).  Training input: "
              "`tools/refit_r2.sh` (round 1's exact fit input + set A + As + the DOT re-sweep with b aligned + "
-             "small diagonals + Sdot lengths + constant-shift TMV candidates).  Sets B and Bs are never "
-             "fitted.  Gates (BJ:north_star): AUTO >= 0.95 x the best fixed variant and >= 0.70 of the "
+             "small diagonals + Sdot lengths + constant-shift TMV, misaligned-MV, long-row and column-chunk "
+             "candidates, the offgrid MV shapes re-swept in full).  Sets B and Bs are never fitted; sections 2 "
+             "and 3 time the FINAL table's AUTO picks (`val_r2_valB3_auto`, `val_r2_valBs3_auto`, measured at "
+             "commit 8a83827) against every fixed candidate swept on those shapes.  Gates (BJ:north_star): AUTO >= 0.95 x the best fixed variant and >= 0.70 of the "
              "measured copy peak (6554.9 GB/s) for inputs >= 256 MiB.\n"]
     parts.append("## 1. Round-1 table, held-out set A (before A entered the training data)\n")
     parts.append("DOT rows of this run placed b right after a, so for R*C % 4 != 0 the two operands differed "
