@@ -45,19 +45,23 @@ def main():
              "`tools/refit_r2.sh` (round 1's exact fit input + set A + As + the DOT re-sweep with b aligned + "
              "small diagonals + Sdot lengths + constant-shift TMV, misaligned-MV, long-row and column-chunk "
              "candidates, the offgrid MV shapes re-swept in full).  Sets B and Bs are never fitted; sections 2 "
-             "and 3 time the FINAL table's AUTO picks (`val_r2_valB3_auto`, `val_r2_valBs3_auto`, measured at "
-             "commit 8a83827) against every fixed candidate swept on those shapes.  Gates (BJ:north_star): AUTO >= 0.95 x the best fixed variant and >= 0.70 of the "
+             "and 3 time the FINAL table's AUTO pick and every fixed candidate of each shape in one run.  Gates (BJ:north_star): AUTO >= 0.95 x the best fixed variant and >= 0.70 of the "
              "measured copy peak (6554.9 GB/s) for inputs >= 256 MiB.\n"]
     parts.append("## 1. Round-1 table, held-out set A (before A entered the training data)\n")
     parts.append("DOT rows of this run placed b right after a, so for R*C % 4 != 0 the two operands differed "
                  "in alignment mod 16 and the misaligned-row DOT kernels (which need equal alignment) fell back "
                  "to scalar loads: those DOT rows understate both AUTO and the best fixed.\n\n```\n")
     parts.append(report([os.path.join(P, "sweep_r2_trainA.jsonl.gz")]).splitlines()[-2] + "\n```\n")
-    parts.append("## 2. Round-2 table, held-out set B (never fitted), >= 256 MiB\n\n")
-    parts.append(report([a.valB, "--best-from"] + best_B))
-    parts.append("\n## 3. Round-2 table, held-out small set Bs (4-64 MiB, device-timed from CUDA graphs)\n\n")
-    parts.append(report([a.valBs, "--best-from", os.path.join(P, "val_r2_heldoutBs.jsonl.gz"), "--min-bytes", "0",
-                         "--no-peak-gate"]))
+    parts.append("## 2. Final round-2 table, held-out set B (never fitted), >= 256 MiB, every candidate and AUTO "
+                 "in ONE run (`val_r2_B_final`, final code)\n\n")
+    parts.append(report([os.path.join(P, "val_r2_B_final.jsonl.gz")]))
+    parts.append("\n## 3. Final round-2 table, held-out small set Bs (4-64 MiB, device-timed from CUDA graphs, one "
+                 "run: `val_r2_Bs_final`)\n\n")
+    parts.append(report([os.path.join(P, "val_r2_Bs_final.jsonl.gz"), "--min-bytes", "0", "--no-peak-gate"]))
+    parts.append("\n## 3b. The same table's AUTO picks timed in another run against the earlier sweeps' best "
+                 "fixed (`val_r2_valB3_auto` vs `val_r2_heldoutB_nodot` + DOT / tshift / misx / rtc / chunk "
+                 "sweeps): cross-run timing, so a ~1 % box-to-box shift moves borderline shapes\n\n```\n")
+    parts.append(report([a.valB, "--best-from"] + best_B).splitlines()[-2] + "\n```\n")
     r = subprocess.run([sys.executable, os.path.join(HERE, "select_sim.py"), "--table",
                         os.path.join(P, "selector_table_r2.json")] + best_B, capture_output=True, text=True)
     parts.append("\n## 4. Offline replica on set B (tools/select_sim.py: the fitted entry's measured GB/s on each "
