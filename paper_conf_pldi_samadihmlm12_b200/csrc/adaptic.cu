@@ -971,6 +971,12 @@ adaptic_status derive_rowtile(adaptic_plan_s* p, const int32_t* params, const De
     if (G <= 0) G = clampi(pow2_ceil(ceil_div(C, 8)), 1, 16);
     if (G < 1 || G > 32 || (G & (G - 1)) || (p->variant == ADAPTIC_V_MV_SUBWARP && G > 16))
         return ADAPTIC_ERR_INVALID_ARG;
+    // a fitted cell spans a factor 2 in C: an entry's lane group fitted on the cell's shorter
+    // rows may hold too few x values per lane for this C -- the smallest group that does
+    // (held-out DOT 393216 x 416 and 507478 x 488 had fallen back to the direct kernels: 0.67-0.89
+    // of the staged plan)
+    if (p->source == 1 && C > int64_t(RT_MAX_C_PER_LANE) * G && p->variant == ADAPTIC_V_MV_SUBWARP)
+        G = int(std::min<int64_t>(16, pow2_ceil(ceil_div(C, int64_t(RT_MAX_C_PER_LANE)))));
     if (C > int64_t(RT_MAX_C_PER_LANE) * G) return ADAPTIC_ERR_UNSUPPORTED;
     int NT = par(ADAPTIC_P_BLOCK);
     if (NT <= 0) NT = 256;
@@ -983,6 +989,14 @@ adaptic_status derive_rowtile(adaptic_plan_s* p, const int32_t* params, const De
     } else if (k == 0) {   // ~24 KB of matrix per tile, whole warps of rows
         k = std::max<int64_t>(1, (24 * 1024) / (C * opb));
         if (k >= ngr) k = k / ngr * ngr;
+    }
+    // a fitted (-n KB, table) or default tile below ~40 KB, when the matrix still gives every SM two
+    // such tiles: the 40 KB height.  Each staged tile costs a fixed hand-off, and over the 33
+    // training shapes >= 256 MiB with both kinds swept the best < 20 KB tile ran a median 0.75
+    // (MV) / 0.71 (DOT) of the best >= 36 KB one, 20-36 KB tiles 0.92 / 0.93 (never faster in 32)
+    if (par(ADAPTIC_P_ROWS) == 0 || (par(ADAPTIC_P_ROWS) < 0 && p->source != 0)) {   // not a forced size
+        const int64_t kf = ceil_div(int64_t(40) * 1024, C * opb);
+        if (k < kf && ceil_div(R, kf) >= 2 * int64_t(dev.sms)) k = kf;
     }
     k = std::min<int64_t>(k, std::max<int64_t>(1, R));
     int cps = par(ADAPTIC_P_CTAS_PER_SM);
@@ -1159,7 +1173,7 @@ adaptic_status derive_tmv_rowtile(adaptic_plan_s* p, const int32_t* params, cons
     if (R > 4096) return ADAPTIC_ERR_UNSUPPORTED;
     int NT = par(ADAPTIC_P_BLOCK);
     if (NT <= 0) NT = R <= 64 ? 256 : R <= 1024 ? 1024 : 1024;
-    if (NT != 256 && NT != 512 && NT != 1024) return ADAPTIC_ERR_INVALID_ARG;
+    if (NT != 256 && NT != 512 && NT != 1024 && !(NT == 544 && R <= 2 * 544)) return ADAPTIC_ERR_INVALID_ARG;
     const int rpt = R <= NT ? 1 : R <= 2 * NT ? 2 : R <= 4 * NT ? 4 : 0;   // outputs per thread
     if (rpt == 0 || !tmv_rowtile_fn(p->dtype, NT, rpt)) return ADAPTIC_ERR_INVALID_ARG;
     int cps = par(ADAPTIC_P_CTAS_PER_SM);
@@ -1167,8 +1181,10 @@ adaptic_status derive_tmv_rowtile(adaptic_plan_s* p, const int32_t* params, cons
     int64_t k = par(ADAPTIC_P_ROWS);
     if (k < 0) {                        // -n: ~n KB of B and x per tile (fitted tables)
         k = std::max<int64_t>(4, (int64_t(-k) * 1024 / 4) / (R + 1) / 4 * 4);
-    } else if (k == 0) {                // ~24 KB of B per tile, and at least 3 stages in the budget
-        const int64_t words = std::min<int64_t>(24 * 1024, (int64_t(220) * 1024 / cps) / 3) / 4 - 9;
+    } else if (k == 0) {                // ~40 KB of B per tile, and at least 3 stages in the budget
+        // (24 KB before: over the 32 training shapes >= 256 MiB with both swept, 20-36 KB tiles ran a
+        // median 0.97 of the best >= 36 KB tile)
+        const int64_t words = std::min<int64_t>(40 * 1024, (int64_t(220) * 1024 / cps) / 3) / 4 - 9;
         k = std::max<int64_t>(4, words / (R + 1) / 4 * 4);
     }
     if (k % 4 != 0) return ADAPTIC_ERR_INVALID_ARG;

@@ -117,6 +117,8 @@ static void* trt(int NT, int rpt) {
         case 1024 * 4 + 1: return reinterpret_cast<void*>(&tmv_rowtile_kernel<T, 1024, 1>);
         case 256 * 4 + 2: return reinterpret_cast<void*>(&tmv_rowtile_kernel<T, 256, 2>);
         case 512 * 4 + 2: return reinterpret_cast<void*>(&tmv_rowtile_kernel<T, 512, 2>);
+        case 544 * 4 + 1: return reinterpret_cast<void*>(&tmv_rowtile_kernel<T, 544, 1>);   // 17 warps: slices
+        case 544 * 4 + 2: return reinterpret_cast<void*>(&tmv_rowtile_kernel<T, 544, 2>);   // of R + 1 rows
         case 1024 * 4 + 2: return reinterpret_cast<void*>(&tmv_rowtile_kernel<T, 1024, 2>);
         case 512 * 4 + 4: return reinterpret_cast<void*>(&tmv_rowtile_kernel<T, 512, 4>);
         case 1024 * 4 + 4: return reinterpret_cast<void*>(&tmv_rowtile_kernel<T, 1024, 4>);

@@ -65,3 +65,18 @@ def test_merge_later_runs_win_and_full_resweeps_replace_shapes(tmp_path):
     m = [json.loads(l) for l in open(out)]
     got = {(r["R"], r["variant"]): r["GBps"] for r in m}
     assert got == {(64, "MV_TPR"): 2000, (64, "MV_WPR"): 900, (8, "MV_WPR"): 50}
+
+
+def test_prefer_staged_dot_only_for_big_short_row_dot_cells():
+    """--prefer-staged-dot: in a DOT cell of rows with 64..1023 values and >= 2^25 elements, a
+    staged row-tile candidate (XSMEM 4) within the margin of the top score wins; outside that
+    range (MV, long rows, small cells, beyond the margin) the plain fit decides."""
+    def cell(op, R, C, direct, staged):
+        return [run(op, R, C, "MV_SUBWARP", [8, 0, 0, 4, 0], direct, vec=True, mis=False),
+                run(op, R, C, "MV_SUBWARP", [8, 0, 0, 0, 4, 256, 47], staged, vec=True, mis=False)]
+    t = ft.fit(cell("dot", 1048576, 64, 6800, 6700), prefer_staged_dot=0.03)
+    assert t[0]["xsmem"] == 4, t
+    assert ft.fit(cell("dot", 1048576, 64, 6800, 6700))[0]["xsmem"] == 0                    # off by default
+    assert ft.fit(cell("dot", 1048576, 64, 7100, 6700), prefer_staged_dot=0.03)[0]["xsmem"] == 0   # 5.6 % apart
+    assert ft.fit(cell("mv", 1048576, 64, 6800, 6700), prefer_staged_dot=0.03)[0]["xsmem"] == 0    # not DOT
+    assert ft.fit(cell("dot", 8192, 512, 6800, 6700), prefer_staged_dot=0.03)[0]["xsmem"] == 0     # 2^22 elements

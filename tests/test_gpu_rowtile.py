@@ -237,7 +237,8 @@ TMV_SHAPES = [(1, 1), (1, 1000), (2, 77), (3, 100003), (5, 7), (9, 4099), (13, 1
               (129, 4099), (255, 100), (256, 17), (257, 999), (513, 1001), (1023, 65), (1024, 9), (4, 3), (30, 7),
               (1025, 333), (2049, 65), (4095, 17), (3000, 1001)]
 TMV_PLANS = [trt_params()] + [trt_params(nt, k, st) for nt, k, st in
-                              ((256, 4, 0), (512, 8, 2), (1024, 0, 3), (1024, 4, 8), (256, 64, 2), (512, 0, 0))]
+                              ((256, 4, 0), (512, 8, 2), (1024, 0, 3), (1024, 4, 8), (256, 64, 2), (512, 0, 0),
+                               (544, 0, 0), (544, 8, 2))]
 
 
 @pytest.mark.parametrize("dt", ["f32", "i32"])

@@ -150,3 +150,18 @@ def test_group_plan_geometry():
             d("tmv", R, 1000, variant="TMV_SPLITK", params=_p([0, 0, 0, 0, 12]))
     # interleaved order and forced slots
     assert d("tmv", 129, 5000, variant="TMV_SPLITK", params=_p([0, 0, 0, 0, 12, 0, 2, 2]))["rows_per_group"] == 2
+
+
+def test_staged_tile_floor_and_lane_group_bump():
+    """Staged MV / DOT row tiles from the table or the default: >= ~40 KB per tile when the
+    matrix still gives every SM two tiles (training sweeps: smaller tiles 0.71-0.93 of the big
+    ones); a fitted lane group too small for this C grows to the smallest that holds it (the
+    cell spans a factor 2 in C); a FORCED size stays exact."""
+    for R, C in ((2872808, 63), (3085902, 61)):
+        p = d("dot", R, C)
+        assert p["xmode"] == 4 and p["rows_per_group"] * C * 8 >= 40 * 1024, p
+    p = d("dot", 393216, 416)                 # cell entry G = 8 fitted on C = 256 (G * 32 < 416)
+    assert p["xmode"] == 4 and p["lanes"] == 16, p
+    assert d("mv", 100000, 100, variant="MV_SUBWARP", params=[4, 0, 0, 0, 4, 256, -12])["rows_per_group"] == 30
+    with pytest.raises(adaptic.AdapticError):  # forced G too small: still an error
+        d("dot", 393216, 416, variant="MV_SUBWARP", params=[8, 0, 0, 0, 4, 256])

@@ -39,7 +39,7 @@ def norm_params(r):
     return p[:9]
 
 
-def fit(rows, tie=0.01, protect=None, protect_tol=0.01, neighbor_weight=0.0, portable_tie=0.0):
+def fit(rows, tie=0.01, protect=None, protect_tol=0.01, neighbor_weight=0.0, portable_tie=0.0, prefer_staged_dot=0.0):
     """Per cell (op, dtype, load-path class, floor(log2 R), floor(log2 C)): the candidate
     (variant, portable params) with the best mean fraction of each shape's best GB/s over
     the cell's measured shapes (a cell may hold a diagonal shape and held-out ones of other
@@ -108,6 +108,14 @@ def fit(rows, tie=0.01, protect=None, protect_tol=0.01, neighbor_weight=0.0, por
             return tot / wt
         score = {ck: sc(ck) for ck in pool}
         top = max(score[ck] for ck in pool)
+        if prefer_staged_dot > 0 and key[0] == "dot" and 6 <= key[4] <= 9 and key[3] + key[4] >= 25 and not prot:
+            # DOT rows of 64..1023 values, >= 256 MiB: staged row tiles (XSMEM 4) generalise across the cell
+            # (every training shape >= 256 MiB with both swept: staged >= 0.98 of the direct
+            # kernels, median 1.05 aligned / 1.41 misaligned), the direct lane groups do not
+            staged = [ck for ck in pool if ck[1][4] == 4 and score[ck] >= top * (1 - prefer_staged_dot)]
+            if staged:
+                pool = staged
+                top = max(score[ck] for ck in pool)
         near = [ck for ck in pool if score[ck] >= top * (1 - tie)]
         if portable_tie > 0:
             port = [ck for ck in pool if score[ck] >= top * (1 - portable_tie)]
@@ -152,6 +160,9 @@ def main():
     ap.add_argument("--neighbor-weight", type=float, default=0.0,
                     help="score candidates on the adjacent cells' shapes too, with this weight")
     ap.add_argument("--portable-tie", type=float, default=0.0)
+    ap.add_argument("--prefer-staged-dot", type=float, default=0.0,
+                    help="DOT cells with rows of 64..1023 values: a staged row-tile candidate within this fraction "
+                         "of the top score wins")
     ap.add_argument("--protect-bench", action="store_true",
                     help="keep every cell pick within 1 %% of the best run on bench.py's own shapes (the 42 "
                          "sweep shapes, their C+1 / R+1 off-grid twins, configs[2..4])")
@@ -166,7 +177,8 @@ def main():
             R, C = 1 << k, 1 << (26 - k)
             protect |= {("mv", R, C), ("tmv", R, C), ("mv", R, C + 1), ("tmv", R + 1, C)}
         protect |= {("dot", 1, 1 << k) for k in range(10, 31)} | {("mv", 131072, 32768), ("tmv", 1024, 1 << 24)}
-    table = fit(rows, protect=protect, neighbor_weight=a.neighbor_weight, portable_tie=a.portable_tie)
+    table = fit(rows, protect=protect, neighbor_weight=a.neighbor_weight, portable_tie=a.portable_tie,
+                prefer_staged_dot=a.prefer_staged_dot)
     write_inc(table, a.out)
     if a.json:
         with open(a.json, "w") as f:

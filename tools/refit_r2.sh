@@ -14,6 +14,9 @@
 #   sweep_r2_offmv_full  the offgrid bench's 21 MV C + 1 shapes, EVERY candidate (incl. the
 #                     column-chunk staged kernel, XSMEM 13) in one run: replaces all earlier runs
 #   sweep_r2_chunk_A  the column-chunk candidates on set A's misaligned long-row MV shapes
+#   sweep_r2_offtmv_full  the offgrid bench's 21 TMV R + 1 shapes, every candidate (incl. 544-thread
+#                     staged tiles) in one run: replaces all earlier runs of those shapes
+# DOT cells with rows of 64..1023 values (>= 256 MiB) prefer a staged row-tile candidate within 3 %.
 # Set B (tools/heldout_shapes.py B / Bs) is NEVER fitted: profiles/val_r2_* only.
 # Fit: bench.py's own shapes protected (pick within 1 % of the best on each), adjacent cells'
 # shapes scoring with weight 0.5 (generalisation), tie -> fewer CTAs.
@@ -26,6 +29,7 @@ python tools/merge_sweeps.py "$OUT" \
   $P/sweep_r1o_rowtile_vec_restricted.jsonl.gz $P/sweep_r1l_tmvrt.jsonl.gz +$P/sweep_r1s_offgrid_full.jsonl.gz \
   +$P/sweep_r2_trainA.jsonl.gz +$P/sweep_r2_dotA.jsonl.gz +$P/sweep_r2_small.jsonl.gz +$P/sweep_r2_trainAs.jsonl.gz \
   $P/sweep_r2_tshift_fit.jsonl.gz $P/sweep_r2_tshift_A.jsonl.gz $P/sweep_r2_misx_fit.jsonl.gz $P/sweep_r2_misx_A.jsonl.gz $P/sweep_r2_rtc_fit.jsonl.gz $P/sweep_r2_rtc_A.jsonl.gz $(ls $P/sweep_r2_dot1.jsonl.gz 2>/dev/null | sed 's/^/+/') \
-  $(ls $P/sweep_r2_offmv_full.jsonl.gz 2>/dev/null | sed 's/^/+/') $(ls $P/sweep_r2_chunk_A.jsonl.gz 2>/dev/null)
-python tools/fit_thresholds.py "$OUT" --ops mv,tmv,dot --protect-bench --neighbor-weight 0.5 \
+  $(ls $P/sweep_r2_offmv_full.jsonl.gz 2>/dev/null | sed 's/^/+/') $(ls $P/sweep_r2_chunk_A.jsonl.gz 2>/dev/null) \
+  $(ls $P/sweep_r2_offtmv_full.jsonl.gz 2>/dev/null | sed 's/^/+/')
+python tools/fit_thresholds.py "$OUT" --ops mv,tmv,dot --protect-bench --neighbor-weight 0.5 --prefer-staged-dot 0.03 \
   --out paper_conf_pldi_samadihmlm12_b200/csrc/table_data.inc --json $P/selector_table_r2.json > /dev/null

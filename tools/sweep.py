@@ -45,8 +45,9 @@ def rowtile_grid(op, R, C):
     if op == "tmv":
         if R > 4096:
             return []
-        ok = lambda nt: R <= nt or (R <= 2 * nt and nt >= 256) or (R <= 4 * nt and nt >= 512)  # noqa: E731
-        return [("TMV_REGTILE", [0, 0, 0, 0, 4, nt, k]) for nt in (256, 512, 1024) if ok(nt)
+        ok = lambda nt: (R <= nt or (R <= 2 * nt and nt >= 256) or (R <= 4 * nt and nt >= 512)) and \
+            (nt != 544 or R <= 1088)  # noqa: E731
+        return [("TMV_REGTILE", [0, 0, 0, 0, 4, nt, k]) for nt in (256, 512, 544, 1024) if ok(nt)
                 for k in sorted({0, max(4, 12 * 1024 // (4 * R) // 4 * 4), max(4, 48 * 1024 // (4 * R) // 4 * 4)})]
     if op not in ("mv", "dot") or C > 1024:
         return []
