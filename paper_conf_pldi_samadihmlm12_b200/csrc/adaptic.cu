@@ -1624,8 +1624,9 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
                                               : pick_splits(tiles, slots, std::max<int64_t>(1, ceil_div(C, int64_t(LC) * U)), 1);
         for (;;) {
             const int64_t iters = ceil_div(ceil_div(C, S), int64_t(LC) * U);
-            p->chain[1] = fold_chain(iters);
-            p->depth[1] = ilog2c(U) + LC + (S > 1 ? ceil_div(S, 2) + 1 : 0) + 1;
+            const int NA = U > 4 ? 2 : U;          // accumulators per thread (tmv_shift_kernel)
+            p->chain[1] = fold_chain(iters * (U / NA));
+            p->depth[1] = ilog2c(NA) + LC + (S > 1 ? ceil_div(S, 2) + 1 : 0) + 1;
             p->path_ok[1] = (dt == DT_I32) || bound_ok(p->chain[1] + p->depth[1]);
             if (p->path_ok[1] || S >= (int64_t(1) << 20)) break;
             S *= 2;

@@ -9,7 +9,9 @@ of timing; 'best fixed' = the fastest of every swept (variant, params) on that s
   2. round-2 table on held-out set B (3/13 multipliers + random, never fitted), >= 256 MiB;
   3. round-2 table on held-out set Bs, the paper's small-input regime (4-64 MiB, CUDA-graph
      device timing; gate: within 5 % of the best fixed only -- these inputs live in L2);
-  4. the offline replica (tools/select_sim.py) on the same sets, as a cross-check.
+  4. the offline replica (tools/select_sim.py) on the same sets, as a cross-check;
+  2c / 3c. the clean sets C / Cs, defined after the last table / planner change (section 2 and 3's
+     set B located the failures that the end-of-round planner rules address).
 
   python tools/selector_report_r2.py --out profiles/r2_selector_report.md
 """
@@ -52,12 +54,18 @@ def main():
                  "in alignment mod 16 and the misaligned-row DOT kernels (which need equal alignment) fell back "
                  "to scalar loads: those DOT rows understate both AUTO and the best fixed.\n\n```\n")
     parts.append(report([os.path.join(P, "sweep_r2_trainA.jsonl.gz")]).splitlines()[-2] + "\n```\n")
-    parts.append("## 2. Final round-2 table, held-out set B (never fitted), >= 256 MiB, every candidate and AUTO "
-                 "in ONE run (`val_r2_B_final`, final code)\n\n")
+    parts.append("## 2. Round-2 table before the end-of-round planner rules (code of commit 8a83827), held-out set "
+                 "B (never fitted), >= 256 MiB, every candidate and AUTO in ONE run (`val_r2_B_final`)\n\n")
     parts.append(report([os.path.join(P, "val_r2_B_final.jsonl.gz")]))
-    parts.append("\n## 3. Final round-2 table, held-out small set Bs (4-64 MiB, device-timed from CUDA graphs, one "
+    parts.append("\n## 3. The same code, held-out small set Bs (4-64 MiB, device-timed from CUDA graphs, one "
                  "run: `val_r2_Bs_final`)\n\n")
     parts.append(report([os.path.join(P, "val_r2_Bs_final.jsonl.gz"), "--min-bytes", "0", "--no-peak-gate"]))
+    parts.append("\n## 2c. CLEAN held-out set C (9 / 11 multipliers + 24 random shapes, new seed; defined AFTER the "
+                 "last table and planner change of round 2 and measured once, every candidate and AUTO in one run: "
+                 "`val_r2_C_final`), >= 256 MiB\n\n")
+    parts.append(report([os.path.join(P, "val_r2_C_final.jsonl.gz")]))
+    parts.append("\n## 3c. CLEAN held-out small set Cs (4-64 MiB, graph-timed, one run: `val_r2_Cs_final`)\n\n")
+    parts.append(report([os.path.join(P, "val_r2_Cs_final.jsonl.gz"), "--min-bytes", "0", "--no-peak-gate"]))
     parts.append("\n## 3b. The same table's AUTO picks timed in another run against the earlier sweeps' best "
                  "fixed (`val_r2_valB3_auto` vs `val_r2_heldoutB_nodot` + DOT / tshift / misx / rtc / chunk "
                  "sweeps): cross-run timing, so a ~1 % box-to-box shift moves borderline shapes\n\n```\n")
