@@ -1617,7 +1617,10 @@ adaptic_status derive(adaptic_plan_s* p, const int32_t* params, const DevInfo& d
         if (!tmv_shift_fn(dt, LR, U)) return ADAPTIC_ERR_INVALID_ARG;
         const int NT = 256, LC = NT / LR, WT = 4 * LR - 4;
         int cps = par(ADAPTIC_P_CTAS_PER_SM);
-        if (cps <= 0) cps = occupancy(tmv_shift_fn(dt, LR, U), NT, 0, dev.present, 2048 / NT);
+        // 3 resident CTAs fit since the kernel keeps 2 accumulators at U = 8 (76 registers); they
+        // pay off for R < 4096 (2049 x 32768: 0.89 -> 0.94 of peak) and cost 8-13 % above, where
+        // more CTAs only add c-splits (16385 x 4096: 0.955 at 2, 0.84 at 3; profiles/r2_exp/r2p_tshift_cmp.jsonl)
+        if (cps <= 0) cps = std::min(R < 4096 ? 3 : 2, occupancy(tmv_shift_fn(dt, LR, U), NT, 0, dev.present, 2));
         const int64_t slots = int64_t(dev.sms) * cps;
         const int64_t tiles = ceil_div(R, int64_t(WT));
         int64_t S = par(ADAPTIC_P_SPLITS) > 0 ? par(ADAPTIC_P_SPLITS)

@@ -162,7 +162,7 @@ namespace adaptic {
 // Tiling, splits and the ticket merge as tmv_kernel; B's first / last 16 bytes are loaded
 // word by word (ld_inside).
 template <class T, int LR, int U, int NT>
-__global__ void __launch_bounds__(NT, U <= 2 ? 4 : U <= 4 ? 3 : 2)
+__global__ void __launch_bounds__(NT, U <= 2 ? 4 : 3)
 tmv_shift_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restrict__ y,
                  int64_t R, int64_t C, int S, T* __restrict__ ws_part, unsigned int* __restrict__ ws_cnt)
 {
@@ -189,9 +189,11 @@ tmv_shift_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restrict
         const int64_t ob = tile * WT;
         const int64_t c0 = int64_t(s) * chunk;
         const int64_t c1 = min(C, c0 + chunk);
-        E acc[U];
+        // NA accumulators (U loads in flight): U = 8 keeps 2, so the 8 loads fit 3 CTAs per SM
+        constexpr int NA = U > 4 ? 2 : U;
+        E acc[NA];
 #pragma unroll
-        for (int u = 0; u < U; ++u) acc[u] = zero_of<E>();
+        for (int u = 0; u < NA; ++u) acc[u] = zero_of<E>();
         E outer = zero_of<E>();
         int it = 0;
         int64_t c = c0 + lc;
@@ -201,11 +203,14 @@ tmv_shift_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restrict
             const int64_t qf = ((b0 + c * R + ob) >> 2) + lr;
             const int64_t ql = ((b0 + (c + int64_t(LC) * (U - 1)) * R + ob) >> 2) + lr;
             if (4 * qf - b0 >= 0 && 4 * ql - b0 + 3 < total) {
+                // LC % 4 == 0: row c + LC u starts LC R / 4 vectors after row c, exactly
+                const E* pa = Ba + qf;
+                const int64_t sv = int64_t(LC) * R / 4;
+                const T* px = X + c;
 #pragma unroll
                 for (int u = 0; u < U; ++u) {
-                    const int64_t cc = c + int64_t(LC) * u;
-                    a[u] = ld_stream(Ba + ((b0 + cc * R + ob) >> 2) + lr);
-                    xs[u] = ld_x(X + cc);
+                    a[u] = ld_stream(pa + sv * u);
+                    xs[u] = ld_x(px + LC * u);
                 }
             } else {
 #pragma unroll
@@ -216,17 +221,17 @@ tmv_shift_kernel(const T* __restrict__ B, const T* __restrict__ X, T* __restrict
                 }
             }
 #pragma unroll
-            for (int u = 0; u < U; ++u) esmac(acc[u], a[u], xs[u]);
-            if (++it == FOLD) {
+            for (int u = 0; u < U; ++u) esmac(acc[u % NA], a[u], xs[u]);
+            if (++it == FOLD * NA / U) {                  // <= FOLD products per accumulator
                 it = 0;
-                outer = eadd(outer, tree_sum<U>(acc));
+                outer = eadd(outer, tree_sum<NA>(acc));
 #pragma unroll
-                for (int u = 0; u < U; ++u) acc[u] = zero_of<E>();
+                for (int u = 0; u < NA; ++u) acc[u] = zero_of<E>();
             }
         }
         for (; c < c1; c += LC)
             esmac(acc[0], ld_inside(Ba, B, ((b0 + c * R + ob) >> 2) + lr, b0, total), ld_x(X + c));
-        const E tot = eadd(outer, tree_sum<U>(acc));
+        const E tot = eadd(outer, tree_sum<NA>(acc));
         T* rl = red + lc * 4 * LR + 4 * lr;
         rl[0] = tot.x; rl[1] = tot.y; rl[2] = tot.z; rl[3] = tot.w;
         __syncthreads();
