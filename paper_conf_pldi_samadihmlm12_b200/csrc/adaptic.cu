@@ -1177,7 +1177,9 @@ adaptic_status derive_tmv_rowtile(adaptic_plan_s* p, const int32_t* params, cons
     const int rpt = R <= NT ? 1 : R <= 2 * NT ? 2 : R <= 4 * NT ? 4 : 0;   // outputs per thread
     if (rpt == 0 || !tmv_rowtile_fn(p->dtype, NT, rpt)) return ADAPTIC_ERR_INVALID_ARG;
     int cps = par(ADAPTIC_P_CTAS_PER_SM);
-    if (cps <= 0) cps = 1024 / NT;
+    // 17-warp CTAs: one per SM up to R = 256, two above (544 threads, 513 x 131072: 0.80 -> 0.85
+    // back to back; below 256 the single CTA was 1-2 % ahead, profiles/r2_exp/r2m_tmv544_cmp.jsonl)
+    if (cps <= 0) cps = NT == 544 ? (R > 256 ? 2 : 1) : 1024 / NT;
     int64_t k = par(ADAPTIC_P_ROWS);
     if (k < 0) {                        // -n: ~n KB of B and x per tile (fitted tables)
         k = std::max<int64_t>(4, (int64_t(-k) * 1024 / 4) / (R + 1) / 4 * 4);

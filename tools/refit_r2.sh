@@ -16,6 +16,8 @@
 #   sweep_r2_chunk_A  the column-chunk candidates on set A's misaligned long-row MV shapes
 #   sweep_r2_offtmv_full  the offgrid bench's 21 TMV R + 1 shapes, every candidate (incl. 544-thread
 #                     staged tiles) in one run: replaces all earlier runs of those shapes
+#   sweep_r2_offtmv_full2 the same shapes re-swept after the constant-shift TMV change (2 accumulators,
+#                     3 CTAs below R = 4096) and the 544-thread CTA count rule: replaces _full's runs
 # DOT cells with rows of 64..1023 values (>= 256 MiB) prefer a staged row-tile candidate within 3 %.
 # Set B (tools/heldout_shapes.py B / Bs) is NEVER fitted: profiles/val_r2_* only.
 # Fit: bench.py's own shapes protected (pick within 1 % of the best on each), adjacent cells'
@@ -30,6 +32,6 @@ python tools/merge_sweeps.py "$OUT" \
   +$P/sweep_r2_trainA.jsonl.gz +$P/sweep_r2_dotA.jsonl.gz +$P/sweep_r2_small.jsonl.gz +$P/sweep_r2_trainAs.jsonl.gz \
   $P/sweep_r2_tshift_fit.jsonl.gz $P/sweep_r2_tshift_A.jsonl.gz $P/sweep_r2_misx_fit.jsonl.gz $P/sweep_r2_misx_A.jsonl.gz $P/sweep_r2_rtc_fit.jsonl.gz $P/sweep_r2_rtc_A.jsonl.gz $(ls $P/sweep_r2_dot1.jsonl.gz 2>/dev/null | sed 's/^/+/') \
   $(ls $P/sweep_r2_offmv_full.jsonl.gz 2>/dev/null | sed 's/^/+/') $(ls $P/sweep_r2_chunk_A.jsonl.gz 2>/dev/null) \
-  $(ls $P/sweep_r2_offtmv_full.jsonl.gz 2>/dev/null | sed 's/^/+/')
+  $(ls $P/sweep_r2_offtmv_full.jsonl.gz 2>/dev/null | sed 's/^/+/') $(ls $P/sweep_r2_offtmv_full2.jsonl.gz 2>/dev/null | sed 's/^/+/')
 python tools/fit_thresholds.py "$OUT" --ops mv,tmv,dot --protect-bench --neighbor-weight 0.5 --prefer-staged-dot 0.03 \
   --out paper_conf_pldi_samadihmlm12_b200/csrc/table_data.inc --json $P/selector_table_r2.json > /dev/null
