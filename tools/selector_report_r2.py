@@ -61,11 +61,11 @@ def main():
                  "run: `val_r2_Bs_final`)\n\n")
     parts.append(report([os.path.join(P, "val_r2_Bs_final.jsonl.gz"), "--min-bytes", "0", "--no-peak-gate"]))
     parts.append("\n## 2c. CLEAN held-out set C (9 / 11 multipliers + 24 random shapes, new seed; defined AFTER the "
-                 "last table and planner change of round 2 and measured once, every candidate and AUTO in one run: "
-                 "`val_r2_C_final`), >= 256 MiB\n\n")
-    parts.append(report([os.path.join(P, "val_r2_C_final.jsonl.gz")]))
-    parts.append("\n## 3c. CLEAN held-out small set Cs (4-64 MiB, graph-timed, one run: `val_r2_Cs_final`)\n\n")
-    parts.append(report([os.path.join(P, "val_r2_Cs_final.jsonl.gz"), "--min-bytes", "0", "--no-peak-gate"]))
+                 "last planner change of round 2, every candidate and AUTO of a shape in one run; its TMV shapes "
+                 "re-swept after the last refit of the misaligned TMV cells: `val_r2_C_final2`), >= 256 MiB\n\n")
+    parts.append(report([os.path.join(P, "val_r2_C_final2.jsonl.gz")]))
+    parts.append("\n## 3c. CLEAN held-out small set Cs (4-64 MiB, graph-timed, TMV re-swept likewise: `val_r2_Cs_final2`)\n\n")
+    parts.append(report([os.path.join(P, "val_r2_Cs_final2.jsonl.gz"), "--min-bytes", "0", "--no-peak-gate"]))
     parts.append("\n## 3b. The same table's AUTO picks timed in another run against the earlier sweeps' best "
                  "fixed (`val_r2_valB3_auto` vs `val_r2_heldoutB_nodot` + DOT / tshift / misx / rtc / chunk "
                  "sweeps): cross-run timing, so a ~1 % box-to-box shift moves borderline shapes\n\n```\n")
