@@ -1778,6 +1778,20 @@ adaptic_status make_plan(int op, int64_t rows, int64_t cols, int dtype, int vari
         int32_t tp[ADAPTIC_NPARAMS] = {e->lanes, projected ? 0 : e->splits, projected ? 0 : e->ctas_per_sm, e->unroll,
                                        e->xsmem, e->block, e->rows, e->order, e->pipe};
         p->variant = e->variant; p->source = 1;
+        // rows off the 16-byte grid, 1024 <= R <= 2^17, >= 2^24 elements: a cell that kept the
+        // funnel kernel (fitted on a smaller or older-kernel shape) runs the constant-shift kernel
+        // (every such training shape with both swept: constant shift 1.03-1.19x the funnel,
+        // median 1.14, 15 of 15)
+        if (op == ADAPTIC_OP_TMV && rows % 4 != 0 && rows >= 1024 && rows <= (int64_t(1) << 17) &&
+            rows * cols >= (int64_t(1) << 24) && e->xsmem == 0 &&
+            (e->variant == ADAPTIC_V_TMV_SPLITK || e->variant == ADAPTIC_V_TMV_COL)) {
+            int32_t ts[ADAPTIC_NPARAMS] = {0};
+            ts[ADAPTIC_P_UNROLL] = 8;
+            ts[ADAPTIC_P_XSMEM] = 7;
+            p->variant = ADAPTIC_V_TMV_SPLITK;
+            if (derive(p, ts, dev) == ADAPTIC_OK) { *out = p; return ADAPTIC_OK; }
+            p->variant = e->variant;
+        }
         if (derive(p, tp, dev) == ADAPTIC_OK) { *out = p; return ADAPTIC_OK; }
         if (derive(p, nullptr, dev) == ADAPTIC_OK) { *out = p; return ADAPTIC_OK; }
     }

@@ -165,3 +165,14 @@ def test_staged_tile_floor_and_lane_group_bump():
     assert d("mv", 100000, 100, variant="MV_SUBWARP", params=[4, 0, 0, 0, 4, 256, -12])["rows_per_group"] == 30
     with pytest.raises(adaptic.AdapticError):  # forced G too small: still an error
         d("dot", 393216, 416, variant="MV_SUBWARP", params=[8, 0, 0, 0, 4, 256])
+
+
+def test_misaligned_tmv_funnel_cells_run_the_constant_shift_kernel():
+    """Rows off the 16-byte grid with 1024 <= R <= 2^17 and >= 2^24 elements: a table cell that
+    kept the funnel kernel (XSMEM 0) runs the constant-shift kernel (XSMEM 7) instead (training
+    sweeps: 1.03-1.19x, 15 of 15); small problems and aligned rows keep their fitted entry."""
+    for R, C in ((27215, 2924), (1950, 44236), (16385, 4096)):
+        p = d("tmv", R, C)
+        assert p["variant"] == "TMV_SPLITK" and p["xmode"] == 7, (R, C, p)
+    assert d("tmv", 1025, 1024)["xmode"] != 7              # 1 Mi elements: the fitted small-cell entry
+    assert d("tmv", 4772, 50180)["xmode"] != 7             # R % 4 == 0: the 128-bit path
