@@ -1786,6 +1786,9 @@ adaptic_status make_plan(int op, int64_t rows, int64_t cols, int dtype, int vari
             rows * cols >= (int64_t(1) << 24) && e->xsmem == 0 &&
             (e->variant == ADAPTIC_V_TMV_SPLITK || e->variant == ADAPTIC_V_TMV_COL)) {
             int32_t ts[ADAPTIC_NPARAMS] = {0};
+            // tile width as the offgrid R + 1 training sweep picked it (sweep_r2_offtmv_full2:
+            // 16 float4 lanes for R = 1025..4097, 32 for 8193..32769, 64 above)
+            ts[ADAPTIC_P_LANES] = rows < 8192 ? 16 : rows < 65536 ? 32 : 64;
             ts[ADAPTIC_P_UNROLL] = 8;
             ts[ADAPTIC_P_XSMEM] = 7;
             p->variant = ADAPTIC_V_TMV_SPLITK;
